@@ -1,0 +1,408 @@
+// The C ABI of libcme (include/cme.h): argument checks, call-order state
+// machine, host-side planning; device work is delegated to device.cu.
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "cme_internal.h"
+#include "comm.h"
+
+namespace cme {
+
+thread_local std::string g_err;
+void set_error(const std::string& msg) { g_err = msg; }
+
+struct Device;
+cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cme_comm_s* comm);
+void device_free(Device* d);
+cme_status device_solve(cme_matrix_s* h, const double* p0, double tol, int64_t max_iter, double* p_out,
+                        int64_t* iters_out);
+cme_status device_spmv(cme_matrix_s* h, const double* x, double* y);
+cme_status device_load(cme_matrix_s* h, const double* p0);
+cme_status device_run(cme_matrix_s* h, int64_t blocks);
+cme_status device_fetch(cme_matrix_s* h, double* p_out);
+
+namespace {
+
+template <typename F>
+cme_status guarded(F&& f) {
+    try {
+        return f();
+    } catch (const std::bad_alloc&) {
+        set_error("out of host memory");
+        return CME_ERR_OOM;
+    } catch (const std::exception& e) {
+        set_error(e.what());
+        return CME_ERR_INVALID_ARG;
+    }
+}
+
+int32_t ell_count(const Csr& B, int64_t r, bool band_on) {
+    int64_t k = B.rp[r + 1] - B.rp[r];
+    if (band_on)
+        for (int64_t p = B.rp[r]; p < B.rp[r + 1]; ++p) k -= (B.ci[p] == r - 1 || B.ci[p] == r + 1);
+    return (int32_t)k;
+}
+
+// Row range [r0, r1) and x-span of every rank; cuts at window multiples,
+// balanced by packed bytes.
+void plan_cuts(cme_matrix_s* h, int nranks) {
+    const Csr& B = h->B;
+    const int64_t n = B.n;
+    const int64_t unit = std::max<int64_t>(32, h->P.window > 1 ? h->P.window : 32);
+    std::vector<double> pre(n + 1, 0.0);
+    for (int64_t i = 0; i < n; ++i) pre[i + 1] = pre[i] + 12.0 * (double)(B.rp[i + 1] - B.rp[i]) + 28.0;
+    h->cuts.assign(nranks + 1, 0);
+    h->cuts[nranks] = n;
+    for (int r = 1; r < nranks; ++r) {
+        const double target = pre[n] * r / nranks;
+        int64_t i = std::lower_bound(pre.begin(), pre.end(), target) - pre.begin();
+        i = std::min<int64_t>(n, (i + unit / 2) / unit * unit);
+        h->cuts[r] = std::max(h->cuts[r - 1], i);
+    }
+    h->span.assign(2 * nranks, 0);
+    for (int r = 0; r < nranks; ++r) {
+        int64_t lo = h->cuts[r], hi = h->cuts[r + 1];
+        for (int64_t i = h->cuts[r]; i < h->cuts[r + 1]; ++i)
+            if (B.rp[i + 1] > B.rp[i]) {
+                lo = std::min<int64_t>(lo, B.ci[B.rp[i]]);
+                hi = std::max<int64_t>(hi, (int64_t)B.ci[B.rp[i + 1] - 1] + 1);
+            }
+        if (h->cuts[r] == h->cuts[r + 1]) lo = hi = h->cuts[r];
+        h->span[2 * r] = lo;
+        h->span[2 * r + 1] = hi;
+    }
+}
+
+HaloPlan halo_plan(const cme_matrix_s* h) {
+    HaloPlan p;
+    const int R = h->nranks, r = h->rank;
+    const int64_t lo = h->span[2 * r], hi = h->span[2 * r + 1];
+    for (int s = 0; s < R; ++s) {
+        if (s == r) continue;
+        // receive the part of s's own rows that falls in my span
+        int64_t a = std::max(lo, h->cuts[s]), b = std::min(hi, h->cuts[s + 1]);
+        if (a < b) { p.recv_peer.push_back(s); p.recv_off.push_back(a - lo); p.recv_cnt.push_back(b - a); }
+        // send the part of my own rows that falls in s's span
+        a = std::max(h->span[2 * s], h->cuts[r]);
+        b = std::min(h->span[2 * s + 1], h->cuts[r + 1]);
+        if (a < b) { p.send_peer.push_back(s); p.send_off.push_back(a - lo); p.send_cnt.push_back(b - a); }
+    }
+    return p;
+}
+
+cme_status build_local(cme_matrix_s* h, int nranks, int rank) {
+    h->nranks = nranks;
+    h->rank = rank;
+    const int64_t n = h->B.n;
+    if (nranks == 1) {
+        h->cuts = {0, n};
+        h->span = {0, n};
+    } else {
+        plan_cuts(h, nranks);
+    }
+    const int64_t r0 = h->cuts[rank], r1 = h->cuts[rank + 1], shift = h->span[2 * rank];
+    if (h->format == CME_FMT_CSR) {
+        pack_csr_rows(h->B, r0, r1, shift, h->P);
+    } else {
+        const bool ell = h->format == CME_FMT_ELL;
+        pack_rows(h->B, r0, r1, shift, ell ? 1 : h->popts.window, h->band_on, ell, h->global_kmax, h->P);
+    }
+    return CME_OK;
+}
+
+bool valid(cme_matrix h, int min_stage) { return h && h->stage >= min_stage; }
+
+}  // namespace
+}  // namespace cme
+
+using namespace cme;
+
+extern "C" {
+
+cme_status cme_matrix_create_coo(int64_t n, int64_t nnz, const int32_t* row, const int32_t* col,
+                                 const double* rate, uint32_t flags, cme_matrix* out) {
+    if (!out) return CME_ERR_INVALID_ARG;
+    *out = nullptr;
+    return guarded([&] {
+        auto* h = new cme_matrix_s();
+        cme_status s = ingest_coo(n, nnz, row, col, rate, flags, h->A);
+        if (s != CME_OK) { delete h; return s; }
+        h->perm.resize(n);
+        for (int64_t i = 0; i < n; ++i) h->perm[i] = (int32_t)i;
+        h->stage = 1;
+        *out = h;
+        return CME_OK;
+    });
+}
+
+cme_status cme_matrix_create_csr(int64_t n, const int64_t* row_ptr, const int32_t* col, const double* rate,
+                                 uint32_t flags, cme_matrix* out) {
+    if (!out || !row_ptr || n <= 0 || n > INT32_MAX) return CME_ERR_INVALID_ARG;
+    *out = nullptr;
+    return guarded([&] {
+        const int64_t nnz = row_ptr[n];
+        if (row_ptr[0] != 0 || nnz < 0) { set_error("row_ptr must start at 0"); return CME_ERR_INVALID_ARG; }
+        std::vector<int32_t> rows(nnz);
+        for (int64_t i = 0; i < n; ++i) {
+            if (row_ptr[i + 1] < row_ptr[i]) { set_error("row_ptr not monotone"); return CME_ERR_INVALID_ARG; }
+            for (int64_t p = row_ptr[i]; p < row_ptr[i + 1]; ++p) rows[p] = (int32_t)i;
+        }
+        return cme_matrix_create_coo(n, nnz, rows.data(), col, rate, flags, out);
+    });
+}
+
+cme_status cme_reorder(cme_matrix h, int method, int64_t root) {
+    if (!valid(h, 1)) return CME_ERR_INVALID_ARG;
+    if (h->stage != 1) { set_error("cme_reorder must precede cme_pack"); return CME_ERR_BAD_STATE; }
+    if (method < CME_ORDER_NONE || method > CME_ORDER_RCM) return CME_ERR_INVALID_ARG;
+    if (method == CME_ORDER_DFS && (root < 0 || root >= h->A.n)) return CME_ERR_INVALID_ARG;
+    return guarded([&] {
+        if (method == CME_ORDER_NONE) {
+            for (int64_t i = 0; i < h->A.n; ++i) h->perm[i] = (int32_t)i;
+        } else if (method == CME_ORDER_DFS) {
+            order_dfs(h->A, root, h->perm);
+        } else {
+            order_rcm(h->A, h->perm);
+        }
+        h->order = method;
+        return CME_OK;
+    });
+}
+
+cme_status cme_pack(cme_matrix h, int format, const cme_pack_opts* opts) {
+    if (!valid(h, 1)) return CME_ERR_INVALID_ARG;
+    if (h->stage == 3) { set_error("matrix already distributed"); return CME_ERR_BAD_STATE; }
+    cme_pack_opts o = opts ? *opts : cme_pack_opts{32, 256, CME_BAND_AUTO, -1};
+    if (format < CME_FMT_DIAG_SELL || format > CME_FMT_CSR || o.slice != 32 || o.band < 0 || o.band > 2 ||
+        o.window < 0 || o.window > (1 << 20) || o.device < CME_DEVICE_HOST_ONLY) {
+        set_error("pack: bad format or options (slice must be 32)");
+        return CME_ERR_INVALID_ARG;
+    }
+    return guarded([&] {
+        h->format = format;
+        h->popts = o;
+        bool identity = true;
+        for (int64_t i = 0; i < h->A.n && identity; ++i) identity = h->perm[i] == i;
+        if (identity) h->B = h->A;
+        else permute(h->A, h->perm, h->B);
+        h->period = directed_period(h->A, 0);
+        double na = 0.0;
+        for (int64_t i = 0; i < h->A.n; ++i) {
+            double s = std::fabs(h->A.d[i]);
+            for (int64_t p = h->A.rp[i]; p < h->A.rp[i + 1]; ++p) s += std::fabs(h->A.v[p]);
+            na = std::max(na, s);
+        }
+        h->norm_inf = na;
+        h->band_on = format != CME_FMT_CSR && band_rule(h->B, o.band);
+        int32_t kmax = 0;
+        for (int64_t i = 0; i < h->B.n; ++i) kmax = std::max(kmax, ell_count(h->B, i, h->band_on));
+        h->global_kmax = kmax;
+        build_local(h, 1, 0);
+        device_free(h->dev);
+        h->dev = nullptr;
+        if (o.device != CME_DEVICE_HOST_ONLY) {
+            cme_status s = device_upload(h, o.device, nullptr, nullptr);
+            if (s != CME_OK) return s;
+        }
+        h->stage = 2;
+        return CME_OK;
+    });
+}
+
+cme_status cme_set_solver_opts(cme_matrix h, const cme_solver_opts* o) {
+    if (!h) return CME_ERR_INVALID_ARG;
+    cme_solver_opts v = o ? *o : cme_solver_opts{0.0, 100, CME_STOP_DELTA_L1, 1e-10, nullptr};
+    if (!(v.omega >= 0.0 && v.omega <= 1.0) || v.check_every < 1 || v.stop < 0 || v.stop > 1 ||
+        !(v.stag_tol >= 0.0)) {
+        set_error("solver opts: omega in [0,1], check_every >= 1, stop in {0,1}, stag_tol >= 0");
+        return CME_ERR_INVALID_ARG;
+    }
+    h->sopts = v;
+    return CME_OK;
+}
+
+cme_status cme_jacobi_solve(cme_matrix h, const double* p0, double tol, int64_t max_iter, double* p_out,
+                            int64_t* iters_out) {
+    if (iters_out) *iters_out = 0;
+    if (!h || !p_out || max_iter < 0 || std::isnan(tol)) return CME_ERR_INVALID_ARG;
+    if (h->stage < 2 || !h->dev) { set_error("solve before pack/distribute"); return CME_ERR_BAD_STATE; }
+    return guarded([&] { return device_solve(h, p0, tol, max_iter, p_out, iters_out); });
+}
+
+cme_status cme_get_report(cme_matrix h, cme_report* r) {
+    if (!h || !r) return CME_ERR_INVALID_ARG;
+    *r = h->report;
+    return CME_OK;
+}
+
+cme_status cme_spmv(cme_matrix h, const double* x, double* y) {
+    if (!h || !x || !y) return CME_ERR_INVALID_ARG;
+    if (h->stage < 2 || !h->dev) return CME_ERR_BAD_STATE;
+    return guarded([&] { return device_spmv(h, x, y); });
+}
+
+cme_status cme_solver_load(cme_matrix h, const double* p0) {
+    if (!h) return CME_ERR_INVALID_ARG;
+    if (h->stage < 2 || !h->dev) return CME_ERR_BAD_STATE;
+    return guarded([&] { return device_load(h, p0); });
+}
+
+cme_status cme_solver_run(cme_matrix h, int64_t blocks) {
+    if (!h || blocks < 0) return CME_ERR_INVALID_ARG;
+    if (h->stage < 2 || !h->dev) return CME_ERR_BAD_STATE;
+    return guarded([&] { return device_run(h, blocks); });
+}
+
+cme_status cme_solver_fetch(cme_matrix h, double* p_out) {
+    if (!h || !p_out) return CME_ERR_INVALID_ARG;
+    if (h->stage < 2 || !h->dev) return CME_ERR_BAD_STATE;
+    return guarded([&] { return device_fetch(h, p_out); });
+}
+
+cme_status cme_get_info(cme_matrix h, cme_info* info) {
+    if (!h || !info || h->stage < 1) return CME_ERR_INVALID_ARG;
+    return guarded([&] {
+        cme_info f{};
+        const Csr& B = h->stage >= 2 ? h->B : h->A;
+        const int64_t n = h->A.n;
+        f.n = n;
+        f.nnz_offdiag = h->A.nnz();
+        f.nnz = f.nnz_offdiag + n;
+        int64_t bw = 0, band = 0;
+        for (int64_t i = 0; i < n; ++i)
+            for (int64_t p = B.rp[i]; p < B.rp[i + 1]; ++p) {
+                bw = std::max<int64_t>(bw, std::llabs(B.ci[p] - i));
+                band += (B.ci[p] == i - 1 || B.ci[p] == i + 1);
+            }
+        f.bandwidth = bw;
+        f.band_density = n > 1 ? (double)band / (double)(2 * n - 2) : 0.0;
+        f.band_density3 = (double)(band + n) / (double)(3 * n - 2);
+        f.format = h->format;
+        f.order = h->order;
+        f.band_on = h->band_on;
+        f.window = h->P.window;
+        f.period = h->stage >= 2 ? h->period : directed_period(h->A, 0);
+        f.norm_inf = h->norm_inf;
+        f.omega = h->sopts.omega > 0 ? h->sopts.omega : (f.period == 1 ? 1.0 : 0.9);
+        const Packed& P = h->P;
+        f.n_slots = P.n_slots;
+        f.n_slices = P.n_slices;
+        f.n_ell = P.n_ell;
+        int64_t ell_nz = 0;
+        for (double v : P.val) ell_nz += v != 0.0;
+        f.ell_efficiency = P.n_ell ? (double)ell_nz / (double)P.n_ell : 1.0;
+        const int64_t nl = P.n;
+        if (h->format == CME_FMT_CSR) {
+            f.packed_bytes = 8 * (int64_t)P.csr_rp.size() + 12 * (int64_t)P.csr_ci.size() + 8 * (int64_t)P.inv_d.size();
+            f.bytes_fmt = 12 * (int64_t)P.csr_ci.size() + 8 * (nl + 1) + 8 * nl + 16 * nl;
+        } else {
+            f.packed_bytes = 12 * P.n_ell + 8 * P.n_slots + (P.band_on ? 16 * P.n_slots : 0) +
+                             (P.window > 1 ? 4 * P.n_slots : 0) + 12 * P.n_slices + 8;
+            f.bytes_fmt = 12 * P.n_ell + 8 * nl + (P.band_on ? 16 * nl : 0) + (P.window > 1 ? 4 * nl : 0) +
+                          12 * P.n_slices + 16 * nl;
+        }
+        f.bytes_alg = 12 * f.nnz + 16 * n;
+        f.rank = h->rank;
+        f.nranks = h->nranks;
+        f.row_begin = h->cuts.empty() ? 0 : h->cuts[h->rank];
+        f.row_end = h->cuts.empty() ? n : h->cuts[h->rank + 1];
+        f.halo_begin = h->span.empty() ? 0 : h->span[2 * h->rank];
+        f.halo_end = h->span.empty() ? n : h->span[2 * h->rank + 1];
+        *info = f;
+        return CME_OK;
+    });
+}
+
+cme_status cme_get_permutation(cme_matrix h, int32_t* new_to_old) {
+    if (!h || !new_to_old || h->stage < 1) return CME_ERR_INVALID_ARG;
+    std::memcpy(new_to_old, h->perm.data(), h->perm.size() * sizeof(int32_t));
+    return CME_OK;
+}
+
+cme_status cme_export_packed(cme_matrix h, cme_packed_view* v) {
+    if (!h || !v) return CME_ERR_INVALID_ARG;
+    if (h->stage < 2) return CME_ERR_BAD_STATE;
+    const Packed& P = h->P;
+    cme_packed_view o{};
+    o.n = P.n; o.n_slots = P.n_slots; o.n_slices = P.n_slices; o.n_ell = P.n_ell;
+    o.band_on = P.band_on; o.window = P.window;
+    o.lo = P.lo.data(); o.up = P.up.data(); o.inv_d = P.inv_d.data(); o.row_of = P.row_of.data();
+    o.slice_off = P.slice_off.data(); o.slice_w = P.slice_w.data(); o.val = P.val.data(); o.col = P.col.data();
+    o.csr_row_ptr = h->format == CME_FMT_CSR ? P.csr_rp.data() : nullptr;
+    if (h->format == CME_FMT_CSR) { o.val = P.csr_v.data(); o.col = P.csr_ci.data(); o.n_ell = (int64_t)P.csr_ci.size(); }
+    *v = o;
+    return CME_OK;
+}
+
+cme_status cme_period(cme_matrix h, int64_t root, int64_t* out) {
+    if (!h || !out || h->stage < 1 || root < 0 || root >= h->A.n) return CME_ERR_INVALID_ARG;
+    return guarded([&] { *out = directed_period(h->A, root); return CME_OK; });
+}
+
+cme_status cme_matrix_plan_partition(cme_matrix h, int nranks, int rank) {
+    if (!h || nranks < 1 || rank < 0 || rank >= nranks) return CME_ERR_INVALID_ARG;
+    if (h->stage < 2) { set_error("plan_partition needs a packed matrix"); return CME_ERR_BAD_STATE; }
+    return guarded([&] {
+        build_local(h, nranks, rank);
+        if (nranks > 1) {  // the single-GPU device copy no longer matches
+            device_free(h->dev);
+            h->dev = nullptr;
+        }
+        return CME_OK;
+    });
+}
+
+cme_status cme_matrix_distribute(cme_matrix h, cme_comm c) {
+    if (!h || !c) return CME_ERR_INVALID_ARG;
+    if (h->stage < 2) { set_error("distribute needs a packed matrix"); return CME_ERR_BAD_STATE; }
+    return guarded([&] {
+        build_local(h, comm_nranks(c), comm_rank(c));
+        HaloPlan p = halo_plan(h);
+        cme_status s = device_upload(h, comm_device(c), &p, c);
+        if (s != CME_OK) return s;
+        h->comm = c;
+        h->stage = 3;
+        return CME_OK;
+    });
+}
+
+cme_status cme_export_halo(cme_matrix h, cme_halo_view* v) {
+    if (!h || !v || h->cuts.empty()) return CME_ERR_INVALID_ARG;
+    v->nranks = h->nranks;
+    v->rank = h->rank;
+    v->row_begin = h->cuts.data();
+    v->span = h->span.data();
+    return CME_OK;
+}
+
+void cme_matrix_destroy(cme_matrix h) {
+    if (!h) return;
+    device_free(h->dev);
+    delete h;
+}
+
+const char* cme_status_string(cme_status s) {
+    switch (s) {
+        case CME_OK: return "CME_OK";
+        case CME_ERR_INVALID_ARG: return "CME_ERR_INVALID_ARG";
+        case CME_ERR_NEGATIVE_RATE: return "CME_ERR_NEGATIVE_RATE";
+        case CME_ERR_ZERO_OUTFLOW: return "CME_ERR_ZERO_OUTFLOW";
+        case CME_ERR_BAD_STATE: return "CME_ERR_BAD_STATE";
+        case CME_ERR_OOM: return "CME_ERR_OOM";
+        case CME_ERR_CUDA: return "CME_ERR_CUDA";
+        case CME_ERR_NCCL: return "CME_ERR_NCCL";
+        case CME_NOT_CONVERGED: return "CME_NOT_CONVERGED";
+        case CME_STAGNATED: return "CME_STAGNATED";
+        case CME_ERR_NUMERIC: return "CME_ERR_NUMERIC";
+        case CME_ERR_NO_DEVICE: return "CME_ERR_NO_DEVICE";
+    }
+    return "CME_UNKNOWN";
+}
+
+const char* cme_last_error(void) { return g_err.c_str(); }
+int cme_abi_version(void) { return 1; }
+
+}  // extern "C"

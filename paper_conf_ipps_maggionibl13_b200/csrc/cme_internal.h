@@ -1,0 +1,83 @@
+// Internal declarations of libcme (not part of the ABI; see include/cme.h).
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "cme.h"
+
+namespace cme {
+
+// Thread-local error detail for cme_last_error().
+void set_error(const std::string& msg);
+
+// Off-diagonal part of A by rows (row i <- col j: transition j -> i) + diagonal.
+struct Csr {
+    int64_t n = 0;
+    std::vector<int64_t> rp;   // n + 1
+    std::vector<int32_t> ci;   // column indices, ascending within a row
+    std::vector<double> v;     // rates
+    std::vector<double> d;     // a_ii (< 0)
+    int64_t nnz() const { return rp.empty() ? 0 : rp.back(); }
+};
+
+// Ingest.  Returns CME_OK or an error status.
+cme_status ingest_coo(int64_t n, int64_t nnz, const int32_t* row, const int32_t* col,
+                      const double* rate, uint32_t flags, Csr& out);
+
+// Orderings and graph tests (R1, R11, R12).
+void order_dfs(const Csr& A, int64_t root, std::vector<int32_t>& new_to_old);
+void order_rcm(const Csr& A, std::vector<int32_t>& new_to_old);
+int64_t directed_period(const Csr& A, int64_t root);
+void permute(const Csr& A, const std::vector<int32_t>& new_to_old, Csr& out);
+
+// Packed layout v0 ("DIAG + warp-grained SELL") of rows
+// [r0, r1) of an ordered matrix, columns shifted by -col_shift.
+struct Packed {
+    int64_t n = 0, n_slots = 0, n_slices = 0, n_ell = 0;
+    int32_t band_on = 0, window = 1, uniform = 0;
+    std::vector<double> lo, up, inv_d;    // slot order
+    std::vector<int32_t> row_of;          // slot -> local row
+    std::vector<int64_t> slice_off;       // n_slices + 1
+    std::vector<int32_t> slice_w;         // n_slices
+    std::vector<double> val;              // n_ell
+    std::vector<int32_t> col;             // n_ell
+    // CSR arm
+    std::vector<int64_t> csr_rp;
+    std::vector<int32_t> csr_ci;
+    std::vector<double> csr_v;
+};
+bool band_rule(const Csr& A, int band_mode);
+void pack_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, int32_t window,
+               bool band_on, bool uniform, int32_t global_kmax, Packed& P);
+void pack_csr_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, Packed& P);
+
+struct Device;  // device state (device.cu)
+
+}  // namespace cme
+
+struct cme_comm_s;
+
+struct cme_matrix_s {
+    int stage = 0;              // 1 created, 2 packed, 3 distributed
+    cme::Csr A;                 // original order
+    int order = CME_ORDER_NONE;
+    std::vector<int32_t> perm;  // new_to_old
+    cme::Csr B;                 // reordered (valid after pack)
+    int format = CME_FMT_DIAG_SELL;
+    cme_pack_opts popts{32, 256, CME_BAND_AUTO, -1};
+    bool band_on = false;
+    int64_t period = 0;
+    double norm_inf = 0.0;
+    cme::Packed P;              // local packed layout (whole matrix unless distributed)
+    int32_t global_kmax = 0;
+    cme_solver_opts sopts{0.0, 100, CME_STOP_DELTA_L1, 1e-10, nullptr};
+    cme_report report{};
+    // partition
+    int nranks = 1, rank = 0;
+    std::vector<int64_t> cuts;  // nranks + 1
+    std::vector<int64_t> span;  // 2 * nranks
+    cme_comm_s* comm = nullptr;
+    cme::Device* dev = nullptr;
+};

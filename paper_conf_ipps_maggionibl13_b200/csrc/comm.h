@@ -1,0 +1,33 @@
+// NCCL glue for the row-sharded multi-GPU Jacobi.
+#pragma once
+#include <cstdint>
+#include <vector>
+#include <cuda_runtime.h>
+
+#include "cme.h"
+
+namespace cme {
+
+// Who sends which contiguous x range to whom after every step.  Offsets are
+// x-span indices of the local buffers (send: own rows; recv: halo slots).
+struct HaloPlan {
+    std::vector<int> send_peer, recv_peer;
+    std::vector<int64_t> send_off, send_cnt, recv_off, recv_cnt;
+    int64_t volume() const {
+        int64_t v = 0;
+        for (auto c : recv_cnt) v += c;
+        return v;
+    }
+};
+
+int comm_rank(const cme_comm_s* c);
+int comm_nranks(const cme_comm_s* c);
+int comm_device(const cme_comm_s* c);
+cme_status comm_halo(cme_comm_s* c, const HaloPlan& p, double* xspan, cudaStream_t s);
+// recv[r*8 .. r*8+7] = send8 of rank r
+cme_status comm_allgather8(cme_comm_s* c, const double* send8, double* recv, cudaStream_t s);
+// every rank r broadcasts buf[cuts[r], cuts[r+1]) to all ranks
+cme_status comm_bcast_segments(cme_comm_s* c, double* buf, const std::vector<int64_t>& cuts,
+                               cudaStream_t s);
+
+}  // namespace cme

@@ -1,0 +1,131 @@
+// Host packer: DIAG band + warp-grained sliced ELL with local rearrangement.
+//
+// Paper: ELL column-major arrays padded to a warp multiple, DIA for
+// the dense {-1,0,+1} band when its density beats 8 B / 12 B = 2/3,
+// sliced ELL with slice = warp decoupled from the block, rows
+// rearranged inside a block to even out slice widths.  The exact
+// layout ("v0") is frozen in DESIGN.md section 5 so that the oracle packer and
+// this one agree byte for byte.
+#include <algorithm>
+
+#include "cme_internal.h"
+
+namespace cme {
+
+namespace {
+// Does row r of A hold column c (columns ascending)?  Returns its value or 0.
+inline double entry(const Csr& A, int64_t r, int64_t c) {
+    const int32_t* b = A.ci.data() + A.rp[r];
+    const int32_t* e = A.ci.data() + A.rp[r + 1];
+    const int32_t* p = std::lower_bound(b, e, (int32_t)c);
+    return (p != e && *p == c) ? A.v[A.rp[r] + (p - b)] : 0.0;
+}
+}  // namespace
+
+bool band_rule(const Csr& A, int band_mode) {
+    if (band_mode == CME_BAND_ALWAYS) return true;
+    if (band_mode == CME_BAND_NEVER) return false;
+    const int64_t n = A.n;
+    int64_t cnt = 0;
+#pragma omp parallel for reduction(+ : cnt) schedule(static)
+    for (int64_t i = 0; i < n; ++i)
+        cnt += (i > 0 && entry(A, i, i - 1) != 0.0) + (i + 1 < n && entry(A, i, i + 1) != 0.0);
+    const int64_t den = 2 * n - 2;
+    return den > 0 && 3 * cnt >= 2 * den;
+}
+
+void pack_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, int32_t window,
+               bool band_on, bool uniform, int32_t global_kmax, Packed& P) {
+    const int64_t n = r1 - r0;  // local rows
+    P = Packed();
+    P.n = n;
+    P.band_on = band_on;
+    P.window = window > 1 ? window : 1;
+    P.uniform = uniform;
+    P.n_slots = (n + 31) / 32 * 32;
+    P.n_slices = P.n_slots / 32;
+    std::vector<int32_t> c(n);
+#pragma omp parallel for schedule(static)
+    for (int64_t l = 0; l < n; ++l) {
+        const int64_t r = r0 + l;
+        int64_t k = A.rp[r + 1] - A.rp[r];
+        if (band_on) k -= (r > 0 && entry(A, r, r - 1) != 0.0) + (r + 1 < A.n && entry(A, r, r + 1) != 0.0);
+        c[l] = (int32_t)k;
+    }
+    // local rearrangement: each window's slots take its rows by (-c, row)
+    P.row_of.resize(P.n_slots);
+    for (int64_t s = 0; s < P.n_slots; ++s) P.row_of[s] = (int32_t)s;
+    if (P.window > 1) {
+        const int64_t W = P.window;
+#pragma omp parallel for schedule(static)
+        for (int64_t w0 = 0; w0 < n; w0 += W) {
+            int32_t* b = P.row_of.data() + w0;
+            int32_t* e = P.row_of.data() + std::min(w0 + W, n);
+            std::stable_sort(b, e, [&](int32_t a, int32_t bb) { return c[a] > c[bb]; });
+        }
+    }
+    P.slice_w.assign(P.n_slices, 0);
+    P.slice_off.assign(P.n_slices + 1, 0);
+    for (int64_t q = 0; q < P.n_slices; ++q) {
+        int32_t w = 0;
+        if (uniform) {
+            w = global_kmax;
+        } else {
+            for (int64_t s = q * 32; s < std::min(q * 32 + 32, n); ++s) w = std::max(w, c[P.row_of[s]]);
+        }
+        P.slice_w[q] = w;
+        P.slice_off[q + 1] = P.slice_off[q] + 32 * (int64_t)w;
+    }
+    P.n_ell = P.slice_off[P.n_slices];
+    P.val.assign(P.n_ell, 0.0);
+    P.col.assign(P.n_ell, 0);
+    P.lo.assign(P.n_slots, 0.0);
+    P.up.assign(P.n_slots, 0.0);
+    P.inv_d.assign(P.n_slots, 0.0);
+#pragma omp parallel for schedule(dynamic, 256)
+    for (int64_t s = 0; s < P.n_slots; ++s) {
+        const int64_t q = s >> 5, lane = s & 31;
+        double* vq = P.val.data() + P.slice_off[q] + lane;
+        int32_t* cq = P.col.data() + P.slice_off[q] + lane;
+        const int32_t w = P.slice_w[q];
+        if (s >= n) {  // pad slot beyond the last row
+            for (int32_t t = 0; t < w; ++t) cq[32 * t] = (int32_t)(r1 - 1 - col_shift);
+            continue;
+        }
+        const int64_t l = P.row_of[s], r = r0 + l;
+        P.inv_d[s] = 1.0 / (-A.d[r]);
+        if (band_on) {
+            P.lo[s] = r > 0 ? entry(A, r, r - 1) : 0.0;
+            P.up[s] = r + 1 < A.n ? entry(A, r, r + 1) : 0.0;
+        }
+        int32_t t = 0;
+        for (int64_t p = A.rp[r]; p < A.rp[r + 1]; ++p) {
+            const int64_t j = A.ci[p];
+            if (band_on && (j == r - 1 || j == r + 1)) continue;
+            vq[32 * t] = A.v[p];
+            cq[32 * t] = (int32_t)(j - col_shift);
+            ++t;
+        }
+        for (; t < w; ++t) cq[32 * t] = (int32_t)(r - col_shift);
+    }
+}
+
+void pack_csr_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, Packed& P) {
+    const int64_t n = r1 - r0;
+    P = Packed();
+    P.n = n;
+    P.n_slots = (n + 31) / 32 * 32;
+    P.n_slices = P.n_slots / 32;
+    P.csr_rp.resize(n + 1);
+    const int64_t base = A.rp[r0];
+    for (int64_t l = 0; l <= n; ++l) P.csr_rp[l] = A.rp[r0 + l] - base;
+    P.csr_ci.resize(P.csr_rp[n]);
+    P.csr_v.assign(A.v.begin() + base, A.v.begin() + base + P.csr_rp[n]);
+    for (int64_t p = 0; p < P.csr_rp[n]; ++p) P.csr_ci[p] = (int32_t)(A.ci[base + p] - col_shift);
+    P.inv_d.assign(P.n_slots, 0.0);
+    for (int64_t l = 0; l < n; ++l) P.inv_d[l] = 1.0 / (-A.d[r0 + l]);
+    P.row_of.resize(P.n_slots);
+    for (int64_t s = 0; s < P.n_slots; ++s) P.row_of[s] = (int32_t)s;
+}
+
+}  // namespace cme

@@ -1,0 +1,223 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle.
+
+Tolerances (north star):
+* one SpMV / Jacobi application: |y_gpu - y_ora| <= 1e-13 * y_ora componentwise
+  for y_ora >= 2^-1000 (absolute 1e-300 below), and L1 <= 1e-13 * ||y||_1;
+* converged landscape: same (omega, tol, C, p0); stop iteration within +-C;
+  ||p_gpu - p_ora||_1 <= 1e-10 (oracle re-run for exactly the GPU's count if
+  the counts differ).
+DESIGN.md section 6 derives why these hold (all terms non-negative: no
+cancellation; expected ~5e-16 per step).
+"""
+import math
+
+import numpy as np
+import pytest
+
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def cme():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.fail("GPU tests need a CUDA device")
+    import paper_conf_ipps_maggionibl13_b200 as m
+    return m
+
+
+def assert_spmv_close(y, ref):
+    y, ref = np.asarray(y), np.asarray(ref)
+    big = ref >= 2.0 ** -1000
+    rel = np.abs(y[big] - ref[big]) / ref[big]
+    assert rel.max(initial=0.0) <= 1e-13, rel.max()
+    assert np.all(np.abs(y[~big] - ref[~big]) <= 1e-300)
+    assert np.abs(y - ref).sum() <= 1e-13 * ref.sum()
+
+
+NETS = [W.toggle_switch(23), W.toggle_switch(60), W.brusselator(40), W.schnakenberg(35),
+        W.birth_death(100), W.schlogl(200), W.cyclic3(5), W.schnakenberg(3)]
+LAYOUTS = [("none", 256, "auto", 0), ("dfs", 256, "auto", 0), ("rcm", 256, "auto", 0),
+           ("rcm", 1, "never", 0), ("dfs", 1, "always", 0), ("none", 1, "auto", 1), ("rcm", 1, "auto", 2)]
+ORD = {"none": 0, "dfs": 1, "rcm": 2}
+BAND = {"auto": 0, "always": 1, "never": 2}
+
+
+def build(cme, oracle_mod, net, order="none", window=256, band="auto", fmt=0):
+    states, r, c, v = oracle_mod.enumerate_network(net)
+    A = oracle_mod.ingest(len(states), r, c, v)
+    m = cme.Matrix(len(states), r, c, v)
+    m.reorder(ORD[order], 0)
+    m.pack(fmt, window, BAND[band])
+    return m, A
+
+
+@pytest.mark.parametrize("net", NETS, ids=lambda n: n.name)
+@pytest.mark.parametrize("layout", LAYOUTS, ids=lambda l: "-".join(map(str, l)))
+@pytest.mark.parametrize("omega", [1.0, 0.9])
+def test_spmv_parity(cme, oracle_mod, net, layout, omega):
+    m, A = build(cme, oracle_mod, net, *layout)
+    m.set_opts(omega=omega)
+    x = W.random_start(A.n, 11)
+    y = m.spmv(x)
+    assert_spmv_close(y, oracle_mod.jacobi_step(A, x, omega))
+
+
+def test_spmv_wide_rates_and_ragged(cme, oracle_mod):
+    """Config-5 generator: irregular widths, rates in [1,2), ragged last slice."""
+    for n, mu, width, irr in [(1000, 10, 64, True), (777, 5, 2, False), (5000, 15, 5000, True), (33, 6, 8, True)]:
+        r, c, v = W.banded_markov(n, mu, width, irr, seed=3)
+        A = oracle_mod.ingest(n, r, c, v)
+        for order in ("none", "rcm"):
+            m = cme.Matrix(n, r, c, v).reorder(ORD[order]).pack()
+            x = W.random_start(n, 5)
+            assert_spmv_close(m.spmv(x), oracle_mod.jacobi_step(A, x, 1.0))
+
+
+def solve_both(cme, oracle_mod, m, A, omega, tol, C=100, max_iter=200000, p0=None, stag=1e-10):
+    m.set_opts(omega=omega, check_every=C, stag_tol=stag)
+    p, st, it = m.solve(p0=p0, tol=tol, max_iter=max_iter)
+    r = oracle_mod.jacobi_solve(A, p0=p0, omega=omega, tol=tol, check_every=C, max_iter=max_iter,
+                                stag_tol=stag)
+    return p, st, it, r
+
+
+@pytest.mark.parametrize("net,omega", [(W.birth_death(100), 0.9), (W.toggle_switch(40), 0.9),
+                                       (W.schnakenberg(30, 8, 1, 5, 1, 0.01), 1.0),
+                                       (W.cyclic3(6), 0.5), (W.schlogl(120, c3=20.0, c4=1.0), 0.9)],
+                         ids=lambda x: getattr(x, "name", str(x)))
+@pytest.mark.parametrize("layout", [("none", 256, "auto", 0), ("rcm", 1, "never", 0), ("dfs", 256, "auto", 2)],
+                         ids=lambda l: "-".join(map(str, l)))
+def test_landscape_parity(cme, oracle_mod, net, omega, layout):
+    m, A = build(cme, oracle_mod, net, *layout)
+    p, st, it, r = solve_both(cme, oracle_mod, m, A, omega, 1e-12)
+    assert st == r.status == "CONVERGED"
+    assert abs(it - r.iters) <= 100
+    if it != r.iters:
+        r = oracle_mod.jacobi_solve(A, omega=omega, tol=0.0, max_iter=it)
+    assert np.abs(p - r.p).sum() <= 1e-10
+    assert abs(p.sum() - 1.0) < 1e-13 and p.min() >= 0
+
+
+def test_closed_forms(cme, oracle_mod):
+    m, A = build(cme, oracle_mod, W.birth_death(100))
+    m.set_opts(omega=0.9)
+    p, st, it = m.solve(tol=1e-14, max_iter=400000)
+    logs = np.array([x * math.log(10.0) - math.lgamma(x + 1) for x in range(101)])
+    pi = np.exp(logs - logs.max()); pi /= pi.sum()
+    assert st == "CONVERGED" and np.abs(p - pi).sum() < 1e-11
+    net = W.schnakenberg(40, 8.0, 1.0, 5.0, 1.0, 0.01)
+    m = cme.Matrix.from_network(net).reorder(cme.CME_ORDER_RCM).pack()
+    p, st, it = m.solve(tol=1e-15, max_iter=400000)
+    logs = np.array([x * math.log(8.0) - math.lgamma(x + 1) + y * math.log(5.0) - math.lgamma(y + 1)
+                     for x, y in m.states])
+    pi = np.exp(logs - logs.max()); pi /= pi.sum()
+    assert st == "CONVERGED" and np.abs(p - pi).sum() < 1e-12
+
+
+def test_stagnation_on_periodic_chain(cme, oracle_mod):
+    m, A = build(cme, oracle_mod, W.birth_death(100))
+    assert m.info().period == 2 and m.info().omega == 0.9
+    p, st, it, r = solve_both(cme, oracle_mod, m, A, 1.0, 1e-14)
+    assert st == r.status == "STAGNATED" and it == r.iters
+    m, A = build(cme, oracle_mod, W.cyclic3(3))
+    assert m.info().period == 3
+    p, st, it, r = solve_both(cme, oracle_mod, m, A, 1.0, 1e-14)
+    assert st == r.status == "STAGNATED"
+
+
+def test_paper_residual_stop(cme, oracle_mod):
+    m, A = build(cme, oracle_mod, W.toggle_switch(30), "rcm")
+    m.set_opts(omega=0.9, stop=cme.CME_STOP_PAPER_RESID)
+    p, st, it = m.solve(tol=1e-8, max_iter=100000)
+    r = oracle_mod.jacobi_solve(A, omega=0.9, tol=1e-8, max_iter=100000, stop_mode=1)
+    assert st == r.status == "CONVERGED" and abs(it - r.iters) <= 100
+    rep = m.report()
+    assert rep.resid <= 1e-8
+    if it == r.iters:
+        assert rep.resid == pytest.approx(r.resid, rel=1e-6)
+
+
+@pytest.mark.parametrize("C", [1, 7, 100])
+def test_max_iter_partial_blocks_and_p0(cme, oracle_mod, C):
+    m, A = build(cme, oracle_mod, W.toggle_switch(25), "rcm", 256)
+    p0 = W.random_start(A.n, 2) * 3.0
+    for max_iter in (0, 1, 5, 250):
+        p, st, it, r = solve_both(cme, oracle_mod, m, A, 0.9, 0.0, C=C, max_iter=max_iter, p0=p0, stag=0.0)
+        assert st == r.status == "NOT_CONVERGED" and it == r.iters == max_iter
+        assert np.abs(p - r.p).sum() <= 1e-12
+
+
+def test_device_pointers_and_streams(cme, oracle_mod):
+    import torch
+    m, A = build(cme, oracle_mod, W.schnakenberg(50), "rcm")
+    s = torch.cuda.Stream()
+    m.set_opts(omega=1.0, stream=s.cuda_stream)
+    p0 = torch.tensor(W.random_start(A.n, 9), device="cuda")
+    out = torch.empty(A.n, dtype=torch.float64, device="cuda")
+    p, st, it = m.solve(p0=p0, tol=1e-12, max_iter=100000, p_out=out)
+    r = oracle_mod.jacobi_solve(A, p0=p0.cpu().numpy(), omega=1.0, tol=1e-12)
+    assert st == r.status and abs(it - r.iters) <= 100
+    if it != r.iters:
+        r = oracle_mod.jacobi_solve(A, p0=p0.cpu().numpy(), omega=1.0, tol=0.0, max_iter=it)
+    assert np.abs(out.cpu().numpy() - r.p).sum() <= 1e-10
+    x = torch.tensor(W.random_start(A.n, 4), device="cuda")
+    y = torch.empty_like(x)
+    cme.cme_spmv(m.h, A.n, x, y)
+    assert_spmv_close(y.cpu().numpy(), oracle_mod.jacobi_step(A, x.cpu().numpy(), 1.0))
+
+
+def test_resident_run_api(cme, oracle_mod):
+    m, A = build(cme, oracle_mod, W.toggle_switch(40), "rcm")
+    m.set_opts(omega=0.9, check_every=50)
+    cme.cme_solver_load(m.h, A.n, None)
+    cme.cme_solver_run(m.h, 3)
+    p = np.empty(A.n)
+    cme.cme_solver_fetch(m.h, A.n, p)
+    r = oracle_mod.jacobi_solve(A, omega=0.9, tol=0.0, check_every=50, max_iter=150, stag_tol=0.0)
+    assert np.abs(p - r.p).sum() <= 1e-12 and m.report().iters == 150
+
+
+def test_invalid_p0(cme, oracle_mod):
+    m, A = build(cme, oracle_mod, W.toggle_switch(10))
+    bad = np.ones(A.n); bad[3] = -1.0
+    with pytest.raises(cme.CmeError) as e:
+        m.solve(p0=bad)
+    assert e.value.status == cme.CME_ERR_INVALID_ARG
+
+
+@pytest.mark.slow
+def test_cfg2_toggle_landscape(cme, oracle_mod):
+    """Config 2: toggle N=224, omega 0.9, tol 1e-12, bimodal landscape."""
+    net = W.toggle_switch(224)
+    m = cme.Matrix.from_network(net).reorder(cme.CME_ORDER_RCM).pack()
+    A = oracle_mod.network_csr(net)
+    m.set_opts(omega=0.9)
+    p, st, it = m.solve(tol=1e-12, max_iter=100000)
+    r = oracle_mod.jacobi_solve(A, omega=0.9, tol=1e-12, nthreads=8)
+    assert st == r.status == "CONVERGED" and abs(it - r.iters) <= 100
+    if it != r.iters:
+        r = oracle_mod.jacobi_solve(A, omega=0.9, tol=0.0, max_iter=it, nthreads=8)
+    assert np.abs(p - r.p).sum() <= 1e-10
+    S = m.states
+    onoff = p[(S[:, 0] >= 20) & (S[:, 1] < 5)].sum()
+    assert 0.40 < onoff < 0.50
+
+
+@pytest.mark.slow
+def test_cfg3a_schnakenberg_closed_form_at_scale(cme):
+    """Config 3a: n = 2,003,001 (Table I size), detailed balance -> product Poisson."""
+    net = W.schnakenberg(2000)
+    m = cme.Matrix.from_network(net).pack()
+    assert m.info().n == 2003001 and m.info().nnz == 14001003
+    p, st, it = m.solve(tol=1e-14, max_iter=2_000_000)
+    assert st == "CONVERGED"
+    S = m.states.astype(np.float64)
+    a, b = 500.0, 400.0
+    from scipy.special import gammaln
+    logs = S[:, 0] * math.log(a) - gammaln(S[:, 0] + 1) + S[:, 1] * math.log(b) - gammaln(S[:, 1] + 1)
+    pi = np.exp(logs - logs.max())
+    pi /= pi.sum()
+    assert np.abs(p - pi).sum() <= 1e-10
