@@ -142,13 +142,17 @@ int oracle_enumerate(int m, const int32_t* x0, int R, const int32_t* reac, const
     if (tab_rehash(&t, 1 << 16)) return ORACLE_OOM;
     int32_t* y = (int32_t*)malloc(sizeof(int32_t) * m);
     int64_t* st_node = NULL; int32_t* st_k = NULL; int64_t st_cap = 0, st_cap2 = 0, sp = 0;
+    int64_t* tgt = NULL; int64_t tgt_cap = 0;   /* tgt[j*R+k]: target of reaction k at j, -1 = disabled */
     int rc = ORACLE_OOM;
     if (!y || tab_add(&t, x0) < 0) goto fail;
     if (grow((void**)&st_node, &st_cap, 1, sizeof(int64_t)) ||
-        grow((void**)&st_k, &st_cap2, 1, sizeof(int32_t))) goto fail;
+        grow((void**)&st_k, &st_cap2, 1, sizeof(int32_t)) ||
+        grow((void**)&tgt, &tgt_cap, R, sizeof(int64_t))) goto fail;
+    for (int k = 0; k < R; k++) tgt[k] = -1;
     st_node[0] = 0; st_k[0] = 0; sp = 1;
     /* recursive DFS preorder with an explicit stack of (state, next reaction):
-     * a state is numbered when first reached and explored at once (reading R9) */
+     * a state is numbered when first reached and explored at once (reading R9).
+     * Every (state, reaction) pair is tried exactly once; its target is kept. */
     while (sp > 0) {
         int64_t j = st_node[sp - 1];
         int k = st_k[sp - 1];
@@ -156,9 +160,13 @@ int oracle_enumerate(int m, const int32_t* x0, int R, const int32_t* reac, const
         st_k[sp - 1] = k + 1;
         const int32_t* xj = t.states + j * m;
         if (!enabled(m, xj, reac + k * m, change + k * m, rates[k], w, cap, y)) continue;
-        if (tab_find(&t, y) >= 0) continue;
-        int64_t id = tab_add(&t, y);
+        int64_t id = tab_find(&t, y);
+        if (id >= 0) { tgt[j * R + k] = id; continue; }
+        id = tab_add(&t, y);
         if (id < 0) goto fail;
+        if (grow((void**)&tgt, &tgt_cap, (id + 1) * R, sizeof(int64_t))) goto fail;
+        for (int q = 0; q < R; q++) tgt[id * R + q] = -1;
+        tgt[j * R + k] = id;
         if (grow((void**)&st_node, &st_cap, sp + 1, sizeof(int64_t)) ||
             grow((void**)&st_k, &st_cap2, sp + 1, sizeof(int32_t))) goto fail;
         st_node[sp] = id; st_k[sp] = 0; sp++;
@@ -167,18 +175,10 @@ int oracle_enumerate(int m, const int32_t* x0, int R, const int32_t* reac, const
 
     {
         int64_t n0 = t.n;
-        int64_t* tgt = (int64_t*)malloc(sizeof(int64_t) * n0 * R);
         uint8_t* alive = (uint8_t*)malloc(n0);
         int64_t* newid = (int64_t*)malloc(sizeof(int64_t) * n0);
-        if (!tgt || !alive || !newid) { free(tgt); free(alive); free(newid); goto fail; }
-        for (int64_t j = 0; j < n0; j++) {
-            alive[j] = 1;
-            for (int k = 0; k < R; k++) {
-                const int32_t* xj = t.states + j * m;
-                tgt[j * R + k] = enabled(m, xj, reac + k * m, change + k * m, rates[k], w, cap, y)
-                                     ? tab_find(&t, y) : -1;
-            }
-        }
+        if (!alive || !newid) { free(alive); free(newid); goto fail; }
+        for (int64_t j = 0; j < n0; j++) alive[j] = 1;
         /* delete zero-outflow states and the edges into them, to a fixpoint (R8) */
         int changed = 1;
         while (changed) {
@@ -207,7 +207,7 @@ int oracle_enumerate(int m, const int32_t* x0, int R, const int32_t* reac, const
         int32_t* Co = (int32_t*)malloc(sizeof(int32_t) * (nnz ? nnz : 1));
         double* Vo = (double*)malloc(sizeof(double) * (nnz ? nnz : 1));
         if (!S || !Ro || !Co || !Vo) {
-            free(S); free(Ro); free(Co); free(Vo); free(tgt); free(alive); free(newid);
+            free(S); free(Ro); free(Co); free(Vo); free(alive); free(newid);
             goto fail;
         }
         int64_t e = 0;
@@ -224,13 +224,13 @@ int oracle_enumerate(int m, const int32_t* x0, int R, const int32_t* reac, const
                 e++;
             }
         }
-        free(tgt); free(alive); free(newid);
+        free(alive); free(newid);
         *n_out = n; *nnz_out = nnz;
         *states_out = S; *row_out = Ro; *col_out = Co; *rate_out = Vo;
         rc = ORACLE_OK;
     }
 fail:
-    free(st_node); free(st_k); free(y); free(t.states); free(t.slot);
+    free(st_node); free(st_k); free(tgt); free(y); free(t.states); free(t.slot);
     return rc;
 }
 

@@ -4,6 +4,9 @@
 // DESIGN.md fix the buffer rule, the zero-outflow pruning, the DFS order and
 // the propensity's index convention.  This is setup (not the hot path); it is
 // checked bit-for-bit against the oracle's independent enumerator.
+#include <sys/mman.h>
+
+#include <cstdlib>
 #include <cstring>
 #include <memory>
 
@@ -57,88 +60,148 @@ inline bool fire(const Net& N, const int32_t* x, int k, int32_t* y) {
     return load <= N.cap;
 }
 
+// Hash set of microstates.  States with m <= 8 species and counts < 2^16 are
+// packed into a 128-bit key kept inside the slot, so a probe touches one cache
+// line (the tables of 20M-state networks are GBs: every miss is a DRAM + TLB
+// miss; the slot array asks for transparent huge pages).
 class StateSet {
   public:
-    explicit StateSet(int m) : m_(m) { rehash(1 << 20); }
+    explicit StateSet(int m) : m_(m), packed_(m <= 8) { rehash(1 << 20); }
+    ~StateSet() { std::free(slot_); }
+    StateSet(const StateSet&) = delete;
+    StateSet& operator=(const StateSet&) = delete;
     int64_t size() const { return n_; }
     const int32_t* at(int64_t s) const { return data_.data() + s * m_; }
-    const std::vector<int32_t>& data() const { return data_; }
+    bool packed() const { return packed_; }
     int64_t find(const int32_t* x) const {
-        const uint64_t h = hash(x);
-        for (uint64_t p = h & mask_;; p = (p + 1) & mask_) {
-            const int64_t s = slot_[p];
-            if (s < 0) return -1;
-            if (hv_[p] == h && std::memcmp(at(s), x, sizeof(int32_t) * m_) == 0) return s;
+        Key k;
+        if (!make_key(x, k)) return -1;
+        for (uint64_t p = k.h & mask_;; p = (p + 1) & mask_) {
+            const Slot& e = slot_[p];
+            if (e.s < 0) return -1;
+            if (e.h == k.h && (packed_ ? (e.a == k.a && e.b == k.b)
+                                       : std::memcmp(at(e.s), x, sizeof(int32_t) * m_) == 0))
+                return e.s;
         }
     }
-    int64_t insert(const int32_t* x) {  // caller checked absence
-        if (2 * (n_ + 1) > (int64_t)slot_.size()) rehash(slot_.size() * 2);
+    // caller checked absence; returns -1 if the state cannot be packed (caller
+    // then restarts in generic mode)
+    int64_t insert(const int32_t* x) {
+        Key k;
+        if (!make_key(x, k)) return -1;
+        if (2 * (n_ + 1) > (int64_t)(mask_ + 1)) rehash(2 * (mask_ + 1));
         data_.insert(data_.end(), x, x + m_);
-        place(n_, hash(x));
+        place(Slot{k.h, n_, k.a, k.b});
         return n_++;
     }
+    void set_generic() { packed_ = false; }
 
   private:
-    uint64_t hash(const int32_t* x) const {
-        uint64_t h = 0x9E3779B97F4A7C15ull;
-        for (int i = 0; i < m_; ++i) {
-            h ^= (uint32_t)x[i] + 0x632BE59BD9B4E019ull + (h << 6) + (h >> 2);
-            h *= 0xFF51AFD7ED558CCDull;
-        }
-        return h ^ (h >> 33);
+    struct Key {
+        uint64_t h, a, b;
+    };
+    struct Slot {
+        uint64_t h;
+        int64_t s;
+        uint64_t a, b;
+    };
+    static uint64_t mix(uint64_t z) {
+        z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+        z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+        return z ^ (z >> 31);
     }
-    void place(int64_t s, uint64_t h) {
-        uint64_t p = h & mask_;
-        while (slot_[p] >= 0) p = (p + 1) & mask_;
-        slot_[p] = s;
-        hv_[p] = h;
+    bool make_key(const int32_t* x, Key& k) const {
+        if (packed_) {
+            uint64_t a = 0, b = 0;
+            for (int i = 0; i < m_; ++i) {
+                if ((uint32_t)x[i] >= 65536u) return false;
+                if (i < 4) a |= (uint64_t)x[i] << (16 * i);
+                else b |= (uint64_t)x[i] << (16 * (i - 4));
+            }
+            k.a = a;
+            k.b = b;
+            k.h = mix(a ^ mix(b + 0x9E3779B97F4A7C15ull));
+            return true;
+        }
+        uint64_t h = 0x9E3779B97F4A7C15ull;
+        for (int i = 0; i < m_; ++i) h = mix(h ^ (uint32_t)x[i]);
+        k.h = h;
+        k.a = k.b = 0;
+        return true;
+    }
+    void place(const Slot& e) {
+        uint64_t p = e.h & mask_;
+        while (slot_[p].s >= 0) p = (p + 1) & mask_;
+        slot_[p] = e;
     }
     void rehash(size_t sz) {
-        slot_.assign(sz, -1);
-        hv_.assign(sz, 0);
+        Slot* old = slot_;
+        const size_t old_n = slot_ ? mask_ + 1 : 0;
+        const size_t bytes = sz * sizeof(Slot);
+        void* mem = nullptr;
+        if (posix_memalign(&mem, 1 << 21, bytes) != 0) throw std::bad_alloc();
+        madvise(mem, bytes, MADV_HUGEPAGE);
+        slot_ = static_cast<Slot*>(mem);
+        for (size_t i = 0; i < sz; ++i) slot_[i].s = -1;
         mask_ = sz - 1;
-        for (int64_t s = 0; s < n_; ++s) place(s, hash(at(s)));
+        for (size_t i = 0; i < old_n; ++i)
+            if (old[i].s >= 0) place(old[i]);
+        std::free(old);
     }
     int m_;
+    bool packed_;
     int64_t n_ = 0;
     uint64_t mask_ = 0;
-    std::vector<int64_t> slot_;
-    std::vector<uint64_t> hv_;
+    Slot* slot_ = nullptr;
     std::vector<int32_t> data_;
 };
 
+struct Unpackable {};
+
 }  // namespace
 
+cme_status enumerate_network(const Net& N, cme_coo_s& out, bool generic);
+
 cme_status enumerate_network(const Net& N, cme_coo_s& out) {
+    try {
+        return enumerate_network(N, out, false);
+    } catch (const Unpackable&) {
+        return enumerate_network(N, out, true);
+    }
+}
+
+cme_status enumerate_network(const Net& N, cme_coo_s& out, bool generic) {
     StateSet S(N.m);
+    if (generic) S.set_generic();
+    const int R = N.R;
     std::vector<int32_t> y(N.m);
-    S.insert(N.x0);
-    // recursive-DFS preorder: (state, next reaction) frames
+    std::vector<int32_t> tgt;                   // tgt[j*R + k]: target of reaction k at j, -1 = disabled
+    std::vector<int32_t> outdeg;
+    auto add = [&](const int32_t* x) {
+        const int64_t id = S.insert(x);
+        if (id < 0) throw Unpackable();
+        tgt.resize((size_t)S.size() * R, -1);
+        outdeg.resize(S.size(), 0);
+        return id;
+    };
+    add(N.x0);
+    // recursive-DFS preorder: (state, next reaction) frames; every (state,
+    // reaction) pair is tried exactly once, so its target is recorded here
     std::vector<std::pair<int64_t, int32_t>> st{{0, 0}};
     while (!st.empty()) {
         auto& f = st.back();
-        if (f.second == N.R) { st.pop_back(); continue; }
+        if (f.second == R) { st.pop_back(); continue; }
         const int k = f.second++;
         const int64_t j = f.first;
-        if (!fire(N, S.at(j), k, y.data()) || S.find(y.data()) >= 0) continue;
-        const int64_t id = S.insert(y.data());
-        st.emplace_back(id, 0);
+        if (!fire(N, S.at(j), k, y.data())) continue;
+        int64_t id = S.find(y.data());   // (an unpackable y is "absent"; add() then restarts)
+        const bool fresh = id < 0;
+        if (fresh) id = add(y.data());
+        tgt[(size_t)j * R + k] = (int32_t)id;
+        ++outdeg[j];
+        if (fresh) st.emplace_back(id, 0);
     }
     const int64_t n0 = S.size();
-    const int R = N.R;
-    std::vector<int32_t> tgt((size_t)n0 * R, -1);
-    std::vector<int32_t> outdeg(n0, 0);
-#pragma omp parallel
-    {
-        std::vector<int32_t> yy(N.m);
-#pragma omp for schedule(static)
-        for (int64_t j = 0; j < n0; ++j)
-            for (int k = 0; k < R; ++k)
-                if (fire(N, S.at(j), k, yy.data())) {
-                    tgt[(size_t)j * R + k] = (int32_t)S.find(yy.data());
-                    ++outdeg[j];
-                }
-    }
     // prune zero-outflow states (and edges into them) to the fixpoint with a
     // worklist over reverse edges
     std::vector<int64_t> rptr(n0 + 1, 0);
