@@ -203,6 +203,11 @@ typedef struct cme_halo_view {
     int32_t nranks, rank;
     const int64_t* row_begin; /* [nranks+1] global row cut points             */
     const int64_t* span;      /* [2*nranks] x-span [lo_r, hi_r) of every rank  */
+    /* this rank's per-iteration exchange: send x-span[off, off+cnt) (own rows)
+     * to peer; receive peer's rows into x-span[off, off+cnt) (halo)          */
+    int32_t n_send, n_recv;
+    const int32_t* send_peer; const int64_t* send_off; const int64_t* send_cnt;
+    const int32_t* recv_peer; const int64_t* recv_off; const int64_t* recv_cnt;
 } cme_halo_view;
 cme_status cme_export_halo(cme_matrix h, cme_halo_view* v);
 

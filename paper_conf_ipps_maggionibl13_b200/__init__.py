@@ -79,7 +79,10 @@ class cme_packed_view(C.Structure):
 
 
 class cme_halo_view(C.Structure):
-    _fields_ = [("nranks", C.c_int32), ("rank", C.c_int32), ("row_begin", i64p), ("span", i64p)]
+    _fields_ = [("nranks", C.c_int32), ("rank", C.c_int32), ("row_begin", i64p), ("span", i64p),
+                ("n_send", C.c_int32), ("n_recv", C.c_int32),
+                ("send_peer", i32p), ("send_off", i64p), ("send_cnt", i64p),
+                ("recv_peer", i32p), ("recv_off", i64p), ("recv_cnt", i64p)]
 
 
 _SIGS = {
@@ -289,7 +292,14 @@ def cme_export_halo(h):
     _chk(_lib.cme_export_halo(h, C.byref(v)), "cme_export_halo")
     cuts = np.ctypeslib.as_array(v.row_begin, shape=(v.nranks + 1,)).copy()
     span = np.ctypeslib.as_array(v.span, shape=(2 * v.nranks,)).copy().reshape(v.nranks, 2)
-    return dict(nranks=v.nranks, rank=v.rank, cuts=cuts, span=span)
+
+    def cp(ptr, k):
+        return np.ctypeslib.as_array(ptr, shape=(k,)).copy() if k else np.zeros(0, np.int64)
+    send = list(zip(cp(v.send_peer, v.n_send).tolist(), cp(v.send_off, v.n_send).tolist(),
+                    cp(v.send_cnt, v.n_send).tolist()))
+    recv = list(zip(cp(v.recv_peer, v.n_recv).tolist(), cp(v.recv_off, v.n_recv).tolist(),
+                    cp(v.recv_cnt, v.n_recv).tolist()))
+    return dict(nranks=v.nranks, rank=v.rank, cuts=cuts, span=span, send=send, recv=recv)
 
 
 def cme_matrix_destroy(h):

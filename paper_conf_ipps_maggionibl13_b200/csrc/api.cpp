@@ -103,6 +103,9 @@ cme_status build_local(cme_matrix_s* h, int nranks, int rank) {
     } else {
         plan_cuts(h, nranks);
     }
+    h->halo = nranks > 1 ? halo_plan(h) : HaloPlan();
+    h->halo_speer.assign(h->halo.send_peer.begin(), h->halo.send_peer.end());
+    h->halo_rpeer.assign(h->halo.recv_peer.begin(), h->halo.recv_peer.end());
     const int64_t r0 = h->cuts[rank], r1 = h->cuts[rank + 1], shift = h->span[2 * rank];
     if (h->format == CME_FMT_CSR) {
         pack_csr_rows(h->B, r0, r1, shift, h->P);
@@ -360,8 +363,7 @@ cme_status cme_matrix_distribute(cme_matrix h, cme_comm c) {
     if (h->stage < 2) { set_error("distribute needs a packed matrix"); return CME_ERR_BAD_STATE; }
     return guarded([&] {
         build_local(h, comm_nranks(c), comm_rank(c));
-        HaloPlan p = halo_plan(h);
-        cme_status s = device_upload(h, comm_device(c), &p, c);
+        cme_status s = device_upload(h, comm_device(c), &h->halo, c);
         if (s != CME_OK) return s;
         h->comm = c;
         h->stage = 3;
@@ -375,6 +377,14 @@ cme_status cme_export_halo(cme_matrix h, cme_halo_view* v) {
     v->rank = h->rank;
     v->row_begin = h->cuts.data();
     v->span = h->span.data();
+    v->n_send = (int32_t)h->halo.send_peer.size();
+    v->n_recv = (int32_t)h->halo.recv_peer.size();
+    v->send_peer = h->halo_speer.data();
+    v->send_off = h->halo.send_off.data();
+    v->send_cnt = h->halo.send_cnt.data();
+    v->recv_peer = h->halo_rpeer.data();
+    v->recv_off = h->halo.recv_off.data();
+    v->recv_cnt = h->halo.recv_cnt.data();
     return CME_OK;
 }
 

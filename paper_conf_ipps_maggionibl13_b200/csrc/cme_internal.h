@@ -6,6 +6,7 @@
 #include <vector>
 
 #include "cme.h"
+#include "comm.h"
 
 namespace cme {
 
@@ -78,6 +79,8 @@ struct cme_matrix_s {
     int nranks = 1, rank = 0;
     std::vector<int64_t> cuts;  // nranks + 1
     std::vector<int64_t> span;  // 2 * nranks
+    cme::HaloPlan halo;         // this rank's exchange plan
+    std::vector<int32_t> halo_speer, halo_rpeer;
     cme_comm_s* comm = nullptr;
     cme::Device* dev = nullptr;
 };

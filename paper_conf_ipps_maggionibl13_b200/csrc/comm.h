@@ -6,6 +6,8 @@
 
 #include "cme.h"
 
+struct cme_comm_s;
+
 namespace cme {
 
 // Who sends which contiguous x range to whom after every step.  Offsets are
