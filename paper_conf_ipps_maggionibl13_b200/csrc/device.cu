@@ -8,12 +8,15 @@
 // the GPU (a decided stop turns the look-ahead block into no-op launches).
 #include <cmath>
 #include <cstddef>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <algorithm>
 
 #include "cme_internal.h"
 #include "comm.h"
 #include "kernels.cuh"
+#include "kernels_tma.cuh"
 
 namespace cme {
 
@@ -70,6 +73,11 @@ struct Device {
     int nranks = 1, rank = 0;
     HaloPlan halo;
     std::vector<int64_t> cuts;
+    // TMA-staged persistent kernel (kernels_tma.cuh)
+    bool use_tma = false;
+    int tma_ncw = 8;
+    int tma_grid = 0, tma_stages = 0, tma_stage_bytes = 0, tma_off_val = 0, tma_off_col = 0;
+    int64_t n_tiles = 0;
     // graphs
     cudaGraphExec_t gexec[2] = {nullptr, nullptr};
     int64_t gC = -1;
@@ -160,7 +168,7 @@ __global__ void __launch_bounds__(kCta) load_kernel(const double* src, const int
         s += v;
         bad += !(v >= 0.0) || isinf(v);
     }
-    cta_check_partials(s, bad, 0.0, 0.0, 0.0, partials);
+    cta_check_partials<kWarpsPerCta>(s, bad, 0.0, 0.0, 0.0, partials);
 }
 
 __global__ void load_decide_kernel(const double* all8, int nranks, Ctrl* c, int32_t normalise) {
@@ -231,6 +239,88 @@ static cme_status select_device(int want, int* out) {
     return CME_OK;
 }
 
+static int env_int(const char* name, int dflt) {
+    const char* v = std::getenv(name);
+    return (v && *v) ? std::atoi(v) : dflt;
+}
+
+template <int W, bool B, bool R, bool D, bool C>
+static cudaError_t tma_attr(int smem) {
+    return cudaFuncSetAttribute(sell_tma_kernel<W, B, R, D, C>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+}
+
+template <int W>
+static cudaError_t tma_attr_all(int smem) {
+    cudaError_t e = cudaSuccess;
+#define A(b, r, dd, c) if (e == cudaSuccess) e = tma_attr<W, b, r, dd, c>(smem);
+    A(0,0,0,0) A(0,0,0,1) A(0,0,1,0) A(0,0,1,1) A(0,1,0,0) A(0,1,0,1) A(0,1,1,0) A(0,1,1,1)
+    A(1,0,0,0) A(1,0,0,1) A(1,0,1,0) A(1,0,1,1) A(1,1,0,0) A(1,1,0,1) A(1,1,1,0) A(1,1,1,1)
+#undef A
+    return e;
+}
+
+template <int W>
+static void launch_tma(const Device& d, const TmaArgs& T, bool damp, bool check, cudaStream_t s) {
+    const int smem = d.tma_stages * d.tma_stage_bytes;
+    const int key = (d.band ? 8 : 0) | (d.rearr ? 4 : 0) | (damp ? 2 : 0) | (check ? 1 : 0);
+    switch (key) {
+#define K(b, r, dd, c) \
+    case (b * 8 + r * 4 + dd * 2 + c): sell_tma_kernel<W, b, r, dd, c><<<d.tma_grid, TmaShape<W>::kThreads, smem, s>>>(T); break;
+        K(0, 0, 0, 0) K(0, 0, 0, 1) K(0, 0, 1, 0) K(0, 0, 1, 1)
+        K(0, 1, 0, 0) K(0, 1, 0, 1) K(0, 1, 1, 0) K(0, 1, 1, 1)
+        K(1, 0, 0, 0) K(1, 0, 0, 1) K(1, 0, 1, 0) K(1, 0, 1, 1)
+        K(1, 1, 0, 0) K(1, 1, 0, 1) K(1, 1, 1, 0) K(1, 1, 1, 1)
+#undef K
+    }
+}
+
+// Choose stages / CTAs per SM for the TMA kernel.  Tuning knobs (environment,
+// read at pack/distribute time): CME_TMA=0 forces the register kernel,
+// CME_TMA_STAGES, CME_TMA_CTAS override the defaults (4 stages, max resident).
+static cme_status configure_tma(Device& d, const Packed& P) {
+    d.use_tma = false;
+    if (env_int("CME_TMA", 1) == 0 || d.n_slices == 0) return CME_OK;
+    const int ncw = env_int("CME_TMA_WARPS", 16) == 8 ? 8 : 16;
+    d.tma_ncw = ncw;
+    d.n_tiles = (d.n_slices + ncw - 1) / ncw;
+    int64_t max_nval = 0;
+    for (int64_t t = 0; t < d.n_tiles; ++t) {
+        const int64_t q0 = t * ncw, q1 = std::min<int64_t>(q0 + ncw, d.n_slices);
+        max_nval = std::max(max_nval, P.slice_off[q1] - P.slice_off[q0]);
+    }
+    auto a128 = [](int64_t b) { return (b + 127) / 128 * 128; };
+    const int64_t off_val = a128(tma_fixed_bytes(ncw, d.band, d.rearr));
+    const int64_t off_col = off_val + a128(8 * max_nval);
+    const int64_t stage = a128(off_col + 4 * max_nval);
+    int dev = 0, smem_max = 0, sms = 0;
+    CUDA_TRY(cudaGetDevice(&dev));
+    CUDA_TRY(cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+    CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    int stages = std::min(8, std::max(2, env_int("CME_TMA_STAGES", 2)));
+    while (stages > 2 && stages * stage > smem_max - 1024) --stages;
+    if (stages * stage > smem_max - 1024) return CME_OK;  // tiles too wide: register kernel
+    const int smem = (int)(stages * stage);
+    CUDA_TRY(ncw == 16 ? tma_attr_all<16>(smem) : tma_attr_all<8>(smem));
+    int occ = 0;
+    if (ncw == 16)
+        CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, sell_tma_kernel<16, false, true, true, true>,
+                                                               TmaShape<16>::kThreads, smem));
+    else
+        CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, sell_tma_kernel<8, false, true, true, true>,
+                                                               TmaShape<8>::kThreads, smem));
+    occ = std::max(1, std::min(occ, env_int("CME_TMA_CTAS", occ)));
+    d.tma_stages = stages;
+    d.tma_stage_bytes = (int)stage;
+    d.tma_off_val = (int)off_val;
+    d.tma_off_col = (int)off_col;
+    d.tma_grid = (int)std::min<int64_t>(d.n_tiles, (int64_t)sms * occ);
+    if (env_int("CME_VERBOSE", 0))
+        std::fprintf(stderr, "[cme] tma: warps=%d stages=%d stage_bytes=%lld occ=%d grid=%d tiles=%lld\n", ncw,
+                     stages, (long long)stage, occ, d.tma_grid, (long long)d.n_tiles);
+    d.use_tma = true;
+    return CME_OK;
+}
+
 // Build the device state from h->P (local layout) and the partition in h.
 cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cme_comm_s* comm) {
     int dev = 0;
@@ -290,6 +380,7 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
     d->grid = d->format == CME_FMT_CSR ? (int)((d->n_own + kCta - 1) / kCta)
                                        : (int)((d->n_slices + kWarpsPerCta - 1) / kWarpsPerCta);
     d->grid = std::max(d->grid, 1);
+    if (d->format != CME_FMT_CSR && (s = configure_tma(*d, P)) != CME_OK) return fail(s);
     d->part_blocks = std::max(d->grid, grid_for(d->n_own));
     if ((s = d->alloc(d->partials, (size_t)d->part_blocks * kPartials)) != CME_OK) return fail(s);
     if ((s = d->alloc(d->gather, (size_t)d->nranks * 8)) != CME_OK) return fail(s);
@@ -350,6 +441,10 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
     if (d.format == CME_FMT_CSR) {
         if (damp) { if (check) csr_step_kernel<true, true><<<d.grid, kCta, 0, s>>>(a); else csr_step_kernel<true, false><<<d.grid, kCta, 0, s>>>(a); }
         else { if (check) csr_step_kernel<false, true><<<d.grid, kCta, 0, s>>>(a); else csr_step_kernel<false, false><<<d.grid, kCta, 0, s>>>(a); }
+    } else if (d.use_tma) {
+        TmaArgs T{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col};
+        if (d.tma_ncw == 16) launch_tma<16>(d, T, damp, check, s);
+        else launch_tma<8>(d, T, damp, check, s);
     } else {
         const int key = (d.band ? 8 : 0) | (d.rearr ? 4 : 0) | (damp ? 2 : 0) | (check ? 1 : 0);
         switch (key) {
@@ -368,8 +463,8 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
 
 // reduce partials of the last CHECK step and decide
 static cme_status launch_finalize(Device& d, cudaStream_t s, int32_t len, int32_t final_partial) {
-    reduce_partials_kernel<<<1, 1024, 0, s>>>(d.partials, d.grid, d.nranks > 1 ? d.local8 : d.gather,
-                                              &d.ctrl->stop);
+    reduce_partials_kernel<<<1, 1024, 0, s>>>(d.partials, d.use_tma ? d.tma_grid : d.grid,
+                                              d.nranks > 1 ? d.local8 : d.gather, &d.ctrl->stop);
     CUDA_TRY(cudaGetLastError());
     if (d.nranks > 1) CME_TRY(comm_allgather8(d.comm, d.local8, d.gather, s));
     decide_kernel<<<1, 1, 0, s>>>(d.gather, d.nranks, d.ctrl, len, final_partial);

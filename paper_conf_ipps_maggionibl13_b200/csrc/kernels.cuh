@@ -90,10 +90,12 @@ __device__ __forceinline__ double warp_max(double v) {
     return v;
 }
 
-// CTA-level deterministic reduction of the 5 check quantities into partials[blockIdx.x].
+// CTA-level deterministic reduction of the 5 check quantities into
+// partials[blockIdx.x]; NW = warps in the CTA (all must call it).
+template <int NW = kWarpsPerCta>
 __device__ __forceinline__ void cta_check_partials(double sy, double sx, double sd, double md,
                                                    double mx, double* partials) {
-    __shared__ double red[kWarpsPerCta][5];
+    __shared__ double red[NW][5];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     sy = warp_sum(sy); sx = warp_sum(sx); sd = warp_sum(sd);
     md = warp_max(md); mx = warp_max(mx);
@@ -101,7 +103,7 @@ __device__ __forceinline__ void cta_check_partials(double sy, double sx, double 
     __syncthreads();
     if (threadIdx.x == 0) {
         double a = 0, b = 0, c = 0, d = 0, e = 0;
-        for (int i = 0; i < kWarpsPerCta; ++i) {
+        for (int i = 0; i < NW; ++i) {
             a += red[i][0]; b += red[i][1]; c += red[i][2];
             d = fmax(d, red[i][3]); e = fmax(e, red[i][4]);
         }
@@ -163,7 +165,7 @@ __global__ void __launch_bounds__(kCta) sell_step_kernel(const StepArgs a) {
             }
         }
     }
-    if (CHECK) cta_check_partials(sy, sx, sd, md, mx, a.partials);
+    if (CHECK) cta_check_partials<kWarpsPerCta>(sy, sx, sd, md, mx, a.partials);
 }
 
 // Plain CSR arm (ablation, CME_FMT_CSR): one thread per row.
@@ -191,7 +193,7 @@ __global__ void __launch_bounds__(kCta) csr_step_kernel(const StepArgs a) {
             sy = yv; sx = xr; sd = df; md = df / id; mx = xr;
         }
     }
-    if (CHECK) cta_check_partials(sy, sx, sd, md, mx, a.partials);
+    if (CHECK) cta_check_partials<kWarpsPerCta>(sy, sx, sd, md, mx, a.partials);
 }
 
 }  // namespace cme

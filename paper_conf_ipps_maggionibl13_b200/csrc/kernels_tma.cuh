@@ -1,0 +1,192 @@
+// TMA-staged persistent variant of the fused Jacobi step (sm_100a).
+//
+// Same arithmetic and layout as sell_step_kernel (kernels.cuh); what changes
+// is how the packed matrix reaches the SM.  A tile is 8 consecutive slices
+// (= 256 rows = one rearrangement window); its val and col entries
+// are ONE contiguous block each (layout v0), and its inv_d / row_of / lo / up
+// entries are contiguous too.  A producer warp streams every tile of the CTA's
+// round-robin share into a ring of S shared-memory stages with 1-D bulk copies
+// (cp.async.bulk ... mbarrier::complete_tx, the TMA engine), each stage
+// guarded by a full/empty mbarrier pair; 8 consumer warps (one slice each)
+// read their rows from shared memory, gather x from global memory (L1/L2),
+// and store y.  The bytes in flight per SM are S x stage bytes x CTAs/SM
+// (~170 KB) instead of whatever the register file of resident warps can
+// hold, so the kernel runs at the HBM limit rather than the latency limit.
+#pragma once
+#include "kernels.cuh"
+
+namespace cme {
+
+// NCW consumer warps (one slice each) + 1 producer warp; a tile = NCW slices.
+template <int NCW>
+struct TmaShape {
+    static constexpr int kThreads = 32 * (NCW + 1);
+    static constexpr int kMinBlocks = NCW == 8 ? 3 : 2;   // register cap: 75 / 60 regs
+};
+
+struct TmaArgs {
+    StepArgs a;
+    int64_t n_tiles;
+    int32_t stages;
+    int32_t stage_bytes;  // bytes per stage (multiple of 128)
+    int32_t off_val;      // byte offsets inside a stage
+    int32_t off_col;
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* b, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+    asm volatile(
+        "{\n"
+        ".reg .pred P1;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+        "@!P1 bra WAIT_%=;\n"
+        "}\n" ::"r"(smem_u32(b)),
+        "r"(parity)
+        : "memory");
+}
+// 1-D bulk copy global -> shared, completion counted on mbarrier `b`
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* b,
+                                         uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::
+            "r"(smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(b)), "l"(pol)
+        : "memory");
+}
+
+// Host/device agreement on the stage layout: returns off_val; off_col and the
+// stage size follow from the largest tile's ELL entry count.
+__host__ __device__ inline int tma_fixed_bytes(int ncw, bool band, bool rearr) {
+    return ncw * 32 * (8 + (rearr ? 4 : 0) + (band ? 16 : 0));
+}
+
+template <int NCW, bool BAND, bool REARR, bool DAMP, bool CHECK>
+__global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBlocks)
+    sell_tma_kernel(const TmaArgs T) {
+    constexpr int kTmaConsumers = NCW, kTileSlices = NCW;
+    const StepArgs& a = T.a;
+    if (a.stop != nullptr && *a.stop) return;
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ uint64_t full[8], empty[8];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int S = T.stages;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < S; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], kTmaConsumers);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+
+    // stage layout: [inv_d][row_of if REARR][lo, up if BAND][val][col], NCW*32 slots
+    // (tma_fixed_bytes() gives the host the same offsets)
+    constexpr int kSlots = NCW * 32;
+    constexpr int kOffInvd = 0, kOffRow = 8 * kSlots, kOffLo = kOffRow + (REARR ? 4 * kSlots : 0),
+                  kOffUp = kOffLo + 8 * kSlots;
+    double sy = 0.0, sx = 0.0, sd = 0.0, md = 0.0, mx = 0.0;
+
+    if (warp == kTmaConsumers) {
+        // ---------------- producer ----------------
+        if (lane == 0) {
+            const uint64_t pol = evict_first_policy();
+            int64_t i = 0;
+            for (int64_t tile = blockIdx.x; tile < T.n_tiles; tile += gridDim.x, ++i) {
+                const int s = (int)(i % S);
+                if (i >= S) mbar_wait(&empty[s], (uint32_t)(((i / S) - 1) & 1));
+                unsigned char* st = smem + (size_t)s * T.stage_bytes;
+                const int64_t q0 = tile * kTileSlices;
+                const int64_t q1 = min(q0 + kTileSlices, a.slice_end);
+                const int64_t e0 = a.slice_off[q0], e1 = a.slice_off[q1];
+                const uint32_t slots = (uint32_t)(q1 - q0) * 32u;
+                const uint32_t nval = (uint32_t)(e1 - e0);
+                uint32_t bytes = nval * 12u + slots * 8u;
+                if (REARR) bytes += slots * 4u;
+                if (BAND) bytes += slots * 16u;
+                mbar_expect_tx(&full[s], bytes);
+                bulk_g2s(st + kOffInvd, a.inv_d + q0 * 32, slots * 8u, &full[s], pol);
+                if (REARR) bulk_g2s(st + kOffRow, a.row_of + q0 * 32, slots * 4u, &full[s], pol);
+                if (BAND) {
+                    bulk_g2s(st + kOffLo, a.lo + q0 * 32, slots * 8u, &full[s], pol);
+                    bulk_g2s(st + kOffUp, a.up + q0 * 32, slots * 8u, &full[s], pol);
+                }
+                if (nval) {
+                    bulk_g2s(st + T.off_val, a.val + e0, nval * 8u, &full[s], pol);
+                    bulk_g2s(st + T.off_col, a.col + e0, nval * 4u, &full[s], pol);
+                }
+            }
+        }
+    } else {
+        // ---------------- consumers ----------------
+        const double* xo = a.x + a.own_off;
+        int64_t i = 0;
+        for (int64_t tile = blockIdx.x; tile < T.n_tiles; tile += gridDim.x, ++i) {
+            const int s = (int)(i % S);
+            const int64_t q0 = tile * kTileSlices;
+            const int64_t q = q0 + warp;
+            const unsigned char* st = smem + (size_t)s * T.stage_bytes;
+            // slice metadata (tiny, L1/L2 resident) before the wait
+            int w = 0;
+            int64_t loff = 0;
+            if (q < a.slice_end) {
+                w = __ldg(a.slice_w + q);
+                loff = __ldg(a.slice_off + q) - __ldg(a.slice_off + q0);
+            }
+            mbar_wait(&full[s], (uint32_t)((i / S) & 1));
+            const int64_t slot = q * 32 + lane;
+            if (q < a.slice_end && slot < a.n_rows) {
+                const int ls = warp * 32 + lane;
+                const double* sval = reinterpret_cast<const double*>(st + T.off_val) + loff + lane;
+                const int32_t* scol = reinterpret_cast<const int32_t*>(st + T.off_col) + loff + lane;
+                const int64_t r = REARR ? (int64_t) reinterpret_cast<const int32_t*>(st + kOffRow)[ls] : slot;
+                double acc = 0.0;
+                for (int t0 = 0; t0 < w; t0 += kUnroll) {
+                    double xv[kUnroll];   // all gathers of the chunk in flight, then FMAs
+#pragma unroll
+                    for (int u = 0; u < kUnroll; ++u)
+                        if (t0 + u < w) xv[u] = ld_x(a.x + scol[32 * (t0 + u)]);
+#pragma unroll
+                    for (int u = 0; u < kUnroll; ++u)
+                        if (t0 + u < w) acc = fma(sval[32 * (t0 + u)], xv[u], acc);
+                }
+                double sum = acc;
+                if (BAND) {
+                    const double l = reinterpret_cast<const double*>(st + kOffLo)[ls];
+                    const double up = reinterpret_cast<const double*>(st + kOffUp)[ls];
+                    sum = fma(l, ld_x(xo + r - 1), up * ld_x(xo + r + 1)) + acc;
+                }
+                const double id = reinterpret_cast<const double*>(st + kOffInvd)[ls];
+                double xr = (DAMP || CHECK) ? ld_x(xo + r) : 0.0;
+                double yv = DAMP ? fma(1.0 - a.omega, xr, a.omega * (id * sum)) : id * sum;
+                if (a.pre_scale != nullptr) {
+                    const double sc = *a.pre_scale;
+                    yv *= sc;
+                    xr *= sc;
+                }
+                a.y[a.own_off + r] = yv;
+                if (CHECK) {
+                    const double df = fabs(yv - xr);
+                    sy += yv; sx += xr; sd += df; md = fmax(md, df / id); mx = fmax(mx, xr);
+                }
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);
+        }
+    }
+    if (CHECK) cta_check_partials<NCW + 1>(sy, sx, sd, md, mx, a.partials);
+}
+
+}  // namespace cme
