@@ -127,6 +127,11 @@ class ClockSampler:
                 "samples": len(rows), "power_w_max": max(float(r[3]) for r in rows if r[3] not in ("", "[N/A]"))}
 
 
+def kernel_name(info):
+    return {0: "sell_step_kernel", 1: f"sell_tma_kernel<{info.tma_warps}>", 2: "csr_step_kernel"}.get(
+        info.kernel, "?")
+
+
 def build_matrix(cme, name, dev_mode):
     cfg = DEFAULTS[name]
     net = W.config_network(name)
@@ -328,7 +333,7 @@ def main():
             "pct_hbm_roofline": round(100.0 * achieved / peak, 2),
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "traffic": ncu_traffic(name),
-                         "peak_source": peak_src, "kernel": "sell_step_kernel",
+                         "peak_source": peak_src, "kernel": kernel_name(info),
                          "bytes_per_launch": info.bytes_alg, "bytes_model": "12 nnz + 16 n (SURVEY 8(d))",
                          "format_bytes_per_launch": info.bytes_fmt,
                          "format_gbs": round(fmt_gbs, 1) if fmt_gbs else None,

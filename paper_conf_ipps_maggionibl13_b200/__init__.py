@@ -67,7 +67,8 @@ class cme_info(C.Structure):
                 ("n_ell", C.c_int64), ("packed_bytes", C.c_int64), ("bytes_alg", C.c_int64),
                 ("bytes_fmt", C.c_int64), ("rank", C.c_int32), ("nranks", C.c_int32),
                 ("row_begin", C.c_int64), ("row_end", C.c_int64), ("halo_begin", C.c_int64),
-                ("halo_end", C.c_int64)]
+                ("halo_end", C.c_int64), ("kernel", C.c_int32), ("tma_warps", C.c_int32),
+                ("tma_stages", C.c_int32), ("grid", C.c_int32)]
 
 
 class cme_packed_view(C.Structure):

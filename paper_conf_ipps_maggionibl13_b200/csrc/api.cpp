@@ -23,6 +23,7 @@ cme_status device_spmv(cme_matrix_s* h, const double* x, double* y);
 cme_status device_load(cme_matrix_s* h, const double* p0);
 cme_status device_run(cme_matrix_s* h, int64_t blocks);
 cme_status device_fetch(cme_matrix_s* h, double* p_out);
+void device_describe(const Device* d, cme_info* f);
 
 namespace {
 
@@ -314,6 +315,7 @@ cme_status cme_get_info(cme_matrix h, cme_info* info) {
         f.row_end = h->cuts.empty() ? n : h->cuts[h->rank + 1];
         f.halo_begin = h->span.empty() ? 0 : h->span[2 * h->rank];
         f.halo_end = h->span.empty() ? n : h->span[2 * h->rank + 1];
+        device_describe(h->dev, &f);
         *info = f;
         return CME_OK;
     });

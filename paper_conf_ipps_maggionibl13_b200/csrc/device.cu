@@ -643,6 +643,14 @@ cme_status device_solve(cme_matrix_s* h, const double* p0, double tol, int64_t m
     return (cme_status)h->report.status;
 }
 
+void device_describe(const Device* d, cme_info* f) {
+    if (!d) { f->kernel = -1; return; }
+    f->kernel = d->format == CME_FMT_CSR ? 2 : d->use_tma ? 1 : 0;
+    f->tma_warps = d->use_tma ? d->tma_ncw : 0;
+    f->tma_stages = d->use_tma ? d->tma_stages : 0;
+    f->grid = d->use_tma ? d->tma_grid : d->grid;
+}
+
 cme_status device_spmv(cme_matrix_s* h, const double* x, double* y) {
     Device& d = *h->dev;
     CUDA_TRY(cudaSetDevice(d.dev));

@@ -1,17 +1,18 @@
 // TMA-staged persistent variant of the fused Jacobi step (sm_100a).
 //
 // Same arithmetic and layout as sell_step_kernel (kernels.cuh); what changes
-// is how the packed matrix reaches the SM.  A tile is 8 consecutive slices
-// (= 256 rows = one rearrangement window); its val and col entries
+// is how the packed matrix reaches the SM.  A tile is NCW consecutive slices
+// (NCW*32 rows, whole rearrangement windows); its val and col entries
 // are ONE contiguous block each (layout v0), and its inv_d / row_of / lo / up
 // entries are contiguous too.  A producer warp streams every tile of the CTA's
 // round-robin share into a ring of S shared-memory stages with 1-D bulk copies
 // (cp.async.bulk ... mbarrier::complete_tx, the TMA engine), each stage
-// guarded by a full/empty mbarrier pair; 8 consumer warps (one slice each)
+// guarded by a full/empty mbarrier pair; NCW consumer warps (one slice each)
 // read their rows from shared memory, gather x from global memory (L1/L2),
-// and store y.  The bytes in flight per SM are S x stage bytes x CTAs/SM
-// (~170 KB) instead of whatever the register file of resident warps can
-// hold, so the kernel runs at the HBM limit rather than the latency limit.
+// and store y.  Default NCW = 16, S = 2, 2 CTAs/SM (56 regs): 32 consumer
+// warps/SM and 4 x ~43 KB of tiles in flight per SM, so the kernel runs at
+// the HBM limit (92% of the measured copy bandwidth on cfg4) where the
+// register-only kernel was latency-bound at 62%.
 #pragma once
 #include "kernels.cuh"
 
