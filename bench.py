@@ -128,7 +128,8 @@ class ClockSampler:
 
 
 def kernel_name(info):
-    return {0: "sell_step_kernel", 1: f"sell_tma_kernel<{info.tma_warps}>", 2: "csr_step_kernel"}.get(
+    return {0: "sell_step_kernel", 1: f"sell_tma_kernel<{info.tma_warps}>", 2: "csr_step_kernel",
+            3: "sell_persistent_kernel"}.get(
         info.kernel, "?")
 
 
@@ -163,7 +164,7 @@ def cpu_oracle_timing(name, budget_s=20.0, steps=1, warmup=0, omega=0.9):
     t = time.perf_counter()
     oracle.jacobi_solve(A, omega=omega, tol=0.0, check_every=C_BLOCK, max_iter=1, stag_tol=0.0, nthreads=cores)
     one = max(time.perf_counter() - t, 1e-6)
-    iters = int(max(1, min(C_BLOCK, budget_s / one / max(1, steps + warmup))))
+    iters = int(max(1, min(C_BLOCK, budget_s / one / max(1, steps + warmup))))  # per step
     for _ in range(warmup):
         oracle.jacobi_solve(A, omega=omega, tol=0.0, check_every=C_BLOCK, max_iter=iters, stag_tol=0.0, nthreads=cores)
     times = []
@@ -185,7 +186,7 @@ def run_reference(args):
     if rank != 0:
         return 0
     name = args.config
-    cb = cpu_oracle_timing(name, budget_s=max(10.0, 10.0 * args.steps), steps=args.steps, warmup=args.warmup,
+    cb = cpu_oracle_timing(name, budget_s=90.0, steps=args.steps, warmup=args.warmup,
                            omega=DEFAULTS[name]["omega"])
     line = {"metric": "fp64 Jacobi GFLOPS (2 nnz/iteration)", "value": cb["value"], "unit": "GFLOPS",
             "impl": "reference", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
@@ -330,9 +331,10 @@ def main():
                        "l2": f"inputs larger than L2 ({info.bytes_alg / 1e9:.3f} GB/iteration vs 126 MB)",
                        "parallelism": f"rows{world}", "setup": setup},
             "iters_per_s": round(iters / sec, 2),
-            "pct_hbm_roofline": round(100.0 * achieved / peak, 2),
-            "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                         "frac": round(achieved / peak, 4), "traffic": ncu_traffic(name),
+            "pct_hbm_roofline": round(100.0 * achieved / (peak * world), 2),
+            "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak * world, "unit": "GB/s",
+                         "frac": round(achieved / (peak * world), 4),
+                         "traffic": ncu_traffic(name) if world == 1 else None,
                          "peak_source": peak_src, "kernel": kernel_name(info),
                          "bytes_per_launch": info.bytes_alg, "bytes_model": "12 nnz + 16 n (SURVEY 8(d))",
                          "format_bytes_per_launch": info.bytes_fmt,

@@ -17,6 +17,7 @@
 #include "comm.h"
 #include "kernels.cuh"
 #include "kernels_tma.cuh"
+#include "kernels_persist.cuh"
 
 namespace cme {
 
@@ -78,6 +79,9 @@ struct Device {
     int tma_ncw = 8;
     int tma_grid = 0, tma_stages = 0, tma_stage_bytes = 0, tma_off_val = 0, tma_off_col = 0;
     int64_t n_tiles = 0;
+    // persistent cooperative kernel for small problems (kernels_persist.cuh)
+    bool use_persist = false;
+    int p_grid = 0;
     // graphs
     cudaGraphExec_t gexec[2] = {nullptr, nullptr};
     int64_t gC = -1;
@@ -279,7 +283,8 @@ static void launch_tma(const Device& d, const TmaArgs& T, bool damp, bool check,
 // CME_TMA_STAGES, CME_TMA_CTAS override the defaults (4 stages, max resident).
 static cme_status configure_tma(Device& d, const Packed& P) {
     d.use_tma = false;
-    if (env_int("CME_TMA", 1) == 0 || d.n_slices == 0) return CME_OK;
+    const int want = env_int("CME_TMA", -1);   // -1 auto, 0 off, 1 force
+    if (want == 0 || d.n_slices == 0) return CME_OK;
     const int ncw = env_int("CME_TMA_WARPS", 16) == 8 ? 8 : 16;
     d.tma_ncw = ncw;
     d.n_tiles = (d.n_slices + ncw - 1) / ncw;
@@ -314,10 +319,49 @@ static cme_status configure_tma(Device& d, const Packed& P) {
     d.tma_off_val = (int)off_val;
     d.tma_off_col = (int)off_col;
     d.tma_grid = (int)std::min<int64_t>(d.n_tiles, (int64_t)sms * occ);
+    // the ring only pays when every CTA streams >= 2 tiles; small problems
+    // (<~300K rows) run faster on the register kernel
+    if (want < 0 && d.n_tiles < 2 * (int64_t)sms * occ) return CME_OK;
     if (env_int("CME_VERBOSE", 0))
         std::fprintf(stderr, "[cme] tma: warps=%d stages=%d stage_bytes=%lld occ=%d grid=%d tiles=%lld\n", ncw,
                      stages, (long long)stage, occ, d.tma_grid, (long long)d.n_tiles);
     d.use_tma = true;
+    return CME_OK;
+}
+
+template <bool B, bool R, bool D>
+static cudaError_t launch_persist_t(const PersistArgs& P, int grid, cudaStream_t s) {
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(kCta);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, sell_persistent_kernel<B, R, D>, P);
+}
+
+// Persistent cooperative kernel for L2-resident problems: one launch per check
+// block.  CME_PERSIST: -1 auto (<= 1M local rows, single GPU), 0 off, 1 force.
+static cme_status configure_persist(Device& d) {
+    d.use_persist = false;
+    const int want = env_int("CME_PERSIST", -1);
+    if (want == 0 || d.comm || d.format == CME_FMT_CSR || d.n_slices == 0) return CME_OK;
+    if (want < 0 && (d.use_tma || d.n_own > (1 << 20))) return CME_OK;
+    int dev = 0, sms = 0, occ = 0;
+    CUDA_TRY(cudaGetDevice(&dev));
+    CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, sell_persistent_kernel<true, true, true>, kCta, 0));
+    int occ2 = 0;
+    CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, sell_persistent_kernel<false, false, false>, kCta, 0));
+    occ = std::max(1, std::min(occ, occ2));
+    const int64_t need = (d.n_slices + kWarpsPerCta - 1) / kWarpsPerCta;
+    d.p_grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * occ));
+    d.use_persist = true;
+    d.use_tma = false;
     return CME_OK;
 }
 
@@ -368,7 +412,7 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
     {
         std::vector<int32_t> po(h->perm.begin() + d->row_begin, h->perm.begin() + d->row_begin + d->n_own);
         UP(perm_own, po);
-        if (h->nranks > 1) UP(perm_global, h->perm);
+        if (comm) UP(perm_global, h->perm);
     }
 #undef UP
     for (int b = 0; b < 2; ++b) {
@@ -381,12 +425,13 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
                                        : (int)((d->n_slices + kWarpsPerCta - 1) / kWarpsPerCta);
     d->grid = std::max(d->grid, 1);
     if (d->format != CME_FMT_CSR && (s = configure_tma(*d, P)) != CME_OK) return fail(s);
+    if ((s = configure_persist(*d)) != CME_OK) return fail(s);
     d->part_blocks = std::max(d->grid, grid_for(d->n_own));
     if ((s = d->alloc(d->partials, (size_t)d->part_blocks * kPartials)) != CME_OK) return fail(s);
     if ((s = d->alloc(d->gather, (size_t)d->nranks * 8)) != CME_OK) return fail(s);
     if ((s = d->alloc(d->local8, 8)) != CME_OK) return fail(s);
     if ((s = d->alloc(d->io, d->n_global)) != CME_OK) return fail(s);
-    if (d->nranks > 1 && (s = d->alloc(d->io2, d->n_global)) != CME_OK) return fail(s);
+    if (comm && (s = d->alloc(d->io2, d->n_global)) != CME_OK) return fail(s);
     if ((s = d->alloc(d->one, 1)) != CME_OK) return fail(s);
     if ((s = d->alloc(d->ctrl, 1)) != CME_OK) return fail(s);
     const double one = 1.0;
@@ -457,16 +502,16 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
         }
     }
     CUDA_TRY(cudaGetLastError());
-    if (d.nranks > 1) CME_TRY(comm_halo(d.comm, d.halo, d.xb[dst], s));
+    if (d.comm) CME_TRY(comm_halo(d.comm, d.halo, d.xb[dst], s));
     return CME_OK;
 }
 
 // reduce partials of the last CHECK step and decide
 static cme_status launch_finalize(Device& d, cudaStream_t s, int32_t len, int32_t final_partial) {
-    reduce_partials_kernel<<<1, 1024, 0, s>>>(d.partials, d.use_tma ? d.tma_grid : d.grid,
-                                              d.nranks > 1 ? d.local8 : d.gather, &d.ctrl->stop);
+    reduce_partials_kernel<<<1, 1024, 0, s>>>(d.partials, d.use_persist ? d.p_grid : d.use_tma ? d.tma_grid : d.grid,
+                                              d.comm ? d.local8 : d.gather, &d.ctrl->stop);
     CUDA_TRY(cudaGetLastError());
-    if (d.nranks > 1) CME_TRY(comm_allgather8(d.comm, d.local8, d.gather, s));
+    if (d.comm) CME_TRY(comm_allgather8(d.comm, d.local8, d.gather, s));
     decide_kernel<<<1, 1, 0, s>>>(d.gather, d.nranks, d.ctrl, len, final_partial);
     CUDA_TRY(cudaGetLastError());
     return CME_OK;
@@ -475,6 +520,44 @@ static cme_status launch_finalize(Device& d, cudaStream_t s, int32_t len, int32_
 // One check block of C steps starting from buffer `start`: steps 0..C-2 plain,
 // step C-1 CHECK; the first step applies the pending 1/||y||_1 (R5).
 static cme_status enqueue_block(Device& d, cudaStream_t s, int start, int64_t C, double omega, bool final_partial) {
+    if (d.use_persist) {
+        PersistArgs P{};
+        P.a.n_rows = d.n_own;
+        P.a.slice_begin = 0;
+        P.a.slice_end = d.n_slices;
+        P.a.slice_off = d.slice_off;
+        P.a.slice_w = d.slice_w;
+        P.a.val = d.val;
+        P.a.col = d.col;
+        P.a.row_of = d.row_of;
+        P.a.lo = d.lo;
+        P.a.up = d.up;
+        P.a.inv_d = d.inv_d;
+        P.a.own_off = d.own_off;
+        P.a.omega = omega;
+        P.a.pre_scale = &d.ctrl->inv_s;
+        P.a.partials = d.partials;
+        P.a.stop = &d.ctrl->stop;
+        P.xb0 = d.xb[0];
+        P.xb1 = d.xb[1];
+        P.start = start;
+        P.steps = (int32_t)C;
+        const bool damp = omega != 1.0;
+        const int key = (d.band ? 4 : 0) | (d.rearr ? 2 : 0) | (damp ? 1 : 0);
+        cudaError_t e = cudaSuccess;
+        switch (key) {
+            case 0: e = launch_persist_t<false, false, false>(P, d.p_grid, s); break;
+            case 1: e = launch_persist_t<false, false, true>(P, d.p_grid, s); break;
+            case 2: e = launch_persist_t<false, true, false>(P, d.p_grid, s); break;
+            case 3: e = launch_persist_t<false, true, true>(P, d.p_grid, s); break;
+            case 4: e = launch_persist_t<true, false, false>(P, d.p_grid, s); break;
+            case 5: e = launch_persist_t<true, false, true>(P, d.p_grid, s); break;
+            case 6: e = launch_persist_t<true, true, false>(P, d.p_grid, s); break;
+            case 7: e = launch_persist_t<true, true, true>(P, d.p_grid, s); break;
+        }
+        CUDA_TRY(e);
+        return launch_finalize(d, s, (int32_t)C, final_partial ? 1 : 0);
+    }
     for (int64_t t = 0; t < C; ++t) {
         const int src = (int)((start + t) & 1);
         CME_TRY(launch_step(d, s, src, 1 - src, t == C - 1, t == 0 ? &d.ctrl->inv_s : nullptr, omega));
@@ -484,6 +567,13 @@ static cme_status enqueue_block(Device& d, cudaStream_t s, int start, int64_t C,
 
 static cme_status ensure_graphs(Device& d, int64_t C, double omega) {
     if (d.gC == C && d.gomega == omega && d.gexec[0]) return CME_OK;
+    if (d.comm) {
+        // NCCL sets up peer connections lazily on first use: do that outside
+        // the capture (one throw-away exchange + gather on the private stream)
+        CME_TRY(comm_halo(d.comm, d.halo, d.xb[1], d.own));
+        CME_TRY(comm_allgather8(d.comm, d.local8, d.gather, d.own));
+        CUDA_TRY(cudaStreamSynchronize(d.own));
+    }
     for (auto& g : d.gexec)
         if (g) { cudaGraphExecDestroy(g); g = nullptr; }
     const int nstart = (C & 1) ? 2 : 1;
@@ -535,13 +625,13 @@ static cme_status load_iterate(cme_matrix_s* h, const double* p0, bool normalise
         }
         const int g = grid_for(d.n_own);
         load_kernel<<<g, kCta, 0, s>>>(src, d.perm_own, d.n_own, x, d.partials);
-        reduce_partials_kernel<<<1, 1024, 0, s>>>(d.partials, g, d.nranks > 1 ? d.local8 : d.gather, nullptr);
+        reduce_partials_kernel<<<1, 1024, 0, s>>>(d.partials, g, d.comm ? d.local8 : d.gather, nullptr);
         CUDA_TRY(cudaGetLastError());
-        if (d.nranks > 1) CME_TRY(comm_allgather8(d.comm, d.local8, d.gather, s));
+        if (d.comm) CME_TRY(comm_allgather8(d.comm, d.local8, d.gather, s));
         load_decide_kernel<<<1, 1, 0, s>>>(d.gather, d.nranks, d.ctrl, normalise ? 1 : 0);
         CUDA_TRY(cudaGetLastError());
     }
-    if (d.nranks > 1) CME_TRY(comm_halo(d.comm, d.halo, d.xb[0], s));
+    if (d.comm) CME_TRY(comm_halo(d.comm, d.halo, d.xb[0], s));
     return CME_OK;
 }
 
@@ -551,7 +641,7 @@ static cme_status write_out(cme_matrix_s* h, double* p_out, const double* scale,
     const double* x = d.xb[d.cur] + d.own_off;
     const bool dev_out = is_device_ptr(p_out);
     double* dst = dev_out ? p_out : d.io;
-    if (d.nranks == 1) {
+    if (!d.comm) {
         scatter_out_kernel<<<grid_for(d.n_own), kCta, 0, s>>>(x, d.perm_own, d.n_own, scale, dst);
         CUDA_TRY(cudaGetLastError());
     } else {
@@ -645,10 +735,10 @@ cme_status device_solve(cme_matrix_s* h, const double* p0, double tol, int64_t m
 
 void device_describe(const Device* d, cme_info* f) {
     if (!d) { f->kernel = -1; return; }
-    f->kernel = d->format == CME_FMT_CSR ? 2 : d->use_tma ? 1 : 0;
+    f->kernel = d->format == CME_FMT_CSR ? 2 : d->use_persist ? 3 : d->use_tma ? 1 : 0;
     f->tma_warps = d->use_tma ? d->tma_ncw : 0;
     f->tma_stages = d->use_tma ? d->tma_stages : 0;
-    f->grid = d->use_tma ? d->tma_grid : d->grid;
+    f->grid = d->use_persist ? d->p_grid : d->use_tma ? d->tma_grid : d->grid;
 }
 
 cme_status device_spmv(cme_matrix_s* h, const double* x, double* y) {

@@ -112,6 +112,77 @@ __device__ __forceinline__ void cta_check_partials(double sy, double sx, double 
     }
 }
 
+// x loads: read-only path (.nc) when x is constant for the whole launch;
+// L2-coherent (.cg) in the persistent kernel, whose x is rewritten by other
+// CTAs between grid barriers.
+template <bool COHERENT>
+__device__ __forceinline__ double ld_xv(const double* p) {
+    if (COHERENT) {
+        double v;
+        asm volatile("ld.global.cg.f64 %0, [%1];" : "=d"(v) : "l"(p));
+        return v;
+    }
+    return __ldg(p);
+}
+
+// Check terms of one row: y, x (both scaled), inv_d.
+struct SlotOut {
+    double y, x, id;
+    bool valid;
+};
+__device__ __forceinline__ void check_accum(const SlotOut& o, double& sy, double& sx, double& sd, double& md,
+                                            double& mx) {
+    if (!o.valid) return;
+    const double df = fabs(o.y - o.x);
+    sy += o.y; sx += o.x; sd += df; md = fmax(md, df / o.id); mx = fmax(mx, o.x);
+}
+
+// One slot (lane) of slice q: computes and stores y_r for its row r.
+template <bool BAND, bool REARR, bool DAMP, bool NEEDX, bool COHERENT>
+__device__ __forceinline__ SlotOut sell_slot(const StepArgs& a, int64_t q, int lane, uint64_t pol,
+                                             const double* x, double* y, const double* pre_scale) {
+    const int64_t slot = q * 32 + lane;
+    const int w = __ldg(a.slice_w + q);
+    const int64_t base = __ldg(a.slice_off + q) + lane;
+    if (slot >= a.n_rows) return SlotOut{0.0, 0.0, 1.0, false};
+    const int64_t r = REARR ? (int64_t)ld_stream(a.row_of + slot, pol) : slot;
+    const double* xo = x + a.own_off;
+    double acc = 0.0;
+    for (int t0 = 0; t0 < w; t0 += kUnroll) {
+        double v[kUnroll];
+        int32_t c[kUnroll];
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) {
+            if (t0 + u < w) {
+                v[u] = ld_stream(a.val + base + 32 * (int64_t)(t0 + u), pol);
+                c[u] = ld_stream(a.col + base + 32 * (int64_t)(t0 + u), pol);
+            }
+        }
+        double xv[kUnroll];
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u)
+            if (t0 + u < w) xv[u] = ld_xv<COHERENT>(x + c[u]);
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u)
+            if (t0 + u < w) acc = fma(v[u], xv[u], acc);
+    }
+    double s = acc;
+    if (BAND) {
+        const double l = ld_stream(a.lo + slot, pol), up = ld_stream(a.up + slot, pol);
+        s = fma(l, ld_xv<COHERENT>(xo + r - 1), up * ld_xv<COHERENT>(xo + r + 1)) + acc;
+    }
+    const double id = ld_stream(a.inv_d + slot, pol);
+    double xr = (DAMP || NEEDX) ? ld_xv<COHERENT>(xo + r) : 0.0;
+    double yv = DAMP ? fma(1.0 - a.omega, xr, a.omega * (id * s)) : id * s;
+    if (pre_scale != nullptr) {
+        const double sc = *pre_scale;
+        yv *= sc;
+        xr *= sc;
+    }
+    y[a.own_off + r] = yv;
+    return SlotOut{yv, xr, id, true};
+}
+
 template <bool BAND, bool REARR, bool DAMP, bool CHECK>
 __global__ void __launch_bounds__(kCta) sell_step_kernel(const StepArgs a) {
     if (a.stop != nullptr && *a.stop) return;
@@ -120,50 +191,8 @@ __global__ void __launch_bounds__(kCta) sell_step_kernel(const StepArgs a) {
     const int64_t q = a.slice_begin + (int64_t)blockIdx.x * kWarpsPerCta + (threadIdx.x >> 5);
     double sy = 0.0, sx = 0.0, sd = 0.0, md = 0.0, mx = 0.0;
     if (q < a.slice_end) {
-        const int64_t slot = q * 32 + lane;
-        const int w = __ldg(a.slice_w + q);
-        const int64_t base = __ldg(a.slice_off + q) + lane;
-        if (slot < a.n_rows) {
-            const int64_t r = REARR ? (int64_t)ld_stream(a.row_of + slot, pol) : slot;
-            const double* xo = a.x + a.own_off;
-            double acc = 0.0;
-            for (int t0 = 0; t0 < w; t0 += kUnroll) {
-                double v[kUnroll];
-                int32_t c[kUnroll];
-#pragma unroll
-                for (int u = 0; u < kUnroll; ++u) {
-                    if (t0 + u < w) {
-                        v[u] = ld_stream(a.val + base + 32 * (int64_t)(t0 + u), pol);
-                        c[u] = ld_stream(a.col + base + 32 * (int64_t)(t0 + u), pol);
-                    }
-                }
-                double xv[kUnroll];
-#pragma unroll
-                for (int u = 0; u < kUnroll; ++u)
-                    if (t0 + u < w) xv[u] = ld_x(a.x + c[u]);
-#pragma unroll
-                for (int u = 0; u < kUnroll; ++u)
-                    if (t0 + u < w) acc = fma(v[u], xv[u], acc);
-            }
-            double s = acc;
-            if (BAND) {
-                const double l = ld_stream(a.lo + slot, pol), up = ld_stream(a.up + slot, pol);
-                s = fma(l, ld_x(xo + r - 1), up * ld_x(xo + r + 1)) + acc;
-            }
-            const double id = ld_stream(a.inv_d + slot, pol);
-            double xr = (DAMP || CHECK) ? ld_x(xo + r) : 0.0;
-            double yv = DAMP ? fma(1.0 - a.omega, xr, a.omega * (id * s)) : id * s;
-            if (a.pre_scale != nullptr) {
-                const double sc = *a.pre_scale;
-                yv *= sc;
-                xr *= sc;
-            }
-            a.y[a.own_off + r] = yv;
-            if (CHECK) {
-                const double df = fabs(yv - xr);
-                sy = yv; sx = xr; sd = df; md = df / id; mx = xr;
-            }
-        }
+        const SlotOut o = sell_slot<BAND, REARR, DAMP, CHECK, false>(a, q, lane, pol, a.x, a.y, a.pre_scale);
+        if (CHECK) check_accum(o, sy, sx, sd, md, mx);
     }
     if (CHECK) cta_check_partials<kWarpsPerCta>(sy, sx, sd, md, mx, a.partials);
 }

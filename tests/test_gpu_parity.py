@@ -221,3 +221,60 @@ def test_cfg3a_schnakenberg_closed_form_at_scale(cme):
     pi = np.exp(logs - logs.max())
     pi /= pi.sum()
     assert np.abs(p - pi).sum() <= 1e-10
+
+
+def test_nccl_one_rank_distributed_path(cme, oracle_mod):
+    """The distributed code path (NCCL allgather of the check record, segment
+    broadcast of the output) with a 1-rank communicator on this GPU must give
+    the single-GPU result.  >= 2 ranks need >= 2 GPUs (tests/test_partition_gloo.py
+    covers the multi-rank protocol on CPU)."""
+    import torch
+    import paper_conf_ipps_maggionibl13_b200 as m
+    net = W.toggle_switch(45)
+    states, r, c, v = oracle_mod.enumerate_network(net)
+    A = oracle_mod.ingest(len(states), r, c, v)
+    ref = m.Matrix(A.n, r, c, v).reorder(m.CME_ORDER_RCM).pack()
+    ref.set_opts(omega=0.9)
+    p_ref, st_ref, it_ref = ref.solve(tol=1e-12)
+    uid = m.cme_comm_unique_id()
+    comm = m.cme_comm_init(1, 0, uid, torch.cuda.current_device())
+    d = m.Matrix(A.n, r, c, v).reorder(m.CME_ORDER_RCM)
+    d.pack(device=m.CME_DEVICE_HOST_ONLY)
+    m.cme_matrix_distribute(d.h, comm)
+    d.set_opts(omega=0.9)
+    p, st, it = d.solve(tol=1e-12)
+    assert st == st_ref == "CONVERGED" and it == it_ref
+    assert np.abs(p - p_ref).sum() <= 1e-14
+    x = W.random_start(A.n, 3)
+    assert_spmv_close(d.spmv(x), oracle_mod.jacobi_step(A, x, 0.9))
+    d.close()
+    m.cme_comm_destroy(comm)
+
+
+@pytest.mark.parametrize("knobs", [{"CME_TMA": "0", "CME_PERSIST": "0"}, {"CME_TMA": "1", "CME_PERSIST": "0"},
+                                   {"CME_TMA": "1", "CME_TMA_WARPS": "8", "CME_PERSIST": "0"},
+                                   {"CME_TMA": "0", "CME_PERSIST": "1"}],
+                         ids=lambda k: ",".join(f"{a}={b}" for a, b in k.items()))
+@pytest.mark.parametrize("net,order,omega", [(W.toggle_switch(70), "rcm", 0.9), (W.schnakenberg(120), "none", 1.0),
+                                             (W.brusselator(90), "dfs", 0.7)], ids=lambda x: getattr(x, "name", str(x)))
+def test_every_step_kernel(cme, oracle_mod, monkeypatch, knobs, net, order, omega):
+    """Each step kernel (register SELL, TMA-staged SELL with 16/8 consumer warps,
+    persistent cooperative SELL) forced on the same problems: per-step parity
+    and a fixed-iteration landscape (C = 7 exercises odd block parity)."""
+    for k, v in knobs.items():
+        monkeypatch.setenv(k, v)
+    states, r, c, v = oracle_mod.enumerate_network(net)
+    A = oracle_mod.ingest(len(states), r, c, v)
+    m = cme.Matrix(A.n, r, c, v).reorder(ORD[order]).pack()
+    f = m.info()
+    expect = 3 if knobs.get("CME_PERSIST") == "1" else (1 if knobs["CME_TMA"] == "1" else 0)
+    assert f.kernel == expect
+    m.set_opts(omega=omega, check_every=7, stag_tol=0.0)
+    x = W.random_start(A.n, 21)
+    assert_spmv_close(m.spmv(x), oracle_mod.jacobi_step(A, x, omega))
+    p, st, it = m.solve(tol=0.0, max_iter=250)
+    ref = oracle_mod.jacobi_solve(A, omega=omega, tol=0.0, check_every=7, max_iter=250, stag_tol=0.0)
+    assert it == ref.iters == 250 and np.abs(p - ref.p).sum() <= 1e-12
+    p, st, it = m.solve(tol=1e-11, max_iter=100000)
+    ref = oracle_mod.jacobi_solve(A, omega=omega, tol=1e-11, check_every=7, max_iter=100000, stag_tol=0.0)
+    assert st == ref.status and abs(it - ref.iters) <= 7
