@@ -239,8 +239,8 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
-    from paper_conf_ipps_maggionibl13_b200 import build as B
-    B.build()
+    import __graft_entry__
+    __graft_entry__.build()
     import paper_conf_ipps_maggionibl13_b200 as cme
 
     comm = None

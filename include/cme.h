@@ -79,9 +79,12 @@ enum { CME_ORDER_NONE = 0, CME_ORDER_DFS = 1, CME_ORDER_RCM = 2 };
  * RCM: reverse Cuthill-McKee of the pattern of A + A^T, George-Liu
  * pseudo-peripheral start per component (root ignored).  Host-only work. */
 cme_status cme_reorder(cme_matrix h, int method, int64_t root);
+/* A caller-chosen ordering (e.g. a seeded random permutation, the locality
+ * stress test of P:L225): new_to_old must be a permutation of 0..n-1. */
+cme_status cme_set_permutation(cme_matrix h, const int32_t* new_to_old);
 
 /* ---- packing ----------------------------------------------- */
-enum { CME_FMT_DIAG_SELL = 0, CME_FMT_ELL = 1, CME_FMT_CSR = 2 };
+enum { CME_FMT_DIAG_SELL = 0, CME_FMT_ELL = 1, CME_FMT_CSR = 2, CME_FMT_SELL256 = 3 };
 enum { CME_BAND_AUTO = 0, CME_BAND_ALWAYS = 1, CME_BAND_NEVER = 2 };
 #define CME_DEVICE_HOST_ONLY (-2)
 typedef struct cme_pack_opts {
@@ -93,8 +96,11 @@ typedef struct cme_pack_opts {
 } cme_pack_opts;
 /* Builds the packed layout on the host, runs the directed
  * period test (R1), uploads to device memory.  opts == NULL: {32, 256, AUTO, -1}.
- * CME_FMT_ELL = one global width (no rearrangement), CME_FMT_CSR = plain CSR
- * (ablation arms).  Errors: INVALID_ARG, BAD_STATE, OOM, CUDA, NO_DEVICE. */
+ * Ablation arms (Tables II-III): CME_FMT_ELL = one global width
+ * (+DIA band per opts.band), CME_FMT_SELL256 = sliced ELL with 256-row slices
+ * ([5], slice = CTA), both without rearrangement; CME_FMT_CSR = plain CSR.
+ * window may be any size (window >= n = the global nnz reordering, pJDS [20]).
+ * Errors: INVALID_ARG, BAD_STATE, OOM, CUDA, NO_DEVICE. */
 cme_status cme_pack(cme_matrix h, int format, const cme_pack_opts* opts);
 
 /* ---- solver -------------------------------------------------------------- */

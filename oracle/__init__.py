@@ -199,10 +199,11 @@ def period(A: CSR, root: int = 0) -> int:
 BAND = {"auto": 0, "always": 1, "never": 2}
 
 
-def pack(A: CSR, window: int = 256, band: str = "auto", uniform: bool = False) -> dict:
-    """Layout v0 arrays of an already-ordered matrix."""
+def pack(A: CSR, window: int = 256, band: str = "auto", uniform: bool = False, group: int = 1) -> dict:
+    """Layout v0 arrays of an already-ordered matrix.
+    group = slices sharing a width (1 warp-grained, 8 block-sliced); uniform = plain ELL."""
     P = _Packed()
-    _check(lib().oracle_pack(A.n, *A._a(), window, BAND[band], int(uniform), C.byref(P)),
+    _check(lib().oracle_pack(A.n, *A._a(), window, BAND[band], 0 if uniform else group, C.byref(P)),
            "oracle_pack")
     try:
         def cp(ptr, k, dt):

@@ -590,9 +590,9 @@ static double find_entry(const int64_t* rp, const int32_t* col, const double* va
 }
 
 int oracle_pack(int64_t n, const int64_t* rp, const int32_t* col, const double* val,
-                const double* diag, int32_t window, int32_t band, int32_t uniform,
+                const double* diag, int32_t window, int32_t band, int32_t group,
                 oracle_packed* out) {
-    if (n <= 0 || !out || band < 0 || band > 2) return ORACLE_INVALID_ARG;
+    if (n <= 0 || !out || band < 0 || band > 2 || group < 0) return ORACLE_INVALID_ARG;
     memset(out, 0, sizeof(*out));
     /* band rule: DIA pays off when the +-1 density exceeds 8/12 = 2/3 */
     int64_t cnt = 0;
@@ -640,15 +640,28 @@ int oracle_pack(int64_t n, const int64_t* rp, const int32_t* col, const double* 
     }
     int32_t kmax = 0;
     for (int64_t i = 0; i < n; i++) if (c[i] > kmax) kmax = c[i];
-    out->slice_off[0] = 0;
+    /* width of a slice = max ELL count of its rows; slices of one
+     * group share the group's max (group 8 = 256-row block-sliced ELL [5]);
+     * group 0 = one global width (plain ELL) */
     for (int64_t q = 0; q < n_slices; q++) {
         int32_t wq = 0;
         for (int64_t s = q * 32; s < q * 32 + 32; s++)
             if (s < n && c[out->row_of[s]] > wq) wq = c[out->row_of[s]];
-        if (uniform) wq = kmax;
         out->slice_w[q] = wq;
-        out->slice_off[q + 1] = out->slice_off[q] + 32 * (int64_t)wq;
     }
+    if (group == 0) {
+        for (int64_t q = 0; q < n_slices; q++) out->slice_w[q] = kmax;
+    } else if (group > 1) {
+        for (int64_t g0 = 0; g0 < n_slices; g0 += group) {
+            int64_t g1 = g0 + group < n_slices ? g0 + group : n_slices;
+            int32_t wg = 0;
+            for (int64_t q = g0; q < g1; q++) if (out->slice_w[q] > wg) wg = out->slice_w[q];
+            for (int64_t q = g0; q < g1; q++) out->slice_w[q] = wg;
+        }
+    }
+    out->slice_off[0] = 0;
+    for (int64_t q = 0; q < n_slices; q++)
+        out->slice_off[q + 1] = out->slice_off[q] + 32 * (int64_t)out->slice_w[q];
     int64_t n_ell = out->slice_off[n_slices];
     out->n_ell = n_ell;
     out->val = (double*)malloc(sizeof(double) * (n_ell ? n_ell : 1));

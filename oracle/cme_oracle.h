@@ -74,9 +74,10 @@ typedef struct {
     int32_t* col;     /* [n_ell]                                                   */
 } oracle_packed;
 /* band: 0 AUTO (+-1 density >= 2/3), 1 ALWAYS, 2 NEVER.  window <= 1 = off.
- * uniform != 0: every slice gets the global max width (plain ELL arm). */
+ * group: slices sharing one width -- 1 warp-grained sliced ELL,
+ * 8 = 256-row block-sliced ELL ([5]), 0 = one global width (plain ELL). */
 int oracle_pack(int64_t n, const int64_t* row_ptr, const int32_t* col, const double* val,
-                const double* diag, int32_t window, int32_t band, int32_t uniform,
+                const double* diag, int32_t window, int32_t band, int32_t group,
                 oracle_packed* out);
 void oracle_packed_free(oracle_packed* p);
 

@@ -20,7 +20,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libcme.so")
 
 if not os.path.exists(LIB_PATH):
-    raise ImportError(f"{LIB_PATH} is not built; run `python -m paper_conf_ipps_maggionibl13_b200.build` "
+    raise ImportError(f"{LIB_PATH} is not built; run `python paper_conf_ipps_maggionibl13_b200/build.py` "
                       "(nvcc, sm_100a).  There is no fallback path.")
 
 _lib = C.CDLL(LIB_PATH, mode=C.RTLD_GLOBAL)
@@ -31,7 +31,7 @@ CME_ERR_BAD_STATE, CME_ERR_OOM, CME_ERR_CUDA, CME_ERR_NCCL = 4, 5, 6, 7
 CME_NOT_CONVERGED, CME_STAGNATED, CME_ERR_NUMERIC, CME_ERR_NO_DEVICE = 8, 9, 10, 11
 CME_DIAG_FROM_COLSUMS, CME_DIAG_GIVEN = 0, 1
 CME_ORDER_NONE, CME_ORDER_DFS, CME_ORDER_RCM = 0, 1, 2
-CME_FMT_DIAG_SELL, CME_FMT_ELL, CME_FMT_CSR = 0, 1, 2
+CME_FMT_DIAG_SELL, CME_FMT_ELL, CME_FMT_CSR, CME_FMT_SELL256 = 0, 1, 2, 3
 CME_BAND_AUTO, CME_BAND_ALWAYS, CME_BAND_NEVER = 0, 1, 2
 CME_DEVICE_HOST_ONLY = -2
 CME_STOP_DELTA_L1, CME_STOP_PAPER_RESID = 0, 1
@@ -90,6 +90,7 @@ _SIGS = {
     "cme_matrix_create_coo": [C.c_int64, C.c_int64, i32p, i32p, f64p, C.c_uint32, _p(vp)],
     "cme_matrix_create_csr": [C.c_int64, i64p, i32p, f64p, C.c_uint32, _p(vp)],
     "cme_reorder": [vp, C.c_int, C.c_int64],
+    "cme_set_permutation": [vp, i32p],
     "cme_pack": [vp, C.c_int, _p(cme_pack_opts)],
     "cme_set_solver_opts": [vp, _p(cme_solver_opts)],
     "cme_jacobi_solve": [vp, vp, C.c_double, C.c_int64, vp, i64p],
@@ -184,6 +185,11 @@ def cme_matrix_create_csr(n, row_ptr, col, rate, flags=CME_DIAG_FROM_COLSUMS):
 
 def cme_reorder(h, method=CME_ORDER_NONE, root=0):
     _chk(_lib.cme_reorder(h, method, root), "cme_reorder")
+
+
+def cme_set_permutation(h, new_to_old):
+    p = _arr(new_to_old, np.int32)
+    _chk(_lib.cme_set_permutation(h, p.ctypes.data_as(i32p)), "cme_set_permutation")
 
 
 def cme_pack(h, fmt=CME_FMT_DIAG_SELL, window=256, band=CME_BAND_AUTO, device=-1):
@@ -362,6 +368,10 @@ class Matrix:
 
     def reorder(self, method=CME_ORDER_NONE, root=0):
         cme_reorder(self.h, method, root)
+        return self
+
+    def set_permutation(self, new_to_old):
+        cme_set_permutation(self.h, new_to_old)
         return self
 
     def pack(self, fmt=CME_FMT_DIAG_SELL, window=256, band=CME_BAND_AUTO, device=-1):

@@ -1,6 +1,8 @@
 """Build libcme.so in-tree with nvcc for sm_100a (no JIT, no torch extension cache).
 
-    python -m paper_conf_ipps_maggionibl13_b200.build [--force]
+    python paper_conf_ipps_maggionibl13_b200/build.py [--force] [-v]
+
+(Run it by path: importing the package loads libcme.so.)
 """
 from __future__ import annotations
 

@@ -52,7 +52,7 @@ int32_t ell_count(const Csr& B, int64_t r, bool band_on) {
 void plan_cuts(cme_matrix_s* h, int nranks) {
     const Csr& B = h->B;
     const int64_t n = B.n;
-    const int64_t unit = std::max<int64_t>(32, h->P.window > 1 ? h->P.window : 32);
+    const int64_t unit = std::max<int64_t>(h->P.group > 1 ? 32 * h->P.group : 32, h->P.window > 1 ? h->P.window : 32);
     std::vector<double> pre(n + 1, 0.0);
     for (int64_t i = 0; i < n; ++i) pre[i + 1] = pre[i] + 12.0 * (double)(B.rp[i + 1] - B.rp[i]) + 28.0;
     h->cuts.assign(nranks + 1, 0);
@@ -111,8 +111,11 @@ cme_status build_local(cme_matrix_s* h, int nranks, int rank) {
     if (h->format == CME_FMT_CSR) {
         pack_csr_rows(h->B, r0, r1, shift, h->P);
     } else {
-        const bool ell = h->format == CME_FMT_ELL;
-        pack_rows(h->B, r0, r1, shift, ell ? 1 : h->popts.window, h->band_on, ell, h->global_kmax, h->P);
+        // DIAG_SELL: warp-grained slices + local rearrangement;
+        // ELL: one global width; SELL256: 256-row block slices [5]
+        const int32_t group = h->format == CME_FMT_ELL ? 0 : h->format == CME_FMT_SELL256 ? 8 : 1;
+        const int32_t window = h->format == CME_FMT_DIAG_SELL ? h->popts.window : 1;
+        pack_rows(h->B, r0, r1, shift, window, h->band_on, group, h->global_kmax, h->P);
     }
     return CME_OK;
 }
@@ -176,12 +179,29 @@ cme_status cme_reorder(cme_matrix h, int method, int64_t root) {
     });
 }
 
+cme_status cme_set_permutation(cme_matrix h, const int32_t* new_to_old) {
+    if (!valid(h, 1) || !new_to_old) return CME_ERR_INVALID_ARG;
+    if (h->stage != 1) { set_error("cme_set_permutation must precede cme_pack"); return CME_ERR_BAD_STATE; }
+    return guarded([&] {
+        const int64_t n = h->A.n;
+        std::vector<char> seen(n, 0);
+        for (int64_t r = 0; r < n; ++r) {
+            const int32_t o = new_to_old[r];
+            if (o < 0 || o >= n || seen[o]) { set_error("not a permutation"); return CME_ERR_INVALID_ARG; }
+            seen[o] = 1;
+        }
+        h->perm.assign(new_to_old, new_to_old + n);
+        h->order = -1;
+        return CME_OK;
+    });
+}
+
 cme_status cme_pack(cme_matrix h, int format, const cme_pack_opts* opts) {
     if (!valid(h, 1)) return CME_ERR_INVALID_ARG;
     if (h->stage == 3) { set_error("matrix already distributed"); return CME_ERR_BAD_STATE; }
     cme_pack_opts o = opts ? *opts : cme_pack_opts{32, 256, CME_BAND_AUTO, -1};
-    if (format < CME_FMT_DIAG_SELL || format > CME_FMT_CSR || o.slice != 32 || o.band < 0 || o.band > 2 ||
-        o.window < 0 || o.window > (1 << 20) || o.device < CME_DEVICE_HOST_ONLY) {
+    if (format < CME_FMT_DIAG_SELL || format > CME_FMT_SELL256 || o.slice != 32 || o.band < 0 || o.band > 2 ||
+        o.window < 0 || o.device < CME_DEVICE_HOST_ONLY) {
         set_error("pack: bad format or options (slice must be 32)");
         return CME_ERR_INVALID_ARG;
     }

@@ -37,7 +37,7 @@ void permute(const Csr& A, const std::vector<int32_t>& new_to_old, Csr& out);
 // [r0, r1) of an ordered matrix, columns shifted by -col_shift.
 struct Packed {
     int64_t n = 0, n_slots = 0, n_slices = 0, n_ell = 0;
-    int32_t band_on = 0, window = 1, uniform = 0;
+    int32_t band_on = 0, window = 1, group = 1;
     std::vector<double> lo, up, inv_d;    // slot order
     std::vector<int32_t> row_of;          // slot -> local row
     std::vector<int64_t> slice_off;       // n_slices + 1
@@ -50,8 +50,9 @@ struct Packed {
     std::vector<double> csr_v;
 };
 bool band_rule(const Csr& A, int band_mode);
+// group: slices sharing one width (1 warp-grained, 8 block-sliced, 0 = global ELL width)
 void pack_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, int32_t window,
-               bool band_on, bool uniform, int32_t global_kmax, Packed& P);
+               bool band_on, int32_t group, int32_t global_kmax, Packed& P);
 void pack_csr_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, Packed& P);
 
 struct Device;  // device state (device.cu)

@@ -35,13 +35,13 @@ bool band_rule(const Csr& A, int band_mode) {
 }
 
 void pack_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, int32_t window,
-               bool band_on, bool uniform, int32_t global_kmax, Packed& P) {
+               bool band_on, int32_t group, int32_t global_kmax, Packed& P) {
     const int64_t n = r1 - r0;  // local rows
     P = Packed();
     P.n = n;
     P.band_on = band_on;
     P.window = window > 1 ? window : 1;
-    P.uniform = uniform;
+    P.group = group;
     P.n_slots = (n + 31) / 32 * 32;
     P.n_slices = P.n_slots / 32;
     std::vector<int32_t> c(n);
@@ -64,18 +64,22 @@ void pack_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, int32_t 
             std::stable_sort(b, e, [&](int32_t a, int32_t bb) { return c[a] > c[bb]; });
         }
     }
+    // slice width = exact max ELL count of its rows; `group` slices
+    // share their max (8 = the 256-row block-sliced ELL of [5]); 0 = global width
     P.slice_w.assign(P.n_slices, 0);
     P.slice_off.assign(P.n_slices + 1, 0);
     for (int64_t q = 0; q < P.n_slices; ++q) {
         int32_t w = 0;
-        if (uniform) {
-            w = global_kmax;
-        } else {
-            for (int64_t s = q * 32; s < std::min(q * 32 + 32, n); ++s) w = std::max(w, c[P.row_of[s]]);
-        }
-        P.slice_w[q] = w;
-        P.slice_off[q + 1] = P.slice_off[q] + 32 * (int64_t)w;
+        for (int64_t s = q * 32; s < std::min(q * 32 + 32, n); ++s) w = std::max(w, c[P.row_of[s]]);
+        P.slice_w[q] = group == 0 ? global_kmax : w;
     }
+    if (group > 1)
+        for (int64_t g0 = 0; g0 < P.n_slices; g0 += group) {
+            const int64_t g1 = std::min<int64_t>(g0 + group, P.n_slices);
+            const int32_t wg = *std::max_element(P.slice_w.begin() + g0, P.slice_w.begin() + g1);
+            std::fill(P.slice_w.begin() + g0, P.slice_w.begin() + g1, wg);
+        }
+    for (int64_t q = 0; q < P.n_slices; ++q) P.slice_off[q + 1] = P.slice_off[q] + 32 * (int64_t)P.slice_w[q];
     P.n_ell = P.slice_off[P.n_slices];
     P.val.assign(P.n_ell, 0.0);
     P.col.assign(P.n_ell, 0);

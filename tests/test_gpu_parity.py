@@ -278,3 +278,29 @@ def test_every_step_kernel(cme, oracle_mod, monkeypatch, knobs, net, order, omeg
     p, st, it = m.solve(tol=1e-11, max_iter=100000)
     ref = oracle_mod.jacobi_solve(A, omega=omega, tol=1e-11, check_every=7, max_iter=100000, stag_tol=0.0)
     assert st == ref.status and abs(it - ref.iters) <= 7
+
+
+@pytest.mark.slow
+def test_cfg4_full_size_parity(cme, oracle_mod):
+    """The bench workload itself (configs[3]: toggle N=3164, n = 20,015,468, RCM,
+    the kernel bench.py times): one SpMV on every row, the |d|-weighted mass
+    invariant, and 300 iterations of the landscape against the
+    oracle's own enumeration + CSR Jacobi (16 host threads)."""
+    import os
+    net = W.config_network("cfg4_toggle_20m")
+    m = cme.Matrix.from_network(net).reorder(cme.CME_ORDER_RCM).pack()
+    info = m.info()
+    assert info.n == 20015468 and info.nnz == 120042194 and info.kernel == 1
+    A = oracle_mod.network_csr(net)
+    x = W.random_start(A.n, 17)
+    m.set_opts(omega=1.0)
+    y = m.spmv(x)
+    assert_spmv_close(y, oracle_mod.jacobi_step(A, x, 1.0))
+    d = -A.diag
+    assert abs((d * y).sum() - (d * x).sum()) <= 1e-12 * (d * x).sum()
+    m.set_opts(omega=0.9, stag_tol=0.0)
+    p, st, it = m.solve(tol=0.0, max_iter=300)
+    ref = oracle_mod.jacobi_solve(A, omega=0.9, tol=0.0, max_iter=300, stag_tol=0.0,
+                                  nthreads=len(os.sched_getaffinity(0)))
+    assert it == ref.iters == 300
+    assert np.abs(p - ref.p).sum() <= 1e-10

@@ -105,6 +105,8 @@ def test_orderings_bit_exact(oracle_mod, net, order):
 
 
 PACK_CASES = [("none", 256, "auto", cme.CME_FMT_DIAG_SELL), ("dfs", 256, "auto", cme.CME_FMT_DIAG_SELL),
+              ("none", 1, "auto", cme.CME_FMT_SELL256), ("rcm", 1, "never", cme.CME_FMT_SELL256),
+              ("rcm", 1 << 30, "never", cme.CME_FMT_DIAG_SELL),
               ("rcm", 256, "auto", cme.CME_FMT_DIAG_SELL), ("none", 1, "never", cme.CME_FMT_DIAG_SELL),
               ("rcm", 64, "always", cme.CME_FMT_DIAG_SELL), ("none", 1, "auto", cme.CME_FMT_ELL),
               ("dfs", 1, "never", cme.CME_FMT_ELL)]
@@ -121,12 +123,28 @@ def test_pack_bit_exact(oracle_mod, net, order, window, band, fmt):
     perm = {"none": np.arange(A.n, dtype=np.int32), "dfs": oracle_mod.order_dfs(A, 0),
             "rcm": oracle_mod.order_rcm(A)}[order]
     ref = oracle_mod.pack(oracle_mod.permute(A, perm), window=window if fmt == cme.CME_FMT_DIAG_SELL else 1,
-                          band=band, uniform=fmt == cme.CME_FMT_ELL)
+                          band=band, uniform=fmt == cme.CME_FMT_ELL,
+                          group=8 if fmt == cme.CME_FMT_SELL256 else 1)
     got = m.packed()
     for key in ("n", "n_slots", "n_slices", "n_ell", "band_on", "window"):
         assert got[key] == ref[key], key
     for key in ("lo", "up", "inv_d", "row_of", "slice_off", "slice_w", "val", "col"):
         assert got[key].dtype == ref[key].dtype and got[key].tobytes() == ref[key].tobytes(), key
+
+
+def test_given_permutation_bit_exact(oracle_mod):
+    """A seeded random ordering (the locality stress test of P:L225) passed to both sides."""
+    states, r, c, v = oracle_mod.enumerate_network(W.toggle_switch(40))
+    A = oracle_mod.ingest(len(states), r, c, v)
+    perm = np.random.default_rng(5).permutation(A.n).astype(np.int32)
+    m = cme.Matrix(A.n, r, c, v).set_permutation(perm)
+    m.pack(cme.CME_FMT_DIAG_SELL, 256, cme.CME_BAND_AUTO, cme.CME_DEVICE_HOST_ONLY)
+    ref = oracle_mod.pack(oracle_mod.permute(A, perm))
+    got = m.packed()
+    for key in ("row_of", "slice_off", "slice_w", "val", "col", "inv_d", "lo", "up"):
+        assert got[key].tobytes() == ref[key].tobytes(), key
+    with pytest.raises(cme.CmeError):
+        cme.Matrix(A.n, r, c, v).set_permutation(np.zeros(A.n, np.int32))
 
 
 @pytest.mark.slow

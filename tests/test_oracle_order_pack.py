@@ -167,6 +167,12 @@ def test_pack_rearrangement_and_efficiency(oracle_mod):
     assert e >= e1   # local rearrangement never lowers the SELL efficiency here
     Pe = oracle_mod.pack(A, window=1, band="never", uniform=True)
     assert Pe["n_ell"] == Pe["n_slots"] * c.max()   # plain ELL: n' x k
+    Pb = oracle_mod.pack(A, window=1, band="never", group=8)   # 256-row block slices [5]
+    for g0 in range(0, Pb["n_slices"], 8):
+        blk = list(range(32 * g0, min(32 * g0 + 256, A.n)))
+        assert set(Pb["slice_w"][g0:g0 + 8]) == {max(c[blk])}
+    Pw = oracle_mod.pack(A, window=1, band="never")
+    assert Pw["n_ell"] <= Pb["n_ell"] <= Pe["n_ell"]   # warp-grained <= block-sliced <= ELL
 
 
 def test_band_rule_threshold(oracle_mod):
