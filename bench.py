@@ -133,11 +133,17 @@ def kernel_name(info):
         info.kernel, "?")
 
 
-def build_matrix(cme, name, dev_mode):
+def build_matrix(cme, name, dev_mode, batch=1):
     cfg = DEFAULTS[name]
-    net = W.config_network(name)
     t0 = time.perf_counter()
-    states, r, c, v = cme.cme_network_enumerate(net)
+    if batch > 1:   # batched sweep: B rate sets on one pattern
+        vs = []
+        for net in W.sweep_networks(name, batch):
+            states, r, c, v = cme.cme_network_enumerate(net)
+            vs.append(v)
+        v = np.stack(vs)
+    else:
+        states, r, c, v = cme.cme_network_enumerate(W.config_network(name))
     t1 = time.perf_counter()
     n = len(states)
     m = cme.Matrix(n, r, c, v)
@@ -227,6 +233,8 @@ def main():
     ap.add_argument("--impl", default="cme", choices=["cme", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-converge", action="store_true")
+    ap.add_argument("--batch", type=int, default=1, choices=[1, 2, 4, 8],
+                    help="solve a sweep of B rate sets on the workload's pattern (SURVEY NEXT-1)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -251,14 +259,15 @@ def main():
         comm = cme.cme_comm_init(world, rank, obj[0], local)
 
     name = args.config
-    m, cfg, setup = build_matrix(cme, name, cme.CME_DEVICE_HOST_ONLY if world > 1 else local)
+    B = args.batch
+    m, cfg, setup = build_matrix(cme, name, cme.CME_DEVICE_HOST_ONLY if world > 1 else local, B)
     if comm is not None:
         cme.cme_matrix_distribute(m.h, comm)
     info = m.info()
     n, nnz = info.n, info.nnz
     stream = torch.cuda.Stream()
     m.set_opts(omega=cfg["omega"], check_every=C_BLOCK, stream=stream.cuda_stream)
-    cme.cme_solver_load(m.h, n, None)
+    cme.cme_solver_load(m.h, n * B, None)
     for _ in range(args.warmup):
         cme.cme_solver_run(m.h, 1)
     torch.cuda.synchronize()
@@ -283,39 +292,39 @@ def main():
         ms = float(t.item())
     iters = args.steps * C_BLOCK
     sec = ms * 1e-3
-    gflops = 2.0 * nnz * iters / sec / 1e9
+    gflops = 2.0 * nnz * B * iters / sec / 1e9
     peak, peak_src = hbm_peak()
     t_iter = sec / iters
     achieved = info.bytes_alg / t_iter / 1e9        # algorithmic bytes per launch / launch time
     fmt_gbs = info.bytes_fmt * world / t_iter / 1e9 if world == 1 else None
 
     # e2e: the public solve call with pinned host buffers, H2D + D2H inside the timed region
-    p0 = torch.empty(n, dtype=torch.float64, pin_memory=True)
-    p0.copy_(torch.from_numpy(W.uniform_start(n)))
-    pout = torch.empty(n, dtype=torch.float64, pin_memory=True)
+    p0 = torch.empty(n * B, dtype=torch.float64, pin_memory=True)
+    p0.copy_(torch.from_numpy(np.tile(W.uniform_start(n), B)))
+    pout = torch.empty(n * B, dtype=torch.float64, pin_memory=True)
     e2e_steps = max(3, min(args.steps, 10))
-    cme.cme_jacobi_solve(m.h, n, p0, 0.0, C_BLOCK, pout)  # warm
+    cme.cme_jacobi_solve(m.h, n * B, p0, 0.0, C_BLOCK, pout)  # warm
     barrier()
     t = time.perf_counter()
     for _ in range(e2e_steps):
-        cme.cme_jacobi_solve(m.h, n, p0, 0.0, C_BLOCK, pout)
+        cme.cme_jacobi_solve(m.h, n * B, p0, 0.0, C_BLOCK, pout)
     barrier()
     e2e_s = time.perf_counter() - t
     if world > 1:
         tt = torch.tensor([e2e_s], device="cuda", dtype=torch.float64)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         e2e_s = float(tt.item())
-    e2e_gflops = 2.0 * nnz * C_BLOCK * e2e_steps / e2e_s / 1e9
+    e2e_gflops = 2.0 * nnz * B * C_BLOCK * e2e_steps / e2e_s / 1e9
     clocks = clk.summary()
 
     conv = None
-    if rank == 0 and world == 1 and not args.no_converge:
+    if rank == 0 and world == 1 and B == 1 and not args.no_converge:
         try:
             conv = converge_line(cme)
         except Exception as ex:  # report, do not hide
             conv = {"error": repr(ex)}
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and B == 1 and not args.no_cpu_baseline:
         cb = cpu_oracle_timing(name, budget_s=20.0, omega=cfg["omega"])
         cpu = {k: cb[k] for k in ("value", "unit", "cores", "kind", "sample")}
 
@@ -325,7 +334,8 @@ def main():
             "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": round(ms / args.steps, 4), "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": name, "n": n, "nnz": nnz, "order": cfg["order"], "format": "diag_sell",
+            "config": {"workload": name if B == 1 else f"{name} x {B}-member sweep", "batch": B,
+                       "n": n, "nnz": nnz, "order": cfg["order"], "format": "diag_sell",
                        "window": cfg["window"], "band_on": bool(info.band_on), "omega": cfg["omega"],
                        "check_every": C_BLOCK, "iters_per_step": C_BLOCK,
                        "l2": f"inputs larger than L2 ({info.bytes_alg / 1e9:.3f} GB/iteration vs 126 MB)",
@@ -336,15 +346,15 @@ def main():
                          "frac": round(achieved / (peak * world), 4),
                          "traffic": ncu_traffic(name) if world == 1 else None,
                          "peak_source": peak_src, "kernel": kernel_name(info),
-                         "bytes_per_launch": info.bytes_alg, "bytes_model": "12 nnz + 16 n (SURVEY 8(d))",
+                         "bytes_per_launch": info.bytes_alg, "bytes_model": "12 nnz + 16 n per member (SURVEY 8(d))" if B == 1 else f"(12 nnz + 16 n) x {B} members: each member counted as if solved alone",
                          "format_bytes_per_launch": info.bytes_fmt,
                          "format_gbs": round(fmt_gbs, 1) if fmt_gbs else None,
                          "launch_time_us": round(t_iter * 1e6, 3),
                          "launch_time_note": "timed-region time / step-kernel launches (includes the 2 tiny "
                                              "check kernels per 100 steps and launch gaps: conservative)"},
             "clocks": clocks,
-            "e2e": {"value": round(e2e_gflops, 3), "unit": "GFLOPS", "h2d_bytes_per_step": 8 * n,
-                    "d2h_bytes_per_step": 8 * n, "steps": e2e_steps,
+            "e2e": {"value": round(e2e_gflops, 3), "unit": "GFLOPS", "h2d_bytes_per_step": 8 * n * B,
+                    "d2h_bytes_per_step": 8 * n * B, "steps": e2e_steps,
                     "call": "cme_jacobi_solve(h, p0_pinned_host, tol=0, max_iter=100, p_out_pinned_host)"},
             "gpu_launches": args.steps * (C_BLOCK + 2) * 1,
             "converge": conv,

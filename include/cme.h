@@ -68,6 +68,20 @@ typedef struct cme_comm_s* cme_comm;     /* opaque; wraps an NCCL communicator *
 cme_status cme_matrix_create_coo(int64_t n, int64_t nnz, const int32_t* row, const int32_t* col,
                                  const double* rate, uint32_t flags, cme_matrix* out);
 
+/* Batched parameter sweep ("the study of the same reaction network
+ * under different conditions"): `batch` rate sets on ONE COO
+ * pattern, rates[b*nnz + e] for member b.  batch in {1, 2, 4, 8}.  An entry is
+ * stored if any member's summed rate is non-zero; every member must have
+ * outflow from every state.  Column indices are stored once; values, the
+ * diagonal and the iterate are member-minor on the device, so one gather
+ * fetches all members.  For a batch handle every vector argument below
+ * (p0, p_out, x, y) holds batch*n doubles, member-major (member b at
+ * [b*n, (b+1)*n)), and the solve stops when every member is converged or
+ * stagnated (per-member results: cme_get_batch_report).  The CSR ablation
+ * format takes batch 1 only. */
+cme_status cme_matrix_create_coo_batch(int64_t n, int64_t nnz, const int32_t* row, const int32_t* col,
+                                       const double* rates, int32_t batch, uint32_t flags, cme_matrix* out);
+
 /* CSR by rows (row_ptr[n+1], col[row_ptr[n]], rate) -- same semantics as COO. */
 cme_status cme_matrix_create_csr(int64_t n, const int64_t* row_ptr, const int32_t* col,
                                  const double* rate, uint32_t flags, cme_matrix* out);
@@ -135,6 +149,10 @@ typedef struct cme_report {
     double seconds;    /* device time of the iteration loop (CUDA events)              */
 } cme_report;
 cme_status cme_get_report(cme_matrix h, cme_report* r);
+/* Per-member reports of the last solve of a batch handle (count <= batch):
+ * status = CME_OK / CME_STAGNATED / CME_NOT_CONVERGED / CME_ERR_NUMERIC of
+ * that member, iters = the iteration at which its status was decided. */
+cme_status cme_get_batch_report(cme_matrix h, cme_report* reports, int32_t count);
 
 /* One application y = M_omega x = (1-omega) x - omega D^-1 (L+U) x, no
  * normalisation (test hook for per-SpMV parity).  x, y: n doubles. */
@@ -171,6 +189,7 @@ typedef struct cme_info {
                                      3 persistent cooperative SELL (small problems), -1 none */
     int32_t tma_warps, tma_stages;/* TMA kernel: consumer warps per CTA, smem stages */
     int32_t grid;                 /* CTAs per step launch                            */
+    int32_t batch;                /* rate sets sharing the pattern (1 = single matrix) */
 } cme_info;
 cme_status cme_get_info(cme_matrix h, cme_info* info);
 
@@ -182,7 +201,7 @@ cme_status cme_get_permutation(cme_matrix h, int32_t* new_to_old);
  * distributed matrix: the local part, columns in local x-span coordinates. */
 typedef struct cme_packed_view {
     int64_t n, n_slots, n_slices, n_ell;
-    int32_t band_on, window;
+    int32_t band_on, window, batch, pad_;   /* val/lo/up/inv_d hold batch values per entry/slot */
     const double* lo;        /* [n_slots] slot order                         */
     const double* up;        /* [n_slots]                                    */
     const double* inv_d;     /* [n_slots] 1/(-A_ii)                          */

@@ -68,13 +68,13 @@ class cme_info(C.Structure):
                 ("bytes_fmt", C.c_int64), ("rank", C.c_int32), ("nranks", C.c_int32),
                 ("row_begin", C.c_int64), ("row_end", C.c_int64), ("halo_begin", C.c_int64),
                 ("halo_end", C.c_int64), ("kernel", C.c_int32), ("tma_warps", C.c_int32),
-                ("tma_stages", C.c_int32), ("grid", C.c_int32)]
+                ("tma_stages", C.c_int32), ("grid", C.c_int32), ("batch", C.c_int32)]
 
 
 class cme_packed_view(C.Structure):
     _fields_ = [("n", C.c_int64), ("n_slots", C.c_int64), ("n_slices", C.c_int64),
                 ("n_ell", C.c_int64), ("band_on", C.c_int32), ("window", C.c_int32),
-                ("lo", f64p), ("up", f64p), ("inv_d", f64p), ("row_of", i32p),
+                ("batch", C.c_int32), ("pad_", C.c_int32), ("lo", f64p), ("up", f64p), ("inv_d", f64p), ("row_of", i32p),
                 ("slice_off", i64p), ("slice_w", i32p), ("val", f64p), ("col", i32p),
                 ("csr_row_ptr", i64p)]
 
@@ -89,6 +89,8 @@ class cme_halo_view(C.Structure):
 _SIGS = {
     "cme_matrix_create_coo": [C.c_int64, C.c_int64, i32p, i32p, f64p, C.c_uint32, _p(vp)],
     "cme_matrix_create_csr": [C.c_int64, i64p, i32p, f64p, C.c_uint32, _p(vp)],
+    "cme_matrix_create_coo_batch": [C.c_int64, C.c_int64, i32p, i32p, f64p, C.c_int32, C.c_uint32, _p(vp)],
+    "cme_get_batch_report": [vp, _p(cme_report), C.c_int32],
     "cme_reorder": [vp, C.c_int, C.c_int64],
     "cme_set_permutation": [vp, i32p],
     "cme_pack": [vp, C.c_int, _p(cme_pack_opts)],
@@ -175,6 +177,25 @@ def cme_matrix_create_coo(n, row, col, rate, flags=CME_DIAG_FROM_COLSUMS):
     return h
 
 
+def cme_matrix_create_coo_batch(n, row, col, rates, flags=CME_DIAG_FROM_COLSUMS):
+    """rates: array (batch, nnz) -- one rate set per member on the (row, col) pattern."""
+    row, col = _arr(row, np.int32), _arr(col, np.int32)
+    rates = np.ascontiguousarray(rates, dtype=np.float64)
+    if rates.ndim != 2 or rates.shape[1] != len(row):
+        raise ValueError("rates must be (batch, nnz)")
+    h = vp()
+    _chk(_lib.cme_matrix_create_coo_batch(n, len(row), row.ctypes.data_as(i32p), col.ctypes.data_as(i32p),
+                                          rates.ctypes.data_as(f64p), rates.shape[0], flags, C.byref(h)),
+         "cme_matrix_create_coo_batch")
+    return h
+
+
+def cme_get_batch_report(h, count):
+    arr = (cme_report * count)()
+    _chk(_lib.cme_get_batch_report(h, arr, count), "cme_get_batch_report")
+    return list(arr)
+
+
 def cme_matrix_create_csr(n, row_ptr, col, rate, flags=CME_DIAG_FROM_COLSUMS):
     row_ptr, col, rate = _arr(row_ptr, np.int64), _arr(col, np.int32), _arr(rate, np.float64)
     h = vp()
@@ -256,11 +277,13 @@ def cme_export_packed(h):
     def cp(ptr, k, dt):
         return np.ctypeslib.as_array(ptr, shape=(k,)).astype(dt, copy=True) if k and ptr else np.zeros(0, dt)
 
+    nb = max(1, v.batch)
     out = dict(n=v.n, n_slots=v.n_slots, n_slices=v.n_slices, n_ell=v.n_ell, band_on=bool(v.band_on),
-               window=v.window, lo=cp(v.lo, v.n_slots, np.float64), up=cp(v.up, v.n_slots, np.float64),
-               inv_d=cp(v.inv_d, v.n_slots, np.float64), row_of=cp(v.row_of, v.n_slots, np.int32),
+               window=v.window, batch=nb, lo=cp(v.lo, v.n_slots * nb, np.float64),
+               up=cp(v.up, v.n_slots * nb, np.float64),
+               inv_d=cp(v.inv_d, v.n_slots * nb, np.float64), row_of=cp(v.row_of, v.n_slots, np.int32),
                slice_off=cp(v.slice_off, v.n_slices + 1, np.int64),
-               slice_w=cp(v.slice_w, v.n_slices, np.int32), val=cp(v.val, v.n_ell, np.float64),
+               slice_w=cp(v.slice_w, v.n_slices, np.int32), val=cp(v.val, v.n_ell * nb, np.float64),
                col=cp(v.col, v.n_ell, np.int32))
     if v.csr_row_ptr:
         out["csr_row_ptr"] = cp(v.csr_row_ptr, v.n + 1, np.int64)
@@ -353,11 +376,20 @@ def cme_network_enumerate(net):
 
 # ---- convenience object ------------------------------------------------------------------
 class Matrix:
-    """Owning wrapper: create -> reorder -> pack -> solve (all work in libcme)."""
+    """Owning wrapper: create -> reorder -> pack -> solve (all work in libcme).
+
+    `rate` of shape (nnz,) is one matrix; shape (batch, nnz) is a batched sweep
+    (vectors then hold batch * n values, member-major)."""
 
     def __init__(self, n, row, col, rate, flags=CME_DIAG_FROM_COLSUMS):
         self.n = int(n)
-        self.h = cme_matrix_create_coo(self.n, row, col, rate, flags)
+        rate = np.asarray(rate, dtype=np.float64)
+        if rate.ndim == 2:
+            self.batch = rate.shape[0]
+            self.h = cme_matrix_create_coo_batch(self.n, row, col, rate, flags)
+        else:
+            self.batch = 1
+            self.h = cme_matrix_create_coo(self.n, row, col, rate, flags)
 
     @classmethod
     def from_network(cls, net):
@@ -384,15 +416,18 @@ class Matrix:
 
     def solve(self, p0=None, tol=1e-12, max_iter=1_000_000, p_out=None):
         if p_out is None:
-            p_out = np.empty(self.n)
-        st, it = cme_jacobi_solve(self.h, self.n, p0, tol, max_iter, p_out)
+            p_out = np.empty(self.n * self.batch)
+        st, it = cme_jacobi_solve(self.h, self.n * self.batch, p0, tol, max_iter, p_out)
         return p_out, SOLVE_STATUS[st], it
 
     def spmv(self, x, y=None):
         if y is None:
-            y = np.empty(self.n)
-        cme_spmv(self.h, self.n, x, y)
+            y = np.empty(self.n * self.batch)
+        cme_spmv(self.h, self.n * self.batch, x, y)
         return y
+
+    def batch_report(self):
+        return cme_get_batch_report(self.h, self.batch)
 
     def info(self):
         return cme_get_info(self.h)

@@ -129,13 +129,33 @@ using namespace cme;
 
 extern "C" {
 
+cme_status cme_matrix_create_coo_batch(int64_t n, int64_t nnz, const int32_t* row, const int32_t* col,
+                                       const double* rates, int32_t batch, uint32_t flags, cme_matrix* out) {
+    if (!out) return CME_ERR_INVALID_ARG;
+    *out = nullptr;
+    if (batch != 1 && batch != 2 && batch != 4 && batch != 8) {
+        set_error("batch must be 1, 2, 4 or 8");
+        return CME_ERR_INVALID_ARG;
+    }
+    return guarded([&] {
+        auto* h = new cme_matrix_s();
+        cme_status s = ingest_coo(n, nnz, row, col, rates, batch, flags, h->A);
+        if (s != CME_OK) { delete h; return s; }
+        h->perm.resize(n);
+        for (int64_t i = 0; i < n; ++i) h->perm[i] = (int32_t)i;
+        h->stage = 1;
+        *out = h;
+        return CME_OK;
+    });
+}
+
 cme_status cme_matrix_create_coo(int64_t n, int64_t nnz, const int32_t* row, const int32_t* col,
                                  const double* rate, uint32_t flags, cme_matrix* out) {
     if (!out) return CME_ERR_INVALID_ARG;
     *out = nullptr;
     return guarded([&] {
         auto* h = new cme_matrix_s();
-        cme_status s = ingest_coo(n, nnz, row, col, rate, flags, h->A);
+        cme_status s = ingest_coo(n, nnz, row, col, rate, 1, flags, h->A);
         if (s != CME_OK) { delete h; return s; }
         h->perm.resize(n);
         for (int64_t i = 0; i < n; ++i) h->perm[i] = (int32_t)i;
@@ -213,13 +233,18 @@ cme_status cme_pack(cme_matrix h, int format, const cme_pack_opts* opts) {
         if (identity) h->B = h->A;
         else permute(h->A, h->perm, h->B);
         h->period = directed_period(h->A, 0);
-        double na = 0.0;
-        for (int64_t i = 0; i < h->A.n; ++i) {
-            double s = std::fabs(h->A.d[i]);
-            for (int64_t p = h->A.rp[i]; p < h->A.rp[i + 1]; ++p) s += std::fabs(h->A.v[p]);
-            na = std::max(na, s);
+        const int32_t nb = h->A.B;
+        if (nb > 1 && format == CME_FMT_CSR) {
+            set_error("the CSR ablation arm takes one rate set (batch 1)");
+            return CME_ERR_INVALID_ARG;
         }
-        h->norm_inf = na;
+        h->norm_inf.assign(nb, 0.0);   // ||A_b||_inf: max row sum of |a_ij| incl. diagonal
+        for (int64_t i = 0; i < h->A.n; ++i)
+            for (int32_t b = 0; b < nb; ++b) {
+                double s = std::fabs(h->A.d[(size_t)i * nb + b]);
+                for (int64_t p = h->A.rp[i]; p < h->A.rp[i + 1]; ++p) s += std::fabs(h->A.v[(size_t)p * nb + b]);
+                h->norm_inf[b] = std::max(h->norm_inf[b], s);
+            }
         h->band_on = format != CME_FMT_CSR && band_rule(h->B, o.band);
         int32_t kmax = 0;
         for (int64_t i = 0; i < h->B.n; ++i) kmax = std::max(kmax, ell_count(h->B, i, h->band_on));
@@ -259,6 +284,16 @@ cme_status cme_jacobi_solve(cme_matrix h, const double* p0, double tol, int64_t 
 cme_status cme_get_report(cme_matrix h, cme_report* r) {
     if (!h || !r) return CME_ERR_INVALID_ARG;
     *r = h->report;
+    return CME_OK;
+}
+
+cme_status cme_get_batch_report(cme_matrix h, cme_report* reports, int32_t count) {
+    if (!h || !reports || count < 0) return CME_ERR_INVALID_ARG;
+    if (count > (int32_t)h->member_reports.size()) {
+        set_error("no solve report for that many members yet");
+        return CME_ERR_INVALID_ARG;
+    }
+    for (int32_t b = 0; b < count; ++b) reports[b] = h->member_reports[b];
     return CME_OK;
 }
 
@@ -309,7 +344,8 @@ cme_status cme_get_info(cme_matrix h, cme_info* info) {
         f.band_on = h->band_on;
         f.window = h->P.window;
         f.period = h->stage >= 2 ? h->period : directed_period(h->A, 0);
-        f.norm_inf = h->norm_inf;
+        f.norm_inf = h->norm_inf.empty() ? 0.0 : h->norm_inf[0];
+        f.batch = h->A.B;
         f.omega = h->sopts.omega > 0 ? h->sopts.omega : (f.period == 1 ? 1.0 : 0.9);
         const Packed& P = h->P;
         f.n_slots = P.n_slots;
@@ -319,16 +355,17 @@ cme_status cme_get_info(cme_matrix h, cme_info* info) {
         for (double v : P.val) ell_nz += v != 0.0;
         f.ell_efficiency = P.n_ell ? (double)ell_nz / (double)P.n_ell : 1.0;
         const int64_t nl = P.n;
+        const int64_t nb = h->A.B;
         if (h->format == CME_FMT_CSR) {
             f.packed_bytes = 8 * (int64_t)P.csr_rp.size() + 12 * (int64_t)P.csr_ci.size() + 8 * (int64_t)P.inv_d.size();
             f.bytes_fmt = 12 * (int64_t)P.csr_ci.size() + 8 * (nl + 1) + 8 * nl + 16 * nl;
         } else {
-            f.packed_bytes = 12 * P.n_ell + 8 * P.n_slots + (P.band_on ? 16 * P.n_slots : 0) +
+            f.packed_bytes = (8 * nb + 4) * P.n_ell + 8 * nb * P.n_slots + (P.band_on ? 16 * nb * P.n_slots : 0) +
                              (P.window > 1 ? 4 * P.n_slots : 0) + 12 * P.n_slices + 8;
-            f.bytes_fmt = 12 * P.n_ell + 8 * nl + (P.band_on ? 16 * nl : 0) + (P.window > 1 ? 4 * nl : 0) +
-                          12 * P.n_slices + 16 * nl;
+            f.bytes_fmt = (8 * nb + 4) * P.n_ell + 8 * nb * nl + (P.band_on ? 16 * nb * nl : 0) +
+                          (P.window > 1 ? 4 * nl : 0) + 12 * P.n_slices + 16 * nb * nl;
         }
-        f.bytes_alg = 12 * f.nnz + 16 * n;
+        f.bytes_alg = (12 * f.nnz + 16 * n) * nb;   // per member, as if solved one by one
         f.rank = h->rank;
         f.nranks = h->nranks;
         f.row_begin = h->cuts.empty() ? 0 : h->cuts[h->rank];
@@ -353,7 +390,7 @@ cme_status cme_export_packed(cme_matrix h, cme_packed_view* v) {
     const Packed& P = h->P;
     cme_packed_view o{};
     o.n = P.n; o.n_slots = P.n_slots; o.n_slices = P.n_slices; o.n_ell = P.n_ell;
-    o.band_on = P.band_on; o.window = P.window;
+    o.band_on = P.band_on; o.window = P.window; o.batch = P.B;
     o.lo = P.lo.data(); o.up = P.up.data(); o.inv_d = P.inv_d.data(); o.row_of = P.row_of.data();
     o.slice_off = P.slice_off.data(); o.slice_w = P.slice_w.data(); o.val = P.val.data(); o.col = P.col.data();
     o.csr_row_ptr = h->format == CME_FMT_CSR ? P.csr_rp.data() : nullptr;

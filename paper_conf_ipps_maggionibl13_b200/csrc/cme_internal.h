@@ -14,18 +14,21 @@ namespace cme {
 void set_error(const std::string& msg);
 
 // Off-diagonal part of A by rows (row i <- col j: transition j -> i) + diagonal.
+// A batch of B rate sets shares the pattern: values are member-minor
+// (v[p*B + b], d[i*B + b]); B = 1 is the ordinary single matrix.
 struct Csr {
     int64_t n = 0;
+    int32_t B = 1;
     std::vector<int64_t> rp;   // n + 1
     std::vector<int32_t> ci;   // column indices, ascending within a row
-    std::vector<double> v;     // rates
-    std::vector<double> d;     // a_ii (< 0)
+    std::vector<double> v;     // rates, nnz * B
+    std::vector<double> d;     // a_ii (< 0), n * B
     int64_t nnz() const { return rp.empty() ? 0 : rp.back(); }
 };
 
-// Ingest.  Returns CME_OK or an error status.
+// Ingest of B rate sets rate[b*nnz + e] on one COO pattern.
 cme_status ingest_coo(int64_t n, int64_t nnz, const int32_t* row, const int32_t* col,
-                      const double* rate, uint32_t flags, Csr& out);
+                      const double* rate, int32_t B, uint32_t flags, Csr& out);
 
 // Orderings and graph tests (R1, R11, R12).
 void order_dfs(const Csr& A, int64_t root, std::vector<int32_t>& new_to_old);
@@ -37,13 +40,13 @@ void permute(const Csr& A, const std::vector<int32_t>& new_to_old, Csr& out);
 // [r0, r1) of an ordered matrix, columns shifted by -col_shift.
 struct Packed {
     int64_t n = 0, n_slots = 0, n_slices = 0, n_ell = 0;
-    int32_t band_on = 0, window = 1, group = 1;
-    std::vector<double> lo, up, inv_d;    // slot order
+    int32_t band_on = 0, window = 1, group = 1, B = 1;
+    std::vector<double> lo, up, inv_d;    // slot order, n_slots * B (member-minor)
     std::vector<int32_t> row_of;          // slot -> local row
     std::vector<int64_t> slice_off;       // n_slices + 1
     std::vector<int32_t> slice_w;         // n_slices
-    std::vector<double> val;              // n_ell
-    std::vector<int32_t> col;             // n_ell
+    std::vector<double> val;              // n_ell * B (member-minor)
+    std::vector<int32_t> col;             // n_ell (shared by the batch)
     // CSR arm
     std::vector<int64_t> csr_rp;
     std::vector<int32_t> csr_ci;
@@ -71,11 +74,12 @@ struct cme_matrix_s {
     cme_pack_opts popts{32, 256, CME_BAND_AUTO, -1};
     bool band_on = false;
     int64_t period = 0;
-    double norm_inf = 0.0;
+    std::vector<double> norm_inf;  // ||A_b||_inf per batch member
     cme::Packed P;              // local packed layout (whole matrix unless distributed)
     int32_t global_kmax = 0;
     cme_solver_opts sopts{0.0, 100, CME_STOP_DELTA_L1, 1e-10, nullptr};
     cme_report report{};
+    std::vector<cme_report> member_reports;  // per batch member
     // partition
     int nranks = 1, rank = 0;
     std::vector<int64_t> cuts;  // nranks + 1

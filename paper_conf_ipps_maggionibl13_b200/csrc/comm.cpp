@@ -100,8 +100,8 @@ cme_status comm_halo(cme_comm_s* c, const HaloPlan& p, double* xspan, cudaStream
     return CME_OK;
 }
 
-cme_status comm_allgather8(cme_comm_s* c, const double* send8, double* recv, cudaStream_t s) {
-    NCCL_TRY(g_api.AllGather(send8, recv, 8, ncclFloat64, c->comm, s));
+cme_status comm_allgather(cme_comm_s* c, const double* send, double* recv, size_t count, cudaStream_t s) {
+    NCCL_TRY(g_api.AllGather(send, recv, count, ncclFloat64, c->comm, s));
     return CME_OK;
 }
 

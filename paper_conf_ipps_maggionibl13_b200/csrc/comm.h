@@ -26,9 +26,9 @@ int comm_rank(const cme_comm_s* c);
 int comm_nranks(const cme_comm_s* c);
 int comm_device(const cme_comm_s* c);
 cme_status comm_halo(cme_comm_s* c, const HaloPlan& p, double* xspan, cudaStream_t s);
-// recv[r*8 .. r*8+7] = send8 of rank r
-cme_status comm_allgather8(cme_comm_s* c, const double* send8, double* recv, cudaStream_t s);
-// every rank r broadcasts buf[cuts[r], cuts[r+1]) to all ranks
+// recv[r*count .. (r+1)*count) = send of rank r
+cme_status comm_allgather(cme_comm_s* c, const double* send, double* recv, size_t count, cudaStream_t s);
+// every rank r broadcasts buf[cuts[r], cuts[r+1]) (in doubles) to all ranks
 cme_status comm_bcast_segments(cme_comm_s* c, double* buf, const std::vector<int64_t>& cuts,
                                cudaStream_t s);
 

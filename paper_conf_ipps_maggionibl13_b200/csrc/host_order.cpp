@@ -187,27 +187,33 @@ int64_t directed_period(const Csr& A, int64_t root) {
 
 void permute(const Csr& A, const std::vector<int32_t>& p, Csr& B) {
     const int64_t n = A.n;
+    const int32_t nb = A.B;
     std::vector<int32_t> inv(n);
     for (int64_t r = 0; r < n; ++r) inv[p[r]] = (int32_t)r;
     B.n = n;
+    B.B = nb;
     B.rp.assign(n + 1, 0);
     for (int64_t r = 0; r < n; ++r) B.rp[r + 1] = B.rp[r] + (A.rp[p[r] + 1] - A.rp[p[r]]);
     B.ci.resize(A.nnz());
-    B.v.resize(A.nnz());
-    B.d.resize(n);
+    B.v.resize((size_t)A.nnz() * nb);
+    B.d.resize((size_t)n * nb);
 #pragma omp parallel
     {
-        std::vector<std::pair<int32_t, double>> row;
+        std::vector<std::pair<int32_t, int64_t>> row;  // (new column, old position)
 #pragma omp for schedule(dynamic, 4096)
         for (int64_t r = 0; r < n; ++r) {
             const int64_t o = p[r];
-            B.d[r] = A.d[o];
+            for (int32_t b = 0; b < nb; ++b) B.d[(size_t)r * nb + b] = A.d[(size_t)o * nb + b];
             row.clear();
-            for (int64_t q = A.rp[o]; q < A.rp[o + 1]; ++q) row.emplace_back(inv[A.ci[q]], A.v[q]);
+            for (int64_t q = A.rp[o]; q < A.rp[o + 1]; ++q) row.emplace_back(inv[A.ci[q]], q);
             std::sort(row.begin(), row.end(),
                       [](const auto& a, const auto& b) { return a.first < b.first; });
             int64_t w = B.rp[r];
-            for (auto& e : row) { B.ci[w] = e.first; B.v[w] = e.second; ++w; }
+            for (auto& e : row) {
+                B.ci[w] = e.first;
+                for (int32_t b = 0; b < nb; ++b) B.v[(size_t)w * nb + b] = A.v[(size_t)e.second * nb + b];
+                ++w;
+            }
         }
     }
 }

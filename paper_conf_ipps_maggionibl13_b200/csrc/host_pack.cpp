@@ -13,12 +13,13 @@
 namespace cme {
 
 namespace {
-// Does row r of A hold column c (columns ascending)?  Returns its value or 0.
-inline double entry(const Csr& A, int64_t r, int64_t c) {
+// Position of column c in row r of A (columns ascending), or -1.  Stored
+// entries are non-zero (in at least one batch member), so presence = A_rc != 0.
+inline int64_t entry(const Csr& A, int64_t r, int64_t c) {
     const int32_t* b = A.ci.data() + A.rp[r];
     const int32_t* e = A.ci.data() + A.rp[r + 1];
     const int32_t* p = std::lower_bound(b, e, (int32_t)c);
-    return (p != e && *p == c) ? A.v[A.rp[r] + (p - b)] : 0.0;
+    return (p != e && *p == c) ? A.rp[r] + (p - b) : -1;
 }
 }  // namespace
 
@@ -29,7 +30,7 @@ bool band_rule(const Csr& A, int band_mode) {
     int64_t cnt = 0;
 #pragma omp parallel for reduction(+ : cnt) schedule(static)
     for (int64_t i = 0; i < n; ++i)
-        cnt += (i > 0 && entry(A, i, i - 1) != 0.0) + (i + 1 < n && entry(A, i, i + 1) != 0.0);
+        cnt += (i > 0 && entry(A, i, i - 1) >= 0) + (i + 1 < n && entry(A, i, i + 1) >= 0);
     const int64_t den = 2 * n - 2;
     return den > 0 && 3 * cnt >= 2 * den;
 }
@@ -42,6 +43,8 @@ void pack_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, int32_t 
     P.band_on = band_on;
     P.window = window > 1 ? window : 1;
     P.group = group;
+    const int32_t nb = A.B;
+    P.B = nb;
     P.n_slots = (n + 31) / 32 * 32;
     P.n_slices = P.n_slots / 32;
     std::vector<int32_t> c(n);
@@ -49,7 +52,7 @@ void pack_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, int32_t 
     for (int64_t l = 0; l < n; ++l) {
         const int64_t r = r0 + l;
         int64_t k = A.rp[r + 1] - A.rp[r];
-        if (band_on) k -= (r > 0 && entry(A, r, r - 1) != 0.0) + (r + 1 < A.n && entry(A, r, r + 1) != 0.0);
+        if (band_on) k -= (r > 0 && entry(A, r, r - 1) >= 0) + (r + 1 < A.n && entry(A, r, r + 1) >= 0);
         c[l] = (int32_t)k;
     }
     // local rearrangement: each window's slots take its rows by (-c, row)
@@ -81,32 +84,36 @@ void pack_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, int32_t 
         }
     for (int64_t q = 0; q < P.n_slices; ++q) P.slice_off[q + 1] = P.slice_off[q] + 32 * (int64_t)P.slice_w[q];
     P.n_ell = P.slice_off[P.n_slices];
-    P.val.assign(P.n_ell, 0.0);
+    // values are member-minor: val[e*B + b], lo/up/inv_d[s*B + b]
+    P.val.assign((size_t)P.n_ell * nb, 0.0);
     P.col.assign(P.n_ell, 0);
-    P.lo.assign(P.n_slots, 0.0);
-    P.up.assign(P.n_slots, 0.0);
-    P.inv_d.assign(P.n_slots, 0.0);
+    P.lo.assign((size_t)P.n_slots * nb, 0.0);
+    P.up.assign((size_t)P.n_slots * nb, 0.0);
+    P.inv_d.assign((size_t)P.n_slots * nb, 0.0);
 #pragma omp parallel for schedule(dynamic, 256)
     for (int64_t s = 0; s < P.n_slots; ++s) {
         const int64_t q = s >> 5, lane = s & 31;
-        double* vq = P.val.data() + P.slice_off[q] + lane;
-        int32_t* cq = P.col.data() + P.slice_off[q] + lane;
+        const int64_t e0 = P.slice_off[q] + lane;   // entry t of this slot: e0 + 32 t
+        int32_t* cq = P.col.data() + e0;
         const int32_t w = P.slice_w[q];
         if (s >= n) {  // pad slot beyond the last row
             for (int32_t t = 0; t < w; ++t) cq[32 * t] = (int32_t)(r1 - 1 - col_shift);
             continue;
         }
         const int64_t l = P.row_of[s], r = r0 + l;
-        P.inv_d[s] = 1.0 / (-A.d[r]);
+        for (int32_t b = 0; b < nb; ++b) P.inv_d[(size_t)s * nb + b] = 1.0 / (-A.d[(size_t)r * nb + b]);
         if (band_on) {
-            P.lo[s] = r > 0 ? entry(A, r, r - 1) : 0.0;
-            P.up[s] = r + 1 < A.n ? entry(A, r, r + 1) : 0.0;
+            const int64_t pl = r > 0 ? entry(A, r, r - 1) : -1, pu = r + 1 < A.n ? entry(A, r, r + 1) : -1;
+            for (int32_t b = 0; b < nb; ++b) {
+                P.lo[(size_t)s * nb + b] = pl >= 0 ? A.v[(size_t)pl * nb + b] : 0.0;
+                P.up[(size_t)s * nb + b] = pu >= 0 ? A.v[(size_t)pu * nb + b] : 0.0;
+            }
         }
         int32_t t = 0;
         for (int64_t p = A.rp[r]; p < A.rp[r + 1]; ++p) {
             const int64_t j = A.ci[p];
             if (band_on && (j == r - 1 || j == r + 1)) continue;
-            vq[32 * t] = A.v[p];
+            for (int32_t b = 0; b < nb; ++b) P.val[(size_t)(e0 + 32 * t) * nb + b] = A.v[(size_t)p * nb + b];
             cq[32 * t] = (int32_t)(j - col_shift);
             ++t;
         }
@@ -124,7 +131,7 @@ void pack_csr_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, Pack
     const int64_t base = A.rp[r0];
     for (int64_t l = 0; l <= n; ++l) P.csr_rp[l] = A.rp[r0 + l] - base;
     P.csr_ci.resize(P.csr_rp[n]);
-    P.csr_v.assign(A.v.begin() + base, A.v.begin() + base + P.csr_rp[n]);
+    P.csr_v.assign(A.v.begin() + base, A.v.begin() + base + P.csr_rp[n]);  // (CSR arm: B = 1 only)
     for (int64_t p = 0; p < P.csr_rp[n]; ++p) P.csr_ci[p] = (int32_t)(A.ci[base + p] - col_shift);
     P.inv_d.assign(P.n_slots, 0.0);
     for (int64_t l = 0; l < n; ++l) P.inv_d[l] = 1.0 / (-A.d[r0 + l]);

@@ -1,19 +1,22 @@
 // sm_100a kernels of the fused Jacobi step.
 //
-// One step computes, for every row r (slot s of the packed layout):
-//   y_r = sc * [ (1-omega) x_r + omega * inv_d_s * ((lo_s x_{r-1} + up_s x_{r+1}) + sum_t val x[col]) ]
-// = sc * M_omega x (eq. 8 with relaxation omega, R1; sc = pending
-// 1/||y||_1 of the previous check, R5).  CHECK steps also emit per-CTA
-// partials of sum y, sum x, sum |y - x|, max |a_ii||y - x| and max x, which
-// are the L1 normalisation, delta (R2) and the paper's normalised
-// residual (r_i = a_ii (x_i - (Mx)_i) = |a_ii| (y_i - x_i) / omega).
+// One step computes, for every row r (slot s of the packed layout) and every
+// batch member b (B rate sets sharing one pattern; B = 1 is the plain solve):
+//   y_rb = sc_b * [ (1-omega) x_rb + omega * inv_d_sb * ((lo_sb x_{r-1,b} + up_sb x_{r+1,b})
+//                                                         + sum_t val_tb x[col_t, b]) ]
+// = sc_b * M_omega x_b (eq. 8 with relaxation omega, R1; sc_b = the
+// pending 1/||y_b||_1 of the previous check, R5).  CHECK steps also emit
+// per-CTA partials of sum y, sum x, sum |y - x|, max |a_ii||y - x| and max x
+// per member: the L1 normalisation, delta (R2) and the paper's
+// normalised residual (r_i = |a_ii| (y_i - x_i) / omega, R21).
 //
 // Mapping: warp = one 32-row slice (slice size decoupled from the
-// 256-thread CTA), lane = slot.  The slice's val/col block is contiguous and
-// column-major, so each t-step of a warp reads 256 B of val and 128 B of col
-// fully coalesced.  Streams are read with L1::no_allocate + an L2 evict-first
-// policy so the gathered iterate x keeps L1/L2; all val/col loads of a chunk
-// of up to 8 t-steps are issued before the dependent x gathers (ILP).
+// CTA), lane = slot.  The slice's val/col block is contiguous and
+// column-major, so each t-step of a warp reads 256*B B of val and 128 B of col,
+// fully coalesced; the iterate is member-minor (x[c*B + b]) so one gather
+// fetches all B members of a column with one 8*B-byte load (B = 4: a 256-bit
+// LDG).  Streams are read with L1::no_allocate + an L2 evict-first policy so
+// the gathered iterate keeps L1/L2.
 #pragma once
 #include <cstdint>
 #include <cuda_runtime.h>
@@ -22,20 +25,23 @@ namespace cme {
 
 constexpr int kWarpsPerCta = 8;
 constexpr int kCta = 32 * kWarpsPerCta;
-constexpr int kPartials = 8;  // doubles per CTA partial record
-constexpr int kUnroll = 8;    // t-steps whose loads are issued together
+constexpr int kPartials = 8;   // doubles per (CTA, member) partial record
+constexpr int kMaxBatch = 8;
 
-// Device control block of a solve (host writes the inputs, finalize the rest).
+// Device control block of a solve (host writes the inputs, decide_kernel the rest).
 struct Ctrl {
-    double omega, tol, stag_tol, norm_inf;
+    double omega, tol, stag_tol;
     int64_t C, max_iter;
-    int32_t stop_mode, nranks;
+    int32_t stop_mode, nranks, batch, pad0_;
     int64_t iter;                 // iterations completed
-    double delta, delta_prev, resid, mass, inv_s;
-    int32_t status;               // -1 running, else cme_status
+    int32_t status;               // -1 running, else overall cme_status
     int32_t stop;                 // 1 -> later step/finalize launches are no-ops
-    int32_t bad_input, pad_;
-    double red[kPartials];        // globally reduced check partials
+    int32_t bad_input, pad1_;
+    double norm_inf[kMaxBatch];
+    double delta[kMaxBatch], delta_prev[kMaxBatch], resid[kMaxBatch], mass[kMaxBatch];
+    double inv_s[kMaxBatch];      // pending 1/sum(y_b), applied by the next step
+    int32_t mstatus[kMaxBatch];   // per member: -1 running, else cme_status
+    int64_t miters[kMaxBatch];    // iteration at which the member's status was set
 };
 
 struct StepArgs {
@@ -43,20 +49,20 @@ struct StepArgs {
     int64_t slice_begin, slice_end;
     const int64_t* slice_off;
     const int32_t* slice_w;
-    const double* val;
+    const double* val;     // [n_ell][B]
     const int32_t* col;    // x-span coordinates
     const int32_t* row_of; // slot -> local row (nullptr: identity)
-    const double* lo;
+    const double* lo;      // [n_slots][B]
     const double* up;
     const double* inv_d;
-    const double* x;       // x-span base (x[-1], x[nx] are zero sentinels)
+    const double* x;       // x-span base, member-minor; x[-B..-1], x[nx*B..] zero sentinels
     double* y;             // x-span base of the output buffer
     int64_t own_off;       // own row r lives at x-span index own_off + r
     double omega;
-    const double* pre_scale;  // nullable
-    double* partials;         // CHECK: [gridDim.x][kPartials]
+    const double* pre_scale;  // nullable: [B] pending scales
+    double* partials;         // CHECK: [gridDim.x][B][kPartials]
     const int32_t* stop;      // nullable
-    // CSR arm
+    // CSR arm (B = 1)
     const int64_t* csr_rp;
     const int32_t* csr_ci;
     const double* csr_v;
@@ -77,7 +83,37 @@ __device__ __forceinline__ int32_t ld_stream(const int32_t* p, uint64_t pol) {
     asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
     return v;
 }
-__device__ __forceinline__ double ld_x(const double* p) { return __ldg(p); }
+
+// B contiguous doubles (B*8-byte aligned): read-only path, vector loads.
+template <int B>
+__device__ __forceinline__ void ld_vec(const double* p, double* v) {
+    if constexpr (B == 1) {
+        v[0] = __ldg(p);
+    } else if constexpr (B == 2) {
+        const double2 t = __ldg(reinterpret_cast<const double2*>(p));
+        v[0] = t.x; v[1] = t.y;
+    } else {
+#pragma unroll
+        for (int k = 0; k < B; k += 4)
+            asm volatile("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];"
+                         : "=d"(v[k]), "=d"(v[k + 1]), "=d"(v[k + 2]), "=d"(v[k + 3]) : "l"(p + k));
+    }
+}
+// B contiguous stream doubles (no L1 allocation, L2 evict-first)
+template <int B>
+__device__ __forceinline__ void ld_stream_vec(const double* p, uint64_t pol, double* v) {
+    if constexpr (B == 1) {
+        v[0] = ld_stream(p, pol);
+    } else if constexpr (B == 2) {
+        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f64 {%0,%1}, [%2], %3;"
+                     : "=d"(v[0]), "=d"(v[1]) : "l"(p), "l"(pol));
+    } else {
+#pragma unroll
+        for (int k = 0; k < B; k += 4)
+            asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f64 {%0,%1,%2,%3}, [%4], %5;"
+                         : "=d"(v[k]), "=d"(v[k + 1]), "=d"(v[k + 2]), "=d"(v[k + 3]) : "l"(p + k), "l"(pol));
+    }
+}
 
 __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
@@ -90,139 +126,158 @@ __device__ __forceinline__ double warp_max(double v) {
     return v;
 }
 
-// CTA-level deterministic reduction of the 5 check quantities into
-// partials[blockIdx.x]; NW = warps in the CTA (all must call it).
-template <int NW = kWarpsPerCta>
-__device__ __forceinline__ void cta_check_partials(double sy, double sx, double sd, double md,
-                                                   double mx, double* partials) {
+// Per-thread check accumulators of B members.
+template <int B>
+struct CheckAcc {
+    double sy[B], sx[B], sd[B], md[B], mx[B];
+    __device__ __forceinline__ CheckAcc() {
+#pragma unroll
+        for (int b = 0; b < B; ++b) sy[b] = sx[b] = sd[b] = md[b] = mx[b] = 0.0;
+    }
+    __device__ __forceinline__ void add(int b, double y, double x, double id) {
+        const double df = fabs(y - x);
+        sy[b] += y; sx[b] += x; sd[b] += df; md[b] = fmax(md[b], df / id); mx[b] = fmax(mx[b], x);
+    }
+};
+
+// CTA-level deterministic reduction of the check quantities of B members into
+// partials[blockIdx.x][b]; NW = warps in the CTA (all threads must call it).
+template <int NW, int B>
+__device__ __forceinline__ void cta_check_partials(const CheckAcc<B>& c, double* partials) {
     __shared__ double red[NW][5];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    sy = warp_sum(sy); sx = warp_sum(sx); sd = warp_sum(sd);
-    md = warp_max(md); mx = warp_max(mx);
-    if (lane == 0) { red[w][0] = sy; red[w][1] = sx; red[w][2] = sd; red[w][3] = md; red[w][4] = mx; }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        double a = 0, b = 0, c = 0, d = 0, e = 0;
-        for (int i = 0; i < NW; ++i) {
-            a += red[i][0]; b += red[i][1]; c += red[i][2];
-            d = fmax(d, red[i][3]); e = fmax(e, red[i][4]);
-        }
-        double* o = partials + (size_t)blockIdx.x * kPartials;
-        o[0] = a; o[1] = b; o[2] = c; o[3] = d; o[4] = e; o[5] = 0; o[6] = 0; o[7] = 0;
-    }
-}
-
-// x loads: read-only path (.nc) when x is constant for the whole launch;
-// L2-coherent (.cg) in the persistent kernel, whose x is rewritten by other
-// CTAs between grid barriers.
-template <bool COHERENT>
-__device__ __forceinline__ double ld_xv(const double* p) {
-    if (COHERENT) {
-        double v;
-        asm volatile("ld.global.cg.f64 %0, [%1];" : "=d"(v) : "l"(p));
-        return v;
-    }
-    return __ldg(p);
-}
-
-// Check terms of one row: y, x (both scaled), inv_d.
-struct SlotOut {
-    double y, x, id;
-    bool valid;
-};
-__device__ __forceinline__ void check_accum(const SlotOut& o, double& sy, double& sx, double& sd, double& md,
-                                            double& mx) {
-    if (!o.valid) return;
-    const double df = fabs(o.y - o.x);
-    sy += o.y; sx += o.x; sd += df; md = fmax(md, df / o.id); mx = fmax(mx, o.x);
-}
-
-// One slot (lane) of slice q: computes and stores y_r for its row r.
-template <bool BAND, bool REARR, bool DAMP, bool NEEDX, bool COHERENT>
-__device__ __forceinline__ SlotOut sell_slot(const StepArgs& a, int64_t q, int lane, uint64_t pol,
-                                             const double* x, double* y, const double* pre_scale) {
-    const int64_t slot = q * 32 + lane;
-    const int w = __ldg(a.slice_w + q);
-    const int64_t base = __ldg(a.slice_off + q) + lane;
-    if (slot >= a.n_rows) return SlotOut{0.0, 0.0, 1.0, false};
-    const int64_t r = REARR ? (int64_t)ld_stream(a.row_of + slot, pol) : slot;
-    const double* xo = x + a.own_off;
-    double acc = 0.0;
-    for (int t0 = 0; t0 < w; t0 += kUnroll) {
-        double v[kUnroll];
-        int32_t c[kUnroll];
-#pragma unroll
-        for (int u = 0; u < kUnroll; ++u) {
-            if (t0 + u < w) {
-                v[u] = ld_stream(a.val + base + 32 * (int64_t)(t0 + u), pol);
-                c[u] = ld_stream(a.col + base + 32 * (int64_t)(t0 + u), pol);
+#pragma unroll 1
+    for (int b = 0; b < B; ++b) {
+        const double sy = warp_sum(c.sy[b]), sx = warp_sum(c.sx[b]), sd = warp_sum(c.sd[b]);
+        const double md = warp_max(c.md[b]), mx = warp_max(c.mx[b]);
+        if (lane == 0) { red[w][0] = sy; red[w][1] = sx; red[w][2] = sd; red[w][3] = md; red[w][4] = mx; }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            double a = 0, bb = 0, cc = 0, d = 0, e = 0;
+            for (int i = 0; i < NW; ++i) {
+                a += red[i][0]; bb += red[i][1]; cc += red[i][2];
+                d = fmax(d, red[i][3]); e = fmax(e, red[i][4]);
             }
+            double* o = partials + ((size_t)blockIdx.x * B + b) * kPartials;
+            o[0] = a; o[1] = bb; o[2] = cc; o[3] = d; o[4] = e; o[5] = 0; o[6] = 0; o[7] = 0;
         }
-        double xv[kUnroll];
-#pragma unroll
-        for (int u = 0; u < kUnroll; ++u)
-            if (t0 + u < w) xv[u] = ld_xv<COHERENT>(x + c[u]);
-#pragma unroll
-        for (int u = 0; u < kUnroll; ++u)
-            if (t0 + u < w) acc = fma(v[u], xv[u], acc);
+        __syncthreads();
     }
-    double s = acc;
-    if (BAND) {
-        const double l = ld_stream(a.lo + slot, pol), up = ld_stream(a.up + slot, pol);
-        s = fma(l, ld_xv<COHERENT>(xo + r - 1), up * ld_xv<COHERENT>(xo + r + 1)) + acc;
-    }
-    const double id = ld_stream(a.inv_d + slot, pol);
-    double xr = (DAMP || NEEDX) ? ld_xv<COHERENT>(xo + r) : 0.0;
-    double yv = DAMP ? fma(1.0 - a.omega, xr, a.omega * (id * s)) : id * s;
-    if (pre_scale != nullptr) {
-        const double sc = *pre_scale;
-        yv *= sc;
-        xr *= sc;
-    }
-    y[a.own_off + r] = yv;
-    return SlotOut{yv, xr, id, true};
 }
 
-template <bool BAND, bool REARR, bool DAMP, bool CHECK>
+// Epilogue of one row shared by all SELL kernels: band term, damping, pending
+// scale, store, check terms.  acc = sum_t val x[col]; lo/up/id = the slot's
+// B-vectors; xo/yo = x-span bases shifted to the own rows (member-minor).
+template <int B, bool BAND, bool CHECK>
+__device__ __forceinline__ void finish_row(const StepArgs& a, int64_t r, const double* xo, double* yo,
+                                           const double (&acc)[B], const double (&lo)[B], const double (&up)[B],
+                                           const double (&id)[B], const double* pre_scale, CheckAcc<B>& ck) {
+    double xl[B], xu[B], xr[B];
+    if (BAND) {
+        ld_vec<B>(xo + (r - 1) * B, xl);
+        ld_vec<B>(xo + (r + 1) * B, xu);
+    }
+    // x_r unconditionally: a guarded load could not be hoisted next to the
+    // gathers (measured 3% slower on cfg4); it shares their L1/L2 lines
+    const bool damp = a.omega != 1.0;
+    ld_vec<B>(xo + r * B, xr);
+    double yv[B];
+#pragma unroll
+    for (int b = 0; b < B; ++b) {
+        const double s = BAND ? fma(lo[b], xl[b], up[b] * xu[b]) + acc[b] : acc[b];
+        double y = damp ? fma(1.0 - a.omega, xr[b], a.omega * (id[b] * s)) : id[b] * s;
+        double x = (damp || CHECK) ? xr[b] : 0.0;
+        if (pre_scale != nullptr) {
+            const double sc = pre_scale[b];
+            y *= sc;
+            x *= sc;
+        }
+        yv[b] = y;
+        if (CHECK) ck.add(b, y, x, id[b]);
+    }
+    double* dst = yo + r * B;
+    if constexpr (B == 1) {
+        dst[0] = yv[0];
+    } else if constexpr (B == 2) {
+        *reinterpret_cast<double2*>(dst) = make_double2(yv[0], yv[1]);
+    } else {
+#pragma unroll
+        for (int k = 0; k < B; k += 4)
+            asm volatile("st.global.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(dst + k), "d"(yv[k]), "d"(yv[k + 1]),
+                         "d"(yv[k + 2]), "d"(yv[k + 3])
+                         : "memory");
+    }
+}
+
+// ILP chunk (t-steps whose loads are issued together) for a batch width.
+template <int B>
+struct Chunk {
+    static constexpr int U = B >= 8 ? 1 : 8 / B;
+};
+
+template <int B, bool BAND, bool REARR, bool CHECK>
 __global__ void __launch_bounds__(kCta) sell_step_kernel(const StepArgs a) {
     if (a.stop != nullptr && *a.stop) return;
     const uint64_t pol = evict_first_policy();
     const int lane = threadIdx.x & 31;
     const int64_t q = a.slice_begin + (int64_t)blockIdx.x * kWarpsPerCta + (threadIdx.x >> 5);
-    double sy = 0.0, sx = 0.0, sd = 0.0, md = 0.0, mx = 0.0;
+    CheckAcc<B> ck;
     if (q < a.slice_end) {
-        const SlotOut o = sell_slot<BAND, REARR, DAMP, CHECK, false>(a, q, lane, pol, a.x, a.y, a.pre_scale);
-        if (CHECK) check_accum(o, sy, sx, sd, md, mx);
+        const int64_t slot = q * 32 + lane;
+        const int w = __ldg(a.slice_w + q);
+        const int64_t base = __ldg(a.slice_off + q) + lane;
+        if (slot < a.n_rows) {
+            const int64_t r = REARR ? (int64_t)ld_stream(a.row_of + slot, pol) : slot;
+            constexpr int U = Chunk<B>::U;
+            double acc[B];
+#pragma unroll
+            for (int b = 0; b < B; ++b) acc[b] = 0.0;
+            for (int t0 = 0; t0 < w; t0 += U) {
+                double v[U][B], xv[U][B];
+                int32_t c[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (t0 + u < w) {
+                        const int64_t e = base + 32 * (int64_t)(t0 + u);
+                        ld_stream_vec<B>(a.val + e * B, pol, v[u]);
+                        c[u] = ld_stream(a.col + e, pol);
+                    }
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (t0 + u < w) ld_vec<B>(a.x + (int64_t)c[u] * B, xv[u]);
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (t0 + u < w)
+#pragma unroll
+                        for (int b = 0; b < B; ++b) acc[b] = fma(v[u][b], xv[u][b], acc[b]);
+            }
+            double lo[B], up[B], id[B];
+            if (BAND) {
+                ld_stream_vec<B>(a.lo + slot * B, pol, lo);
+                ld_stream_vec<B>(a.up + slot * B, pol, up);
+            }
+            ld_stream_vec<B>(a.inv_d + slot * B, pol, id);
+            finish_row<B, BAND, CHECK>(a, r, a.x + a.own_off * B, a.y + a.own_off * B, acc, lo, up, id,
+                                       a.pre_scale, ck);
+        }
     }
-    if (CHECK) cta_check_partials<kWarpsPerCta>(sy, sx, sd, md, mx, a.partials);
+    if (CHECK) cta_check_partials<kWarpsPerCta, B>(ck, a.partials);
 }
 
-// Plain CSR arm (ablation, CME_FMT_CSR): one thread per row.
-template <bool DAMP, bool CHECK>
+// Plain CSR arm (ablation, CME_FMT_CSR, B = 1): one thread per row.
+template <bool CHECK>
 __global__ void __launch_bounds__(kCta) csr_step_kernel(const StepArgs a) {
     if (a.stop != nullptr && *a.stop) return;
     const int64_t r = a.slice_begin * 32 + (int64_t)blockIdx.x * kCta + threadIdx.x;
-    double sy = 0.0, sx = 0.0, sd = 0.0, md = 0.0, mx = 0.0;
+    CheckAcc<1> ck;
     if (r < a.n_rows && r < a.slice_end * 32) {
         const int64_t b = __ldg(a.csr_rp + r), e = __ldg(a.csr_rp + r + 1);
-        double acc = 0.0;
-        for (int64_t p = b; p < e; ++p) acc = fma(__ldg(a.csr_v + p), ld_x(a.x + __ldg(a.csr_ci + p)), acc);
-        const double id = __ldg(a.inv_d + r);
-        const double* xo = a.x + a.own_off;
-        double xr = (DAMP || CHECK) ? ld_x(xo + r) : 0.0;
-        double yv = DAMP ? fma(1.0 - a.omega, xr, a.omega * (id * acc)) : id * acc;
-        if (a.pre_scale != nullptr) {
-            const double sc = *a.pre_scale;
-            yv *= sc;
-            xr *= sc;
-        }
-        a.y[a.own_off + r] = yv;
-        if (CHECK) {
-            const double df = fabs(yv - xr);
-            sy = yv; sx = xr; sd = df; md = df / id; mx = xr;
-        }
+        double acc[1] = {0.0};
+        for (int64_t p = b; p < e; ++p) acc[0] = fma(__ldg(a.csr_v + p), __ldg(a.x + __ldg(a.csr_ci + p)), acc[0]);
+        const double id[1] = {__ldg(a.inv_d + r)}, z[1] = {0.0};
+        finish_row<1, false, CHECK>(a, r, a.x + a.own_off, a.y + a.own_off, acc, z, z, id, a.pre_scale, ck);
     }
-    if (CHECK) cta_check_partials<kWarpsPerCta>(sy, sx, sd, md, mx, a.partials);
+    if (CHECK) cta_check_partials<kWarpsPerCta, 1>(ck, a.partials);
 }
 
 }  // namespace cme

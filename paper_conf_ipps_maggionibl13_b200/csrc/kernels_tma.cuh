@@ -68,16 +68,19 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
         : "memory");
 }
 
-// Host/device agreement on the stage layout: returns off_val; off_col and the
-// stage size follow from the largest tile's ELL entry count.
-__host__ __device__ inline int tma_fixed_bytes(int ncw, bool band, bool rearr) {
-    return ncw * 32 * (8 + (rearr ? 4 : 0) + (band ? 16 : 0));
+// Stage layout: [inv_d][row_of if REARR][lo, up if BAND][val][col] for
+// NCW*32 slots and B members; the host computes the same offsets from
+// tma_fixed_bytes() and the widest tile.
+__host__ __device__ inline int tma_fixed_bytes(int ncw, int B, bool band, bool rearr) {
+    return ncw * 32 * (8 * B + (rearr ? 4 : 0) + (band ? 16 * B : 0));
 }
 
-template <int NCW, bool BAND, bool REARR, bool DAMP, bool CHECK>
+template <int NCW, int B, bool BAND, bool REARR, bool CHECK>
 __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBlocks)
     sell_tma_kernel(const TmaArgs T) {
-    constexpr int kTmaConsumers = NCW, kTileSlices = NCW;
+    constexpr int kConsumers = NCW, kTileSlices = NCW, kSlots = NCW * 32;
+    constexpr int kOffInvd = 0, kOffRow = 8 * B * kSlots, kOffLo = kOffRow + (REARR ? 4 * kSlots : 0),
+                  kOffUp = kOffLo + 8 * B * kSlots;
     const StepArgs& a = T.a;
     if (a.stop != nullptr && *a.stop) return;
     extern __shared__ __align__(128) unsigned char smem[];
@@ -87,20 +90,14 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
             mbar_init(&full[s], 1);
-            mbar_init(&empty[s], kTmaConsumers);
+            mbar_init(&empty[s], kConsumers);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
+    CheckAcc<B> ck;
 
-    // stage layout: [inv_d][row_of if REARR][lo, up if BAND][val][col], NCW*32 slots
-    // (tma_fixed_bytes() gives the host the same offsets)
-    constexpr int kSlots = NCW * 32;
-    constexpr int kOffInvd = 0, kOffRow = 8 * kSlots, kOffLo = kOffRow + (REARR ? 4 * kSlots : 0),
-                  kOffUp = kOffLo + 8 * kSlots;
-    double sy = 0.0, sx = 0.0, sd = 0.0, md = 0.0, mx = 0.0;
-
-    if (warp == kTmaConsumers) {
+    if (warp == kConsumers) {
         // ---------------- producer ----------------
         if (lane == 0) {
             const uint64_t pol = evict_first_policy();
@@ -114,25 +111,26 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
                 const int64_t e0 = a.slice_off[q0], e1 = a.slice_off[q1];
                 const uint32_t slots = (uint32_t)(q1 - q0) * 32u;
                 const uint32_t nval = (uint32_t)(e1 - e0);
-                uint32_t bytes = nval * 12u + slots * 8u;
+                uint32_t bytes = nval * (8u * B + 4u) + slots * 8u * B;
                 if (REARR) bytes += slots * 4u;
-                if (BAND) bytes += slots * 16u;
+                if (BAND) bytes += slots * 16u * B;
                 mbar_expect_tx(&full[s], bytes);
-                bulk_g2s(st + kOffInvd, a.inv_d + q0 * 32, slots * 8u, &full[s], pol);
+                bulk_g2s(st + kOffInvd, a.inv_d + q0 * 32 * B, slots * 8u * B, &full[s], pol);
                 if (REARR) bulk_g2s(st + kOffRow, a.row_of + q0 * 32, slots * 4u, &full[s], pol);
                 if (BAND) {
-                    bulk_g2s(st + kOffLo, a.lo + q0 * 32, slots * 8u, &full[s], pol);
-                    bulk_g2s(st + kOffUp, a.up + q0 * 32, slots * 8u, &full[s], pol);
+                    bulk_g2s(st + kOffLo, a.lo + q0 * 32 * B, slots * 8u * B, &full[s], pol);
+                    bulk_g2s(st + kOffUp, a.up + q0 * 32 * B, slots * 8u * B, &full[s], pol);
                 }
                 if (nval) {
-                    bulk_g2s(st + T.off_val, a.val + e0, nval * 8u, &full[s], pol);
+                    bulk_g2s(st + T.off_val, a.val + e0 * B, nval * 8u * B, &full[s], pol);
                     bulk_g2s(st + T.off_col, a.col + e0, nval * 4u, &full[s], pol);
                 }
             }
         }
     } else {
         // ---------------- consumers ----------------
-        const double* xo = a.x + a.own_off;
+        const double* xo = a.x + a.own_off * B;
+        double* yo = a.y + a.own_off * B;
         int64_t i = 0;
         for (int64_t tile = blockIdx.x; tile < T.n_tiles; tile += gridDim.x, ++i) {
             const int s = (int)(i % S);
@@ -150,44 +148,38 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
             const int64_t slot = q * 32 + lane;
             if (q < a.slice_end && slot < a.n_rows) {
                 const int ls = warp * 32 + lane;
-                const double* sval = reinterpret_cast<const double*>(st + T.off_val) + loff + lane;
+                const double* sval = reinterpret_cast<const double*>(st + T.off_val) + (loff + lane) * B;
                 const int32_t* scol = reinterpret_cast<const int32_t*>(st + T.off_col) + loff + lane;
                 const int64_t r = REARR ? (int64_t) reinterpret_cast<const int32_t*>(st + kOffRow)[ls] : slot;
-                double acc = 0.0;
-                for (int t0 = 0; t0 < w; t0 += kUnroll) {
-                    double xv[kUnroll];   // all gathers of the chunk in flight, then FMAs
+                constexpr int U = Chunk<B>::U;
+                double acc[B];
 #pragma unroll
-                    for (int u = 0; u < kUnroll; ++u)
-                        if (t0 + u < w) xv[u] = ld_x(a.x + scol[32 * (t0 + u)]);
+                for (int b = 0; b < B; ++b) acc[b] = 0.0;
+                for (int t0 = 0; t0 < w; t0 += U) {
+                    double xv[U][B];   // all gathers of the chunk in flight, then FMAs
 #pragma unroll
-                    for (int u = 0; u < kUnroll; ++u)
-                        if (t0 + u < w) acc = fma(sval[32 * (t0 + u)], xv[u], acc);
+                    for (int u = 0; u < U; ++u)
+                        if (t0 + u < w) ld_vec<B>(a.x + (int64_t)scol[32 * (t0 + u)] * B, xv[u]);
+#pragma unroll
+                    for (int u = 0; u < U; ++u)
+                        if (t0 + u < w)
+#pragma unroll
+                            for (int b = 0; b < B; ++b) acc[b] = fma(sval[32 * (t0 + u) * B + b], xv[u][b], acc[b]);
                 }
-                double sum = acc;
-                if (BAND) {
-                    const double l = reinterpret_cast<const double*>(st + kOffLo)[ls];
-                    const double up = reinterpret_cast<const double*>(st + kOffUp)[ls];
-                    sum = fma(l, ld_x(xo + r - 1), up * ld_x(xo + r + 1)) + acc;
+                double lo[B], up[B], id[B];
+#pragma unroll
+                for (int b = 0; b < B; ++b) {
+                    id[b] = reinterpret_cast<const double*>(st + kOffInvd)[ls * B + b];
+                    lo[b] = BAND ? reinterpret_cast<const double*>(st + kOffLo)[ls * B + b] : 0.0;
+                    up[b] = BAND ? reinterpret_cast<const double*>(st + kOffUp)[ls * B + b] : 0.0;
                 }
-                const double id = reinterpret_cast<const double*>(st + kOffInvd)[ls];
-                double xr = (DAMP || CHECK) ? ld_x(xo + r) : 0.0;
-                double yv = DAMP ? fma(1.0 - a.omega, xr, a.omega * (id * sum)) : id * sum;
-                if (a.pre_scale != nullptr) {
-                    const double sc = *a.pre_scale;
-                    yv *= sc;
-                    xr *= sc;
-                }
-                a.y[a.own_off + r] = yv;
-                if (CHECK) {
-                    const double df = fabs(yv - xr);
-                    sy += yv; sx += xr; sd += df; md = fmax(md, df / id); mx = fmax(mx, xr);
-                }
+                finish_row<B, BAND, CHECK>(a, r, xo, yo, acc, lo, up, id, a.pre_scale, ck);
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);
         }
     }
-    if (CHECK) cta_check_partials<NCW + 1>(sy, sx, sd, md, mx, a.partials);
+    if (CHECK) cta_check_partials<NCW + 1, B>(ck, a.partials);
 }
 
 }  // namespace cme

@@ -1,0 +1,73 @@
+// Definitions of the launchers declared in launch.h (included by step_b*.cu).
+#pragma once
+#include "launch.h"
+
+namespace cme {
+
+template <int B>
+cudaError_t launch_sell(const StepArgs& a, int grid, bool band, bool rearr, bool check, cudaStream_t s) {
+    const int key = (band ? 4 : 0) | (rearr ? 2 : 0) | (check ? 1 : 0);
+    switch (key) {
+#define K(bd, r, c) \
+    case bd * 4 + r * 2 + c: sell_step_kernel<B, bd, r, c><<<grid, kCta, 0, s>>>(a); break;
+        K(0, 0, 0) K(0, 0, 1) K(0, 1, 0) K(0, 1, 1) K(1, 0, 0) K(1, 0, 1) K(1, 1, 0) K(1, 1, 1)
+#undef K
+    }
+    return cudaGetLastError();
+}
+
+template <int W, int B>
+static cudaError_t launch_tma_w(const TmaArgs& T, int grid, int smem, bool band, bool rearr, bool check,
+                                cudaStream_t s) {
+    const int key = (band ? 4 : 0) | (rearr ? 2 : 0) | (check ? 1 : 0);
+    switch (key) {
+#define K(bd, r, c)                                                                                  \
+    case bd * 4 + r * 2 + c:                                                                         \
+        sell_tma_kernel<W, B, bd, r, c><<<grid, TmaShape<W>::kThreads, smem, s>>>(T);                \
+        break;
+        K(0, 0, 0) K(0, 0, 1) K(0, 1, 0) K(0, 1, 1) K(1, 0, 0) K(1, 0, 1) K(1, 1, 0) K(1, 1, 1)
+#undef K
+    }
+    return cudaGetLastError();
+}
+
+template <int B>
+cudaError_t launch_tma(const TmaArgs& T, int ncw, int grid, int smem, bool band, bool rearr, bool check,
+                       cudaStream_t s) {
+    return ncw == 16 ? launch_tma_w<16, B>(T, grid, smem, band, rearr, check, s)
+                     : launch_tma_w<8, B>(T, grid, smem, band, rearr, check, s);
+}
+
+template <int W, int B>
+static cudaError_t tma_prepare_w(int smem) {
+    cudaError_t e = cudaSuccess;
+#define A(bd, r, c) \
+    if (e == cudaSuccess)  \
+        e = cudaFuncSetAttribute(sell_tma_kernel<W, B, bd, r, c>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    A(0, 0, 0) A(0, 0, 1) A(0, 1, 0) A(0, 1, 1) A(1, 0, 0) A(1, 0, 1) A(1, 1, 0) A(1, 1, 1)
+#undef A
+    return e;
+}
+
+template <int B>
+cudaError_t tma_prepare(int ncw, int smem) {
+    return ncw == 16 ? tma_prepare_w<16, B>(smem) : tma_prepare_w<8, B>(smem);
+}
+
+template <int B>
+cudaError_t tma_occupancy(int ncw, int smem, int* occ) {
+    // the heaviest variant (band + rearrangement + check) bounds the residency
+    if (ncw == 16)
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_tma_kernel<16, B, true, true, true>,
+                                                             TmaShape<16>::kThreads, smem);
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_tma_kernel<8, B, true, true, true>,
+                                                         TmaShape<8>::kThreads, smem);
+}
+
+#define CME_INSTANTIATE_LAUNCHERS(B)                                                                       \
+    template cudaError_t launch_sell<B>(const StepArgs&, int, bool, bool, bool, cudaStream_t);              \
+    template cudaError_t launch_tma<B>(const TmaArgs&, int, int, int, bool, bool, bool, cudaStream_t);      \
+    template cudaError_t tma_prepare<B>(int, int);                                                          \
+    template cudaError_t tma_occupancy<B>(int, int, int*);
+
+}  // namespace cme

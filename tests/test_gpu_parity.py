@@ -251,23 +251,21 @@ def test_nccl_one_rank_distributed_path(cme, oracle_mod):
     m.cme_comm_destroy(comm)
 
 
-@pytest.mark.parametrize("knobs", [{"CME_TMA": "0", "CME_PERSIST": "0"}, {"CME_TMA": "1", "CME_PERSIST": "0"},
-                                   {"CME_TMA": "1", "CME_TMA_WARPS": "8", "CME_PERSIST": "0"},
-                                   {"CME_TMA": "0", "CME_PERSIST": "1"}],
+@pytest.mark.parametrize("knobs", [{"CME_TMA": "0"}, {"CME_TMA": "1"}, {"CME_TMA": "1", "CME_TMA_WARPS": "8"}],
                          ids=lambda k: ",".join(f"{a}={b}" for a, b in k.items()))
 @pytest.mark.parametrize("net,order,omega", [(W.toggle_switch(70), "rcm", 0.9), (W.schnakenberg(120), "none", 1.0),
                                              (W.brusselator(90), "dfs", 0.7)], ids=lambda x: getattr(x, "name", str(x)))
 def test_every_step_kernel(cme, oracle_mod, monkeypatch, knobs, net, order, omega):
-    """Each step kernel (register SELL, TMA-staged SELL with 16/8 consumer warps,
-    persistent cooperative SELL) forced on the same problems: per-step parity
-    and a fixed-iteration landscape (C = 7 exercises odd block parity)."""
+    """Each step kernel (register SELL, TMA-staged SELL with 16/8 consumer
+    warps) forced on the same problems: per-step parity and a fixed-iteration
+    landscape (C = 7 exercises odd block parity)."""
     for k, v in knobs.items():
         monkeypatch.setenv(k, v)
     states, r, c, v = oracle_mod.enumerate_network(net)
     A = oracle_mod.ingest(len(states), r, c, v)
     m = cme.Matrix(A.n, r, c, v).reorder(ORD[order]).pack()
     f = m.info()
-    expect = 3 if knobs.get("CME_PERSIST") == "1" else (1 if knobs["CME_TMA"] == "1" else 0)
+    expect = 1 if knobs["CME_TMA"] == "1" else 0
     assert f.kernel == expect
     m.set_opts(omega=omega, check_every=7, stag_tol=0.0)
     x = W.random_start(A.n, 21)

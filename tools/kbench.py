@@ -15,6 +15,7 @@ import time
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
+import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
 import workloads as W  # noqa: E402
@@ -28,6 +29,7 @@ ap.add_argument("--band", type=int, default=0)
 ap.add_argument("--fmt", type=int, default=0)
 ap.add_argument("--blocks", type=int, default=10)
 ap.add_argument("--C", type=int, default=100)
+ap.add_argument("--batch", type=int, default=1)
 ap.add_argument("variants", nargs="*", default=[""])
 a = ap.parse_args()
 
@@ -38,9 +40,15 @@ if a.config.startswith("banded"):
     omega = 1.0
     order = a.order or "none"
 else:
-    net = W.config_network(a.config)
     t = time.time()
-    s, r, c, v = cme.cme_network_enumerate(net)
+    if a.batch > 1:
+        vs = []
+        for net in W.sweep_networks(a.config, a.batch):
+            s, r, c, v = cme.cme_network_enumerate(net)
+            vs.append(v)
+        v = np.stack(vs)
+    else:
+        s, r, c, v = cme.cme_network_enumerate(W.config_network(a.config))
     n = len(s)
     omega = W.CONFIGS[a.config]["omega"]
     order = a.order or ("rcm" if "toggle" in a.config else "none")
@@ -62,7 +70,7 @@ for var in a.variants:
     f = m.info()
     st = torch.cuda.Stream()
     m.set_opts(omega=omega, check_every=a.C, stream=st.cuda_stream)
-    cme.cme_solver_load(m.h, n, None)
+    cme.cme_solver_load(m.h, n * a.batch, None)
     cme.cme_solver_run(m.h, 3)
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -73,7 +81,7 @@ for var in a.variants:
     ms = e0.elapsed_time(e1)
     it = a.blocks * a.C
     ti = ms * 1e-3 / it
-    print(f"[{var or 'default'}] {a.config} order={order} n={f.n} nnz={f.nnz} band={f.band_on} "
-          f"t/iter={ti * 1e6:.1f}us GFLOPS={2 * f.nnz / ti / 1e9:.1f} "
+    print(f"[{var or 'default'}] {a.config} B={a.batch} kernel={f.kernel} order={order} n={f.n} nnz={f.nnz} "
+          f"band={f.band_on} t/iter={ti * 1e6:.1f}us GFLOPS={2 * f.nnz * a.batch / ti / 1e9:.1f} "
           f"alg={f.bytes_alg / ti / 1e9:.0f}GB/s ({100 * f.bytes_alg / ti / 1e9 / peak:.1f}%) "
           f"fmt={f.bytes_fmt / ti / 1e9:.0f}GB/s", flush=True)

@@ -180,6 +180,26 @@ def config_network(name: str) -> Network:
     return CONFIGS[name]["network"]()
 
 
+# Batched sweeps: member b of a sweep over a config scales the
+# network's rates by these per-reaction factors (all > 0, so every member has
+# the same reachable states and sparsity pattern).
+SWEEP_FACTORS = [1.0, 0.7, 1.3, 2.0, 0.5, 1.1, 0.9, 1.6]
+
+
+def sweep_networks(name: str, batch: int):
+    """`batch` variants of config `name`: reaction k of member b has rate
+    r_k * SWEEP_FACTORS[b] ** (+1 for even k, -0.5 for odd k)."""
+    base = config_network(name)
+    out = []
+    for b in range(batch):
+        f = SWEEP_FACTORS[b % len(SWEEP_FACTORS)]
+        rates = [r * (f if k % 2 == 0 else f ** -0.5) for k, r in enumerate(base.rates)]
+        out.append(Network(name=f"{base.name}_sweep{b}", species=base.species, x0=base.x0,
+                           reactants=base.reactants, change=base.change, rates=rates,
+                           weights=base.weights, cap=base.cap, meta=dict(base.meta, sweep=b)))
+    return out
+
+
 # ----------------------------------------------------------------------------
 # Config 5: synthetic banded Markov generator (SURVEY.md 8(d), "Config 5
 # generator").  Counter-based splitmix64; every source state j owns the stream
