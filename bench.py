@@ -244,6 +244,9 @@ def main():
     import torch
     import torch.distributed as dist
     world = int(os.environ.get("WORLD_SIZE", "1"))
+    # under torchrun (RANK set) the row-sharded path runs even with one rank:
+    # NCCL communicator, distribute, halo/allgather in the graphs
+    dist_path = "RANK" in os.environ
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
@@ -252,7 +255,7 @@ def main():
     import paper_conf_ipps_maggionibl13_b200 as cme
 
     comm = None
-    if world > 1:
+    if dist_path:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         obj = [cme.cme_comm_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
@@ -260,7 +263,7 @@ def main():
 
     name = args.config
     B = args.batch
-    m, cfg, setup = build_matrix(cme, name, cme.CME_DEVICE_HOST_ONLY if world > 1 else local, B)
+    m, cfg, setup = build_matrix(cme, name, cme.CME_DEVICE_HOST_ONLY if dist_path else local, B)
     if comm is not None:
         cme.cme_matrix_distribute(m.h, comm)
     info = m.info()
@@ -273,7 +276,7 @@ def main():
     torch.cuda.synchronize()
 
     def barrier():
-        if world > 1:
+        if dist_path:
             dist.barrier()
         torch.cuda.synchronize()
 
