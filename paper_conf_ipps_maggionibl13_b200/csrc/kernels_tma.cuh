@@ -101,10 +101,13 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
         // ---------------- producer ----------------
         if (lane == 0) {
             const uint64_t pol = evict_first_policy();
-            int64_t i = 0;
-            for (int64_t tile = blockIdx.x; tile < T.n_tiles; tile += gridDim.x, ++i) {
-                const int s = (int)(i % S);
-                if (i >= S) mbar_wait(&empty[s], (uint32_t)(((i / S) - 1) & 1));
+            // stage s and the parity of its current use, advanced incrementally
+            // (no 64-bit division per tile)
+            int s = 0;
+            uint32_t phase = 0;
+            bool wrapped = false;
+            for (int64_t tile = blockIdx.x; tile < T.n_tiles; tile += gridDim.x) {
+                if (wrapped) mbar_wait(&empty[s], phase ^ 1u);   // consumers released the previous use
                 unsigned char* st = smem + (size_t)s * T.stage_bytes;
                 const int64_t q0 = tile * kTileSlices;
                 const int64_t q1 = min(q0 + kTileSlices, a.slice_end);
@@ -125,15 +128,16 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
                     bulk_g2s(st + T.off_val, a.val + e0 * B, nval * 8u * B, &full[s], pol);
                     bulk_g2s(st + T.off_col, a.col + e0, nval * 4u, &full[s], pol);
                 }
+                if (++s == S) { s = 0; phase ^= 1u; wrapped = true; }
             }
         }
     } else {
         // ---------------- consumers ----------------
         const double* xo = a.x + a.own_off * B;
         double* yo = a.y + a.own_off * B;
-        int64_t i = 0;
-        for (int64_t tile = blockIdx.x; tile < T.n_tiles; tile += gridDim.x, ++i) {
-            const int s = (int)(i % S);
+        int s = 0;
+        uint32_t phase = 0;
+        for (int64_t tile = blockIdx.x; tile < T.n_tiles; tile += gridDim.x) {
             const int64_t q0 = tile * kTileSlices;
             const int64_t q = q0 + warp;
             const unsigned char* st = smem + (size_t)s * T.stage_bytes;
@@ -144,7 +148,7 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
                 w = __ldg(a.slice_w + q);
                 loff = __ldg(a.slice_off + q) - __ldg(a.slice_off + q0);
             }
-            mbar_wait(&full[s], (uint32_t)((i / S) & 1));
+            mbar_wait(&full[s], phase);
             const int64_t slot = q * 32 + lane;
             if (q < a.slice_end && slot < a.n_rows) {
                 const int ls = warp * 32 + lane;
@@ -177,6 +181,7 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);
+            if (++s == S) { s = 0; phase ^= 1u; }
         }
     }
     if (CHECK) cta_check_partials<NCW + 1, B>(ck, a.partials);

@@ -1,3 +1,4 @@
 set -x
-timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 1 --master-addr 127.0.0.1 --master-port 29511 bench.py --gpus 1 --steps 10 --warmup 3 --no-cpu-baseline --no-converge 2>&1 | tail -3
-NCCL_DEBUG=WARN timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 1 --master-addr 127.0.0.1 --master-port 29512 bench.py --gpus 1 --steps 5 --warmup 3 --no-cpu-baseline --no-converge --batch 2 2>&1 | tail -3
+timeout 1500 python -m pytest tests -x -q -m "gpu and not slow" 2>&1 | tail -2
+timeout 900 python tools/kbench.py --config cfg4_toggle_20m --blocks 20 CME_TMA=1 CME_TMA=1 2>&1
+timeout 600 python tools/kbench.py --config cfg3a_schnakenberg_2m CME_TMA=1 2>&1
