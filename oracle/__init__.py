@@ -80,6 +80,8 @@ def lib():
                                           C.c_double, C.c_int64, C.c_int64, C.c_int, C.c_double,
                                           C.c_int, f64p, i64p, f64p, f64p]
         L.oracle_lu_steady.argtypes = [C.c_int64, i64p, i32p, f64p, f64p, f64p]
+        L.oracle_transient.argtypes = [C.c_int64, i64p, i32p, f64p, f64p, f64p, C.c_double, C.c_double,
+                                       f64p, i64p, f64p]
         _lib = L
     return _lib
 
@@ -258,3 +260,16 @@ def lu_steady(A: CSR) -> np.ndarray:
     p = np.empty(A.n)
     _check(lib().oracle_lu_steady(A.n, *A._a(), _ptr(p, f64p)), "oracle_lu_steady")
     return p
+
+
+def transient(A: CSR, t: float, p0=None, eps: float = 1e-14):
+    """p(t) = exp(A t) p0 by uniformization; returns (p, terms, Lambda)."""
+    p = np.empty(A.n)
+    terms, lam = C.c_int64(), C.c_double()
+    p0p = None
+    if p0 is not None:
+        p0 = np.ascontiguousarray(p0, dtype=np.float64)
+        p0p = _ptr(p0, f64p)
+    _check(lib().oracle_transient(A.n, *A._a(), p0p, t, eps, _ptr(p, f64p), C.byref(terms), C.byref(lam)),
+           "oracle_transient")
+    return p, terms.value, lam.value

@@ -833,7 +833,57 @@ int oracle_jacobi_solve(int64_t n, const int64_t* rp, const int32_t* col, const 
 }
 
 /* ------------------------------------------------------------------------ */
-/* 7. Dense LU null-space solve for tiny state spaces (north star)            */
+/* 7. Transient landscape by uniformization (P:L277 future work; R22)         */
+/* ------------------------------------------------------------------------ */
+int oracle_transient(int64_t n, const int64_t* rp, const int32_t* col, const double* val,
+                     const double* diag, const double* p0, double t, double eps, double* p_out,
+                     int64_t* terms_out, double* lambda_out) {
+    if (n <= 0 || !p_out || !(t >= 0.0) || !(eps > 0.0 && eps < 1.0)) return ORACLE_INVALID_ARG;
+    double lam = 0.0;
+    for (int64_t i = 0; i < n; i++) if (-diag[i] > lam) lam = -diag[i];
+    double* x = (double*)malloc(sizeof(double) * n);
+    double* y = (double*)malloc(sizeof(double) * n);
+    if (!x || !y) { free(x); free(y); return ORACLE_OOM; }
+    for (int64_t i = 0; i < n; i++) { x[i] = p0 ? p0[i] : (i == 0 ? 1.0 : 0.0); p_out[i] = 0.0; }
+    /* Poisson(k; mu = Lambda t) weights (R22): w_k ~ exp(k ln mu - lgamma(k+1))
+     * for k <= Kmax = ceil(mu + 10 sqrt(mu) + 40), normalised to sum 1;
+     * K = the smallest k with sum_{j>k} w_j <= eps */
+    const double mu = lam * t;
+    const int64_t kmax = (int64_t)ceil(mu + 10.0 * sqrt(mu) + 40.0);
+    double* w = (double*)malloc(sizeof(double) * (kmax + 1));
+    if (!w) { free(x); free(y); return ORACLE_OOM; }
+    double lmax = -INFINITY;
+    for (int64_t k = 0; k <= kmax; k++) {
+        w[k] = mu > 0.0 ? (double)k * log(mu) - lgamma((double)k + 1.0) : (k == 0 ? 0.0 : -INFINITY);
+        if (w[k] > lmax) lmax = w[k];
+    }
+    double W = 0.0;
+    for (int64_t k = 0; k <= kmax; k++) { w[k] = exp(w[k] - lmax); W += w[k]; }
+    for (int64_t k = 0; k <= kmax; k++) w[k] /= W;
+    int64_t K = kmax;
+    double tail = 0.0;
+    while (K > 0 && tail + w[K] <= eps) { tail += w[K]; K--; }
+    int64_t k = 0;
+    for (;; k++) {
+        for (int64_t i = 0; i < n; i++) p_out[i] += w[k] * x[i];
+        if (k == K) break;
+        /* x <- P x = x + A x / Lambda */
+        for (int64_t i = 0; i < n; i++) {
+            double s = 0.0;
+            for (int64_t p = rp[i]; p < rp[i + 1]; p++) s += val[p] * x[col[p]];
+            y[i] = x[i] + (s + diag[i] * x[i]) / lam;
+        }
+        double* tmp = x; x = y; y = tmp;
+    }
+    free(w);
+    if (terms_out) *terms_out = k + 1;
+    if (lambda_out) *lambda_out = lam;
+    free(x); free(y);
+    return ORACLE_OK;
+}
+
+/* ------------------------------------------------------------------------ */
+/* 8. Dense LU null-space solve for tiny state spaces (north star)            */
 /* ------------------------------------------------------------------------ */
 int oracle_lu_steady(int64_t n, const int64_t* rp, const int32_t* col, const double* val,
                      const double* diag, double* p_out) {

@@ -96,6 +96,14 @@ int oracle_jacobi_solve(int64_t n, const int64_t* row_ptr, const int32_t* col, c
                         int nthreads, double* p_out, int64_t* iters_out, double* delta_out,
                         double* resid_out);
 
+/* Transient landscape p(t) = exp(A t) p0 by uniformization (the paper's
+ * future work; R22): Lambda = max_i |a_ii|, P = I + A/Lambda,
+ * p(t) = sum_{k=0}^{K} Pois(k; Lambda t) P^k p0 with K the smallest k whose
+ * cumulative Poisson weight reaches 1 - eps.  p0 NULL = all mass on state 0. */
+int oracle_transient(int64_t n, const int64_t* row_ptr, const int32_t* col, const double* val,
+                     const double* diag, const double* p0, double t, double eps, double* p_out,
+                     int64_t* terms_out, double* lambda_out);
+
 /* Dense GEPP null-space solve of A p = 0, sum p = 1 (last row of A replaced by
  * ones, rhs e_n), n <= 4096. */
 int oracle_lu_steady(int64_t n, const int64_t* row_ptr, const int32_t* col, const double* val,
