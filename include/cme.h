@@ -139,6 +139,17 @@ cme_status cme_set_solver_opts(cme_matrix h, const cme_solver_opts* o);
 cme_status cme_jacobi_solve(cme_matrix h, const double* p0, double tol, int64_t max_iter,
                             double* p_out, int64_t* iters_out);
 
+/* Transient landscape p(t) = exp(A t) p0 (dP/dt = A P) by
+ * uniformization -- the paper's stated future work, on the same
+ * fused step (I + A/Lambda is a Jacobi step with per-row omega = |a_ii|/Lambda):
+ * Lambda = max_i |a_ii|, p(t) = sum_{k<=K} w_k (I + A/Lambda)^k p0 with the
+ * Poisson(Lambda t) weights of reading R22 (normalised on k <= ceil(mu +
+ * 10 sqrt(mu) + 40), right tail <= eps cut).  p0 (n doubles, used as given) or
+ * NULL = all mass on original state 0 (the enumeration's initial microstate).
+ * *terms_out = K + 1 fused steps.  Batch 1, SELL formats.  Synchronous. */
+cme_status cme_transient(cme_matrix h, const double* p0, double t, double eps, double* p_out,
+                         int64_t* terms_out);
+
 typedef struct cme_report {
     int32_t status;    /* cme_status of the last solve                                 */
     int64_t iters;     /* iterations done                                              */

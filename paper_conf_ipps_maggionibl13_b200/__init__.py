@@ -97,6 +97,7 @@ _SIGS = {
     "cme_set_solver_opts": [vp, _p(cme_solver_opts)],
     "cme_jacobi_solve": [vp, vp, C.c_double, C.c_int64, vp, i64p],
     "cme_get_report": [vp, _p(cme_report)],
+    "cme_transient": [vp, vp, C.c_double, C.c_double, vp, i64p],
     "cme_spmv": [vp, vp, vp],
     "cme_solver_load": [vp, vp],
     "cme_solver_run": [vp, C.c_int64],
@@ -230,6 +231,14 @@ def cme_jacobi_solve(h, n, p0, tol, max_iter, p_out):
     st = _lib.cme_jacobi_solve(h, pp, tol, max_iter, po, C.byref(it))
     _chk(st, "cme_jacobi_solve", ok=tuple(SOLVE_STATUS))
     return st, it.value
+
+
+def cme_transient(h, n, p0, t, eps, p_out):
+    pp, _k0 = _vec_ptr(p0, n)
+    po, _k1 = _vec_ptr(p_out, n, writable=True)
+    k = C.c_int64()
+    _chk(_lib.cme_transient(h, pp, t, eps, po, C.byref(k)), "cme_transient")
+    return k.value
 
 
 def cme_get_report(h):
@@ -425,6 +434,13 @@ class Matrix:
             y = np.empty(self.n * self.batch)
         cme_spmv(self.h, self.n * self.batch, x, y)
         return y
+
+    def transient(self, t, p0=None, eps=1e-14, p_out=None):
+        """p(t) = exp(A t) p0 by uniformization; returns (p, terms)."""
+        if p_out is None:
+            p_out = np.empty(self.n)
+        terms = cme_transient(self.h, self.n, p0, t, eps, p_out)
+        return p_out, terms
 
     def batch_report(self):
         return cme_get_batch_report(self.h, self.batch)

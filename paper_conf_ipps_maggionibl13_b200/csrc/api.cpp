@@ -23,6 +23,8 @@ cme_status device_spmv(cme_matrix_s* h, const double* x, double* y);
 cme_status device_load(cme_matrix_s* h, const double* p0);
 cme_status device_run(cme_matrix_s* h, int64_t blocks);
 cme_status device_fetch(cme_matrix_s* h, double* p_out);
+cme_status device_transient(cme_matrix_s* h, const double* p0, double t, double eps, double* p_out,
+                            int64_t* terms_out);
 void device_describe(const Device* d, cme_info* f);
 
 namespace {
@@ -279,6 +281,15 @@ cme_status cme_jacobi_solve(cme_matrix h, const double* p0, double tol, int64_t 
     if (!h || !p_out || max_iter < 0 || std::isnan(tol)) return CME_ERR_INVALID_ARG;
     if (h->stage < 2 || !h->dev) { set_error("solve before pack/distribute"); return CME_ERR_BAD_STATE; }
     return guarded([&] { return device_solve(h, p0, tol, max_iter, p_out, iters_out); });
+}
+
+cme_status cme_transient(cme_matrix h, const double* p0, double t, double eps, double* p_out,
+                         int64_t* terms_out) {
+    if (terms_out) *terms_out = 0;
+    if (!h || !p_out || !(t >= 0.0) || std::isinf(t) || !(eps > 0.0 && eps < 1.0)) return CME_ERR_INVALID_ARG;
+    if (h->stage < 2 || !h->dev) { set_error("transient before pack/distribute"); return CME_ERR_BAD_STATE; }
+    if (h->format == CME_FMT_CSR) { set_error("transient runs on the SELL formats"); return CME_ERR_INVALID_ARG; }
+    return guarded([&] { return device_transient(h, p0, t, eps, p_out, terms_out); });
 }
 
 cme_status cme_get_report(cme_matrix h, cme_report* r) {

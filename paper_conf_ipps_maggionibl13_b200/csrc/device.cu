@@ -68,6 +68,8 @@ struct Device {
     double* io = nullptr;            // n_global * B staging
     double* io2 = nullptr;           // second staging (distributed output)
     double* one = nullptr;           // constant 1.0 x kMaxBatch
+    double* acc_base = nullptr;      // transient accumulator allocation (lazily)
+    double* accb = nullptr;          //   its x-span base (one sentinel row in front)
     Ctrl* ctrl = nullptr;
     Ctrl* ctrl_host = nullptr;       // pinned, 2 slots
     int64_t n_global = 0, n_own = 0, nx = 0, own_off = 0, row_begin = 0;
@@ -478,8 +480,11 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
 // launches
 // ------------------------------------------------------------------------------
 static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool check, const double* pre,
-                              double omega) {
+                              double omega, double unif_lam_inv = 0.0, double acc_w = 0.0) {
     StepArgs a{};
+    a.unif_lam_inv = unif_lam_inv;
+    a.acc = unif_lam_inv != 0.0 ? d.accb : nullptr;
+    a.acc_w = acc_w;
     a.n_rows = d.n_own;
     a.slice_begin = 0;
     a.slice_end = d.n_slices;
@@ -745,6 +750,74 @@ cme_status device_solve(cme_matrix_s* h, const double* p0, double tol, int64_t m
     if (iters_out) *iters_out = f.iter;
     CME_TRY(write_out(h, p_out, d.ctrl->inv_s, s));
     return (cme_status)overall;
+}
+
+// Transient landscape p(t) = exp(A t) p0 by uniformization (R22):
+// step k adds w_k x_k to the accumulator and forms x_{k+1} = (I + A/Lambda) x_k
+// in the same fused kernel.  Weights: Poisson(mu = Lambda t) on k <= Kmax =
+// ceil(mu + 10 sqrt(mu) + 40), normalised to sum 1, right-truncated at the
+// first K whose tail mass is <= eps.
+cme_status device_transient(cme_matrix_s* h, const double* p0, double t, double eps, double* p_out,
+                            int64_t* terms_out) {
+    Device& d = *h->dev;
+    if (d.B != 1) { set_error("transient solves take one rate set (batch 1)"); return CME_ERR_INVALID_ARG; }
+    CUDA_TRY(cudaSetDevice(d.dev));
+    cudaStream_t s = stream_of(h);
+    double lam = 0.0;
+    for (double v : h->A.d) lam = std::max(lam, -v);
+    const double mu = lam * t;
+    const int64_t kmax = (int64_t)std::ceil(mu + 10.0 * std::sqrt(mu) + 40.0);
+    std::vector<double> w(kmax + 1);
+    double lmax = -INFINITY;
+    for (int64_t k = 0; k <= kmax; ++k) {
+        w[k] = mu > 0.0 ? (double)k * std::log(mu) - std::lgamma((double)k + 1.0) : (k == 0 ? 0.0 : -INFINITY);
+        lmax = std::max(lmax, w[k]);
+    }
+    double W = 0.0;
+    for (double& v : w) { v = std::exp(v - lmax); W += v; }
+    for (double& v : w) v /= W;
+    int64_t K = kmax;
+    double tail = 0.0;
+    while (K > 0 && tail + w[K] <= eps) { tail += w[K]; --K; }
+    if (!d.acc_base) {
+        CME_TRY(d.alloc(d.acc_base, (size_t)(d.nx + 2)));
+        d.accb = d.acc_base + 1;
+    }
+    CUDA_TRY(cudaMemsetAsync(d.acc_base, 0, (size_t)(d.nx + 2) * sizeof(double), s));
+    if (p0) {
+        CME_TRY(load_iterate(h, p0, false, s));
+    } else {  // all mass on the initial microstate (original state 0)
+        std::vector<double> e0(d.n_global, 0.0);
+        e0[0] = 1.0;
+        CME_TRY(load_iterate(h, e0.data(), false, s));
+    }
+    for (int64_t k = 0; k <= K; ++k)
+        CME_TRY(launch_step(d, s, (int)(k & 1), (int)((k + 1) & 1), false, nullptr, 1.0, 1.0 / lam, w[k]));
+    // p(t) = accumulator (own rows), original order
+    const double* xacc = d.accb + d.own_off;
+    const bool dev_out = is_device_ptr(p_out);
+    double* dst = dev_out ? p_out : d.io;
+    if (!d.comm) {
+        scatter_out_kernel<<<grid_for(d.n_own), kCta, 0, s>>>(xacc, d.perm_own, d.n_own, 1, d.n_global, d.one, dst);
+        CUDA_TRY(cudaGetLastError());
+    } else {
+        scale_copy_kernel<<<grid_for(d.n_own), kCta, 0, s>>>(xacc, d.n_own, 1, d.one, d.io + d.row_begin);
+        CUDA_TRY(cudaGetLastError());
+        CME_TRY(comm_bcast_segments(d.comm, d.io, d.cuts, s));
+        dst = dev_out ? p_out : d.io2;
+        scatter_out_kernel<<<grid_for(d.n_global), kCta, 0, s>>>(d.io, d.perm_global, d.n_global, 1, d.n_global,
+                                                                 d.one, dst);
+        CUDA_TRY(cudaGetLastError());
+    }
+    if (!dev_out) CUDA_TRY(cudaMemcpyAsync(p_out, dst, (size_t)d.n_global * sizeof(double), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    d.cur = (int)((K + 1) & 1);
+    if (terms_out) *terms_out = K + 1;
+    h->report = cme_report{};
+    h->report.status = CME_OK;
+    h->report.iters = K + 1;
+    h->report.omega = lam;   // the uniformization rate
+    return CME_OK;
 }
 
 void device_describe(const Device* d, cme_info* f) {

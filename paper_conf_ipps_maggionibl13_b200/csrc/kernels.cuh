@@ -66,6 +66,11 @@ struct StepArgs {
     const int64_t* csr_rp;
     const int32_t* csr_ci;
     const double* csr_v;
+    // transient mode (uniformization, R22): y = x + (A x)/Lambda and
+    // acc += acc_w * x; unif_lam_inv = 0 selects the Jacobi step
+    double unif_lam_inv;
+    double* acc;           // x-span base of the accumulator (nullable)
+    double acc_w;
 };
 
 __device__ __forceinline__ uint64_t evict_first_policy() {
@@ -182,10 +187,16 @@ __device__ __forceinline__ void finish_row(const StepArgs& a, int64_t r, const d
     const bool damp = a.omega != 1.0;
     ld_vec<B>(xo + r * B, xr);
     double yv[B];
+    const bool unif = a.unif_lam_inv != 0.0;
 #pragma unroll
     for (int b = 0; b < B; ++b) {
         const double s = BAND ? fma(lo[b], xl[b], up[b] * xu[b]) + acc[b] : acc[b];
         double y = damp ? fma(1.0 - a.omega, xr[b], a.omega * (id[b] * s)) : id[b] * s;
+        if (unif) {   // transient: (I + A/Lambda) x with a_rr = -1/id
+            y = fma(a.unif_lam_inv, s - xr[b] / id[b], xr[b]);
+            double* ac = a.acc + (a.own_off + r) * B + b;
+            *ac = fma(a.acc_w, xr[b], *ac);
+        }
         double x = (damp || CHECK) ? xr[b] : 0.0;
         if (pre_scale != nullptr) {
             const double sc = pre_scale[b];
