@@ -17,7 +17,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libcme.so")
+# CME_LIBRARY: load another build of libcme.so (kernel A/B experiments in tools/)
+LIB_PATH = os.environ.get("CME_LIBRARY") or os.path.join(_HERE, "libcme.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} is not built; run `python paper_conf_ipps_maggionibl13_b200/build.py` "

@@ -117,6 +117,8 @@ struct Device {
 // over nblocks partial records, in a fixed order (deterministic).  1 CTA x 1024.
 __global__ void __launch_bounds__(1024) reduce_partials_kernel(const double* partials, int nblocks, int B,
                                                                double* out, const int32_t* stop) {
+    pdl_trigger();
+    pdl_wait();
     if (stop != nullptr && *stop) return;
     __shared__ double s[32][5];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -144,6 +146,8 @@ __global__ void __launch_bounds__(1024) reduce_partials_kernel(const double* par
 // Check decision (readings R2-R5), per member.
 // all holds one [B][8] record per rank, combined in rank order.
 __global__ void decide_kernel(const double* all, int nranks, Ctrl* c, int32_t len, int32_t final_partial) {
+    pdl_trigger();
+    pdl_wait();
     if (c->stop) return;
     const int B = c->batch;
     const int64_t k = c->iter + len;
@@ -506,28 +510,30 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
     a.csr_rp = d.csr_rp;
     a.csr_ci = d.csr_ci;
     a.csr_v = d.csr_v;
+    // programmatic dependent launch between consecutive steps (not across the
+    // NCCL calls of a distributed solve, which are ordinary stream work)
+    const bool pdl = !d.comm && env_int("CME_PDL", 1) != 0;
     if (d.format == CME_FMT_CSR) {
-        if (check) csr_step_kernel<true><<<d.grid, kCta, 0, s>>>(a);
-        else csr_step_kernel<false><<<d.grid, kCta, 0, s>>>(a);
-        CUDA_TRY(cudaGetLastError());
+        CUDA_TRY(check ? launch_ex(csr_step_kernel<true>, dim3(d.grid), dim3(kCta), 0, pdl, s, a)
+                       : launch_ex(csr_step_kernel<false>, dim3(d.grid), dim3(kCta), 0, pdl, s, a));
     } else if (d.use_tma) {
         TmaArgs T{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col};
         const int smem = d.tma_stages * d.tma_stage_bytes;
         cudaError_t e;
         switch (d.B) {
-            case 1: e = launch_tma<1>(T, d.tma_ncw, d.tma_grid, smem, d.band, d.rearr, check, s); break;
-            case 2: e = launch_tma<2>(T, d.tma_ncw, d.tma_grid, smem, d.band, d.rearr, check, s); break;
-            case 4: e = launch_tma<4>(T, d.tma_ncw, d.tma_grid, smem, d.band, d.rearr, check, s); break;
-            default: e = launch_tma<8>(T, d.tma_ncw, d.tma_grid, smem, d.band, d.rearr, check, s); break;
+            case 1: e = launch_tma<1>(T, d.tma_ncw, d.tma_grid, smem, d.band, d.rearr, check, pdl, s); break;
+            case 2: e = launch_tma<2>(T, d.tma_ncw, d.tma_grid, smem, d.band, d.rearr, check, pdl, s); break;
+            case 4: e = launch_tma<4>(T, d.tma_ncw, d.tma_grid, smem, d.band, d.rearr, check, pdl, s); break;
+            default: e = launch_tma<8>(T, d.tma_ncw, d.tma_grid, smem, d.band, d.rearr, check, pdl, s); break;
         }
         CUDA_TRY(e);
     } else {
         cudaError_t e;
         switch (d.B) {
-            case 1: e = launch_sell<1>(a, d.grid, d.band, d.rearr, check, s); break;
-            case 2: e = launch_sell<2>(a, d.grid, d.band, d.rearr, check, s); break;
-            case 4: e = launch_sell<4>(a, d.grid, d.band, d.rearr, check, s); break;
-            default: e = launch_sell<8>(a, d.grid, d.band, d.rearr, check, s); break;
+            case 1: e = launch_sell<1>(a, d.grid, d.band, d.rearr, check, pdl, s); break;
+            case 2: e = launch_sell<2>(a, d.grid, d.band, d.rearr, check, pdl, s); break;
+            case 4: e = launch_sell<4>(a, d.grid, d.band, d.rearr, check, pdl, s); break;
+            default: e = launch_sell<8>(a, d.grid, d.band, d.rearr, check, pdl, s); break;
         }
         CUDA_TRY(e);
     }
@@ -537,12 +543,12 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
 
 // reduce partials of the last CHECK step and decide
 static cme_status launch_finalize(Device& d, cudaStream_t s, int32_t len, int32_t final_partial) {
-    reduce_partials_kernel<<<1, 1024, 0, s>>>(d.partials, d.step_grid(), d.B, d.comm ? d.local8 : d.gather,
-                                              &d.ctrl->stop);
-    CUDA_TRY(cudaGetLastError());
+    const bool pdl = !d.comm && env_int("CME_PDL", 1) != 0;
+    CUDA_TRY(launch_ex(reduce_partials_kernel, dim3(1), dim3(1024), 0, pdl, s, (const double*)d.partials,
+                       d.step_grid(), d.B, d.comm ? d.local8 : d.gather, (const int32_t*)&d.ctrl->stop));
     if (d.comm) CME_TRY(comm_allgather(d.comm, d.local8, d.gather, (size_t)8 * d.B, s));
-    decide_kernel<<<1, 1, 0, s>>>(d.gather, d.nranks, d.ctrl, len, final_partial);
-    CUDA_TRY(cudaGetLastError());
+    CUDA_TRY(launch_ex(decide_kernel, dim3(1), dim3(1), 0, pdl, s, (const double*)d.gather, d.nranks, d.ctrl, len,
+                       final_partial));
     return CME_OK;
 }
 

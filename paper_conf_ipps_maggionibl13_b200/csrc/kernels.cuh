@@ -73,6 +73,14 @@ struct StepArgs {
     double acc_w;
 };
 
+// Programmatic dependent launch (the step kernels and the check kernels are
+// launched with cudaLaunchAttributeProgrammaticStreamSerialization): let the
+// next grid in the stream be scheduled early, and wait for the previous grid's
+// results before touching anything it wrote (x, ctrl).  Both are no-ops for a
+// normal launch.
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 __device__ __forceinline__ uint64_t evict_first_policy() {
     uint64_t p;
     asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
@@ -226,8 +234,30 @@ struct Chunk {
     static constexpr int U = B >= 8 ? 1 : 8 / B;
 };
 
+// Sum over the W ELL entries of one slot: all stream loads, then all gathers,
+// then the FMAs in t order (W known at compile time: no predicated-off slots).
+template <int B, int W>
+__device__ __forceinline__ void ell_row_global(const StepArgs& a, int64_t base, uint64_t pol, double (&acc)[B]) {
+    double v[W][B], xv[W][B];
+    int32_t c[W];
+#pragma unroll
+    for (int u = 0; u < W; ++u) {
+        const int64_t e = base + 32 * (int64_t)u;
+        ld_stream_vec<B>(a.val + e * B, pol, v[u]);
+        c[u] = ld_stream(a.col + e, pol);
+    }
+#pragma unroll
+    for (int u = 0; u < W; ++u) ld_vec<B>(a.x + (int64_t)c[u] * B, xv[u]);
+#pragma unroll
+    for (int u = 0; u < W; ++u)
+#pragma unroll
+        for (int b = 0; b < B; ++b) acc[b] = fma(v[u][b], xv[u][b], acc[b]);
+}
+
 template <int B, bool BAND, bool REARR, bool CHECK>
 __global__ void __launch_bounds__(kCta) sell_step_kernel(const StepArgs a) {
+    pdl_trigger();
+    pdl_wait();
     if (a.stop != nullptr && *a.stop) return;
     const uint64_t pol = evict_first_policy();
     const int lane = threadIdx.x & 31;
@@ -239,28 +269,40 @@ __global__ void __launch_bounds__(kCta) sell_step_kernel(const StepArgs a) {
         const int64_t base = __ldg(a.slice_off + q) + lane;
         if (slot < a.n_rows) {
             const int64_t r = REARR ? (int64_t)ld_stream(a.row_of + slot, pol) : slot;
-            constexpr int U = Chunk<B>::U;
             double acc[B];
 #pragma unroll
             for (int b = 0; b < B; ++b) acc[b] = 0.0;
-            for (int t0 = 0; t0 < w; t0 += U) {
-                double v[U][B], xv[U][B];
-                int32_t c[U];
+            constexpr int U = Chunk<B>::U;
+            switch (B == 1 ? w : -1) {   // warp-uniform exact widths for the common B = 1 case
+                case 0: break;
+                case 1: ell_row_global<B, 1>(a, base, pol, acc); break;
+                case 2: ell_row_global<B, 2>(a, base, pol, acc); break;
+                case 3: ell_row_global<B, 3>(a, base, pol, acc); break;
+                case 4: ell_row_global<B, 4>(a, base, pol, acc); break;
+                case 5: ell_row_global<B, 5>(a, base, pol, acc); break;
+                case 6: ell_row_global<B, 6>(a, base, pol, acc); break;
+                case 7: ell_row_global<B, 7>(a, base, pol, acc); break;
+                case 8: ell_row_global<B, 8>(a, base, pol, acc); break;
+                default:
+                    for (int t0 = 0; t0 < w; t0 += U) {
+                        double v[U][B], xv[U][B];
+                        int32_t c[U];
 #pragma unroll
-                for (int u = 0; u < U; ++u)
-                    if (t0 + u < w) {
-                        const int64_t e = base + 32 * (int64_t)(t0 + u);
-                        ld_stream_vec<B>(a.val + e * B, pol, v[u]);
-                        c[u] = ld_stream(a.col + e, pol);
+                        for (int u = 0; u < U; ++u)
+                            if (t0 + u < w) {
+                                const int64_t e = base + 32 * (int64_t)(t0 + u);
+                                ld_stream_vec<B>(a.val + e * B, pol, v[u]);
+                                c[u] = ld_stream(a.col + e, pol);
+                            }
+#pragma unroll
+                        for (int u = 0; u < U; ++u)
+                            if (t0 + u < w) ld_vec<B>(a.x + (int64_t)c[u] * B, xv[u]);
+#pragma unroll
+                        for (int u = 0; u < U; ++u)
+                            if (t0 + u < w)
+#pragma unroll
+                                for (int b = 0; b < B; ++b) acc[b] = fma(v[u][b], xv[u][b], acc[b]);
                     }
-#pragma unroll
-                for (int u = 0; u < U; ++u)
-                    if (t0 + u < w) ld_vec<B>(a.x + (int64_t)c[u] * B, xv[u]);
-#pragma unroll
-                for (int u = 0; u < U; ++u)
-                    if (t0 + u < w)
-#pragma unroll
-                        for (int b = 0; b < B; ++b) acc[b] = fma(v[u][b], xv[u][b], acc[b]);
             }
             double lo[B], up[B], id[B];
             if (BAND) {
@@ -278,6 +320,8 @@ __global__ void __launch_bounds__(kCta) sell_step_kernel(const StepArgs a) {
 // Plain CSR arm (ablation, CME_FMT_CSR, B = 1): one thread per row.
 template <bool CHECK>
 __global__ void __launch_bounds__(kCta) csr_step_kernel(const StepArgs a) {
+    pdl_trigger();
+    pdl_wait();
     if (a.stop != nullptr && *a.stop) return;
     const int64_t r = a.slice_begin * 32 + (int64_t)blockIdx.x * kCta + threadIdx.x;
     CheckAcc<1> ck;

@@ -75,6 +75,83 @@ __host__ __device__ inline int tma_fixed_bytes(int ncw, int B, bool band, bool r
     return ncw * 32 * (8 * B + (rearr ? 4 : 0) + (band ? 16 * B : 0));
 }
 
+// Sum over the W ELL entries of one slot from shared memory: all x gathers
+// first, then the FMAs in t order (W known at compile time).
+template <int B, int W>
+__device__ __forceinline__ void ell_row_smem(const int32_t* scol, const double* sval, const double* x,
+                                             double (&acc)[B]) {
+    double xv[W][B];
+#pragma unroll
+    for (int u = 0; u < W; ++u) ld_vec<B>(x + (int64_t)scol[32 * u] * B, xv[u]);
+#pragma unroll
+    for (int u = 0; u < W; ++u)
+#pragma unroll
+        for (int b = 0; b < B; ++b) acc[b] = fma(sval[32 * u * B + b], xv[u][b], acc[b]);
+}
+
+// Producer: one tile -> one stage (inv_d, row_of, lo/up, val, col blocks, all
+// contiguous in HBM), completion counted on `bar`.  Scalar arguments only, so
+// the call neither copies the kernel parameters to local memory nor carries
+// the producer's addressing into the consumers' register allocation.
+#ifndef CME_TMA_PRODUCER_INLINE
+#define CME_TMA_PRODUCER_INLINE 0
+#endif
+template <int NCW, int B, bool BAND, bool REARR>
+__device__ __forceinline__ void tma_issue_body(unsigned char* st, uint64_t* bar, const int64_t* slice_off,
+                                               int64_t slice_end, const double* inv_d, const int32_t* row_of,
+                                               const double* lo, const double* up, const double* val,
+                                               const int32_t* col, int off_val, int off_col, int64_t tile,
+                                               uint64_t pol) {
+    constexpr int kSlots = NCW * 32;
+    constexpr int kOffInvd = 0, kOffRow = 8 * B * kSlots, kOffLo = kOffRow + (REARR ? 4 * kSlots : 0),
+                  kOffUp = kOffLo + 8 * B * kSlots;
+    const int64_t q0 = tile * NCW;
+    const int64_t q1 = min(q0 + NCW, slice_end);
+    const int64_t e0 = slice_off[q0], e1 = slice_off[q1];
+    const uint32_t slots = (uint32_t)(q1 - q0) * 32u;
+    const uint32_t nval = (uint32_t)(e1 - e0);
+    uint32_t bytes = nval * (8u * B + 4u) + slots * 8u * B;
+    if (REARR) bytes += slots * 4u;
+    if (BAND) bytes += slots * 16u * B;
+    mbar_expect_tx(bar, bytes);
+    bulk_g2s(st + kOffInvd, inv_d + q0 * 32 * B, slots * 8u * B, bar, pol);
+    if (REARR) bulk_g2s(st + kOffRow, row_of + q0 * 32, slots * 4u, bar, pol);
+    if (BAND) {
+        bulk_g2s(st + kOffLo, lo + q0 * 32 * B, slots * 8u * B, bar, pol);
+        bulk_g2s(st + kOffUp, up + q0 * 32 * B, slots * 8u * B, bar, pol);
+    }
+    if (nval) {
+        bulk_g2s(st + off_val, val + e0 * B, nval * 8u * B, bar, pol);
+        bulk_g2s(st + off_col, col + e0, nval * 4u, bar, pol);
+    }
+}
+template <int NCW, int B, bool BAND, bool REARR>
+__device__ __noinline__ void tma_issue_call(unsigned char* st, uint64_t* bar, const int64_t* slice_off,
+                                            int64_t slice_end, const double* inv_d, const int32_t* row_of,
+                                            const double* lo, const double* up, const double* val,
+                                            const int32_t* col, int off_val, int off_col, int64_t tile,
+                                            uint64_t pol) {
+    tma_issue_body<NCW, B, BAND, REARR>(st, bar, slice_off, slice_end, inv_d, row_of, lo, up, val, col, off_val,
+                                        off_col, tile, pol);
+}
+template <int NCW, int B, bool BAND, bool REARR>
+__device__ __forceinline__ void tma_issue(const TmaArgs& T, unsigned char* smem, uint64_t* full, int64_t tile, int s,
+                                          uint64_t pol) {
+    const StepArgs& a = T.a;
+    unsigned char* st = smem + (size_t)s * T.stage_bytes;
+    if (CME_TMA_PRODUCER_INLINE)
+        tma_issue_body<NCW, B, BAND, REARR>(st, &full[s], a.slice_off, a.slice_end, a.inv_d, a.row_of, a.lo, a.up,
+                                            a.val, a.col, T.off_val, T.off_col, tile, pol);
+    else
+        tma_issue_call<NCW, B, BAND, REARR>(st, &full[s], a.slice_off, a.slice_end, a.inv_d, a.row_of, a.lo, a.up,
+                                            a.val, a.col, T.off_val, T.off_col, tile, pol);
+}
+
+#ifndef CME_TMA_EXACT_WIDTHS
+#define CME_TMA_EXACT_WIDTHS 1
+#endif
+constexpr bool kExactWidths = CME_TMA_EXACT_WIDTHS;
+
 template <int NCW, int B, bool BAND, bool REARR, bool CHECK>
 __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBlocks)
     sell_tma_kernel(const TmaArgs T) {
@@ -82,7 +159,7 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
     constexpr int kOffInvd = 0, kOffRow = 8 * B * kSlots, kOffLo = kOffRow + (REARR ? 4 * kSlots : 0),
                   kOffUp = kOffLo + 8 * B * kSlots;
     const StepArgs& a = T.a;
-    if (a.stop != nullptr && *a.stop) return;
+    pdl_trigger();
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ uint64_t full[8], empty[8];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -95,40 +172,36 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
+    const bool producer = warp == kConsumers && lane == 0;
+    uint64_t pol = 0;
+    // Prologue: the packed matrix is constant across steps, so the first S
+    // tiles stream in while the previous step (programmatic dependency) drains.
+    const int64_t my_tiles = (int64_t)blockIdx.x < T.n_tiles ? (T.n_tiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    const int pro = (int)(my_tiles < (int64_t)S ? my_tiles : (int64_t)S);
+    if (producer) {
+        pol = evict_first_policy();
+        for (int i = 0; i < pro; ++i)
+            tma_issue<NCW, B, BAND, REARR>(T, smem, full, (int64_t)blockIdx.x + (int64_t)i * gridDim.x, i, pol);
+    }
+    pdl_wait();   // x / ctrl of the previous step are final from here on
+    if (a.stop != nullptr && *a.stop) {
+        // a decided solve: drain the prologue copies before the CTA exits
+        if (producer)
+            for (int i = 0; i < pro; ++i) mbar_wait(&full[i], 0u);
+        return;
+    }
     CheckAcc<B> ck;
 
     if (warp == kConsumers) {
         // ---------------- producer ----------------
-        if (lane == 0) {
-            const uint64_t pol = evict_first_policy();
+        if (lane == 0 && my_tiles > pro) {
             // stage s and the parity of its current use, advanced incrementally
-            // (no 64-bit division per tile)
             int s = 0;
-            uint32_t phase = 0;
-            bool wrapped = false;
-            for (int64_t tile = blockIdx.x; tile < T.n_tiles; tile += gridDim.x) {
-                if (wrapped) mbar_wait(&empty[s], phase ^ 1u);   // consumers released the previous use
-                unsigned char* st = smem + (size_t)s * T.stage_bytes;
-                const int64_t q0 = tile * kTileSlices;
-                const int64_t q1 = min(q0 + kTileSlices, a.slice_end);
-                const int64_t e0 = a.slice_off[q0], e1 = a.slice_off[q1];
-                const uint32_t slots = (uint32_t)(q1 - q0) * 32u;
-                const uint32_t nval = (uint32_t)(e1 - e0);
-                uint32_t bytes = nval * (8u * B + 4u) + slots * 8u * B;
-                if (REARR) bytes += slots * 4u;
-                if (BAND) bytes += slots * 16u * B;
-                mbar_expect_tx(&full[s], bytes);
-                bulk_g2s(st + kOffInvd, a.inv_d + q0 * 32 * B, slots * 8u * B, &full[s], pol);
-                if (REARR) bulk_g2s(st + kOffRow, a.row_of + q0 * 32, slots * 4u, &full[s], pol);
-                if (BAND) {
-                    bulk_g2s(st + kOffLo, a.lo + q0 * 32 * B, slots * 8u * B, &full[s], pol);
-                    bulk_g2s(st + kOffUp, a.up + q0 * 32 * B, slots * 8u * B, &full[s], pol);
-                }
-                if (nval) {
-                    bulk_g2s(st + T.off_val, a.val + e0 * B, nval * 8u * B, &full[s], pol);
-                    bulk_g2s(st + T.off_col, a.col + e0, nval * 4u, &full[s], pol);
-                }
-                if (++s == S) { s = 0; phase ^= 1u; wrapped = true; }
+            uint32_t phase = 1;   // pro == S here: every stage holds its first use
+            for (int64_t tile = (int64_t)blockIdx.x + (int64_t)pro * gridDim.x; tile < T.n_tiles; tile += gridDim.x) {
+                mbar_wait(&empty[s], phase ^ 1u);   // consumers released the previous use
+                tma_issue<NCW, B, BAND, REARR>(T, smem, full, tile, s, pol);
+                if (++s == S) { s = 0; phase ^= 1u; }
             }
         }
     } else {
@@ -155,20 +228,34 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
                 const double* sval = reinterpret_cast<const double*>(st + T.off_val) + (loff + lane) * B;
                 const int32_t* scol = reinterpret_cast<const int32_t*>(st + T.off_col) + loff + lane;
                 const int64_t r = REARR ? (int64_t) reinterpret_cast<const int32_t*>(st + kOffRow)[ls] : slot;
-                constexpr int U = Chunk<B>::U;
                 double acc[B];
 #pragma unroll
                 for (int b = 0; b < B; ++b) acc[b] = 0.0;
-                for (int t0 = 0; t0 < w; t0 += U) {
-                    double xv[U][B];   // all gathers of the chunk in flight, then FMAs
+                switch (kExactWidths && B <= 2 ? w : -1) {   // warp-uniform exact widths
+                    case 0: break;
+                    case 1: ell_row_smem<B, 1>(scol, sval, a.x, acc); break;
+                    case 2: ell_row_smem<B, 2>(scol, sval, a.x, acc); break;
+                    case 3: ell_row_smem<B, 3>(scol, sval, a.x, acc); break;
+                    case 4: ell_row_smem<B, 4>(scol, sval, a.x, acc); break;
+                    case 5: ell_row_smem<B, 5>(scol, sval, a.x, acc); break;
+                    case 6: ell_row_smem<B, 6>(scol, sval, a.x, acc); break;
+                    case 7: ell_row_smem<B, 7>(scol, sval, a.x, acc); break;
+                    case 8: ell_row_smem<B, 8>(scol, sval, a.x, acc); break;
+                    default: {
+                        constexpr int U = Chunk<B>::U;
+                        for (int t0 = 0; t0 < w; t0 += U) {
+                            double xv[U][B];   // all gathers of the chunk in flight, then FMAs
 #pragma unroll
-                    for (int u = 0; u < U; ++u)
-                        if (t0 + u < w) ld_vec<B>(a.x + (int64_t)scol[32 * (t0 + u)] * B, xv[u]);
+                            for (int u = 0; u < U; ++u)
+                                if (t0 + u < w) ld_vec<B>(a.x + (int64_t)scol[32 * (t0 + u)] * B, xv[u]);
 #pragma unroll
-                    for (int u = 0; u < U; ++u)
-                        if (t0 + u < w)
+                            for (int u = 0; u < U; ++u)
+                                if (t0 + u < w)
 #pragma unroll
-                            for (int b = 0; b < B; ++b) acc[b] = fma(sval[32 * (t0 + u) * B + b], xv[u][b], acc[b]);
+                                    for (int b = 0; b < B; ++b)
+                                        acc[b] = fma(sval[32 * (t0 + u) * B + b], xv[u][b], acc[b]);
+                        }
+                    }
                 }
                 double lo[B], up[B], id[B];
 #pragma unroll

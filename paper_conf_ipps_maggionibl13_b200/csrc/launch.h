@@ -2,16 +2,36 @@
 // step_b{1,2,4,8}.cu (so nvcc compiles them in parallel).
 #pragma once
 #include <cuda_runtime.h>
+#include <utility>
 
 #include "kernels_tma.cuh"
 
 namespace cme {
 
+// pdl: launch with programmatic stream serialization (the kernel may start
+// while the previous kernel in the stream drains; it waits in-kernel).
 template <int B>
-cudaError_t launch_sell(const StepArgs& a, int grid, bool band, bool rearr, bool check, cudaStream_t s);
+cudaError_t launch_sell(const StepArgs& a, int grid, bool band, bool rearr, bool check, bool pdl, cudaStream_t s);
 template <int B>
-cudaError_t launch_tma(const TmaArgs& T, int ncw, int grid, int smem, bool band, bool rearr, bool check,
+cudaError_t launch_tma(const TmaArgs& T, int ncw, int grid, int smem, bool band, bool rearr, bool check, bool pdl,
                        cudaStream_t s);
+
+// cudaLaunchKernelEx with an optional programmatic-dependency attribute
+template <typename... KArgs, typename... Args>
+cudaError_t launch_ex(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, bool pdl, cudaStream_t s,
+                      Args&&... args) {
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = pdl ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
 // cudaFuncSetAttribute(max dynamic smem) on every TMA variant of (B, ncw)
 template <int B>
 cudaError_t tma_prepare(int ncw, int smem);

@@ -5,37 +5,36 @@
 namespace cme {
 
 template <int B>
-cudaError_t launch_sell(const StepArgs& a, int grid, bool band, bool rearr, bool check, cudaStream_t s) {
+cudaError_t launch_sell(const StepArgs& a, int grid, bool band, bool rearr, bool check, bool pdl, cudaStream_t s) {
     const int key = (band ? 4 : 0) | (rearr ? 2 : 0) | (check ? 1 : 0);
     switch (key) {
 #define K(bd, r, c) \
-    case bd * 4 + r * 2 + c: sell_step_kernel<B, bd, r, c><<<grid, kCta, 0, s>>>(a); break;
+    case bd * 4 + r * 2 + c: return launch_ex(sell_step_kernel<B, bd, r, c>, dim3(grid), dim3(kCta), 0, pdl, s, a);
         K(0, 0, 0) K(0, 0, 1) K(0, 1, 0) K(0, 1, 1) K(1, 0, 0) K(1, 0, 1) K(1, 1, 0) K(1, 1, 1)
 #undef K
     }
-    return cudaGetLastError();
+    return cudaErrorInvalidValue;
 }
 
 template <int W, int B>
-static cudaError_t launch_tma_w(const TmaArgs& T, int grid, int smem, bool band, bool rearr, bool check,
+static cudaError_t launch_tma_w(const TmaArgs& T, int grid, int smem, bool band, bool rearr, bool check, bool pdl,
                                 cudaStream_t s) {
     const int key = (band ? 4 : 0) | (rearr ? 2 : 0) | (check ? 1 : 0);
     switch (key) {
-#define K(bd, r, c)                                                                                  \
-    case bd * 4 + r * 2 + c:                                                                         \
-        sell_tma_kernel<W, B, bd, r, c><<<grid, TmaShape<W>::kThreads, smem, s>>>(T);                \
-        break;
+#define K(bd, r, c)                                                                                          \
+    case bd * 4 + r * 2 + c:                                                                                 \
+        return launch_ex(sell_tma_kernel<W, B, bd, r, c>, dim3(grid), dim3(TmaShape<W>::kThreads), smem, pdl, s, T);
         K(0, 0, 0) K(0, 0, 1) K(0, 1, 0) K(0, 1, 1) K(1, 0, 0) K(1, 0, 1) K(1, 1, 0) K(1, 1, 1)
 #undef K
     }
-    return cudaGetLastError();
+    return cudaErrorInvalidValue;
 }
 
 template <int B>
-cudaError_t launch_tma(const TmaArgs& T, int ncw, int grid, int smem, bool band, bool rearr, bool check,
+cudaError_t launch_tma(const TmaArgs& T, int ncw, int grid, int smem, bool band, bool rearr, bool check, bool pdl,
                        cudaStream_t s) {
-    return ncw == 16 ? launch_tma_w<16, B>(T, grid, smem, band, rearr, check, s)
-                     : launch_tma_w<8, B>(T, grid, smem, band, rearr, check, s);
+    return ncw == 16 ? launch_tma_w<16, B>(T, grid, smem, band, rearr, check, pdl, s)
+                     : launch_tma_w<8, B>(T, grid, smem, band, rearr, check, pdl, s);
 }
 
 template <int W, int B>
@@ -65,8 +64,8 @@ cudaError_t tma_occupancy(int ncw, int smem, int* occ) {
 }
 
 #define CME_INSTANTIATE_LAUNCHERS(B)                                                                       \
-    template cudaError_t launch_sell<B>(const StepArgs&, int, bool, bool, bool, cudaStream_t);              \
-    template cudaError_t launch_tma<B>(const TmaArgs&, int, int, int, bool, bool, bool, cudaStream_t);      \
+    template cudaError_t launch_sell<B>(const StepArgs&, int, bool, bool, bool, bool, cudaStream_t);        \
+    template cudaError_t launch_tma<B>(const TmaArgs&, int, int, int, bool, bool, bool, bool, cudaStream_t); \
     template cudaError_t tma_prepare<B>(int, int);                                                          \
     template cudaError_t tma_occupancy<B>(int, int, int*);
 
