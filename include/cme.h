@@ -234,6 +234,16 @@ cme_status cme_period(cme_matrix h, int64_t root, int64_t* period_out);
  * with dlopen (the copy torch already loaded, else libnccl.so.2). */
 cme_status cme_comm_unique_id(uint8_t id[128]);
 cme_status cme_comm_init(int nranks, int rank, const uint8_t id[128], int device, cme_comm* out);
+/* Peer-memory transport (NEXT-4; no NCCL on the iteration path): an
+ * in-process group of nranks communicators on devices[r] (distinct GPUs with
+ * NVLink/NVSwitch peer access, or the same GPU repeated).  After
+ * cme_matrix_distribute every step kernel stores the halo rows its
+ * neighbours need straight into their iterate buffers (st.global to peer
+ * memory), and a one-thread flag kernel (st.release.sys / ld.acquire.sys,
+ * bounded spin) orders consecutive steps; check records and the output are
+ * exchanged the same way.  Each rank's handle must be driven by its own host
+ * thread; comms_out[nranks]; nranks <= 9. */
+cme_status cme_comm_init_local(int nranks, const int* devices, cme_comm* comms_out);
 /* Host-only partition plan for (nranks, rank): contiguous reordered rows cut
  * at window boundaries, balanced by packed bytes; local layout with columns
  * remapped to the local x span.  cme_matrix_distribute = plan + upload. */
@@ -251,6 +261,8 @@ typedef struct cme_halo_view {
 } cme_halo_view;
 cme_status cme_export_halo(cme_matrix h, cme_halo_view* v);
 
+/* For a handle distributed over a peer-memory (cme_comm_init_local) group,
+ * destroy is collective: it returns when every rank has called it. */
 void cme_matrix_destroy(cme_matrix h);
 void cme_comm_destroy(cme_comm c);
 

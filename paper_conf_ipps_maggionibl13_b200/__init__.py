@@ -109,6 +109,7 @@ _SIGS = {
     "cme_period": [vp, C.c_int64, i64p],
     "cme_comm_unique_id": [u8p],
     "cme_comm_init": [C.c_int, C.c_int, u8p, C.c_int, _p(vp)],
+    "cme_comm_init_local": [C.c_int, i32p, _p(vp)],
     "cme_matrix_plan_partition": [vp, C.c_int, C.c_int],
     "cme_matrix_distribute": [vp, vp],
     "cme_export_halo": [vp, _p(cme_halo_view)],
@@ -317,6 +318,14 @@ def cme_comm_init(nranks, rank, uid: bytes, device=-1):
     c = vp()
     _chk(_lib.cme_comm_init(nranks, rank, buf, device, C.byref(c)), "cme_comm_init")
     return c
+
+
+def cme_comm_init_local(devices):
+    """In-process peer-memory group: one communicator per entry of `devices`."""
+    devs = np.asarray(devices, dtype=np.int32)
+    out = (vp * len(devs))()
+    _chk(_lib.cme_comm_init_local(len(devs), devs.ctypes.data_as(i32p), out), "cme_comm_init_local")
+    return [vp(c) for c in out]
 
 
 def cme_matrix_plan_partition(h, nranks, rank):

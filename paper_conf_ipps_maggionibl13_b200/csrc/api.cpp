@@ -6,6 +6,8 @@
 #include <new>
 #include <string>
 
+#include <cuda_runtime.h>
+
 #include "cme_internal.h"
 #include "comm.h"
 
@@ -16,6 +18,7 @@ void set_error(const std::string& msg) { g_err = msg; }
 
 struct Device;
 cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cme_comm_s* comm);
+cme_status device_p2p_setup(cme_matrix_s* h);
 void device_free(Device* d);
 cme_status device_solve(cme_matrix_s* h, const double* p0, double tol, int64_t max_iter, double* p_out,
                         int64_t* iters_out);
@@ -435,6 +438,7 @@ cme_status cme_matrix_distribute(cme_matrix h, cme_comm c) {
         build_local(h, comm_nranks(c), comm_rank(c));
         cme_status s = device_upload(h, comm_device(c), &h->halo, c);
         if (s != CME_OK) return s;
+        if (comm_transport(c) == kTransportP2P && (s = device_p2p_setup(h)) != CME_OK) return s;
         h->comm = c;
         h->stage = 3;
         return CME_OK;
@@ -460,6 +464,12 @@ cme_status cme_export_halo(cme_matrix h, cme_halo_view* v) {
 
 void cme_matrix_destroy(cme_matrix h) {
     if (!h) return;
+    // peer-memory transport: peers may still address this rank's buffers
+    // until every rank of the group reaches its destroy (collective)
+    if (h->comm && comm_transport(h->comm) == kTransportP2P) {
+        cudaDeviceSynchronize();
+        comm_p2p_host_barrier(h->comm);
+    }
     device_free(h->dev);
     delete h;
 }

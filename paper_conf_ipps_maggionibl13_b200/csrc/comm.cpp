@@ -13,7 +13,10 @@
 #include <dlfcn.h>
 #include <cstdlib>
 #include <cstring>
+#include <condition_variable>
+#include <memory>
 #include <mutex>
+#include <vector>
 #include <string>
 
 #include <nccl.h>
@@ -69,9 +72,35 @@ cme_status load_nccl() {
 }  // namespace
 }  // namespace cme
 
+namespace cme {
+// In-process group of the peer-memory transport: ranks are host threads that
+// publish their buffers here; a generation barrier orders setup/teardown.
+struct LocalGroup {
+    int n = 0;
+    std::mutex mu;
+    std::condition_variable cv;
+    int count = 0;
+    uint64_t gen = 0;
+    std::vector<P2PRank> slots;
+    void barrier() {
+        std::unique_lock<std::mutex> lk(mu);
+        const uint64_t g = gen;
+        if (++count == n) {
+            count = 0;
+            ++gen;
+            cv.notify_all();
+        } else {
+            cv.wait(lk, [&] { return gen != g; });
+        }
+    }
+};
+}  // namespace cme
+
 struct cme_comm_s {
+    int transport = cme::kTransportNccl;
     ncclComm_t comm = nullptr;
     int nranks = 1, rank = 0, device = 0;
+    std::shared_ptr<cme::LocalGroup> group;   // P2P transport
 };
 
 namespace cme {
@@ -84,6 +113,27 @@ namespace cme {
             return CME_ERR_NCCL;                                                     \
         }                                                                            \
     } while (0)
+
+int comm_transport(const cme_comm_s* c) { return c->transport; }
+
+cme_status comm_p2p_exchange(cme_comm_s* c, const P2PRank& mine, std::vector<P2PRank>& all) {
+    if (c->transport != kTransportP2P || !c->group) return CME_ERR_INVALID_ARG;
+    {
+        std::lock_guard<std::mutex> lk(c->group->mu);
+        c->group->slots[c->rank] = mine;
+    }
+    c->group->barrier();
+    {
+        std::lock_guard<std::mutex> lk(c->group->mu);
+        all = c->group->slots;
+    }
+    c->group->barrier();   // nobody republishes before everyone has read
+    return CME_OK;
+}
+
+void comm_p2p_host_barrier(cme_comm_s* c) {
+    if (c->group) c->group->barrier();
+}
 
 int comm_rank(const cme_comm_s* c) { return c->rank; }
 int comm_nranks(const cme_comm_s* c) { return c->nranks; }
@@ -159,8 +209,51 @@ extern "C" cme_status cme_comm_init(int nranks, int rank, const uint8_t id[128],
     return CME_OK;
 }
 
+extern "C" cme_status cme_comm_init_local(int nranks, const int* devices, cme_comm* comms_out) {
+    if (nranks < 1 || nranks > cme::kMaxPeers + 1 || !devices || !comms_out) return CME_ERR_INVALID_ARG;
+    int count = 0;
+    if (cudaGetDeviceCount(&count) != cudaSuccess || count == 0) {
+        cudaGetLastError();
+        cme::set_error("no CUDA device visible");
+        return CME_ERR_NO_DEVICE;
+    }
+    for (int r = 0; r < nranks; ++r)
+        if (devices[r] < 0 || devices[r] >= count) return CME_ERR_INVALID_ARG;
+    // peer access between distinct devices (NVLink / NVSwitch); same device needs none
+    for (int a = 0; a < nranks; ++a)
+        for (int b = 0; b < nranks; ++b) {
+            if (devices[a] == devices[b]) continue;
+            int ok = 0;
+            cudaDeviceCanAccessPeer(&ok, devices[a], devices[b]);
+            if (!ok) {
+                cme::set_error("devices without peer access");
+                return CME_ERR_NCCL;
+            }
+            cudaSetDevice(devices[a]);
+            cudaError_t e = cudaDeviceEnablePeerAccess(devices[b], 0);
+            if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) {
+                cme::set_error(std::string("cudaDeviceEnablePeerAccess: ") + cudaGetErrorString(e));
+                return CME_ERR_CUDA;
+            }
+            cudaGetLastError();
+        }
+    auto group = std::make_shared<cme::LocalGroup>();
+    group->n = nranks;
+    group->slots.resize(nranks);
+    for (int r = 0; r < nranks; ++r) {
+        auto* c = new cme_comm_s();
+        c->transport = cme::kTransportP2P;
+        c->nranks = nranks;
+        c->rank = r;
+        c->device = devices[r];
+        c->group = group;
+        comms_out[r] = c;
+    }
+    return CME_OK;
+}
+
 extern "C" void cme_comm_destroy(cme_comm c) {
     if (!c) return;
-    if (c->comm) cme::g_api.CommDestroy(c->comm);
+    if (c->comm && cme::g_api.CommDestroy) cme::g_api.CommDestroy(c->comm);
     delete c;
 }

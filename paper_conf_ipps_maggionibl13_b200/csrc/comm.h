@@ -22,6 +22,27 @@ struct HaloPlan {
     }
 };
 
+enum { kTransportNccl = 0, kTransportP2P = 1 };
+constexpr int kMaxPeers = 8;
+
+// One rank's device buffers, published to the group by the peer-memory
+// transport: the two x-span iterate buffers, the sync flags, the check
+// gather array and the output staging vector (+ geometry to address them).
+struct P2PRank {
+    double* xb[2] = {nullptr, nullptr};
+    int64_t* flags = nullptr;   // [nranks] latest sync epoch signalled by each rank
+    double* gather = nullptr;   // [nranks][B][8]
+    double* io = nullptr;       // [n_global * B] reordered staging
+    int64_t span_lo = 0;        // first global row of the x-span
+    int device = 0;
+};
+
+int comm_transport(const cme_comm_s* c);
+// Publish `mine`, block until every rank of the group has, return all ranks'.
+cme_status comm_p2p_exchange(cme_comm_s* c, const P2PRank& mine, std::vector<P2PRank>& all);
+// Host-side barrier over the group (setup / teardown only).
+void comm_p2p_host_barrier(cme_comm_s* c);
+
 int comm_rank(const cme_comm_s* c);
 int comm_nranks(const cme_comm_s* c);
 int comm_device(const cme_comm_s* c);

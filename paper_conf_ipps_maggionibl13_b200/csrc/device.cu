@@ -79,6 +79,17 @@ struct Device {
     // distributed
     cme_comm_s* comm = nullptr;
     int nranks = 1, rank = 0;
+    bool p2p = false;                // peer-memory transport (no NCCL on the iteration path)
+    int64_t* flags = nullptr;        // [nranks] sync epochs signalled by each rank (written by peers)
+    int64_t* epoch = nullptr;        // [1] this rank's sync counter
+    int npeer = 0;                   // other ranks
+    int peer_rank[kMaxPushPeers] = {};
+    int64_t* peer_flags[kMaxPushPeers] = {};
+    double* peer_gather[kMaxPushPeers] = {};
+    double* peer_io[kMaxPushPeers] = {};
+    int npush = 0;                   // peers that need some of my rows
+    int64_t push_lo[kMaxPushPeers] = {}, push_hi[kMaxPushPeers] = {};   // local rows
+    double* push_y[2][kMaxPushPeers] = {};   // peer buffer (parity b) shifted to my local rows
     HaloPlan halo;                   // counts/offsets in doubles (rows x B)
     std::vector<int64_t> cuts;       // in doubles (rows x B) for the output broadcast
     // TMA-staged persistent kernel (kernels_tma.cuh)
@@ -255,6 +266,61 @@ __global__ void scatter_out_kernel(const double* x, const int32_t* perm, int64_t
 __global__ void scale_copy_kernel(const double* x, int64_t n, int B, const double* scale, double* out) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n * B; i += (int64_t)gridDim.x * blockDim.x)
         out[i] = x[i] * scale[i % B];
+}
+
+// Peer-memory barrier (NEXT-4): one thread bumps this rank's epoch, publishes
+// it into every peer's flag slot (release, system scope: the step's halo
+// stores into that peer are ordered before it) and waits (acquire) until every
+// peer has published the same epoch.  Bounded spin: a peer that never arrives
+// turns the solve into CME_ERR_NCCL instead of a hung GPU.
+struct BarrierArgs {
+    int64_t* flags;
+    int64_t* epoch;
+    int64_t* peer_flags[kMaxPushPeers];
+    int peer_rank[kMaxPushPeers];
+    int npeer, rank;
+    const int32_t* stop;   // nullable: skip when the solve has stopped (all ranks agree)
+    Ctrl* ctrl;
+};
+__global__ void p2p_barrier_kernel(const BarrierArgs a) {
+    if (threadIdx.x != 0) return;
+    if (a.stop != nullptr && *a.stop) return;
+    const int64_t e = *a.epoch + 1;
+    *a.epoch = e;
+    __threadfence_system();
+    for (int p = 0; p < a.npeer; ++p)
+        asm volatile("st.release.sys.global.s64 [%0], %1;" ::"l"(a.peer_flags[p] + a.rank), "l"(e) : "memory");
+    for (int p = 0; p < a.npeer; ++p) {
+        const int64_t* f = a.flags + a.peer_rank[p];
+        int64_t v = 0;
+        long long spins = 0;
+        for (;;) {
+            asm volatile("ld.acquire.sys.global.s64 %0, [%1];" : "=l"(v) : "l"(f) : "memory");
+            if (v >= e) break;
+            if (++spins > (1LL << 28)) {   // ~ tens of seconds: a peer is gone
+                a.ctrl->status = CME_ERR_NCCL;
+                a.ctrl->stop = 1;
+                return;
+            }
+            __nanosleep(64);
+        }
+    }
+}
+
+// dst[j][0..count) = src[0..count) for every destination (local and/or peer)
+struct CopyArgs {
+    const double* src;
+    double* dst[kMaxPushPeers + 1];
+    int ndst;
+    int64_t count;
+    const int32_t* stop;
+};
+__global__ void multicast_copy_kernel(const CopyArgs a) {
+    if (a.stop != nullptr && *a.stop) return;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.count; i += (int64_t)gridDim.x * blockDim.x) {
+        const double v = a.src[i];
+        for (int j = 0; j < a.ndst; ++j) a.dst[j][i] = v;
+    }
 }
 
 // ------------------------------------------------------------------------------
@@ -463,6 +529,14 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
     if ((s = d->alloc(d->io, (size_t)d->n_global * B)) != CME_OK) return fail(s);
     if (comm && (s = d->alloc(d->io2, (size_t)d->n_global * B)) != CME_OK) return fail(s);
     if ((s = d->alloc(d->one, kMaxBatch)) != CME_OK) return fail(s);
+    d->p2p = comm && comm_transport(comm) == kTransportP2P;
+    if (d->p2p) {
+        if ((s = d->alloc(d->flags, (size_t)d->nranks)) != CME_OK) return fail(s);
+        if ((s = d->alloc(d->epoch, 1)) != CME_OK) return fail(s);
+        if (cudaMemset(d->flags, 0, d->nranks * sizeof(int64_t)) != cudaSuccess ||
+            cudaMemset(d->epoch, 0, sizeof(int64_t)) != cudaSuccess)
+            return fail(CME_ERR_CUDA);
+    }
     if ((s = d->alloc(d->ctrl, 1)) != CME_OK) return fail(s);
     const double ones[kMaxBatch] = {1, 1, 1, 1, 1, 1, 1, 1};
     if (cudaMemcpy(d->one, ones, sizeof(ones), cudaMemcpyHostToDevice) != cudaSuccess) return fail(CME_ERR_CUDA);
@@ -480,6 +554,125 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
     return CME_OK;
 }
 
+
+// ------------------------------------------------------------------------------
+// exchanges of the row-sharded solve: NCCL (grouped send/recv, allgather,
+// broadcast) or the peer-memory transport (direct stores + flag barriers)
+// ------------------------------------------------------------------------------
+static cme_status p2p_barrier(Device& d, cudaStream_t s, bool respect_stop) {
+    BarrierArgs b{};
+    b.flags = d.flags;
+    b.epoch = d.epoch;
+    for (int p = 0; p < d.npeer; ++p) {
+        b.peer_flags[p] = d.peer_flags[p];
+        b.peer_rank[p] = d.peer_rank[p];
+    }
+    b.npeer = d.npeer;
+    b.rank = d.rank;
+    b.stop = respect_stop ? &d.ctrl->stop : nullptr;
+    b.ctrl = d.ctrl;
+    p2p_barrier_kernel<<<1, 32, 0, s>>>(b);
+    CUDA_TRY(cudaGetLastError());
+    return CME_OK;
+}
+
+// after a step wrote buffer `dst`: halo exchange (NCCL) / step barrier (P2P;
+// the halo rows were already stored into the peers by the step kernel)
+static cme_status exch_after_step(Device& d, int dst, cudaStream_t s) {
+    if (!d.comm) return CME_OK;
+    if (d.p2p) return p2p_barrier(d, s, true);
+    return comm_halo(d.comm, d.halo, d.xb[dst], s);
+}
+
+// every rank's [B][8] check record (local8) into gather[rank] on all ranks
+static cme_status exch_records(Device& d, cudaStream_t s, bool respect_stop) {
+    if (!d.comm) return CME_OK;
+    const size_t cnt = (size_t)8 * d.B;
+    if (!d.p2p) return comm_allgather(d.comm, d.local8, d.gather, cnt, s);
+    CopyArgs c{};
+    c.src = d.local8;
+    c.dst[0] = d.gather + (size_t)d.rank * cnt;
+    for (int p = 0; p < d.npeer; ++p) c.dst[p + 1] = d.peer_gather[p] + (size_t)d.rank * cnt;
+    c.ndst = d.npeer + 1;
+    c.count = (int64_t)cnt;
+    c.stop = respect_stop ? &d.ctrl->stop : nullptr;
+    multicast_copy_kernel<<<1, 64, 0, s>>>(c);
+    CUDA_TRY(cudaGetLastError());
+    return p2p_barrier(d, s, respect_stop);
+}
+
+// fill the halo of buffer `buf` from the peers' own rows (load time)
+static cme_status exch_halo_full(Device& d, int buf, cudaStream_t s) {
+    if (!d.comm) return CME_OK;
+    if (!d.p2p) return comm_halo(d.comm, d.halo, d.xb[buf], s);
+    const double* own = d.xb[buf] + d.own_off * d.B;
+    for (int p = 0; p < d.npush; ++p) {
+        CopyArgs c{};
+        c.src = own + d.push_lo[p] * d.B;
+        c.dst[0] = d.push_y[buf][p] + d.push_lo[p] * d.B;
+        c.ndst = 1;
+        c.count = (d.push_hi[p] - d.push_lo[p]) * d.B;
+        multicast_copy_kernel<<<64, 256, 0, s>>>(c);
+        CUDA_TRY(cudaGetLastError());
+    }
+    return p2p_barrier(d, s, false);
+}
+
+// every rank's own segment of the reordered staging vector io to all ranks
+static cme_status exch_segments(Device& d, cudaStream_t s) {
+    if (!d.p2p) return comm_bcast_segments(d.comm, d.io, d.cuts, s);
+    CopyArgs c{};
+    const int64_t off = d.cuts[d.rank];
+    c.src = d.io + off;
+    for (int p = 0; p < d.npeer; ++p) c.dst[p] = d.peer_io[p] + off;
+    c.ndst = d.npeer;
+    c.count = d.cuts[d.rank + 1] - off;
+    if (c.ndst) {
+        multicast_copy_kernel<<<grid_for(c.count), kCta, 0, s>>>(c);
+        CUDA_TRY(cudaGetLastError());
+    }
+    return p2p_barrier(d, s, false);
+}
+
+// Peer-memory transport setup (NEXT-4): publish this rank's buffers to the
+// in-process group, then derive the peers' flag/gather/io pointers and, for
+// every peer that needs some of my rows, where in its x-span they go.
+cme_status device_p2p_setup(cme_matrix_s* h) {
+    Device& d = *h->dev;
+    if (!d.p2p) return CME_OK;
+    P2PRank mine;
+    mine.xb[0] = d.xb[0];
+    mine.xb[1] = d.xb[1];
+    mine.flags = d.flags;
+    mine.gather = d.gather;
+    mine.io = d.io;
+    mine.span_lo = h->span[2 * h->rank];
+    mine.device = d.dev;
+    std::vector<P2PRank> all;
+    CME_TRY(comm_p2p_exchange(d.comm, mine, all));
+    d.npeer = 0;
+    for (int r = 0; r < d.nranks; ++r) {
+        if (r == d.rank) continue;
+        d.peer_rank[d.npeer] = r;
+        d.peer_flags[d.npeer] = all[r].flags;
+        d.peer_gather[d.npeer] = all[r].gather;
+        d.peer_io[d.npeer] = all[r].io;
+        ++d.npeer;
+    }
+    const HaloPlan& hp = h->halo;   // rows (not yet scaled by B)
+    d.npush = 0;
+    for (size_t i = 0; i < hp.send_peer.size(); ++i) {
+        const int sp = hp.send_peer[i];
+        const int64_t lo_local = hp.send_off[i] - d.own_off;   // x-span offset -> own local row
+        d.push_lo[d.npush] = lo_local;
+        d.push_hi[d.npush] = lo_local + hp.send_cnt[i];
+        const int64_t shift = (d.row_begin - all[sp].span_lo) * d.B;   // my local row 0 in peer's x-span
+        for (int b = 0; b < 2; ++b) d.push_y[b][d.npush] = all[sp].xb[b] + shift;
+        ++d.npush;
+    }
+    return CME_OK;
+}
+
 // ------------------------------------------------------------------------------
 // launches
 // ------------------------------------------------------------------------------
@@ -489,6 +682,12 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
     a.unif_lam_inv = unif_lam_inv;
     a.acc = unif_lam_inv != 0.0 ? d.accb : nullptr;
     a.acc_w = acc_w;
+    a.npush = d.p2p ? d.npush : 0;
+    for (int p = 0; p < a.npush; ++p) {
+        a.push_lo[p] = d.push_lo[p];
+        a.push_hi[p] = d.push_hi[p];
+        a.push_y[p] = d.push_y[dst][p];
+    }
     a.n_rows = d.n_own;
     a.slice_begin = 0;
     a.slice_end = d.n_slices;
@@ -512,7 +711,7 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
     a.csr_v = d.csr_v;
     // programmatic dependent launch between consecutive steps (not across the
     // NCCL calls of a distributed solve, which are ordinary stream work)
-    const bool pdl = !d.comm && env_int("CME_PDL", 1) != 0;
+    const bool pdl = (!d.comm || d.p2p) && env_int("CME_PDL", 1) != 0;
     if (d.format == CME_FMT_CSR) {
         CUDA_TRY(check ? launch_ex(csr_step_kernel<true>, dim3(d.grid), dim3(kCta), 0, pdl, s, a)
                        : launch_ex(csr_step_kernel<false>, dim3(d.grid), dim3(kCta), 0, pdl, s, a));
@@ -537,16 +736,15 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
         }
         CUDA_TRY(e);
     }
-    if (d.comm) CME_TRY(comm_halo(d.comm, d.halo, d.xb[dst], s));
-    return CME_OK;
+    return exch_after_step(d, dst, s);
 }
 
 // reduce partials of the last CHECK step and decide
 static cme_status launch_finalize(Device& d, cudaStream_t s, int32_t len, int32_t final_partial) {
-    const bool pdl = !d.comm && env_int("CME_PDL", 1) != 0;
+    const bool pdl = (!d.comm || d.p2p) && env_int("CME_PDL", 1) != 0;
     CUDA_TRY(launch_ex(reduce_partials_kernel, dim3(1), dim3(1024), 0, pdl, s, (const double*)d.partials,
                        d.step_grid(), d.B, d.comm ? d.local8 : d.gather, (const int32_t*)&d.ctrl->stop));
-    if (d.comm) CME_TRY(comm_allgather(d.comm, d.local8, d.gather, (size_t)8 * d.B, s));
+    CME_TRY(exch_records(d, s, true));
     CUDA_TRY(launch_ex(decide_kernel, dim3(1), dim3(1), 0, pdl, s, (const double*)d.gather, d.nranks, d.ctrl, len,
                        final_partial));
     return CME_OK;
@@ -564,7 +762,7 @@ static cme_status enqueue_block(Device& d, cudaStream_t s, int start, int64_t C,
 
 static cme_status ensure_graphs(Device& d, int64_t C, double omega) {
     if (d.gC == C && d.gomega == omega && d.gexec[0]) return CME_OK;
-    if (d.comm) {
+    if (d.comm && !d.p2p) {
         // NCCL sets up peer connections lazily on first use: do that outside
         // the capture (one throw-away exchange + gather on the private stream)
         CME_TRY(comm_halo(d.comm, d.halo, d.xb[1], d.own));
@@ -642,12 +840,11 @@ static cme_status load_iterate(cme_matrix_s* h, const double* p0, bool normalise
         }
         reduce_partials_kernel<<<1, 1024, 0, s>>>(d.partials, g, B, d.comm ? d.local8 : d.gather, nullptr);
         CUDA_TRY(cudaGetLastError());
-        if (d.comm) CME_TRY(comm_allgather(d.comm, d.local8, d.gather, (size_t)8 * B, s));
+        CME_TRY(exch_records(d, s, false));
         load_decide_kernel<<<1, 1, 0, s>>>(d.gather, d.nranks, d.ctrl, normalise ? 1 : 0);
         CUDA_TRY(cudaGetLastError());
     }
-    if (d.comm) CME_TRY(comm_halo(d.comm, d.halo, d.xb[0], s));
-    return CME_OK;
+    return exch_halo_full(d, 0, s);
 }
 
 // p_out[b][original order] <- x[cur] * scale[b]
@@ -666,7 +863,7 @@ static cme_status write_out(cme_matrix_s* h, double* p_out, const double* scale,
         // then un-permute into the caller's buffer (or the second staging buffer)
         scale_copy_kernel<<<grid_for(d.n_own * B), kCta, 0, s>>>(x, d.n_own, B, scale, d.io + d.row_begin * B);
         CUDA_TRY(cudaGetLastError());
-        CME_TRY(comm_bcast_segments(d.comm, d.io, d.cuts, s));
+        CME_TRY(exch_segments(d, s));
         dst = dev_out ? p_out : d.io2;
         scatter_out_kernel<<<grid_for(d.n_global), kCta, 0, s>>>(d.io, d.perm_global, d.n_global, B, d.n_global,
                                                                  d.one, dst);
@@ -809,7 +1006,7 @@ cme_status device_transient(cme_matrix_s* h, const double* p0, double t, double 
     } else {
         scale_copy_kernel<<<grid_for(d.n_own), kCta, 0, s>>>(xacc, d.n_own, 1, d.one, d.io + d.row_begin);
         CUDA_TRY(cudaGetLastError());
-        CME_TRY(comm_bcast_segments(d.comm, d.io, d.cuts, s));
+        CME_TRY(exch_segments(d, s));
         dst = dev_out ? p_out : d.io2;
         scatter_out_kernel<<<grid_for(d.n_global), kCta, 0, s>>>(d.io, d.perm_global, d.n_global, 1, d.n_global,
                                                                  d.one, dst);

@@ -27,6 +27,7 @@ constexpr int kWarpsPerCta = 8;
 constexpr int kCta = 32 * kWarpsPerCta;
 constexpr int kPartials = 8;   // doubles per (CTA, member) partial record
 constexpr int kMaxBatch = 8;
+constexpr int kMaxPushPeers = 8;
 
 // Device control block of a solve (host writes the inputs, decide_kernel the rest).
 struct Ctrl {
@@ -71,6 +72,11 @@ struct StepArgs {
     double unif_lam_inv;
     double* acc;           // x-span base of the accumulator (nullable)
     double acc_w;
+    // peer-memory halo (NEXT-4): own rows [push_lo[p], push_hi[p]) are also
+    // stored at push_y[p] + r*B, i.e. into peer p's output buffer (NVLink)
+    int32_t npush;
+    int64_t push_lo[kMaxPushPeers], push_hi[kMaxPushPeers];
+    double* push_y[kMaxPushPeers];
 };
 
 // Programmatic dependent launch (the step kernels and the check kernels are
@@ -178,6 +184,21 @@ __device__ __forceinline__ void cta_check_partials(const CheckAcc<B>& c, double*
     }
 }
 
+template <int B>
+__device__ __forceinline__ void store_vec(double* dst, const double (&yv)[B]) {
+    if constexpr (B == 1) {
+        dst[0] = yv[0];
+    } else if constexpr (B == 2) {
+        *reinterpret_cast<double2*>(dst) = make_double2(yv[0], yv[1]);
+    } else {
+#pragma unroll
+        for (int k = 0; k < B; k += 4)
+            asm volatile("st.global.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(dst + k), "d"(yv[k]), "d"(yv[k + 1]),
+                         "d"(yv[k + 2]), "d"(yv[k + 3])
+                         : "memory");
+    }
+}
+
 // Epilogue of one row shared by all SELL kernels: band term, damping, pending
 // scale, store, check terms.  acc = sum_t val x[col]; lo/up/id = the slot's
 // B-vectors; xo/yo = x-span bases shifted to the own rows (member-minor).
@@ -214,18 +235,9 @@ __device__ __forceinline__ void finish_row(const StepArgs& a, int64_t r, const d
         yv[b] = y;
         if (CHECK) ck.add(b, y, x, id[b]);
     }
-    double* dst = yo + r * B;
-    if constexpr (B == 1) {
-        dst[0] = yv[0];
-    } else if constexpr (B == 2) {
-        *reinterpret_cast<double2*>(dst) = make_double2(yv[0], yv[1]);
-    } else {
-#pragma unroll
-        for (int k = 0; k < B; k += 4)
-            asm volatile("st.global.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(dst + k), "d"(yv[k]), "d"(yv[k + 1]),
-                         "d"(yv[k + 2]), "d"(yv[k + 3])
-                         : "memory");
-    }
+    store_vec<B>(yo + r * B, yv);
+    for (int p = 0; p < a.npush; ++p)   // halo rows straight into the peer's buffer
+        if (r >= a.push_lo[p] && r < a.push_hi[p]) store_vec<B>(a.push_y[p] + r * B, yv);
 }
 
 // ILP chunk (t-steps whose loads are issued together) for a batch width.
