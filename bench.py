@@ -235,6 +235,9 @@ def main():
     ap.add_argument("--no-converge", action="store_true")
     ap.add_argument("--batch", type=int, default=1, choices=[1, 2, 4, 8],
                     help="solve a sweep of B rate sets on the workload's pattern (SURVEY NEXT-1)")
+    ap.add_argument("--transport", choices=["p2p", "nccl"], default=os.environ.get("CME_TRANSPORT", "p2p"),
+                    help="multi-rank halo/record exchange: peer-memory stores from the step kernel + flag "
+                         "barriers over CUDA IPC (p2p), or NCCL send/recv + allgather in the graphs (nccl)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -245,7 +248,7 @@ def main():
     import torch.distributed as dist
     world = int(os.environ.get("WORLD_SIZE", "1"))
     # under torchrun (RANK set) the row-sharded path runs even with one rank:
-    # NCCL communicator, distribute, halo/allgather in the graphs
+    # communicator, distribute, halo/record exchange in the graphs
     dist_path = "RANK" in os.environ
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
@@ -257,15 +260,22 @@ def main():
     comm = None
     if dist_path:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        obj = [cme.cme_comm_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(obj, src=0)
-        comm = cme.cme_comm_init(world, rank, obj[0], local)
+        if args.transport == "nccl":
+            obj = [cme.cme_comm_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(obj, src=0)
+            comm = cme.cme_comm_init(world, rank, obj[0], local)
+        else:
+            comm = cme.cme_comm_init_ipc(world, rank, local)
 
     name = args.config
     B = args.batch
     m, cfg, setup = build_matrix(cme, name, cme.CME_DEVICE_HOST_ONLY if dist_path else local, B)
     if comm is not None:
         cme.cme_matrix_distribute(m.h, comm)
+        if args.transport == "p2p":
+            blobs = [None] * world
+            dist.all_gather_object(blobs, cme.cme_matrix_ipc_export(m.h))
+            cme.cme_matrix_ipc_attach(m.h, blobs)
     info = m.info()
     n, nnz = info.n, info.nnz
     stream = torch.cuda.Stream()
@@ -342,7 +352,8 @@ def main():
                        "window": cfg["window"], "band_on": bool(info.band_on), "omega": cfg["omega"],
                        "check_every": C_BLOCK, "iters_per_step": C_BLOCK,
                        "l2": f"inputs larger than L2 ({info.bytes_alg / 1e9:.3f} GB/iteration vs 126 MB)",
-                       "parallelism": f"rows{world}", "setup": setup},
+                       "parallelism": f"rows{world}", "setup": setup,
+                       "transport": args.transport if dist_path else None},
             "iters_per_s": round(iters / sec, 2),
             "pct_hbm_roofline": round(100.0 * achieved / (peak * world), 2),
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak * world, "unit": "GB/s",
@@ -365,6 +376,7 @@ def main():
         }
         print(json.dumps(line), flush=True)
     if comm is not None:
+        dist.barrier()   # peers may address this rank's buffers until everyone is done
         m.close()
         cme.cme_comm_destroy(comm)
         dist.destroy_process_group()

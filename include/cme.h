@@ -244,6 +244,17 @@ cme_status cme_comm_init(int nranks, int rank, const uint8_t id[128], int device
  * exchanged the same way.  Each rank's handle must be driven by its own host
  * thread; comms_out[nranks]; nranks <= 9. */
 cme_status cme_comm_init_local(int nranks, const int* devices, cme_comm* comms_out);
+/* The same transport across processes (one per GPU): cme_comm_init_ipc for
+ * this rank, cme_matrix_distribute, then cme_matrix_ipc_export fills this
+ * rank's CME_IPC_BLOB_BYTES blob (CUDA IPC handles of its iterate buffers,
+ * flags, gather and staging arrays); the caller all-gathers the blobs in rank
+ * order (e.g. torch.distributed) and passes them to cme_matrix_ipc_attach.
+ * Until attach, solving returns BAD_STATE.  Before cme_matrix_destroy the
+ * caller barriers the ranks (peers map this rank's memory). */
+#define CME_IPC_BLOB_BYTES 512
+cme_status cme_comm_init_ipc(int nranks, int rank, int device, cme_comm* out);
+cme_status cme_matrix_ipc_export(cme_matrix h, uint8_t blob[CME_IPC_BLOB_BYTES]);
+cme_status cme_matrix_ipc_attach(cme_matrix h, const uint8_t* blobs /* [nranks][CME_IPC_BLOB_BYTES] */);
 /* Host-only partition plan for (nranks, rank): contiguous reordered rows cut
  * at window boundaries, balanced by packed bytes; local layout with columns
  * remapped to the local x span.  cme_matrix_distribute = plan + upload. */

@@ -110,6 +110,9 @@ _SIGS = {
     "cme_comm_unique_id": [u8p],
     "cme_comm_init": [C.c_int, C.c_int, u8p, C.c_int, _p(vp)],
     "cme_comm_init_local": [C.c_int, i32p, _p(vp)],
+    "cme_comm_init_ipc": [C.c_int, C.c_int, C.c_int, _p(vp)],
+    "cme_matrix_ipc_export": [vp, u8p],
+    "cme_matrix_ipc_attach": [vp, u8p],
     "cme_matrix_plan_partition": [vp, C.c_int, C.c_int],
     "cme_matrix_distribute": [vp, vp],
     "cme_export_halo": [vp, _p(cme_halo_view)],
@@ -326,6 +329,31 @@ def cme_comm_init_local(devices):
     out = (vp * len(devs))()
     _chk(_lib.cme_comm_init_local(len(devs), devs.ctypes.data_as(i32p), out), "cme_comm_init_local")
     return [vp(c) for c in out]
+
+
+CME_IPC_BLOB_BYTES = 512
+
+
+def cme_comm_init_ipc(nranks, rank, device=-1):
+    """Multi-process peer-memory transport (one process per GPU)."""
+    c = vp()
+    _chk(_lib.cme_comm_init_ipc(nranks, rank, device, C.byref(c)), "cme_comm_init_ipc")
+    return c
+
+
+def cme_matrix_ipc_export(h) -> bytes:
+    buf = (C.c_uint8 * CME_IPC_BLOB_BYTES)()
+    _chk(_lib.cme_matrix_ipc_export(h, buf), "cme_matrix_ipc_export")
+    return bytes(buf)
+
+
+def cme_matrix_ipc_attach(h, blobs):
+    """blobs: every rank's cme_matrix_ipc_export bytes, in rank order."""
+    data = b"".join(blobs)
+    if any(len(b) != CME_IPC_BLOB_BYTES for b in blobs):
+        raise ValueError("IPC blobs must be CME_IPC_BLOB_BYTES each")
+    buf = (C.c_uint8 * len(data)).from_buffer_copy(data)
+    _chk(_lib.cme_matrix_ipc_attach(h, buf), "cme_matrix_ipc_attach")
 
 
 def cme_matrix_plan_partition(h, nranks, rank):

@@ -19,6 +19,8 @@ void set_error(const std::string& msg) { g_err = msg; }
 struct Device;
 cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cme_comm_s* comm);
 cme_status device_p2p_setup(cme_matrix_s* h);
+cme_status device_ipc_export(cme_matrix_s* h, uint8_t* out);
+cme_status device_ipc_attach(cme_matrix_s* h, const uint8_t* blobs);
 void device_free(Device* d);
 cme_status device_solve(cme_matrix_s* h, const double* p0, double tol, int64_t max_iter, double* p_out,
                         int64_t* iters_out);
@@ -445,6 +447,18 @@ cme_status cme_matrix_distribute(cme_matrix h, cme_comm c) {
     });
 }
 
+cme_status cme_matrix_ipc_export(cme_matrix h, uint8_t* blob) {
+    if (!h || !blob) return CME_ERR_INVALID_ARG;
+    if (h->stage != 3 || !h->dev) return CME_ERR_BAD_STATE;
+    return guarded([&] { return device_ipc_export(h, blob); });
+}
+
+cme_status cme_matrix_ipc_attach(cme_matrix h, const uint8_t* blobs) {
+    if (!h || !blobs) return CME_ERR_INVALID_ARG;
+    if (h->stage != 3 || !h->dev) return CME_ERR_BAD_STATE;
+    return guarded([&] { return device_ipc_attach(h, blobs); });
+}
+
 cme_status cme_export_halo(cme_matrix h, cme_halo_view* v) {
     if (!h || !v || h->cuts.empty()) return CME_ERR_INVALID_ARG;
     v->nranks = h->nranks;
@@ -466,7 +480,7 @@ void cme_matrix_destroy(cme_matrix h) {
     if (!h) return;
     // peer-memory transport: peers may still address this rank's buffers
     // until every rank of the group reaches its destroy (collective)
-    if (h->comm && comm_transport(h->comm) == kTransportP2P) {
+    if (h->comm && comm_transport(h->comm) == kTransportP2P) {   // (IPC: the caller barriers)
         cudaDeviceSynchronize();
         comm_p2p_host_barrier(h->comm);
     }

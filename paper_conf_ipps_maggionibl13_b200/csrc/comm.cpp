@@ -252,6 +252,26 @@ extern "C" cme_status cme_comm_init_local(int nranks, const int* devices, cme_co
     return CME_OK;
 }
 
+extern "C" cme_status cme_comm_init_ipc(int nranks, int rank, int device, cme_comm* out) {
+    if (!out || nranks < 1 || nranks > cme::kMaxPeers + 1 || rank < 0 || rank >= nranks) return CME_ERR_INVALID_ARG;
+    *out = nullptr;
+    int count = 0;
+    if (cudaGetDeviceCount(&count) != cudaSuccess || count == 0) {
+        cudaGetLastError();
+        cme::set_error("no CUDA device visible");
+        return CME_ERR_NO_DEVICE;
+    }
+    if (device < 0 && cudaGetDevice(&device) != cudaSuccess) return CME_ERR_CUDA;
+    if (device >= count) return CME_ERR_INVALID_ARG;
+    auto* c = new cme_comm_s();
+    c->transport = cme::kTransportIpc;
+    c->nranks = nranks;
+    c->rank = rank;
+    c->device = device;
+    *out = c;
+    return CME_OK;
+}
+
 extern "C" void cme_comm_destroy(cme_comm c) {
     if (!c) return;
     if (c->comm && cme::g_api.CommDestroy) cme::g_api.CommDestroy(c->comm);

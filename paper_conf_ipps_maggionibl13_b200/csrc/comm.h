@@ -22,7 +22,7 @@ struct HaloPlan {
     }
 };
 
-enum { kTransportNccl = 0, kTransportP2P = 1 };
+enum { kTransportNccl = 0, kTransportP2P = 1, kTransportIpc = 2 };
 constexpr int kMaxPeers = 8;
 
 // One rank's device buffers, published to the group by the peer-memory
@@ -38,6 +38,7 @@ struct P2PRank {
 };
 
 int comm_transport(const cme_comm_s* c);
+inline bool transport_is_peer(int t) { return t == kTransportP2P || t == kTransportIpc; }
 // Publish `mine`, block until every rank of the group has, return all ranks'.
 cme_status comm_p2p_exchange(cme_comm_s* c, const P2PRank& mine, std::vector<P2PRank>& all);
 // Host-side barrier over the group (setup / teardown only).

@@ -90,6 +90,8 @@ struct Device {
     int npush = 0;                   // peers that need some of my rows
     int64_t push_lo[kMaxPushPeers] = {}, push_hi[kMaxPushPeers] = {};   // local rows
     double* push_y[2][kMaxPushPeers] = {};   // peer buffer (parity b) shifted to my local rows
+    bool peers_ready = false;        // IPC transport: attach done
+    std::vector<void*> ipc_opened;   // peer allocations mapped into this process
     HaloPlan halo;                   // counts/offsets in doubles (rows x B)
     std::vector<int64_t> cuts;       // in doubles (rows x B) for the output broadcast
     // TMA-staged persistent kernel (kernels_tma.cuh)
@@ -336,6 +338,7 @@ static int grid_for(int64_t n) {
 void device_free(Device* d) {
     if (!d) return;
     if (d->dev >= 0) cudaSetDevice(d->dev);
+    for (void* p : d->ipc_opened) cudaIpcCloseMemHandle(p);
     for (auto& g : d->gexec)
         if (g) cudaGraphExecDestroy(g);
     for (auto& e : d->ev)
@@ -529,7 +532,7 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
     if ((s = d->alloc(d->io, (size_t)d->n_global * B)) != CME_OK) return fail(s);
     if (comm && (s = d->alloc(d->io2, (size_t)d->n_global * B)) != CME_OK) return fail(s);
     if ((s = d->alloc(d->one, kMaxBatch)) != CME_OK) return fail(s);
-    d->p2p = comm && comm_transport(comm) == kTransportP2P;
+    d->p2p = comm && transport_is_peer(comm_transport(comm));
     if (d->p2p) {
         if ((s = d->alloc(d->flags, (size_t)d->nranks)) != CME_OK) return fail(s);
         if ((s = d->alloc(d->epoch, 1)) != CME_OK) return fail(s);
@@ -560,6 +563,7 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
 // broadcast) or the peer-memory transport (direct stores + flag barriers)
 // ------------------------------------------------------------------------------
 static cme_status p2p_barrier(Device& d, cudaStream_t s, bool respect_stop) {
+    if (d.npeer == 0) return CME_OK;   // a group of one
     BarrierArgs b{};
     b.flags = d.flags;
     b.epoch = d.epoch;
@@ -634,22 +638,11 @@ static cme_status exch_segments(Device& d, cudaStream_t s) {
     return p2p_barrier(d, s, false);
 }
 
-// Peer-memory transport setup (NEXT-4): publish this rank's buffers to the
-// in-process group, then derive the peers' flag/gather/io pointers and, for
-// every peer that needs some of my rows, where in its x-span they go.
-cme_status device_p2p_setup(cme_matrix_s* h) {
+// Peer-memory transport: given every rank's published buffers, derive the
+// peers' flag/gather/io pointers and, for every peer that needs some of my
+// rows, where in its x-span they go.
+static void p2p_wire(cme_matrix_s* h, const std::vector<P2PRank>& all) {
     Device& d = *h->dev;
-    if (!d.p2p) return CME_OK;
-    P2PRank mine;
-    mine.xb[0] = d.xb[0];
-    mine.xb[1] = d.xb[1];
-    mine.flags = d.flags;
-    mine.gather = d.gather;
-    mine.io = d.io;
-    mine.span_lo = h->span[2 * h->rank];
-    mine.device = d.dev;
-    std::vector<P2PRank> all;
-    CME_TRY(comm_p2p_exchange(d.comm, mine, all));
     d.npeer = 0;
     for (int r = 0; r < d.nranks; ++r) {
         if (r == d.rank) continue;
@@ -659,7 +652,7 @@ cme_status device_p2p_setup(cme_matrix_s* h) {
         d.peer_io[d.npeer] = all[r].io;
         ++d.npeer;
     }
-    const HaloPlan& hp = h->halo;   // rows (not yet scaled by B)
+    const HaloPlan& hp = h->halo;   // rows (not scaled by B)
     d.npush = 0;
     for (size_t i = 0; i < hp.send_peer.size(); ++i) {
         const int sp = hp.send_peer[i];
@@ -670,6 +663,91 @@ cme_status device_p2p_setup(cme_matrix_s* h) {
         for (int b = 0; b < 2; ++b) d.push_y[b][d.npush] = all[sp].xb[b] + shift;
         ++d.npush;
     }
+    d.peers_ready = true;
+}
+
+static P2PRank p2p_mine(cme_matrix_s* h) {
+    Device& d = *h->dev;
+    P2PRank mine;
+    mine.xb[0] = d.xb[0];
+    mine.xb[1] = d.xb[1];
+    mine.flags = d.flags;
+    mine.gather = d.gather;
+    mine.io = d.io;
+    mine.span_lo = h->span[2 * h->rank];
+    mine.device = d.dev;
+    return mine;
+}
+
+// In-process group (cme_comm_init_local): exchange through the group object.
+cme_status device_p2p_setup(cme_matrix_s* h) {
+    Device& d = *h->dev;
+    if (!d.p2p || comm_transport(d.comm) != kTransportP2P) return CME_OK;
+    std::vector<P2PRank> all;
+    CME_TRY(comm_p2p_exchange(d.comm, p2p_mine(h), all));
+    p2p_wire(h, all);
+    return CME_OK;
+}
+
+// Multi-process group (cme_comm_init_ipc): this rank's buffers as CUDA IPC
+// handles + offsets (allocation bases are exported; the x-span pointers sit
+// one sentinel row past them).
+struct IpcBlob {
+    uint64_t magic;
+    int32_t rank, device;
+    int64_t span_lo;
+    cudaIpcMemHandle_t h[5];   // xb[0] base, xb[1] base, flags, gather, io
+    int64_t off[5];            // byte offset of the published pointer in its allocation
+};
+static_assert(sizeof(IpcBlob) <= CME_IPC_BLOB_BYTES, "IPC blob too large");
+constexpr uint64_t kIpcMagic = 0x434d45495043ull;   // "CMEIPC"
+
+cme_status device_ipc_export(cme_matrix_s* h, uint8_t* out) {
+    Device& d = *h->dev;
+    if (!d.p2p || comm_transport(d.comm) != kTransportIpc) { set_error("not an IPC-distributed handle"); return CME_ERR_BAD_STATE; }
+    CUDA_TRY(cudaSetDevice(d.dev));
+    IpcBlob b{};
+    b.magic = kIpcMagic;
+    b.rank = d.rank;
+    b.device = d.dev;
+    b.span_lo = h->span[2 * h->rank];
+    // allocation bases (device_upload): xb[b] sits one sentinel row of B doubles in
+    void* bases[5] = {d.xb[0] - d.B, d.xb[1] - d.B, d.flags, d.gather, d.io};
+    const int64_t offs[5] = {(int64_t)(d.B * sizeof(double)), (int64_t)(d.B * sizeof(double)), 0, 0, 0};
+    for (int i = 0; i < 5; ++i) {
+        CUDA_TRY(cudaIpcGetMemHandle(&b.h[i], bases[i]));
+        b.off[i] = offs[i];
+    }
+    std::memset(out, 0, CME_IPC_BLOB_BYTES);
+    std::memcpy(out, &b, sizeof(b));
+    return CME_OK;
+}
+
+cme_status device_ipc_attach(cme_matrix_s* h, const uint8_t* blobs) {
+    Device& d = *h->dev;
+    if (!d.p2p || comm_transport(d.comm) != kTransportIpc) { set_error("not an IPC-distributed handle"); return CME_ERR_BAD_STATE; }
+    CUDA_TRY(cudaSetDevice(d.dev));
+    std::vector<P2PRank> all(d.nranks);
+    for (int r = 0; r < d.nranks; ++r) {
+        IpcBlob b;
+        std::memcpy(&b, blobs + (size_t)r * CME_IPC_BLOB_BYTES, sizeof(b));
+        if (b.magic != kIpcMagic || b.rank != r) { set_error("bad IPC blob order/content"); return CME_ERR_INVALID_ARG; }
+        if (r == d.rank) { all[r] = p2p_mine(h); continue; }
+        void* mapped[5];
+        for (int i = 0; i < 5; ++i) {
+            CUDA_TRY(cudaIpcOpenMemHandle(&mapped[i], b.h[i], cudaIpcMemLazyEnablePeerAccess));
+            d.ipc_opened.push_back(mapped[i]);
+            mapped[i] = (char*)mapped[i] + b.off[i];
+        }
+        all[r].xb[0] = (double*)mapped[0];
+        all[r].xb[1] = (double*)mapped[1];
+        all[r].flags = (int64_t*)mapped[2];
+        all[r].gather = (double*)mapped[3];
+        all[r].io = (double*)mapped[4];
+        all[r].span_lo = b.span_lo;
+        all[r].device = b.device;
+    }
+    p2p_wire(h, all);
     return CME_OK;
 }
 
@@ -897,9 +975,15 @@ static void fill_reports(cme_matrix_s* h, const Ctrl& f, double omega, double se
     h->report.iters = f.iter;
 }
 
+static cme_status peers_check(const Device& d) {
+    if (d.p2p && !d.peers_ready) { set_error("peer-memory transport: cme_matrix_ipc_attach first"); return CME_ERR_BAD_STATE; }
+    return CME_OK;
+}
+
 cme_status device_solve(cme_matrix_s* h, const double* p0, double tol, int64_t max_iter, double* p_out,
                         int64_t* iters_out) {
     Device& d = *h->dev;
+    CME_TRY(peers_check(d));
     CUDA_TRY(cudaSetDevice(d.dev));
     cudaStream_t s = stream_of(h);
     const int64_t C = h->sopts.check_every;
@@ -963,6 +1047,7 @@ cme_status device_solve(cme_matrix_s* h, const double* p0, double tol, int64_t m
 cme_status device_transient(cme_matrix_s* h, const double* p0, double t, double eps, double* p_out,
                             int64_t* terms_out) {
     Device& d = *h->dev;
+    CME_TRY(peers_check(d));
     if (d.B != 1) { set_error("transient solves take one rate set (batch 1)"); return CME_ERR_INVALID_ARG; }
     CUDA_TRY(cudaSetDevice(d.dev));
     cudaStream_t s = stream_of(h);
@@ -1033,6 +1118,7 @@ void device_describe(const Device* d, cme_info* f) {
 
 cme_status device_spmv(cme_matrix_s* h, const double* x, double* y) {
     Device& d = *h->dev;
+    CME_TRY(peers_check(d));
     CUDA_TRY(cudaSetDevice(d.dev));
     cudaStream_t s = stream_of(h);
     CME_TRY(load_iterate(h, x, false, s));
@@ -1043,6 +1129,7 @@ cme_status device_spmv(cme_matrix_s* h, const double* x, double* y) {
 
 cme_status device_load(cme_matrix_s* h, const double* p0) {
     Device& d = *h->dev;
+    CME_TRY(peers_check(d));
     CUDA_TRY(cudaSetDevice(d.dev));
     cudaStream_t s = stream_of(h);
     CME_TRY(load_iterate(h, p0, true, s));
@@ -1063,6 +1150,7 @@ cme_status device_load(cme_matrix_s* h, const double* p0) {
 
 cme_status device_run(cme_matrix_s* h, int64_t blocks) {
     Device& d = *h->dev;
+    CME_TRY(peers_check(d));
     CUDA_TRY(cudaSetDevice(d.dev));
     cudaStream_t s = stream_of(h);
     const int64_t C = h->sopts.check_every;
