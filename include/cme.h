@@ -197,7 +197,8 @@ typedef struct cme_info {
     int64_t row_begin, row_end;   /* local rows in the reordered numbering          */
     int64_t halo_begin, halo_end; /* local x span [halo_begin, halo_end)             */
     int32_t kernel;               /* step kernel: 0 register SELL, 1 TMA-staged SELL, 2 CSR,
-                                     3 persistent cooperative SELL (small problems), -1 none */
+                                     3 SMEM-resident persistent SELL (matrix in shared memory,
+                                     neighbour-flag sync; problems that fit), -1 none */
     int32_t tma_warps, tma_stages;/* TMA kernel: consumer warps per CTA, smem stages */
     int32_t grid;                 /* CTAs per step launch                            */
     int32_t batch;                /* rate sets sharing the pattern (1 = single matrix) */

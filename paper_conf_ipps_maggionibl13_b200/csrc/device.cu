@@ -21,6 +21,7 @@
 #include "cme_internal.h"
 #include "comm.h"
 #include "launch.h"
+#include "kernels_resident.cuh"
 
 namespace cme {
 
@@ -99,6 +100,14 @@ struct Device {
     int tma_ncw = 16;
     int tma_grid = 0, tma_stages = 0, tma_stage_bytes = 0, tma_off_val = 0, tma_off_col = 0;
     int64_t n_tiles = 0;
+    // SMEM-resident persistent kernel (kernels_resident.cuh)
+    bool use_res = false;
+    int res_grid = 0, res_smem = 0, res_rps = 1;
+    int32_t* res_q = nullptr;        // [res_grid + 1] slice cuts
+    int32_t* res_row = nullptr;      // [res_grid + 1] first own row per CTA
+    int32_t* res_dep = nullptr;      // [2 res_grid] CTA ranges to probe
+    uint32_t* res_sync = nullptr;    // [4] grid-barrier words
+    int64_t res_timeout_ns = 0;
     // graphs
     cudaGraphExec_t gexec[2] = {nullptr, nullptr};
     int64_t gC = -1;
@@ -156,64 +165,13 @@ __global__ void __launch_bounds__(1024) reduce_partials_kernel(const double* par
     }
 }
 
-// Check decision (readings R2-R5), per member.
-// all holds one [B][8] record per rank, combined in rank order.
+// Check decision (readings R2-R5): decide_apply
+// (kernels.cuh) on the rank-ordered check records.
 __global__ void decide_kernel(const double* all, int nranks, Ctrl* c, int32_t len, int32_t final_partial) {
     pdl_trigger();
     pdl_wait();
     if (c->stop) return;
-    const int B = c->batch;
-    const int64_t k = c->iter + len;
-    c->iter = k;
-    bool numeric = false, running = false;
-    for (int b = 0; b < B; ++b) {
-        double s = 0, sx = 0, sd = 0, md = 0, mx = 0;
-        for (int r = 0; r < nranks; ++r) {
-            const double* p = all + ((size_t)r * B + b) * 8;
-            s += p[0]; sx += p[1]; sd += p[2]; md = fmax(md, p[3]); mx = fmax(mx, p[4]);
-        }
-        const double delta = sd / sx;
-        const double resid = md / (c->omega * c->norm_inf[b] * mx);
-        c->mass[b] = s;
-        c->delta[b] = delta;
-        c->resid[b] = resid;
-        if (!(s > 0.0) || isinf(s) || isnan(delta)) {
-            c->mstatus[b] = CME_ERR_NUMERIC;
-            c->miters[b] = k;
-            numeric = true;
-            continue;
-        }
-        c->inv_s[b] = 1.0 / s;  // L1 normalisation, applied by the next step (R5)
-        if (final_partial || c->mstatus[b] != -1) continue;
-        const double crit = c->stop_mode == CME_STOP_DELTA_L1 ? delta : resid;
-        if (crit <= c->tol) {
-            c->mstatus[b] = CME_OK;
-            c->miters[b] = k;
-        } else if (c->stag_tol > 0.0 && k >= 2 * c->C &&
-                   fabs(delta - c->delta_prev[b]) <= c->stag_tol * c->delta_prev[b]) {
-            c->mstatus[b] = CME_STAGNATED;
-            c->miters[b] = k;
-        } else {
-            c->delta_prev[b] = delta;
-            running = true;
-        }
-    }
-    int32_t overall = -1;
-    if (numeric) {
-        overall = CME_ERR_NUMERIC;
-    } else if (final_partial || (running && k >= c->max_iter)) {
-        overall = CME_NOT_CONVERGED;
-    } else if (!running) {
-        overall = CME_OK;
-        for (int b = 0; b < B; ++b)
-            if (c->mstatus[b] == CME_STAGNATED) overall = CME_STAGNATED;
-    }
-    if (overall != -1) {
-        for (int b = 0; b < B; ++b)
-            if (c->mstatus[b] == -1) { c->mstatus[b] = CME_NOT_CONVERGED; c->miters[b] = k; }
-        c->status = overall;
-        c->stop = 1;
-    }
+    decide_apply(all, nranks, c, len, final_partial);
 }
 
 // x_own[l*B + b] = src[b*n_global + perm[l]] (original -> reordered,
@@ -456,6 +414,101 @@ static cme_status configure_tma(Device& d, const Packed& P) {
     return CME_OK;
 }
 
+// Plan the SMEM-resident kernel (kernels_resident.cuh): one CTA per SM, each
+// owning a window-aligned run of slices (<= 128) whose packed image fits in
+// shared memory; its probe range = owners of the columns it reads plus the
+// CTAs reading its rows.  Single GPU, B = 1, SELL formats.  CME_RESIDENT = -1
+// auto (use it whenever it fits), 0 off, 1 force (error if it does not fit);
+// CME_RES_TIMEOUT_MS bounds every wait (default 2000).
+static cme_status configure_resident(Device& d, const Packed& P, bool distributed) {
+    d.use_res = false;
+    const int want = env_int("CME_RESIDENT", -1);
+    if (want == 0) return CME_OK;
+    auto refuse = [&](const char* why) {
+        if (want == 1) { set_error(std::string("CME_RESIDENT=1: ") + why); return CME_ERR_INVALID_ARG; }
+        return CME_OK;
+    };
+    if (distributed || d.B != 1 || d.format == CME_FMT_CSR || d.n_slices == 0)
+        return refuse("needs one GPU, batch 1 and a sliced format");
+    int dev = 0, smem_max = 0, sms = 0;
+    CUDA_TRY(cudaGetDevice(&dev));
+    CUDA_TRY(cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+    CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    const int64_t win = std::max<int32_t>(P.window, 1);
+    int64_t g32 = 32, ww = win;
+    while (ww) { const int64_t t = g32 % ww; g32 = ww; ww = t; }
+    const int64_t unit = win > 1 ? win / g32 : 1;           // slices per window-aligned unit
+    const int64_t units = (d.n_slices + unit - 1) / unit;
+    const int G = (int)std::min<int64_t>(sms, units);
+    std::vector<int32_t> q(G + 1);
+    for (int b = 0; b <= G; ++b) q[b] = (int32_t)std::min<int64_t>(d.n_slices, (int64_t)b * units / G * unit);
+    int64_t smem = 0, max_nsl = 0;
+    for (int b = 0; b < G; ++b) {
+        const int64_t nsl = q[b + 1] - q[b], nval = P.slice_off[q[b + 1]] - P.slice_off[q[b]];
+        smem = std::max(smem, res_smem_bytes(nval, nsl, d.band, d.rearr));
+        max_nsl = std::max(max_nsl, nsl);
+    }
+    if (max_nsl > 4 * kResWarps) return refuse("more than 128 slices per CTA");
+    const int rps = max_nsl <= kResWarps ? 1 : max_nsl <= 2 * kResWarps ? 2 : 4;
+    smem = (smem + 15) / 16 * 16;
+    if (smem > smem_max - 4096) return refuse("packed matrix does not fit in shared memory");
+    // own-row and column hulls per CTA (local rows = x-span on one GPU)
+    const int64_t n = d.n_own;
+    std::vector<int64_t> rlo(G), rhi(G), clo(G), chi(G);
+    for (int b = 0; b < G; ++b) {
+        int64_t lo = INT64_MAX, hi = -1, cl = INT64_MAX, ch = -1, cnt = 0;
+        for (int64_t slot = (int64_t)q[b] * 32; slot < std::min<int64_t>((int64_t)q[b + 1] * 32, n); ++slot) {
+            const int64_t r = d.rearr ? P.row_of[slot] : slot;
+            lo = std::min(lo, r); hi = std::max(hi, r); ++cnt;
+        }
+        if (cnt != hi - lo + 1) return refuse("CTA rows are not contiguous");
+        cl = lo; ch = hi;
+        if (d.band) { cl = std::max<int64_t>(0, lo - 1); ch = std::min<int64_t>(n - 1, hi + 1); }
+        for (int64_t e = P.slice_off[q[b]]; e < P.slice_off[q[b + 1]]; ++e) {
+            cl = std::min<int64_t>(cl, P.col[e]); ch = std::max<int64_t>(ch, P.col[e]);
+        }
+        rlo[b] = lo; rhi[b] = hi; clo[b] = std::max<int64_t>(cl, 0); chi[b] = std::min<int64_t>(ch, n - 1);
+    }
+    for (int b = 1; b < G; ++b)
+        if (rlo[b] != rhi[b - 1] + 1) return refuse("CTA row runs are not consecutive");
+    auto owner = [&](int64_t row) {
+        return (int)(std::upper_bound(rlo.begin(), rlo.end(), row) - rlo.begin()) - 1;
+    };
+    std::vector<int> ilo(G), ihi(G);
+    for (int b = 0; b < G; ++b) { ilo[b] = owner(clo[b]); ihi[b] = owner(chi[b]); }
+    std::vector<int32_t> dep(2 * G);
+    for (int b = 0; b < G; ++b) {
+        int lo = std::min(ilo[b], b), hi = std::max(ihi[b], b);
+        for (int c = 0; c < G; ++c)   // readers of b's rows (WAR on the double buffer)
+            if (ilo[c] <= b && b <= ihi[c]) { lo = std::min(lo, c); hi = std::max(hi, c); }
+        dep[2 * b] = lo;
+        dep[2 * b + 1] = hi;
+    }
+    CUDA_TRY(resident_prepare((int)smem));
+    int occ = 0;
+    CUDA_TRY(resident_occupancy((int)smem, &occ));
+    if (occ < 1) return refuse("resident kernel cannot be resident");
+    std::vector<int32_t> first(G + 1);
+    for (int b = 0; b < G; ++b) first[b] = (int32_t)rlo[b];
+    first[G] = (int32_t)n;
+    CME_TRY(d.upload(d.res_q, q));
+    CME_TRY(d.upload(d.res_row, first));
+    CME_TRY(d.upload(d.res_dep, dep));
+    CME_TRY(d.alloc(d.res_sync, 4));
+    d.res_grid = G;
+    d.res_smem = (int)smem;
+    d.res_rps = rps;
+    d.res_timeout_ns = (int64_t)std::max(1, env_int("CME_RES_TIMEOUT_MS", 2000)) * 1000000;
+    d.use_res = true;
+    if (env_int("CME_VERBOSE", 0)) {
+        int64_t mx = 0;
+        for (int b = 0; b < G; ++b) mx = std::max<int64_t>(mx, dep[2 * b + 1] - dep[2 * b] + 1);
+        std::fprintf(stderr, "[cme] resident: grid=%d smem=%lld unit=%lld rows/thread=%d max_probes=%lld\n", G,
+                     (long long)smem, (long long)unit, rps, (long long)mx);
+    }
+    return CME_OK;
+}
+
 // Build the device state from h->P (local layout) and the partition in h.
 cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cme_comm_s* comm) {
     int dev = 0;
@@ -525,7 +578,8 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
                                        : (int)((d->n_slices + kWarpsPerCta - 1) / kWarpsPerCta);
     d->grid = std::max(d->grid, 1);
     if (d->format != CME_FMT_CSR && (s = configure_tma(*d, P)) != CME_OK) return fail(s);
-    d->part_blocks = std::max(d->grid, grid_for(d->n_own));
+    if ((s = configure_resident(*d, P, comm != nullptr || h->nranks > 1)) != CME_OK) return fail(s);
+    d->part_blocks = std::max(std::max(d->grid, d->res_grid), grid_for(d->n_own));
     if ((s = d->alloc(d->partials, (size_t)d->part_blocks * B * kPartials)) != CME_OK) return fail(s);
     if ((s = d->alloc(d->gather, (size_t)d->nranks * B * 8)) != CME_OK) return fail(s);
     if ((s = d->alloc(d->local8, (size_t)B * 8)) != CME_OK) return fail(s);
@@ -817,6 +871,52 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
     return exch_after_step(d, dst, s);
 }
 
+// nsteps Jacobi steps from buffer `start` in SMEM-resident launches (chunks of
+// 2^20 check blocks, so the 32-bit grid-barrier counters cannot wrap); solve:
+// the last step closes a partial check block (max_iter).  Stops early when a
+// check decides (ctrl.stop).
+static cme_status launch_res(Device& d, cudaStream_t s, int start, int64_t nsteps, bool solve, int64_t C,
+                             double omega) {
+    const int64_t chunk = C >= (int64_t(1) << 40) ? std::max<int64_t>(nsteps, 1) : (int64_t(1) << 20) * C;
+    for (int64_t done = 0; done < nsteps;) {
+        const int64_t len = std::min(chunk, nsteps - done);
+        CUDA_TRY(cudaMemsetAsync(d.res_sync, 0, 4 * sizeof(uint32_t), s));
+        ResArgs a{};
+        a.n_rows = d.n_own;
+        a.slice_off = d.slice_off;
+        a.slice_w = d.slice_w;
+        a.val = d.val;
+        a.col = d.col;
+        a.row_of = d.row_of;
+        a.lo = d.lo;
+        a.up = d.up;
+        a.inv_d = d.inv_d;
+        a.xb0 = d.xb[0];
+        a.xb1 = d.xb[1];
+        a.cta_q = d.res_q;
+        a.cta_row = d.res_row;
+        a.dep = d.res_dep;
+        a.sync = d.res_sync;
+        a.partials = d.partials;
+        a.ctrl = d.ctrl;
+        a.nsteps = len;
+        a.C = C;
+        a.omega = omega;
+        a.start = (int)((start + done) & 1);
+        a.solve = solve && done + len == nsteps ? 1 : 0;
+        a.timeout_ns = d.res_timeout_ns;
+        CUDA_TRY(launch_resident(a, d.res_grid, d.res_smem, d.band, d.rearr, d.res_rps, s));
+        done += len;
+        if (done < nsteps) {   // a later chunk only if no check stopped the solve
+            int32_t stop = 0;
+            CUDA_TRY(cudaMemcpyAsync(&stop, &d.ctrl->stop, sizeof(stop), cudaMemcpyDeviceToHost, s));
+            CUDA_TRY(cudaStreamSynchronize(s));
+            if (stop) break;
+        }
+    }
+    return CME_OK;
+}
+
 // reduce partials of the last CHECK step and decide
 static cme_status launch_finalize(Device& d, cudaStream_t s, int32_t len, int32_t final_partial) {
     const bool pdl = (!d.comm || d.p2p) && env_int("CME_PDL", 1) != 0;
@@ -922,6 +1022,10 @@ static cme_status load_iterate(cme_matrix_s* h, const double* p0, bool normalise
         load_decide_kernel<<<1, 1, 0, s>>>(d.gather, d.nranks, d.ctrl, normalise ? 1 : 0);
         CUDA_TRY(cudaGetLastError());
     }
+    if (d.use_res) {   // epoch state of the resident kernel: the other buffer's rows negative
+        fill_kernel<<<grid_for(d.n_own), kCta, 0, s>>>(d.xb[1] + d.own_off, d.n_own, -0.0);
+        CUDA_TRY(cudaGetLastError());
+    }
     return exch_halo_full(d, 0, s);
 }
 
@@ -980,6 +1084,29 @@ static cme_status peers_check(const Device& d) {
     return CME_OK;
 }
 
+// End of a solve: time, control block, reports, output (P:L125 final L1 scale).
+static cme_status solve_epilogue(cme_matrix_s* h, cudaStream_t s, double omega, int64_t max_iter, double* p_out,
+                                 int64_t* iters_out) {
+    Device& d = *h->dev;
+    CUDA_TRY(cudaEventRecord(d.t1, s));
+    CUDA_TRY(cudaMemcpyAsync(&d.ctrl_host[0], d.ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    const Ctrl& f = d.ctrl_host[0];
+    d.cur = (int)(f.iter & 1);
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, d.t0, d.t1);
+    if (f.status == CME_ERR_CUDA && d.use_res) {
+        set_error("resident kernel: a dependency wait timed out (CME_RES_TIMEOUT_MS)");
+        if (iters_out) *iters_out = f.iter;
+        return CME_ERR_CUDA;
+    }
+    const int32_t overall = max_iter == 0 ? CME_NOT_CONVERGED : f.status;
+    fill_reports(h, f, omega, ms * 1e-3, overall);
+    if (iters_out) *iters_out = f.iter;
+    CME_TRY(write_out(h, p_out, d.ctrl->inv_s, s));
+    return (cme_status)overall;
+}
+
 cme_status device_solve(cme_matrix_s* h, const double* p0, double tol, int64_t max_iter, double* p_out,
                         int64_t* iters_out) {
     Device& d = *h->dev;
@@ -1005,6 +1132,11 @@ cme_status device_solve(cme_matrix_s* h, const double* p0, double tol, int64_t m
         set_error("p0 has a negative/NaN entry or no positive mass");
         return CME_ERR_INVALID_ARG;
     }
+    if (d.use_res) {   // one persistent launch runs the whole solve
+        CUDA_TRY(cudaEventRecord(d.t0, s));
+        CME_TRY(launch_res(d, s, 0, max_iter, true, C, omega));
+        return solve_epilogue(h, s, omega, max_iter, p_out, iters_out);
+    }
     CME_TRY(ensure_graphs(d, C, omega));
     const int64_t nfull = max_iter / C, rem = max_iter % C;
     CUDA_TRY(cudaEventRecord(d.t0, s));
@@ -1025,18 +1157,7 @@ cme_status device_solve(cme_matrix_s* h, const double* p0, double tol, int64_t m
         if (status != -1) break;
     }
     if (status == -1 && rem > 0) CME_TRY(enqueue_block(d, s, start, rem, omega, true));
-    CUDA_TRY(cudaEventRecord(d.t1, s));
-    CUDA_TRY(cudaMemcpyAsync(&d.ctrl_host[0], d.ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost, s));
-    CUDA_TRY(cudaStreamSynchronize(s));
-    const Ctrl& f = d.ctrl_host[0];
-    d.cur = (int)(f.iter & 1);
-    float ms = 0.f;
-    cudaEventElapsedTime(&ms, d.t0, d.t1);
-    const int32_t overall = max_iter == 0 ? CME_NOT_CONVERGED : f.status;
-    fill_reports(h, f, omega, ms * 1e-3, overall);
-    if (iters_out) *iters_out = f.iter;
-    CME_TRY(write_out(h, p_out, d.ctrl->inv_s, s));
-    return (cme_status)overall;
+    return solve_epilogue(h, s, omega, max_iter, p_out, iters_out);
 }
 
 // Transient landscape p(t) = exp(A t) p0 by uniformization (R22):
@@ -1110,10 +1231,10 @@ cme_status device_transient(cme_matrix_s* h, const double* p0, double t, double 
 
 void device_describe(const Device* d, cme_info* f) {
     if (!d) { f->kernel = -1; return; }
-    f->kernel = d->format == CME_FMT_CSR ? 2 : d->use_tma ? 1 : 0;
+    f->kernel = d->format == CME_FMT_CSR ? 2 : d->use_res ? 3 : d->use_tma ? 1 : 0;
     f->tma_warps = d->use_tma ? d->tma_ncw : 0;
     f->tma_stages = d->use_tma ? d->tma_stages : 0;
-    f->grid = d->step_grid();
+    f->grid = d->use_res ? d->res_grid : d->step_grid();
 }
 
 cme_status device_spmv(cme_matrix_s* h, const double* x, double* y) {
@@ -1122,7 +1243,10 @@ cme_status device_spmv(cme_matrix_s* h, const double* x, double* y) {
     CUDA_TRY(cudaSetDevice(d.dev));
     cudaStream_t s = stream_of(h);
     CME_TRY(load_iterate(h, x, false, s));
-    CME_TRY(launch_step(d, s, 0, 1, false, nullptr, effective_omega(h)));
+    if (d.use_res)   // one resident step (C beyond reach: no check)
+        CME_TRY(launch_res(d, s, 0, 1, false, INT64_MAX / 4, effective_omega(h)));
+    else
+        CME_TRY(launch_step(d, s, 0, 1, false, nullptr, effective_omega(h)));
     d.cur = 1;
     return write_out(h, y, d.one, s);
 }
@@ -1145,7 +1269,7 @@ cme_status device_load(cme_matrix_s* h, const double* p0) {
     CUDA_TRY(cudaMemcpyAsync(&d.ctrl->omega, &omega, sizeof(double), cudaMemcpyHostToDevice, s));
     CUDA_TRY(cudaMemcpyAsync(&d.ctrl->C, &C, sizeof(int64_t), cudaMemcpyHostToDevice, s));
     CUDA_TRY(cudaStreamSynchronize(s));
-    return ensure_graphs(d, C, omega);
+    return d.use_res ? CME_OK : ensure_graphs(d, C, omega);
 }
 
 cme_status device_run(cme_matrix_s* h, int64_t blocks) {
@@ -1154,6 +1278,11 @@ cme_status device_run(cme_matrix_s* h, int64_t blocks) {
     CUDA_TRY(cudaSetDevice(d.dev));
     cudaStream_t s = stream_of(h);
     const int64_t C = h->sopts.check_every;
+    if (d.use_res) {
+        CME_TRY(launch_res(d, s, d.cur, blocks * C, false, C, effective_omega(h)));
+        d.cur = (int)((d.cur + blocks * C) & 1);
+        return CME_OK;
+    }
     CME_TRY(ensure_graphs(d, C, effective_omega(h)));
     for (int64_t b = 0; b < blocks; ++b) {
         CUDA_TRY(cudaGraphLaunch(d.gexec[d.cur], s));

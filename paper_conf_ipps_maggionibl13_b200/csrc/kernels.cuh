@@ -21,6 +21,8 @@
 #include <cstdint>
 #include <cuda_runtime.h>
 
+#include "cme.h"   // status codes (decide_apply)
+
 namespace cme {
 
 constexpr int kWarpsPerCta = 8;
@@ -238,6 +240,64 @@ __device__ __forceinline__ void finish_row(const StepArgs& a, int64_t r, const d
     store_vec<B>(yo + r * B, yv);
     for (int p = 0; p < a.npush; ++p)   // halo rows straight into the peer's buffer
         if (r >= a.push_lo[p] && r < a.push_hi[p]) store_vec<B>(a.push_y[p] + r * B, yv);
+}
+
+// Check decision (readings R2-R5), per member.
+// all holds one [B][8] record per rank, combined in rank order.  Runs on one
+// thread (decide_kernel, or the last-arriving CTA of the resident kernel).
+static __device__ __noinline__ void decide_apply(const double* all, int nranks, Ctrl* c, int32_t len, int32_t final_partial) {
+    const int B = c->batch;
+    const int64_t k = c->iter + len;
+    c->iter = k;
+    bool numeric = false, running = false;
+    for (int b = 0; b < B; ++b) {
+        double s = 0, sx = 0, sd = 0, md = 0, mx = 0;
+        for (int r = 0; r < nranks; ++r) {
+            const double* p = all + ((size_t)r * B + b) * 8;
+            s += p[0]; sx += p[1]; sd += p[2]; md = fmax(md, p[3]); mx = fmax(mx, p[4]);
+        }
+        const double delta = sd / sx;
+        const double resid = md / (c->omega * c->norm_inf[b] * mx);
+        c->mass[b] = s;
+        c->delta[b] = delta;
+        c->resid[b] = resid;
+        if (!(s > 0.0) || isinf(s) || isnan(delta)) {
+            c->mstatus[b] = CME_ERR_NUMERIC;
+            c->miters[b] = k;
+            numeric = true;
+            continue;
+        }
+        c->inv_s[b] = 1.0 / s;  // L1 normalisation, applied by the next step (R5)
+        if (final_partial || c->mstatus[b] != -1) continue;
+        const double crit = c->stop_mode == CME_STOP_DELTA_L1 ? delta : resid;
+        if (crit <= c->tol) {
+            c->mstatus[b] = CME_OK;
+            c->miters[b] = k;
+        } else if (c->stag_tol > 0.0 && k >= 2 * c->C &&
+                   fabs(delta - c->delta_prev[b]) <= c->stag_tol * c->delta_prev[b]) {
+            c->mstatus[b] = CME_STAGNATED;
+            c->miters[b] = k;
+        } else {
+            c->delta_prev[b] = delta;
+            running = true;
+        }
+    }
+    int32_t overall = -1;
+    if (numeric) {
+        overall = CME_ERR_NUMERIC;
+    } else if (final_partial || (running && k >= c->max_iter)) {
+        overall = CME_NOT_CONVERGED;
+    } else if (!running) {
+        overall = CME_OK;
+        for (int b = 0; b < B; ++b)
+            if (c->mstatus[b] == CME_STAGNATED) overall = CME_STAGNATED;
+    }
+    if (overall != -1) {
+        for (int b = 0; b < B; ++b)
+            if (c->mstatus[b] == -1) { c->mstatus[b] = CME_NOT_CONVERGED; c->miters[b] = k; }
+        c->status = overall;
+        c->stop = 1;
+    }
 }
 
 // ILP chunk (t-steps whose loads are issued together) for a batch width.

@@ -39,3 +39,11 @@ template <int B>
 cudaError_t tma_occupancy(int ncw, int smem, int* blocks_per_sm);
 
 }  // namespace cme
+
+namespace cme {
+struct ResArgs;
+// SMEM-resident persistent Jacobi kernel (resident.cu)
+cudaError_t resident_prepare(int smem);
+cudaError_t resident_occupancy(int smem, int* blocks_per_sm);
+cudaError_t launch_resident(const ResArgs& a, int grid, int smem, bool band, bool rearr, int rps, cudaStream_t s);
+}  // namespace cme

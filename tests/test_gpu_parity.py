@@ -251,21 +251,24 @@ def test_nccl_one_rank_distributed_path(cme, oracle_mod):
     m.cme_comm_destroy(comm)
 
 
-@pytest.mark.parametrize("knobs", [{"CME_TMA": "0"}, {"CME_TMA": "1"}, {"CME_TMA": "1", "CME_TMA_WARPS": "8"}],
+@pytest.mark.parametrize("knobs", [{"CME_TMA": "0", "CME_RESIDENT": "0"}, {"CME_TMA": "1", "CME_RESIDENT": "0"},
+                                   {"CME_TMA": "1", "CME_TMA_WARPS": "8", "CME_RESIDENT": "0"},
+                                   {"CME_RESIDENT": "1"}],
                          ids=lambda k: ",".join(f"{a}={b}" for a, b in k.items()))
 @pytest.mark.parametrize("net,order,omega", [(W.toggle_switch(70), "rcm", 0.9), (W.schnakenberg(120), "none", 1.0),
                                              (W.brusselator(90), "dfs", 0.7)], ids=lambda x: getattr(x, "name", str(x)))
 def test_every_step_kernel(cme, oracle_mod, monkeypatch, knobs, net, order, omega):
     """Each step kernel (register SELL, TMA-staged SELL with 16/8 consumer
-    warps) forced on the same problems: per-step parity and a fixed-iteration
-    landscape (C = 7 exercises odd block parity)."""
+    warps, SMEM-resident persistent with epoch-tagged iterates) forced on the
+    same problems: per-step parity and a fixed-iteration landscape (C = 7
+    exercises odd block parity and, with max_iter = 250, a partial final block)."""
     for k, v in knobs.items():
         monkeypatch.setenv(k, v)
     states, r, c, v = oracle_mod.enumerate_network(net)
     A = oracle_mod.ingest(len(states), r, c, v)
     m = cme.Matrix(A.n, r, c, v).reorder(ORD[order]).pack()
     f = m.info()
-    expect = 1 if knobs["CME_TMA"] == "1" else 0
+    expect = 3 if knobs.get("CME_RESIDENT") == "1" else 1 if knobs["CME_TMA"] == "1" else 0
     assert f.kernel == expect
     m.set_opts(omega=omega, check_every=7, stag_tol=0.0)
     x = W.random_start(A.n, 21)
@@ -302,3 +305,42 @@ def test_cfg4_full_size_parity(cme, oracle_mod):
                                   nthreads=len(os.sched_getaffinity(0)))
     assert it == ref.iters == 300
     assert np.abs(p - ref.p).sum() <= 1e-10
+
+
+@pytest.mark.parametrize("width", [16, 5000])
+def test_resident_dependency_ranges(cme, oracle_mod, monkeypatch, width):
+    """SMEM-resident kernel on config-5 generator matrices whose column reach
+    is narrow (a few neighbour CTAs) or global (every CTA depends on every
+    other): SpMV, a fixed-iteration landscape with a partial last block, and
+    a solve to convergence, all against the oracle; the free-running API
+    (cme_solver_load/run/fetch) continues across launches."""
+    monkeypatch.setenv("CME_RESIDENT", "1")
+    n = 20000
+    r, c, v = W.banded_markov(n, 10, width, True, seed=5)
+    A = oracle_mod.ingest(n, r, c, v)
+    m = cme.Matrix(n, r, c, v).pack()
+    f = m.info()
+    assert f.kernel == 3 and f.grid > 1
+    x = W.random_start(n, 2)
+    m.set_opts(omega=0.8, check_every=10, stag_tol=0.0)
+    assert_spmv_close(m.spmv(x), oracle_mod.jacobi_step(A, x, 0.8))
+    p, st, it = m.solve(tol=0.0, max_iter=95)
+    ref = oracle_mod.jacobi_solve(A, omega=0.8, tol=0.0, check_every=10, max_iter=95, stag_tol=0.0)
+    assert st == ref.status == "NOT_CONVERGED" and it == ref.iters == 95
+    assert np.abs(p - ref.p).sum() <= 1e-12
+    # width 16 mixes too slowly to converge in 20000 iterations (both sides
+    # report NOT_CONVERGED); width 5000 converges in a few hundred
+    p, st, it = m.solve(tol=1e-12, max_iter=20000)
+    ref = oracle_mod.jacobi_solve(A, omega=0.8, tol=1e-12, check_every=10, max_iter=20000, stag_tol=0.0)
+    assert st == ref.status == ("CONVERGED" if width > 1000 else "NOT_CONVERGED") and abs(it - ref.iters) <= 10
+    if it != ref.iters:
+        ref = oracle_mod.jacobi_solve(A, omega=0.8, tol=0.0, check_every=10, max_iter=it, stag_tol=0.0)
+    assert np.abs(p - ref.p).sum() <= 1e-10
+    # free-running: 3 blocks, then 4 more in a second launch == 70 iterations
+    cme.cme_solver_load(m.h, n, x)
+    cme.cme_solver_run(m.h, 3)
+    cme.cme_solver_run(m.h, 4)
+    q = np.empty(n)
+    cme.cme_solver_fetch(m.h, n, q)
+    ref = oracle_mod.jacobi_solve(A, p0=x, omega=0.8, tol=0.0, check_every=10, max_iter=70, stag_tol=0.0)
+    assert np.abs(q - ref.p).sum() <= 1e-12

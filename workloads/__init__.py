@@ -25,7 +25,7 @@ import numpy as np
 __all__ = [
     "Network", "birth_death", "toggle_switch", "brusselator", "schnakenberg",
     "schlogl", "cyclic3", "CONFIGS", "config_network", "banded_markov",
-    "uniform_start", "random_start",
+    "uniform_start", "random_start", "banded_markov_fast", "build_generator",
 ]
 
 
@@ -301,3 +301,54 @@ def random_start(n: int, seed: int = 0) -> np.ndarray:
     """A strictly positive seeded start vector (not normalised)."""
     g = np.random.default_rng(seed)
     return g.random(n) + 0.5
+
+
+# ----------------------------------------------------------------------------
+# The same config-5 generator in C (workloads/banded_markov.c, OpenMP over
+# source states) for the 1M-100M-row sweep; tests/test_workloads.py checks it
+# against banded_markov above array for array.
+# ----------------------------------------------------------------------------
+import ctypes as _C  # noqa: E402
+import os as _os  # noqa: E402
+import subprocess as _sp  # noqa: E402
+
+_HERE = _os.path.dirname(_os.path.abspath(__file__))
+_GEN_SRC = _os.path.join(_HERE, "banded_markov.c")
+_GEN_LIB = _os.path.join(_HERE, "libwl_gen.so")
+_gen = None
+
+
+def build_generator(force: bool = False) -> str:
+    """Compile libwl_gen.so (gcc, OpenMP; input generation only)."""
+    if force or not _os.path.exists(_GEN_LIB) or _os.path.getmtime(_GEN_LIB) < _os.path.getmtime(_GEN_SRC):
+        tmp = _GEN_LIB + f".tmp{_os.getpid()}"
+        _sp.check_call(["gcc", "-O2", "-std=c99", "-fopenmp", "-fPIC", "-shared", "-Wall", "-o", tmp, _GEN_SRC])
+        _os.replace(tmp, _GEN_LIB)
+    return _GEN_LIB
+
+
+def banded_markov_fast(n: int, mu: int = 10, width: int = 1024, irregular: bool = False, seed: int = 1):
+    """banded_markov(...) computed by the C generator: identical arrays."""
+    global _gen
+    if n < 2 or mu < 3 or width < 2:
+        raise ValueError("banded_markov needs n >= 2, mu >= 3, width >= 2")
+    if _gen is None:
+        L = _C.CDLL(build_generator())
+        L.wl_banded_markov.restype = _C.c_int64
+        L.wl_banded_markov.argtypes = [_C.c_int64, _C.c_int, _C.c_int64, _C.c_int, _C.c_uint64,
+                                       _C.POINTER(_C.POINTER(_C.c_int32)), _C.POINTER(_C.POINTER(_C.c_int32)),
+                                       _C.POINTER(_C.POINTER(_C.c_double))]
+        L.wl_free.argtypes = [_C.c_void_p]
+        _gen = L
+    r, c, v = _C.POINTER(_C.c_int32)(), _C.POINTER(_C.c_int32)(), _C.POINTER(_C.c_double)()
+    nnz = _gen.wl_banded_markov(n, mu, width, 1 if irregular else 0, seed, _C.byref(r), _C.byref(c), _C.byref(v))
+    if nnz < 0:
+        raise ValueError("wl_banded_markov failed (arguments or memory)")
+    try:
+        rows = np.ctypeslib.as_array(r, shape=(nnz,)).copy()
+        cols = np.ctypeslib.as_array(c, shape=(nnz,)).copy()
+        rates = np.ctypeslib.as_array(v, shape=(nnz,)).copy()
+    finally:
+        for p in (r, c, v):
+            _gen.wl_free(_C.cast(p, _C.c_void_p))
+    return rows, cols, rates
