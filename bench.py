@@ -129,7 +129,7 @@ class ClockSampler:
 
 def kernel_name(info):
     return {0: "sell_step_kernel", 1: f"sell_tma_kernel<{info.tma_warps}>", 2: "csr_step_kernel",
-            3: "sell_persistent_kernel"}.get(
+            3: "sell_resident_kernel"}.get(
         info.kernel, "?")
 
 
@@ -210,7 +210,7 @@ def converge_line(cme, name="cfg2_toggle_100k", tol=1e-12):
     """configs[1]: time-to-converge of the ~100K-state toggle on 1 GPU (resident matrix)."""
     m, cfg, setup = build_matrix(cme, name, -1)
     m.set_opts(omega=cfg["omega"], check_every=C_BLOCK)
-    m.solve(tol=tol, max_iter=200000)   # warm (graph build)
+    m.solve(tol=tol, max_iter=200000)   # warm (graph build / first resident launch)
     t = time.perf_counter()
     p, st, it = m.solve(tol=tol, max_iter=200000)
     wall = time.perf_counter() - t

@@ -39,6 +39,11 @@ if a.config.startswith("banded"):
     n = int(n)
     omega = 1.0
     order = a.order or "none"
+elif a.config.startswith("toggle:"):   # toggle switch with buffer N (Table I toggle-switch-1: N = 400)
+    s, r, c, v = cme.cme_network_enumerate(W.toggle_switch(int(a.config.split(":")[1])))
+    n = len(s)
+    omega = 0.9
+    order = a.order or "rcm"
 else:
     t = time.time()
     if a.batch > 1:

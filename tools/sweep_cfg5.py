@@ -92,7 +92,15 @@ def main():
     a = ap.parse_args()
     peak, src = peak_gbs()
     rows = []
+    import psutil
     for p in points(a.quick):
+        need = 60 * p[0] * p[1]          # ~60 B of host memory per generated entry (COO + ingest + pack)
+        avail = psutil.virtual_memory().available
+        if need > 0.7 * avail:
+            print(json.dumps(dict(n=p[0], mu=p[1], width=p[2], irregular=p[3],
+                                  skipped=f"needs ~{need / 1e9:.0f} GB host memory, {avail / 1e9:.0f} GB free")),
+                  flush=True)
+            continue
         o = run_point(*p, blocks=a.blocks)
         o["frac_alg"] = o["alg_gbs"] / peak
         o["frac_fmt"] = o["fmt_gbs"] / peak

@@ -334,21 +334,24 @@ def banded_markov_fast(n: int, mu: int = 10, width: int = 1024, irregular: bool 
         raise ValueError("banded_markov needs n >= 2, mu >= 3, width >= 2")
     if _gen is None:
         L = _C.CDLL(build_generator())
-        L.wl_banded_markov.restype = _C.c_int64
-        L.wl_banded_markov.argtypes = [_C.c_int64, _C.c_int, _C.c_int64, _C.c_int, _C.c_uint64,
-                                       _C.POINTER(_C.POINTER(_C.c_int32)), _C.POINTER(_C.POINTER(_C.c_int32)),
-                                       _C.POINTER(_C.POINTER(_C.c_double))]
-        L.wl_free.argtypes = [_C.c_void_p]
+        i64p = _C.POINTER(_C.c_int64)
+        L.wl_banded_markov_count.restype = _C.c_int64
+        L.wl_banded_markov_count.argtypes = [_C.c_int64, _C.c_int, _C.c_int64, _C.c_int, _C.c_uint64, i64p]
+        L.wl_banded_markov_fill.restype = None
+        L.wl_banded_markov_fill.argtypes = [_C.c_int64, _C.c_int, _C.c_int64, _C.c_int, _C.c_uint64, i64p,
+                                            _C.POINTER(_C.c_int32), _C.POINTER(_C.c_int32),
+                                            _C.POINTER(_C.c_double)]
         _gen = L
-    r, c, v = _C.POINTER(_C.c_int32)(), _C.POINTER(_C.c_int32)(), _C.POINTER(_C.c_double)()
-    nnz = _gen.wl_banded_markov(n, mu, width, 1 if irregular else 0, seed, _C.byref(r), _C.byref(c), _C.byref(v))
+    off = np.empty(n + 1, dtype=np.int64)
+    args = (n, mu, width, 1 if irregular else 0, seed)
+    nnz = _gen.wl_banded_markov_count(*args, off.ctypes.data_as(_C.POINTER(_C.c_int64)))
     if nnz < 0:
-        raise ValueError("wl_banded_markov failed (arguments or memory)")
-    try:
-        rows = np.ctypeslib.as_array(r, shape=(nnz,)).copy()
-        cols = np.ctypeslib.as_array(c, shape=(nnz,)).copy()
-        rates = np.ctypeslib.as_array(v, shape=(nnz,)).copy()
-    finally:
-        for p in (r, c, v):
-            _gen.wl_free(_C.cast(p, _C.c_void_p))
+        raise ValueError("wl_banded_markov_count: bad arguments")
+    rows = np.empty(nnz, dtype=np.int32)
+    cols = np.empty(nnz, dtype=np.int32)
+    rates = np.empty(nnz, dtype=np.float64)
+    _gen.wl_banded_markov_fill(*args, off.ctypes.data_as(_C.POINTER(_C.c_int64)),
+                               rows.ctypes.data_as(_C.POINTER(_C.c_int32)),
+                               cols.ctypes.data_as(_C.POINTER(_C.c_int32)),
+                               rates.ctypes.data_as(_C.POINTER(_C.c_double)))
     return rows, cols, rates

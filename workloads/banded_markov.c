@@ -13,8 +13,8 @@
  *   k = r % (2w-2); delta = k < w-1 ? k-w : k-w+3; accept j+delta if in range
  *   and not already emitted, with rate(next(s)).
  * rate(r) = 1 + (r >> 11) 2^-53.  Output sorted by column j, then emission. */
+#include <stddef.h>
 #include <stdint.h>
-#include <stdlib.h>
 
 #define GOLDEN 0x9E3779B97F4A7C15ULL
 
@@ -67,37 +67,32 @@ static int emit(int64_t j, int64_t n, int mu, int64_t w, int irregular, uint64_t
     return cnt;
 }
 
-/* Two passes: counts per source (offsets), then emission into place.
- * Returns the number of entries, or -1 on bad arguments / allocation failure.
- * *row/*col/*rate are malloc'ed (free with wl_free). */
-int64_t wl_banded_markov(int64_t n, int mu, int64_t width, int irregular, uint64_t seed, int32_t** row,
-                         int32_t** col, double** rate) {
+/* Pass 1: off[j+1] = number of targets of source j, then the prefix sum
+ * (off[0] = 0; off has n+1 entries, caller-allocated).  Returns nnz, or -1 on
+ * bad arguments. */
+int64_t wl_banded_markov_count(int64_t n, int mu, int64_t width, int irregular, uint64_t seed, int64_t* off) {
     if (n < 2 || mu < 3 || width < 2 || 2 * (mu - 3) + 2 > 64) return -1;
     const int64_t w = width < n ? width : n;
-    int64_t* off = (int64_t*)malloc((size_t)(n + 1) * sizeof(int64_t));
-    if (!off) return -1;
 #pragma omp parallel for schedule(static)
     for (int64_t j = 0; j < n; ++j) off[j + 1] = emit(j, n, mu, w, irregular, seed, 0, NULL, NULL);
     off[0] = 0;
     for (int64_t j = 0; j < n; ++j) off[j + 1] += off[j];
-    const int64_t nnz = off[n];
-    *row = (int32_t*)malloc((size_t)(nnz ? nnz : 1) * sizeof(int32_t));
-    *col = (int32_t*)malloc((size_t)(nnz ? nnz : 1) * sizeof(int32_t));
-    *rate = (double*)malloc((size_t)(nnz ? nnz : 1) * sizeof(double));
-    if (!*row || !*col || !*rate) { free(off); free(*row); free(*col); free(*rate); return -1; }
+    return off[n];
+}
+
+/* Pass 2: emission into caller-allocated row/col/rate (off from pass 1). */
+void wl_banded_markov_fill(int64_t n, int mu, int64_t width, int irregular, uint64_t seed, const int64_t* off,
+                           int32_t* row, int32_t* col, double* rate) {
+    const int64_t w = width < n ? width : n;
 #pragma omp parallel for schedule(static)
     for (int64_t j = 0; j < n; ++j) {
         int64_t t[64];
         double r[64];
         const int c = emit(j, n, mu, w, irregular, seed, 64, t, r);
         for (int i = 0; i < c; ++i) {
-            (*row)[off[j] + i] = (int32_t)t[i];
-            (*col)[off[j] + i] = (int32_t)j;
-            (*rate)[off[j] + i] = r[i];
+            row[off[j] + i] = (int32_t)t[i];
+            col[off[j] + i] = (int32_t)j;
+            rate[off[j] + i] = r[i];
         }
     }
-    free(off);
-    return nnz;
 }
-
-void wl_free(void* p) { free(p); }
