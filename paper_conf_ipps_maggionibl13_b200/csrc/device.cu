@@ -98,7 +98,7 @@ struct Device {
     // TMA-staged persistent kernel (kernels_tma.cuh)
     bool use_tma = false;
     int tma_ncw = 16;
-    int tma_grid = 0, tma_stages = 0, tma_stage_bytes = 0, tma_off_val = 0, tma_off_col = 0;
+    int tma_grid = 0, tma_stages = 0, tma_stage_bytes = 0, tma_off_val = 0, tma_off_col = 0, tma_contig = 1;
     int64_t n_tiles = 0;
     // SMEM-resident persistent kernel (kernels_resident.cuh)
     bool use_res = false;
@@ -407,6 +407,7 @@ static cme_status configure_tma(Device& d, const Packed& P) {
     d.tma_off_val = (int)best.off_val;
     d.tma_off_col = (int)best.off_col;
     d.tma_grid = best.grid;
+    d.tma_contig = env_int("CME_TMA_CONTIG", 0) != 0;   // measured: round robin wins on cfg4 (+3%)
     d.use_tma = true;
     if (env_int("CME_VERBOSE", 0))
         std::fprintf(stderr, "[cme] tma: B=%d warps=%d stages=%d stage_bytes=%lld occ=%d grid=%d tiles=%lld\n",
@@ -852,7 +853,7 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
         CUDA_TRY(check ? launch_ex(csr_step_kernel<true>, dim3(d.grid), dim3(kCta), 0, pdl, s, a)
                        : launch_ex(csr_step_kernel<false>, dim3(d.grid), dim3(kCta), 0, pdl, s, a));
     } else if (d.use_tma) {
-        TmaArgs T{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col};
+        TmaArgs T{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col, d.tma_contig};
         const int smem = d.tma_stages * d.tma_stage_bytes;
         cudaError_t e;
         switch (d.B) {

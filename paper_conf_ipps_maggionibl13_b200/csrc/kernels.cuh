@@ -204,19 +204,30 @@ __device__ __forceinline__ void store_vec(double* dst, const double (&yv)[B]) {
 // Epilogue of one row shared by all SELL kernels: band term, damping, pending
 // scale, store, check terms.  acc = sum_t val x[col]; lo/up/id = the slot's
 // B-vectors; xo/yo = x-span bases shifted to the own rows (member-minor).
-template <int B, bool BAND, bool CHECK>
-__device__ __forceinline__ void finish_row(const StepArgs& a, int64_t r, const double* xo, double* yo,
-                                           const double (&acc)[B], const double (&lo)[B], const double (&up)[B],
-                                           const double (&id)[B], const double* pre_scale, CheckAcc<B>& ck) {
+// Own-row and band loads of row r (issued before the gathers by callers that
+// want them in flight together).
+template <int B, bool BAND>
+struct RowX {
     double xl[B], xu[B], xr[B];
-    if (BAND) {
-        ld_vec<B>(xo + (r - 1) * B, xl);
-        ld_vec<B>(xo + (r + 1) * B, xu);
+    __device__ __forceinline__ void load(const double* xo, int64_t r) {
+        if (BAND) {
+            ld_vec<B>(xo + (r - 1) * B, xl);
+            ld_vec<B>(xo + (r + 1) * B, xu);
+        }
+        // x_r unconditionally: a guarded load could not be hoisted next to the
+        // gathers (measured 3% slower on cfg4); it shares their L1/L2 lines
+        ld_vec<B>(xo + r * B, xr);
     }
-    // x_r unconditionally: a guarded load could not be hoisted next to the
-    // gathers (measured 3% slower on cfg4); it shares their L1/L2 lines
+};
+
+template <int B, bool BAND, bool CHECK>
+__device__ __forceinline__ void finish_row_x(const StepArgs& a, int64_t r, double* yo, const double (&acc)[B],
+                                             const double (&lo)[B], const double (&up)[B], const double (&id)[B],
+                                             const double* pre_scale, CheckAcc<B>& ck, const RowX<B, BAND>& X) {
+    const double(&xl)[B] = X.xl;
+    const double(&xu)[B] = X.xu;
+    const double(&xr)[B] = X.xr;
     const bool damp = a.omega != 1.0;
-    ld_vec<B>(xo + r * B, xr);
     double yv[B];
     const bool unif = a.unif_lam_inv != 0.0;
 #pragma unroll
@@ -240,6 +251,15 @@ __device__ __forceinline__ void finish_row(const StepArgs& a, int64_t r, const d
     store_vec<B>(yo + r * B, yv);
     for (int p = 0; p < a.npush; ++p)   // halo rows straight into the peer's buffer
         if (r >= a.push_lo[p] && r < a.push_hi[p]) store_vec<B>(a.push_y[p] + r * B, yv);
+}
+
+template <int B, bool BAND, bool CHECK>
+__device__ __forceinline__ void finish_row(const StepArgs& a, int64_t r, const double* xo, double* yo,
+                                           const double (&acc)[B], const double (&lo)[B], const double (&up)[B],
+                                           const double (&id)[B], const double* pre_scale, CheckAcc<B>& ck) {
+    RowX<B, BAND> X;
+    X.load(xo, r);
+    finish_row_x<B, BAND, CHECK>(a, r, yo, acc, lo, up, id, pre_scale, ck, X);
 }
 
 // Check decision (readings R2-R5), per member.

@@ -32,7 +32,26 @@ struct TmaArgs {
     int32_t stage_bytes;  // bytes per stage (multiple of 128)
     int32_t off_val;      // byte offsets inside a stage
     int32_t off_col;
+    int32_t contig;       // 1: CTA b takes a contiguous run of tiles, 0: round robin (default, CME_TMA_CONTIG)
 };
+
+// Tile sequence of one CTA: contiguous runs keep consecutive tiles -- whose x
+// gather windows overlap -- on the same SM, so the window stays in L1;
+// round robin interleaves the CTAs.  Returns the first tile, the count and
+// the stride.
+__device__ __forceinline__ void tma_tile_range(const TmaArgs& T, int64_t* first, int64_t* count, int64_t* stride) {
+    const int64_t b = blockIdx.x, G = gridDim.x;
+    if (T.contig) {
+        const int64_t lo = b * T.n_tiles / G, hi = (b + 1) * T.n_tiles / G;
+        *first = lo;
+        *count = hi - lo;
+        *stride = 1;
+    } else {
+        *first = b;
+        *count = b < T.n_tiles ? (T.n_tiles - 1 - b) / G + 1 : 0;
+        *stride = G;
+    }
+}
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -151,6 +170,10 @@ __device__ __forceinline__ void tma_issue(const TmaArgs& T, unsigned char* smem,
 #define CME_TMA_EXACT_WIDTHS 1
 #endif
 constexpr bool kExactWidths = CME_TMA_EXACT_WIDTHS;
+#ifndef CME_TMA_EARLY_X
+#define CME_TMA_EARLY_X 1
+#endif
+constexpr bool kEarlyX = CME_TMA_EARLY_X;
 
 template <int NCW, int B, bool BAND, bool REARR, bool CHECK>
 __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBlocks)
@@ -176,12 +199,14 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
     uint64_t pol = 0;
     // Prologue: the packed matrix is constant across steps, so the first S
     // tiles stream in while the previous step (programmatic dependency) drains.
-    const int64_t my_tiles = (int64_t)blockIdx.x < T.n_tiles ? (T.n_tiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    int64_t t_first, my_tiles, t_stride;
+    tma_tile_range(T, &t_first, &my_tiles, &t_stride);
+    const int64_t t_end = t_first + my_tiles * t_stride;
     const int pro = (int)(my_tiles < (int64_t)S ? my_tiles : (int64_t)S);
     if (producer) {
         pol = evict_first_policy();
         for (int i = 0; i < pro; ++i)
-            tma_issue<NCW, B, BAND, REARR>(T, smem, full, (int64_t)blockIdx.x + (int64_t)i * gridDim.x, i, pol);
+            tma_issue<NCW, B, BAND, REARR>(T, smem, full, t_first + (int64_t)i * t_stride, i, pol);
     }
     pdl_wait();   // x / ctrl of the previous step are final from here on
     if (a.stop != nullptr && *a.stop) {
@@ -198,7 +223,7 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
             // stage s and the parity of its current use, advanced incrementally
             int s = 0;
             uint32_t phase = 1;   // pro == S here: every stage holds its first use
-            for (int64_t tile = (int64_t)blockIdx.x + (int64_t)pro * gridDim.x; tile < T.n_tiles; tile += gridDim.x) {
+            for (int64_t tile = t_first + (int64_t)pro * t_stride; tile < t_end; tile += t_stride) {
                 mbar_wait(&empty[s], phase ^ 1u);   // consumers released the previous use
                 tma_issue<NCW, B, BAND, REARR>(T, smem, full, tile, s, pol);
                 if (++s == S) { s = 0; phase ^= 1u; }
@@ -210,7 +235,7 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
         double* yo = a.y + a.own_off * B;
         int s = 0;
         uint32_t phase = 0;
-        for (int64_t tile = blockIdx.x; tile < T.n_tiles; tile += gridDim.x) {
+        for (int64_t tile = t_first; tile < t_end; tile += t_stride) {
             const int64_t q0 = tile * kTileSlices;
             const int64_t q = q0 + warp;
             const unsigned char* st = smem + (size_t)s * T.stage_bytes;
@@ -228,6 +253,9 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
                 const double* sval = reinterpret_cast<const double*>(st + T.off_val) + (loff + lane) * B;
                 const int32_t* scol = reinterpret_cast<const int32_t*>(st + T.off_col) + loff + lane;
                 const int64_t r = REARR ? (int64_t) reinterpret_cast<const int32_t*>(st + kOffRow)[ls] : slot;
+                // own/band x loads in flight with the gathers (CME_TMA_EARLY_X)
+                RowX<B, BAND> X;
+                if (kEarlyX) X.load(xo, r);
                 double acc[B];
 #pragma unroll
                 for (int b = 0; b < B; ++b) acc[b] = 0.0;
@@ -264,7 +292,8 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
                     lo[b] = BAND ? reinterpret_cast<const double*>(st + kOffLo)[ls * B + b] : 0.0;
                     up[b] = BAND ? reinterpret_cast<const double*>(st + kOffUp)[ls * B + b] : 0.0;
                 }
-                finish_row<B, BAND, CHECK>(a, r, xo, yo, acc, lo, up, id, a.pre_scale, ck);
+                if (!kEarlyX) X.load(xo, r);
+                finish_row_x<B, BAND, CHECK>(a, r, yo, acc, lo, up, id, a.pre_scale, ck, X);
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);
