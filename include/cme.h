@@ -293,6 +293,19 @@ typedef struct cme_coo_s* cme_coo;
 cme_status cme_network_enumerate(int m, const int32_t* x0, int R, const int32_t* reac,
                                  const int32_t* change, const double* rates, const int32_t* w,
                                  int64_t cap, cme_coo* out);
+/* GPU enumerator: the same reachable set, rates and
+ * zero-outflow pruning as cme_network_enumerate (eq. 1, R7-R10),
+ * computed on CUDA device `device` (-1: current) by a level-synchronous BFS
+ * over a 128-bit-key hash table (16 bits per species).  States are numbered in
+ * LEXICOGRAPHIC order of (x_0, ..., x_{m-1}) -- deterministic -- instead of
+ * DFS preorder; triplets are emitted per source state in reaction order, rates
+ * bit-identical to the host enumerator's.  Limits: m <= 8 species, R <= 64
+ * reactions, counts <= 65534 (CME_ERR_INVALID_ARG otherwise: use
+ * cme_network_enumerate).  CME_ERR_NO_DEVICE / CME_ERR_OOM / CME_ERR_CUDA on
+ * device failures.  Output object and ownership as cme_network_enumerate. */
+cme_status cme_network_enumerate_gpu(int m, const int32_t* x0, int R, const int32_t* reac,
+                                     const int32_t* change, const double* rates, const int32_t* w,
+                                     int64_t cap, int device, cme_coo* out);
 cme_status cme_coo_get(cme_coo c, int64_t* n, int64_t* nnz, int32_t m[1], const int32_t** states,
                        const int32_t** row, const int32_t** col, const double** rate);
 void cme_coo_destroy(cme_coo c);

@@ -117,6 +117,7 @@ _SIGS = {
     "cme_matrix_distribute": [vp, vp],
     "cme_export_halo": [vp, _p(cme_halo_view)],
     "cme_network_enumerate": [C.c_int, i32p, C.c_int, i32p, i32p, f64p, i32p, C.c_int64, _p(vp)],
+    "cme_network_enumerate_gpu": [C.c_int, i32p, C.c_int, i32p, i32p, f64p, i32p, C.c_int64, C.c_int, _p(vp)],
     "cme_coo_get": [vp, i64p, i64p, i32p, _p(i32p), _p(i32p), _p(i32p), _p(f64p)],
 }
 for _name, _args in _SIGS.items():
@@ -407,6 +408,22 @@ def cme_network_enumerate(net):
     _chk(_lib.cme_network_enumerate(net.m, x0.ctypes.data_as(i32p), net.R, reac.ctypes.data_as(i32p),
                                     chg.ctypes.data_as(i32p), rates.ctypes.data_as(f64p),
                                     w.ctypes.data_as(i32p), cap, C.byref(c)), "cme_network_enumerate")
+    return _coo_take(c)
+
+
+def cme_network_enumerate_gpu(net, device=-1):
+    """GPU enumerator (lexicographic state order) -> (states, row, col, rate)."""
+    x0, reac, chg, rates, w, cap = net.arrays()
+    reac, chg = np.ascontiguousarray(reac), np.ascontiguousarray(chg)
+    c = vp()
+    _chk(_lib.cme_network_enumerate_gpu(net.m, x0.ctypes.data_as(i32p), net.R, reac.ctypes.data_as(i32p),
+                                        chg.ctypes.data_as(i32p), rates.ctypes.data_as(f64p),
+                                        w.ctypes.data_as(i32p), cap, device, C.byref(c)),
+         "cme_network_enumerate_gpu")
+    return _coo_take(c)
+
+
+def _coo_take(c):
     try:
         n, nnz, m = C.c_int64(), C.c_int64(), (C.c_int32 * 1)()
         S, R_, Cc, V = i32p(), i32p(), i32p(), f64p()
@@ -439,8 +456,9 @@ class Matrix:
             self.h = cme_matrix_create_coo(self.n, row, col, rate, flags)
 
     @classmethod
-    def from_network(cls, net):
-        states, r, c, v = cme_network_enumerate(net)
+    def from_network(cls, net, gpu=False):
+        """gpu=True: the GPU enumerator (lexicographic state order)."""
+        states, r, c, v = cme_network_enumerate_gpu(net) if gpu else cme_network_enumerate(net)
         m = cls(len(states), r, c, v)
         m.states = states
         return m

@@ -89,3 +89,11 @@ struct cme_matrix_s {
     cme_comm_s* comm = nullptr;
     cme::Device* dev = nullptr;
 };
+
+// Enumerated network (cme_network_enumerate / cme_network_enumerate_gpu).
+struct cme_coo_s {
+    int64_t n = 0, nnz = 0;
+    int32_t m = 0;
+    std::vector<int32_t> states, row, col;
+    std::vector<double> rate;
+};

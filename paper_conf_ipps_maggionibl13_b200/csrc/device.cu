@@ -98,7 +98,7 @@ struct Device {
     // TMA-staged persistent kernel (kernels_tma.cuh)
     bool use_tma = false;
     int tma_ncw = 16;
-    int tma_grid = 0, tma_stages = 0, tma_stage_bytes = 0, tma_off_val = 0, tma_off_col = 0, tma_contig = 1;
+    int tma_grid = 0, tma_stages = 0, tma_stage_bytes = 0, tma_off_val = 0, tma_off_col = 0, tma_contig = 0;
     int64_t n_tiles = 0;
     // SMEM-resident persistent kernel (kernels_resident.cuh)
     bool use_res = false;

@@ -12,13 +12,6 @@
 
 #include "cme_internal.h"
 
-struct cme_coo_s {
-    int64_t n = 0, nnz = 0;
-    int32_t m = 0;
-    std::vector<int32_t> states, row, col;
-    std::vector<double> rate;
-};
-
 namespace cme {
 namespace {
 
