@@ -16,7 +16,8 @@ molecule buffer, ~20M states" (N = 3164: n = 20,015,468, nnz = 120,042,194),
 RCM order, DIAG+SELL layout, omega = 0.9 -- the >= 10M-state network of the
 north-star target, whose 1.76 GB/iteration exceeds the 126 MB L2 (no flush
 needed).  configs[1] (~100K states, L2-resident) is reported as the
-time-to-converge line in "converge".
+time-to-converge line in "converge"; configs[2] (Schnakenberg, 2M states) is solved to
+tol 1e-12 and compared with its closed form in "converge_closed_form".
 
 --impl reference times the oracle (oracle/, plain C, all host cores) on the
 same workload and metric: the reference arm of this paper-only tier.
@@ -224,6 +225,36 @@ def converge_line(cme, name="cfg2_toggle_100k", tol=1e-12):
     return out
 
 
+def converge_closed_form(cme, name="cfg3a_schnakenberg_2m", tol=1e-12):
+    """configs[2] (Schnakenberg, n = 2,003,001, Table I size) solved to tol on 1 GPU,
+    plus its L1 distance to the exact stationary law: the network satisfies
+    detailed balance, so pi(x, y) is product Poisson with means k1/k2 and
+    k3/k4, evaluated in log space."""
+    import math
+    from scipy.special import gammaln
+    m, cfg, setup = build_matrix(cme, name, -1)
+    m.set_opts(omega=cfg["omega"], check_every=C_BLOCK)
+    t = time.perf_counter()
+    p, st, it = m.solve(tol=tol, max_iter=2_000_000)
+    wall = time.perf_counter() - t
+    rep = m.report()
+    info = m.info()
+    meta = W.config_network(name).meta
+    S = m.states.astype(np.float64)
+    a, b = meta["k1"] / meta["k2"], meta["k3"] / meta["k4"]
+    logs = S[:, 0] * math.log(a) - gammaln(S[:, 0] + 1) + S[:, 1] * math.log(b) - gammaln(S[:, 1] + 1)
+    pi = np.exp(logs - logs.max())
+    pi /= pi.sum()
+    out = {"workload": name, "n": info.n, "nnz": info.nnz, "tol": tol, "omega": cfg["omega"], "status": st,
+           "iters": it, "device_seconds": round(rep.seconds, 4), "wall_seconds": round(wall, 4),
+           "iters_per_s": round(it / rep.seconds, 1) if rep.seconds > 0 else None,
+           "gflops": round(2 * info.nnz * it / rep.seconds / 1e9, 2) if rep.seconds > 0 else None,
+           "kernel": kernel_name(info), "l1_to_closed_form": float(np.abs(p - pi).sum()),
+           "closed_form": "product Poisson (detailed balance), means k1/k2, k3/k4"}
+    m.close()
+    return out
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -336,6 +367,12 @@ def main():
             conv = converge_line(cme)
         except Exception as ex:  # report, do not hide
             conv = {"error": repr(ex)}
+    conv3 = None
+    if rank == 0 and world == 1 and B == 1 and not args.no_converge:
+        try:
+            conv3 = converge_closed_form(cme)
+        except Exception as ex:  # report, do not hide
+            conv3 = {"error": repr(ex)}
     cpu = None
     if rank == 0 and world == 1 and B == 1 and not args.no_cpu_baseline:
         cb = cpu_oracle_timing(name, budget_s=20.0, omega=cfg["omega"])
@@ -372,6 +409,7 @@ def main():
                     "call": "cme_jacobi_solve(h, p0_pinned_host, tol=0, max_iter=100, p_out_pinned_host)"},
             "gpu_launches": args.steps * (C_BLOCK + 2) * 1,
             "converge": conv,
+            "converge_closed_form": conv3,
             "cpu_baseline": cpu,
         }
         print(json.dumps(line), flush=True)

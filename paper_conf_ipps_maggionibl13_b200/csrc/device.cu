@@ -390,7 +390,11 @@ static cme_status configure_tma(Device& d, const Packed& P) {
         while (sh.stages > 2 && sh.stages * sh.stage > smem_max - 1024) --sh.stages;
         if (sh.stages * sh.stage > smem_max - 1024) continue;   // tiles too wide for this shape
         const int smem = (int)(sh.stages * sh.stage);
-        CUDA_TRY(tma_prepare_b(d.B, ncw, smem));
+        // the attribute is process-wide per kernel: always raise it to the
+        // largest size any handle may use (handles on several host threads --
+        // an in-process rank group -- would otherwise lower it under each
+        // other's launches: "invalid argument")
+        CUDA_TRY(tma_prepare_b(d.B, ncw, smem_max - 1024));
         CUDA_TRY(tma_occupancy_b(d.B, ncw, smem, &sh.occ));
         if (sh.occ < 1) continue;
         sh.occ = std::max(1, std::min(sh.occ, env_int("CME_TMA_CTAS", sh.occ)));
@@ -489,7 +493,7 @@ static cme_status configure_resident(Device& d, const Packed& P, bool distribute
         dep[2 * b] = lo;
         dep[2 * b + 1] = hi;
     }
-    CUDA_TRY(resident_prepare((int)smem));
+    CUDA_TRY(resident_prepare(smem_max - 4096));   // process-wide cap (see configure_tma)
     int occ = 0;
     CUDA_TRY(resident_occupancy((int)smem, &occ));
     if (occ < 1) return refuse("resident kernel cannot be resident");

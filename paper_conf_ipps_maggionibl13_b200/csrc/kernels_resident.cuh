@@ -93,11 +93,16 @@ __device__ __forceinline__ double with_sign(double v, bool neg) {
     const long long b = __double_as_longlong(v) & 0x7fffffffffffffffLL;
     return __longlong_as_double(neg ? (b | (long long)0x8000000000000000ULL) : b);
 }
-// |x[p]| once its epoch sign is `neg` (re-load until then; `bad` on timeout)
-__device__ __forceinline__ double settle(const double* p, double v, bool neg, uint64_t deadline, bool& bad) {
-    while (neg_bit(v) != neg) {
-        if (global_ns() > deadline) { bad = true; return 0.0; }
-        v = ld_x(p);
+// |x[p]| once its epoch sign is `neg` (re-load until then; `bad` after
+// `timeout` ns).  The clock is read only on the slow path: the fast path is
+// one sign test.
+__device__ __forceinline__ double settle(const double* p, double v, bool neg, uint64_t timeout, bool& bad) {
+    if (neg_bit(v) != neg) {
+        const uint64_t t0 = global_ns();
+        do {
+            v = ld_x(p);
+            if (global_ns() - t0 > timeout) { bad = true; break; }
+        } while (neg_bit(v) != neg);
     }
     return fabs(v);
 }
@@ -138,7 +143,8 @@ __device__ __forceinline__ double res_ell(const double* sval, const int32_t* sco
     return acc;
 }
 
-// y of row slot (local slice ql, lane) from the epoch-checked iterate x.
+// y of row slot (local slice ql, lane) from the epoch-checked iterate x
+// (dl = the per-spin timeout in ns).
 template <bool BAND, bool REARR>
 __device__ __forceinline__ double res_row(const ResArgs& a, const ResSmem& s, int ql, int64_t slot, const double* x,
                                           bool neg, double sc, uint64_t dl, bool& bad, int64_t& r, double& xr_out,
@@ -277,7 +283,7 @@ __global__ void __launch_bounds__(kResThreads, 1) sell_resident_kernel(const Res
     __syncthreads();
     int64_t k = 0;
     while (k < a.nsteps) {
-        const uint64_t dl = global_ns() + (uint64_t)a.timeout_ns;
+        const uint64_t dl = (uint64_t)a.timeout_ns;   // per-spin budget (settle)
         const int src = (int)((a.start + k) & 1);
         const double* x = src ? a.xb1 : a.xb0;
         double* y = src ? a.xb0 : a.xb1;
@@ -315,7 +321,7 @@ __global__ void __launch_bounds__(kResThreads, 1) sell_resident_kernel(const Res
         // grid-wide check: the last CTA to arrive reduces the partials in CTA
         // order and decides
         const int32_t len = full ? (int32_t)a.C : (int32_t)(done % a.C);
-        const bool ok = res_grid_barrier(a.sync, ++gen, dl, s_flag, [&](int t) {
+        const bool ok = res_grid_barrier(a.sync, ++gen, global_ns() + dl, s_flag, [&](int t) {
             double v0 = 0, v1 = 0, v2 = 0, v3 = 0, v4 = 0;
             for (int i = t; i < G; i += kResThreads) {
                 const double* p = a.partials + (size_t)i * kPartials;
