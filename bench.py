@@ -361,6 +361,24 @@ def main():
     e2e_gflops = 2.0 * nnz * B * C_BLOCK * e2e_steps / e2e_s / 1e9
     clocks = clk.summary()
 
+    # time-to-converge of the benchmark workload itself (BASELINE metric), on
+    # every rank of a row-sharded run; device time from the solver's events
+    conv_main = None
+    if B == 1 and not args.no_converge:
+        t = time.perf_counter()
+        p_c, st_c, it_c = m.solve(tol=1e-12, max_iter=200000)
+        wall_c = time.perf_counter() - t
+        rep_c = m.report()
+        dev_s = rep_c.seconds
+        if world > 1:
+            tt = torch.tensor([dev_s], device="cuda", dtype=torch.float64)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            dev_s = float(tt.item())
+        conv_main = {"workload": name, "tol": 1e-12, "omega": cfg["omega"], "status": st_c, "iters": it_c,
+                     "device_seconds": round(dev_s, 4), "wall_seconds": round(wall_c, 4),
+                     "delta": rep_c.delta, "mass": float(p_c.sum()),
+                     "note": "cme_jacobi_solve from uniform p0; device_seconds = the solve's iteration loop "
+                             "(max over ranks), wall includes the p0 load and the D2H of p"}
     conv = None
     if rank == 0 and world == 1 and B == 1 and not args.no_converge:
         try:
@@ -408,6 +426,7 @@ def main():
                     "d2h_bytes_per_step": 8 * n * B, "steps": e2e_steps,
                     "call": "cme_jacobi_solve(h, p0_pinned_host, tol=0, max_iter=100, p_out_pinned_host)"},
             "gpu_launches": args.steps * (C_BLOCK + 2) * 1,
+            "time_to_converge": conv_main,
             "converge": conv,
             "converge_closed_form": conv3,
             "cpu_baseline": cpu,

@@ -105,7 +105,8 @@ struct Device {
     int res_grid = 0, res_smem = 0, res_rps = 1;
     int32_t* res_q = nullptr;        // [res_grid + 1] slice cuts
     int32_t* res_row = nullptr;      // [res_grid + 1] first own row per CTA
-    int32_t* res_dep = nullptr;      // [2 res_grid] CTA ranges to probe
+    int32_t* res_probe_off = nullptr;   // [res_grid + 1] CSR offsets of the probe lists
+    int32_t* res_probe = nullptr;       // CTAs each CTA probes (readers it does not read)
     uint32_t* res_sync = nullptr;    // [4] grid-barrier words
     int64_t res_timeout_ns = 0;
     // graphs
@@ -428,7 +429,7 @@ static cme_status configure_tma(Device& d, const Packed& P) {
 static cme_status configure_resident(Device& d, const Packed& P, bool distributed) {
     d.use_res = false;
     const int want = env_int("CME_RESIDENT", -1);
-    if (want == 0) return CME_OK;
+    if (want == 0 || (want < 0 && env_int("CME_TMA", -1) == 1)) return CME_OK;   // a forced TMA kernel wins
     auto refuse = [&](const char* why) {
         if (want == 1) { set_error(std::string("CME_RESIDENT=1: ") + why); return CME_ERR_INVALID_ARG; }
         return CME_OK;
@@ -483,16 +484,24 @@ static cme_status configure_resident(Device& d, const Packed& P, bool distribute
     auto owner = [&](int64_t row) {
         return (int)(std::upper_bound(rlo.begin(), rlo.end(), row) - rlo.begin()) - 1;
     };
-    std::vector<int> ilo(G), ihi(G);
-    for (int b = 0; b < G; ++b) { ilo[b] = owner(clo[b]); ihi[b] = owner(chi[b]); }
-    std::vector<int32_t> dep(2 * G);
+    // D[b] = CTAs whose rows b reads (its gathers see their outputs), R[b] =
+    // CTAs reading b's rows; b probes R[b] \ D[b] (WAR, kernels_resident.cuh)
+    std::vector<std::vector<char>> D(G, std::vector<char>(G, 0));
     for (int b = 0; b < G; ++b) {
-        int lo = std::min(ilo[b], b), hi = std::max(ihi[b], b);
-        for (int c = 0; c < G; ++c)   // readers of b's rows (WAR on the double buffer)
-            if (ilo[c] <= b && b <= ihi[c]) { lo = std::min(lo, c); hi = std::max(hi, c); }
-        dep[2 * b] = lo;
-        dep[2 * b + 1] = hi;
+        auto mark = [&](int64_t c) { if (c >= 0 && c < n) D[b][owner(c)] = 1; };
+        for (int64_t e = P.slice_off[q[b]]; e < P.slice_off[q[b + 1]]; ++e) mark(P.col[e]);
+        if (d.band) { mark(rlo[b] - 1); mark(rhi[b] + 1); }
+        D[b][b] = 1;
     }
+    std::vector<int32_t> probe_off(G + 1, 0), probe_cta;
+    int64_t max_probes = 0;
+    for (int b = 0; b < G; ++b) {
+        for (int c = 0; c < G; ++c)
+            if (c != b && D[c][b] && !D[b][c]) probe_cta.push_back(c);
+        probe_off[b + 1] = (int32_t)probe_cta.size();
+        max_probes = std::max<int64_t>(max_probes, probe_off[b + 1] - probe_off[b]);
+    }
+    if (max_probes > kResThreads) return refuse("too many probe CTAs");
     CUDA_TRY(resident_prepare(smem_max - 4096));   // process-wide cap (see configure_tma)
     int occ = 0;
     CUDA_TRY(resident_occupancy((int)smem, &occ));
@@ -502,19 +511,17 @@ static cme_status configure_resident(Device& d, const Packed& P, bool distribute
     first[G] = (int32_t)n;
     CME_TRY(d.upload(d.res_q, q));
     CME_TRY(d.upload(d.res_row, first));
-    CME_TRY(d.upload(d.res_dep, dep));
+    CME_TRY(d.upload(d.res_probe_off, probe_off));
+    CME_TRY(d.upload(d.res_probe, probe_cta));
     CME_TRY(d.alloc(d.res_sync, 4));
     d.res_grid = G;
     d.res_smem = (int)smem;
     d.res_rps = rps;
     d.res_timeout_ns = (int64_t)std::max(1, env_int("CME_RES_TIMEOUT_MS", 2000)) * 1000000;
     d.use_res = true;
-    if (env_int("CME_VERBOSE", 0)) {
-        int64_t mx = 0;
-        for (int b = 0; b < G; ++b) mx = std::max<int64_t>(mx, dep[2 * b + 1] - dep[2 * b] + 1);
-        std::fprintf(stderr, "[cme] resident: grid=%d smem=%lld unit=%lld rows/thread=%d max_probes=%lld\n", G,
-                     (long long)smem, (long long)unit, rps, (long long)mx);
-    }
+    if (env_int("CME_VERBOSE", 0))
+        std::fprintf(stderr, "[cme] resident: grid=%d smem=%lld unit=%lld rows/thread=%d probes=%lld (max %lld)\n", G,
+                     (long long)smem, (long long)unit, rps, (long long)probe_cta.size(), (long long)max_probes);
     return CME_OK;
 }
 
@@ -904,7 +911,8 @@ static cme_status launch_res(Device& d, cudaStream_t s, int start, int64_t nstep
         a.xb1 = d.xb[1];
         a.cta_q = d.res_q;
         a.cta_row = d.res_row;
-        a.dep = d.res_dep;
+        a.probe_off = d.res_probe_off;
+        a.probe = d.res_probe;
         a.sync = d.res_sync;
         a.partials = d.partials;
         a.ctrl = d.ctrl;

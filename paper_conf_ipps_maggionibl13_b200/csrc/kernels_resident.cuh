@@ -18,9 +18,10 @@
 //   RAW is thus carried by the data itself (an 8-byte store is single-copy
 //   atomic).  WAR (step k overwrites the buffer neighbours read in step k-1)
 //   holds because every CTA finishes ALL its gathers of a step (one CTA
-//   barrier) before storing any row of it, and checks one row ("probe") of
-//   every CTA whose rows it reads or that reads its rows: seeing that CTA's
-//   step-(k-1) output proves it finished its step-(k-1) gathers;
+//   barrier) before storing any row of it, and observes a step-(k-1) output
+//   of every CTA that reads its rows -- which proves that CTA finished its
+//   step-(k-1) gathers: through its own gathers when it also reads that
+//   CTA's rows, else through one extra "probe" load of that CTA's first row;
 // * every C-th step (and the last step of a solve cut short by max_iter) the
 //   CTAs write their check partials and meet at one grid barrier whose last
 //   arriver reduces the partials in CTA order and runs decide_apply (the same
@@ -54,7 +55,8 @@ struct ResArgs {
     double* xb1;
     const int32_t* cta_q;    // [G+1] slice cuts
     const int32_t* cta_row;  // [G+1] first own row of each CTA (cta_row[G] = n)
-    const int32_t* dep;      // [2G] inclusive CTA range each CTA probes
+    const int32_t* probe_off;   // [G+1] CSR offsets into probe
+    const int32_t* probe;       // CTAs that read CTA b's rows but whose rows b does not read
     uint32_t* sync;          // [0] grid-barrier arrivals, [1] released generation (zeroed)
     double* partials;        // [G][kPartials]
     Ctrl* ctrl;
@@ -79,10 +81,19 @@ __device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t* p) {
 __device__ __forceinline__ void st_release_u32(uint32_t* p, uint32_t v) {
     asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
-// iterate accesses: strong (relaxed, gpu scope) -- coherent in L2, no stale L1
+// iterate accesses: strong (relaxed, gpu scope) -- coherent in L2, no stale L1.
+// CME_RES_LD (A/B builds only): 1 = ld.global.cg, 2 = ld.volatile.global.
+#ifndef CME_RES_LD
+#define CME_RES_LD 0
+#endif
 __device__ __forceinline__ double ld_x(const double* p) {
     double v;
-    asm volatile("ld.relaxed.gpu.global.f64 %0, [%1];" : "=d"(v) : "l"(p) : "memory");
+    if (CME_RES_LD == 1)
+        asm volatile("ld.global.cg.f64 %0, [%1];" : "=d"(v) : "l"(p) : "memory");
+    else if (CME_RES_LD == 2)
+        asm volatile("ld.volatile.global.f64 %0, [%1];" : "=d"(v) : "l"(p) : "memory");
+    else
+        asm volatile("ld.relaxed.gpu.global.f64 %0, [%1];" : "=d"(v) : "l"(p) : "memory");
     return v;
 }
 __device__ __forceinline__ void st_x(double* p, double v) {
@@ -273,9 +284,10 @@ __global__ void __launch_bounds__(kResThreads, 1) sell_resident_kernel(const Res
             s.off[i] = (int32_t)(__ldg(a.slice_off + q0 + i) - e0);
         }
     }
-    // probe: thread tid < ndep checks the first row of CTA dep_lo + tid
-    const int dlo = a.dep[2 * b], ndep = a.dep[2 * b + 1] - dlo + 1;
-    const int64_t probe = tid < ndep ? (int64_t)a.cta_row[dlo + tid] : -1;
+    // probe: thread tid < nprobe checks the first row of one reader CTA that
+    // this CTA's gathers do not already observe
+    const int p0 = a.probe_off[b], nprobe = a.probe_off[b + 1] - p0;
+    const int64_t probe = tid < nprobe ? (int64_t)a.cta_row[a.probe[p0 + tid]] : -1;
     const int64_t it0 = *(volatile const int64_t*)&a.ctrl->iter;
     double sc = *(volatile const double*)&a.ctrl->inv_s[0];   // pending 1/sum(y) (R5)
     uint32_t gen = 0;
@@ -292,7 +304,9 @@ __global__ void __launch_bounds__(kResThreads, 1) sell_resident_kernel(const Res
         const bool full = done % a.C == 0;
         const bool check = full || (a.solve && k + 1 == a.nsteps);
         bool bad = false;
+#ifndef CME_RES_NOPROBE   // (A/B measurement only: without probes WAR is not guaranteed)
         if (probe >= 0) (void)settle(x + probe, ld_x(x + probe), in_neg, dl, bad);
+#endif
         double yv[R], xr[R], id[R];
         int64_t rr[R];
 #pragma unroll

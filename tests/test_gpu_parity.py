@@ -307,7 +307,20 @@ def test_cfg4_full_size_parity(cme, oracle_mod):
     assert np.abs(p - ref.p).sum() <= 1e-10
 
 
-@pytest.mark.parametrize("width", [16, 5000])
+def directed_ring(n, hops=(1, 5), rates=(1.0, 0.5)):
+    """Off-diagonal COO of a one-way ring: j -> j+h (mod n) for each hop h.
+    Column j's entries are read by rows ahead of it only, so with contiguous
+    row blocks every block is read by the NEXT block but reads only the
+    PREVIOUS one: the resident kernel's WAR protection needs its probes."""
+    j = np.arange(n, dtype=np.int64)
+    rows = np.concatenate([(j + h) % n for h in hops]).astype(np.int32)
+    cols = np.concatenate([j for _ in hops]).astype(np.int32)
+    vals = np.concatenate([np.full(n, r) for r in rates])
+    order = np.lexsort((rows, cols))
+    return rows[order], cols[order], vals[order]
+
+
+@pytest.mark.parametrize("width", [16, 5000, "ring"])
 def test_resident_dependency_ranges(cme, oracle_mod, monkeypatch, width):
     """SMEM-resident kernel on config-5 generator matrices whose column reach
     is narrow (a few neighbour CTAs) or global (every CTA depends on every
@@ -316,7 +329,7 @@ def test_resident_dependency_ranges(cme, oracle_mod, monkeypatch, width):
     (cme_solver_load/run/fetch) continues across launches."""
     monkeypatch.setenv("CME_RESIDENT", "1")
     n = 20000
-    r, c, v = W.banded_markov(n, 10, width, True, seed=5)
+    r, c, v = directed_ring(n) if width == "ring" else W.banded_markov(n, 10, width, True, seed=5)
     A = oracle_mod.ingest(n, r, c, v)
     m = cme.Matrix(n, r, c, v).pack()
     f = m.info()
@@ -324,17 +337,18 @@ def test_resident_dependency_ranges(cme, oracle_mod, monkeypatch, width):
     x = W.random_start(n, 2)
     m.set_opts(omega=0.8, check_every=10, stag_tol=0.0)
     assert_spmv_close(m.spmv(x), oracle_mod.jacobi_step(A, x, 0.8))
-    p, st, it = m.solve(tol=0.0, max_iter=95)
-    ref = oracle_mod.jacobi_solve(A, omega=0.8, tol=0.0, check_every=10, max_iter=95, stag_tol=0.0)
+    p, st, it = m.solve(p0=x, tol=0.0, max_iter=95)
+    ref = oracle_mod.jacobi_solve(A, p0=x, omega=0.8, tol=0.0, check_every=10, max_iter=95, stag_tol=0.0)
     assert st == ref.status == "NOT_CONVERGED" and it == ref.iters == 95
     assert np.abs(p - ref.p).sum() <= 1e-12
     # width 16 mixes too slowly to converge in 20000 iterations (both sides
     # report NOT_CONVERGED); width 5000 converges in a few hundred
-    p, st, it = m.solve(tol=1e-12, max_iter=20000)
-    ref = oracle_mod.jacobi_solve(A, omega=0.8, tol=1e-12, check_every=10, max_iter=20000, stag_tol=0.0)
-    assert st == ref.status == ("CONVERGED" if width > 1000 else "NOT_CONVERGED") and abs(it - ref.iters) <= 10
+    p, st, it = m.solve(p0=x, tol=1e-12, max_iter=20000)
+    ref = oracle_mod.jacobi_solve(A, p0=x, omega=0.8, tol=1e-12, check_every=10, max_iter=20000, stag_tol=0.0)
+    assert st == ref.status and abs(it - ref.iters) <= 10
+    assert st == ("NOT_CONVERGED" if width == 16 else st)
     if it != ref.iters:
-        ref = oracle_mod.jacobi_solve(A, omega=0.8, tol=0.0, check_every=10, max_iter=it, stag_tol=0.0)
+        ref = oracle_mod.jacobi_solve(A, p0=x, omega=0.8, tol=0.0, check_every=10, max_iter=it, stag_tol=0.0)
     assert np.abs(p - ref.p).sum() <= 1e-10
     # free-running: 3 blocks, then 4 more in a second launch == 70 iterations
     cme.cme_solver_load(m.h, n, x)
