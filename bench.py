@@ -129,6 +129,8 @@ class ClockSampler:
 
 
 def kernel_name(info):
+    if info.kernel == 1 and info.compact:
+        return f"sell_cpt_kernel<{info.tma_warps}>"
     return {0: "sell_step_kernel", 1: f"sell_tma_kernel<{info.tma_warps}>", 2: "csr_step_kernel",
             3: "sell_resident_kernel"}.get(
         info.kernel, "?")
@@ -341,6 +343,11 @@ def main():
     t_iter = sec / iters
     achieved = info.bytes_alg / t_iter / 1e9        # algorithmic bytes per launch / launch time
     fmt_gbs = info.bytes_fmt * world / t_iter / 1e9 if world == 1 else None
+    compact_note = ("compact encoding (DESIGN.md sec. 5b): the kernel streams the rows of M = |D|^-1 O with "
+                    "int16 column and uint8 row offsets, 10 B per ELL slot + 17 B per row (format_bytes_per_launch) "
+                    "instead of the model's 12 B per non-zero + 16 B per row; frac > 1 therefore means fewer bytes "
+                    "than the SURVEY 8(d) byte model, not a faster-than-HBM kernel -- format_frac is the kernel's "
+                    "own DRAM efficiency") if info.compact else None
 
     # e2e: the public solve call with pinned host buffers, H2D + D2H inside the timed region
     p0 = torch.empty(n * B, dtype=torch.float64, pin_memory=True)
@@ -418,6 +425,8 @@ def main():
                          "bytes_per_launch": info.bytes_alg, "bytes_model": "12 nnz + 16 n per member (SURVEY 8(d))" if B == 1 else f"(12 nnz + 16 n) x {B} members: each member counted as if solved alone",
                          "format_bytes_per_launch": info.bytes_fmt,
                          "format_gbs": round(fmt_gbs, 1) if fmt_gbs else None,
+                         "format_frac": round(fmt_gbs / peak, 4) if fmt_gbs else None,
+                         "encoding": "compact" if info.compact else "layout v0", "note": compact_note,
                          "launch_time_us": round(t_iter * 1e6, 3),
                          "launch_time_note": "timed-region time / step-kernel launches (includes the 2 tiny "
                                              "check kernels per 100 steps and launch gaps: conservative)"},

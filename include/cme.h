@@ -202,6 +202,9 @@ typedef struct cme_info {
     int32_t tma_warps, tma_stages;/* TMA kernel: consumer warps per CTA, smem stages */
     int32_t grid;                 /* CTAs per step launch                            */
     int32_t batch;                /* rate sets sharing the pattern (1 = single matrix) */
+    int32_t compact;              /* 1: the TMA kernel streams the compact encoding (rows of
+                                     M = |D|^-1 O, int16 column and uint8 row offsets,
+                                     DESIGN.md sec. 5b); bytes_fmt/packed_bytes count it */
 } cme_info;
 cme_status cme_get_info(cme_matrix h, cme_info* info);
 
@@ -225,6 +228,29 @@ typedef struct cme_packed_view {
     const int64_t* csr_row_ptr; /* CME_FMT_CSR only (else NULL): [n+1]       */
 } cme_packed_view;
 cme_status cme_export_packed(cme_matrix h, cme_packed_view* v);
+
+/* Compact encoding of the current SELL pack (what the TMA
+ * kernel streams when cme_info.compact = 1): the rows of M = |D|^-1 O, the
+ * matrix of the Jacobi iteration (eq. 8), plus offsets instead of
+ * indices.  val[e] = a_rj / (-a_rr) (one IEEE division), lo/up likewise;
+ * col16[e] = j - r (x-span column minus the entry's own row, int16); row8[s]
+ * = r - (s >> win_shift << win_shift) (row inside its rearrangement window).
+ * Pad entries: val 0, col16 0; pad slots: all 0.  Library-owned host arrays,
+ * valid until destroy or the next pack/distribute; computed on demand when
+ * the device does not use it (so host-only packs can be checked too).
+ * Errors: BAD_STATE before cme_pack; INVALID_ARG when the pack does not
+ * qualify (batch > 1, CSR format, window not a power of two <= 256, or an
+ * offset outside int16). */
+typedef struct cme_compact_view {
+    int64_t n, n_slots, n_slices, n_ell;
+    int32_t band_on, win_shift;
+    const double* val;       /* [n_ell]                                      */
+    const int16_t* col16;    /* [n_ell]                                      */
+    const uint8_t* row8;     /* [n_slots], NULL when win_shift == 0          */
+    const double* lo;        /* [n_slots], NULL when the band is off         */
+    const double* up;        /* [n_slots], NULL when the band is off         */
+} cme_compact_view;
+cme_status cme_export_compact(cme_matrix h, cme_compact_view* v);
 
 /* Directed period of the ingested graph from `root` (R1); host-only. */
 cme_status cme_period(cme_matrix h, int64_t root, int64_t* period_out);

@@ -222,6 +222,43 @@ def pack(A: CSR, window: int = 256, band: str = "auto", uniform: bool = False, g
     return out
 
 
+def compact(A: CSR, P: dict):
+    """Compact encoding of a layout-v0 pack P = pack(A, ...)
+    of the already-ordered matrix A, from its definition: the stored rows are
+    those of M = |D|^-1 O, the Jacobi iteration matrix of P:L111 eq. 8
+    (x_i <- sum_{j!=i} a_ij x_j / (-a_ii)), i.e. val_c[e] = a_rj / (-a_rr)
+    for the entry e of row r (one IEEE division), lo/up likewise; col16[e] =
+    j - r; row8[s] = r - (s // window) * window.  Pad entries and pad slots
+    hold 0.  Returns None when the encoding does not apply (window not a power
+    of two <= 256, or some |j - r| > 32767)."""
+    n, W = P["n"], P["window"]
+    if W > 1 and (W > 256 or W & (W - 1)):
+        return None
+    q_of_e = np.repeat(np.arange(P["n_slices"], dtype=np.int64), 32 * P["slice_w"].astype(np.int64))
+    lane = (np.arange(P["n_ell"], dtype=np.int64) - P["slice_off"][q_of_e]) % 32
+    slot = 32 * q_of_e + lane                      # slot of every stored entry
+    real = slot < n
+    row = np.where(real, P["row_of"][np.minimum(slot, P["n_slots"] - 1)], 0).astype(np.int64)
+    dneg = -A.diag[row]                            # -a_rr of the entry's row
+    delta = np.where(real, P["col"].astype(np.int64) - row, 0)
+    if delta.size and np.abs(delta).max() > 32767:
+        return None
+    val = np.where(real, P["val"] / np.where(real, dneg, 1.0), 0.0)
+    out = dict(val=val, col16=delta.astype(np.int16),
+               win_shift=int(W).bit_length() - 1 if W > 1 else 0)
+    srow = P["row_of"][:n].astype(np.int64)
+    if W > 1:
+        r8 = np.zeros(P["n_slots"], np.uint8)
+        r8[:n] = (srow - (np.arange(n) // W) * W).astype(np.uint8)
+        out["row8"] = r8
+    if P["band_on"]:
+        for k in ("lo", "up"):
+            v = np.zeros(P["n_slots"])
+            v[:n] = P[k][:n] / (-A.diag[srow])
+            out[k] = v
+    return out
+
+
 def jacobi_step(A: CSR, x: np.ndarray, omega: float = 1.0) -> np.ndarray:
     x = np.ascontiguousarray(x, dtype=np.float64)
     y = np.empty(A.n)

@@ -69,7 +69,8 @@ class cme_info(C.Structure):
                 ("bytes_fmt", C.c_int64), ("rank", C.c_int32), ("nranks", C.c_int32),
                 ("row_begin", C.c_int64), ("row_end", C.c_int64), ("halo_begin", C.c_int64),
                 ("halo_end", C.c_int64), ("kernel", C.c_int32), ("tma_warps", C.c_int32),
-                ("tma_stages", C.c_int32), ("grid", C.c_int32), ("batch", C.c_int32)]
+                ("tma_stages", C.c_int32), ("grid", C.c_int32), ("batch", C.c_int32),
+                ("compact", C.c_int32)]
 
 
 class cme_packed_view(C.Structure):
@@ -78,6 +79,13 @@ class cme_packed_view(C.Structure):
                 ("batch", C.c_int32), ("pad_", C.c_int32), ("lo", f64p), ("up", f64p), ("inv_d", f64p), ("row_of", i32p),
                 ("slice_off", i64p), ("slice_w", i32p), ("val", f64p), ("col", i32p),
                 ("csr_row_ptr", i64p)]
+
+
+class cme_compact_view(C.Structure):
+    _fields_ = [("n", C.c_int64), ("n_slots", C.c_int64), ("n_slices", C.c_int64),
+                ("n_ell", C.c_int64), ("band_on", C.c_int32), ("win_shift", C.c_int32),
+                ("val", f64p), ("col16", C.POINTER(C.c_int16)), ("row8", C.POINTER(C.c_uint8)),
+                ("lo", f64p), ("up", f64p)]
 
 
 class cme_halo_view(C.Structure):
@@ -107,6 +115,7 @@ _SIGS = {
     "cme_get_permutation": [vp, i32p],
     "cme_export_packed": [vp, _p(cme_packed_view)],
     "cme_period": [vp, C.c_int64, i64p],
+    "cme_export_compact": [vp, _p(cme_compact_view)],
     "cme_comm_unique_id": [u8p],
     "cme_comm_init": [C.c_int, C.c_int, u8p, C.c_int, _p(vp)],
     "cme_comm_init_local": [C.c_int, i32p, _p(vp)],
@@ -302,6 +311,24 @@ def cme_export_packed(h):
                col=cp(v.col, v.n_ell, np.int32))
     if v.csr_row_ptr:
         out["csr_row_ptr"] = cp(v.csr_row_ptr, v.n + 1, np.int64)
+    return out
+
+
+def cme_export_compact(h):
+    """Host copies of the compact encoding (include/cme.h cme_export_compact)."""
+    v = cme_compact_view()
+    _chk(_lib.cme_export_compact(h, C.byref(v)), "cme_export_compact")
+
+    def cp(ptr, k, dt):
+        return np.ctypeslib.as_array(ptr, shape=(k,)).astype(dt, copy=True) if k and ptr else np.zeros(0, dt)
+
+    out = dict(val=cp(v.val, v.n_ell, np.float64), col16=cp(v.col16, v.n_ell, np.int16),
+               win_shift=v.win_shift)
+    if v.row8:
+        out["row8"] = cp(v.row8, v.n_slots, np.uint8)
+    if v.lo:
+        out["lo"] = cp(v.lo, v.n_slots, np.float64)
+        out["up"] = cp(v.up, v.n_slots, np.float64)
     return out
 
 
@@ -512,6 +539,9 @@ class Matrix:
 
     def packed(self):
         return cme_export_packed(self.h)
+
+    def compact(self):
+        return cme_export_compact(self.h)
 
     def close(self):
         if getattr(self, "h", None):

@@ -124,6 +124,7 @@ cme_status build_local(cme_matrix_s* h, int nranks, int rank) {
         const int32_t window = h->format == CME_FMT_DIAG_SELL ? h->popts.window : 1;
         pack_rows(h->B, r0, r1, shift, window, h->band_on, group, h->global_kmax, h->P);
     }
+    h->Cpt = Compact();   // re-encoded by device_upload / cme_export_compact
     return CME_OK;
 }
 
@@ -413,6 +414,32 @@ cme_status cme_export_packed(cme_matrix h, cme_packed_view* v) {
     if (h->format == CME_FMT_CSR) { o.val = P.csr_v.data(); o.col = P.csr_ci.data(); o.n_ell = (int64_t)P.csr_ci.size(); }
     *v = o;
     return CME_OK;
+}
+
+cme_status cme_export_compact(cme_matrix h, cme_compact_view* v) {
+    if (!h || !v) return CME_ERR_INVALID_ARG;
+    if (h->stage < 2) return CME_ERR_BAD_STATE;
+    return guarded([&] {
+        if (h->format == CME_FMT_CSR) { set_error("compact encoding: SELL formats only"); return CME_ERR_INVALID_ARG; }
+        if (!h->Cpt.valid) {
+            const int64_t own_off = h->nranks > 1 ? h->cuts[h->rank] - h->span[2 * h->rank] : 0;
+            if (!encode_compact(h->P, own_off, h->Cpt)) {
+                set_error("compact encoding: batch, window or column offsets do not qualify");
+                return CME_ERR_INVALID_ARG;
+            }
+        }
+        const Packed& P = h->P;
+        const Compact& Q = h->Cpt;
+        cme_compact_view o{};
+        o.n = P.n; o.n_slots = P.n_slots; o.n_slices = P.n_slices; o.n_ell = P.n_ell;
+        o.band_on = P.band_on; o.win_shift = Q.win_shift;
+        o.val = Q.val.data(); o.col16 = Q.col16.data();
+        o.row8 = Q.row8.empty() ? nullptr : Q.row8.data();
+        o.lo = Q.lo.empty() ? nullptr : Q.lo.data();
+        o.up = Q.up.empty() ? nullptr : Q.up.data();
+        *v = o;
+        return CME_OK;
+    });
 }
 
 cme_status cme_period(cme_matrix h, int64_t root, int64_t* out) {

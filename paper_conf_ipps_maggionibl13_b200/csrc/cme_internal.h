@@ -42,6 +42,7 @@ struct Packed {
     int64_t n = 0, n_slots = 0, n_slices = 0, n_ell = 0;
     int32_t band_on = 0, window = 1, group = 1, B = 1;
     std::vector<double> lo, up, inv_d;    // slot order, n_slots * B (member-minor)
+    std::vector<double> dneg;             // slot order: -A_rr (0 for pad slots), for the compact encoding
     std::vector<int32_t> row_of;          // slot -> local row
     std::vector<int64_t> slice_off;       // n_slices + 1
     std::vector<int32_t> slice_w;         // n_slices
@@ -57,6 +58,22 @@ bool band_rule(const Csr& A, int band_mode);
 void pack_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, int32_t window,
                bool band_on, int32_t group, int32_t global_kmax, Packed& P);
 void pack_csr_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, Packed& P);
+
+// Compact encoding of a B = 1 layout-v0 pack: the rows of
+// M = |D|^-1 O instead of O + inv_d (val_c = a_rj / (-a_rr), lo/up likewise),
+// 16-bit column offsets relative to the row (col16 = j - r), 8-bit row offsets
+// inside the rearrangement window (row8 = r - window base).  Returns false
+// (and leaves C empty) when the pack does not qualify: batch, a window that is
+// not a power of two <= 256, or an offset outside int16.  own_off: x-span
+// index of local row 0 (the column coordinates of P.col).
+struct Compact {
+    bool valid = false;                   // encoded
+    int32_t win_shift = 0;                // log2(window), 0 = no rearrangement
+    std::vector<double> val, lo, up;      // val: n_ell; lo/up: n_slots (band only)
+    std::vector<int16_t> col16;           // n_ell
+    std::vector<uint8_t> row8;            // n_slots (rearranged packs only)
+};
+bool encode_compact(const Packed& P, int64_t own_off, Compact& C);
 
 struct Device;  // device state (device.cu)
 
@@ -76,6 +93,7 @@ struct cme_matrix_s {
     int64_t period = 0;
     std::vector<double> norm_inf;  // ||A_b||_inf per batch member
     cme::Packed P;              // local packed layout (whole matrix unless distributed)
+    cme::Compact Cpt;           // its compact encoding when the device uses it (else empty)
     int32_t global_kmax = 0;
     cme_solver_opts sopts{0.0, 100, CME_STOP_DELTA_L1, 1e-10, nullptr};
     cme_report report{};

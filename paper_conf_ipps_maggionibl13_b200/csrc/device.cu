@@ -22,6 +22,7 @@
 #include "comm.h"
 #include "launch.h"
 #include "kernels_resident.cuh"
+#include "kernels_cpt.cuh"
 
 namespace cme {
 
@@ -99,7 +100,15 @@ struct Device {
     bool use_tma = false;
     int tma_ncw = 16;
     int tma_grid = 0, tma_stages = 0, tma_stage_bytes = 0, tma_off_val = 0, tma_off_col = 0, tma_contig = 0;
+    int tma_xpf = 0;
     int64_t n_tiles = 0;
+    // compact encoding (kernels_cpt.cuh): the TMA kernel streams M's rows,
+    // 16-bit column offsets and 8-bit row offsets
+    bool cpt = false;
+    double *cval = nullptr, *clo = nullptr, *cup = nullptr;
+    int16_t* col16 = nullptr;
+    uint8_t* row8 = nullptr;
+    int32_t win_shift = 0;
     // SMEM-resident persistent kernel (kernels_resident.cuh)
     bool use_res = false;
     int res_grid = 0, res_smem = 0, res_rps = 1;
@@ -358,6 +367,11 @@ static int64_t tma_stage_bytes(const Device& d, const Packed& P, int ncw, int64_
         max_nval = std::max(max_nval, P.slice_off[q1] - P.slice_off[q0]);
     }
     auto a128 = [](int64_t b) { return (b + 127) / 128 * 128; };
+    if (d.cpt) {   // [row8][lo, up][val][col16]
+        *off_val = a128(cpt_fixed_bytes(ncw, d.band, d.rearr));
+        *off_col = *off_val + a128(8 * max_nval);
+        return a128(*off_col + 2 * max_nval);
+    }
     *off_val = a128(tma_fixed_bytes(ncw, d.B, d.band, d.rearr));
     *off_col = *off_val + a128(8 * d.B * max_nval);
     return a128(*off_col + 4 * max_nval);
@@ -378,7 +392,8 @@ static cme_status configure_tma(Device& d, const Packed& P) {
     CUDA_TRY(cudaGetDevice(&dev));
     CUDA_TRY(cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
     CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-    const int stages_req = std::min(8, std::max(2, env_int("CME_TMA_STAGES", 2)));
+    const int stages_env = env_int("CME_TMA_STAGES", 0);   // 0 = auto
+    const int stages_req = stages_env > 0 ? std::min(8, std::max(2, stages_env)) : 0;
     const int force_w = env_int("CME_TMA_WARPS", 0);
     struct Shape { int ncw, stages, occ, grid; int64_t stage, off_val, off_col, n_tiles; };
     Shape best{};
@@ -387,17 +402,37 @@ static cme_status configure_tma(Device& d, const Packed& P) {
         Shape sh{};
         sh.ncw = ncw;
         sh.stage = tma_stage_bytes(d, P, ncw, &sh.off_val, &sh.off_col, &sh.n_tiles);
-        sh.stages = stages_req;
-        while (sh.stages > 2 && sh.stages * sh.stage > smem_max - 1024) --sh.stages;
-        if (sh.stages * sh.stage > smem_max - 1024) continue;   // tiles too wide for this shape
-        const int smem = (int)(sh.stages * sh.stage);
         // the attribute is process-wide per kernel: always raise it to the
         // largest size any handle may use (handles on several host threads --
         // an in-process rank group -- would otherwise lower it under each
         // other's launches: "invalid argument")
-        CUDA_TRY(tma_prepare_b(d.B, ncw, smem_max - 1024));
-        CUDA_TRY(tma_occupancy_b(d.B, ncw, smem, &sh.occ));
-        if (sh.occ < 1) continue;
+        if (d.cpt) CUDA_TRY(cpt_prepare(ncw, smem_max - 1024));
+        else CUDA_TRY(tma_prepare_b(d.B, ncw, smem_max - 1024));
+        auto occ_of = [&](int stages, int* occ) -> cudaError_t {
+            *occ = 0;
+            if (stages * sh.stage > smem_max - 1024) return cudaSuccess;
+            return d.cpt ? cpt_occupancy(ncw, (int)(stages * sh.stage), occ)
+                         : tma_occupancy_b(d.B, ncw, (int)(stages * sh.stage), occ);
+        };
+        if (stages_req > 0) {
+            sh.stages = stages_req;
+            while (sh.stages > 2 && sh.stages * sh.stage > smem_max - 1024) --sh.stages;
+            CUDA_TRY(occ_of(sh.stages, &sh.occ));
+        } else {
+            // auto: the deepest ring (<= 4 stages) that keeps the residency of
+            // 2 stages (measured on B200: 3 stages of the ~31 KB compact cfg4
+            // tiles at 2 CTAs/SM 222 vs 235 us; a 3rd stage that drops a CTA
+            // per SM loses 7% on the band-on config-5 matrices)
+            sh.stages = 2;
+            CUDA_TRY(occ_of(2, &sh.occ));
+            for (int st = 3; st <= 4 && sh.occ > 0; ++st) {
+                int o = 0;
+                CUDA_TRY(occ_of(st, &o));
+                if (o < sh.occ) break;
+                sh.stages = st;
+            }
+        }
+        if (sh.occ < 1) continue;   // tiles too wide for this shape
         sh.occ = std::max(1, std::min(sh.occ, env_int("CME_TMA_CTAS", sh.occ)));
         sh.grid = (int)std::min<int64_t>(sh.n_tiles, (int64_t)sms * sh.occ);
         if (sh.ncw * sh.occ > best.ncw * best.occ) best = sh;
@@ -413,10 +448,15 @@ static cme_status configure_tma(Device& d, const Packed& P) {
     d.tma_off_col = (int)best.off_col;
     d.tma_grid = best.grid;
     d.tma_contig = env_int("CME_TMA_CONTIG", 0) != 0;   // measured: round robin wins on cfg4 (+3%)
+    // L2 prefetch of each tile's x rows: pays when the iterate does not stay
+    // L2-resident across steps (measured: cfg4, 160 MB of x, 235 vs 241 us;
+    // cfg3a, 16 MB, 21.5 vs 20.5 us).  CME_TMA_XPF = -1 auto / 0 / 1.
+    const int xpf = env_int("CME_TMA_XPF", -1);
+    d.tma_xpf = xpf >= 0 ? xpf != 0 : (d.nx + 2) * 8 * d.B > (int64_t)48 << 20;
     d.use_tma = true;
     if (env_int("CME_VERBOSE", 0))
-        std::fprintf(stderr, "[cme] tma: B=%d warps=%d stages=%d stage_bytes=%lld occ=%d grid=%d tiles=%lld\n",
-                     d.B, best.ncw, best.stages, (long long)best.stage, best.occ, best.grid, (long long)best.n_tiles);
+        std::fprintf(stderr, "[cme] tma: B=%d compact=%d warps=%d stages=%d stage_bytes=%lld occ=%d grid=%d tiles=%lld\n",
+                     d.B, (int)d.cpt, best.ncw, best.stages, (long long)best.stage, best.occ, best.grid, (long long)best.n_tiles);
     return CME_OK;
 }
 
@@ -571,18 +611,13 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
     } else {
         UP(slice_off, P.slice_off);
         UP(slice_w, P.slice_w);
-        UP(val, P.val);
-        UP(col, P.col);
         UP(inv_d, P.inv_d);
-        if (d->band) { UP(lo, P.lo); UP(up, P.up); }
-        if (d->rearr) UP(row_of, P.row_of);
     }
     {
         std::vector<int32_t> po(h->perm.begin() + d->row_begin, h->perm.begin() + d->row_begin + d->n_own);
         UP(perm_own, po);
         if (comm) UP(perm_global, h->perm);
     }
-#undef UP
     for (int b = 0; b < 2; ++b) {
         double* base = nullptr;
         const size_t len = (size_t)(d->nx + 2) * B;
@@ -594,7 +629,32 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
                                        : (int)((d->n_slices + kWarpsPerCta - 1) / kWarpsPerCta);
     d->grid = std::max(d->grid, 1);
     if (d->format != CME_FMT_CSR && (s = configure_tma(*d, P)) != CME_OK) return fail(s);
+    // compact encoding when the TMA kernel streams a single matrix
+    // (CME_COMPACT = 0 keeps layout v0 on the TMA kernel too)
+    h->Cpt = Compact();
+    if (d->use_tma && d->B == 1 && d->format == CME_FMT_DIAG_SELL && env_int("CME_COMPACT", 1) != 0 &&
+        encode_compact(P, d->own_off, h->Cpt)) {
+        d->cpt = true;
+        d->win_shift = h->Cpt.win_shift;
+        if ((s = configure_tma(*d, P)) != CME_OK) return fail(s);   // compact stage geometry
+        if (!d->use_tma) d->cpt = false;
+    }
     if ((s = configure_resident(*d, P, comm != nullptr || h->nranks > 1)) != CME_OK) return fail(s);
+    if (d->format != CME_FMT_CSR) {
+        if (d->cpt) {
+            UP(cval, h->Cpt.val);
+            UP(col16, h->Cpt.col16);
+            if (d->band) { UP(clo, h->Cpt.lo); UP(cup, h->Cpt.up); }
+            if (d->rearr) UP(row8, h->Cpt.row8);
+        }
+        if (!d->cpt || d->use_res) {   // layout v0 arrays (register / resident kernels)
+            UP(val, P.val);
+            UP(col, P.col);
+            if (d->band) { UP(lo, P.lo); UP(up, P.up); }
+            if (d->rearr) UP(row_of, P.row_of);
+        }
+    }
+#undef UP
     d->part_blocks = std::max(std::max(d->grid, d->res_grid), grid_for(d->n_own));
     if ((s = d->alloc(d->partials, (size_t)d->part_blocks * B * kPartials)) != CME_OK) return fail(s);
     if ((s = d->alloc(d->gather, (size_t)d->nranks * B * 8)) != CME_OK) return fail(s);
@@ -863,8 +923,17 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
     if (d.format == CME_FMT_CSR) {
         CUDA_TRY(check ? launch_ex(csr_step_kernel<true>, dim3(d.grid), dim3(kCta), 0, pdl, s, a)
                        : launch_ex(csr_step_kernel<false>, dim3(d.grid), dim3(kCta), 0, pdl, s, a));
+    } else if (d.use_tma && d.cpt) {
+        a.val = d.cval;
+        a.lo = d.clo;
+        a.up = d.cup;
+        a.col = nullptr;
+        a.row_of = nullptr;
+        CptArgs K{TmaArgs{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col, d.tma_contig, d.tma_xpf},
+                  d.col16, d.row8, d.win_shift};
+        CUDA_TRY(launch_cpt(K, d.tma_ncw, d.tma_grid, d.tma_stages * d.tma_stage_bytes, d.band, d.rearr, check, pdl, s));
     } else if (d.use_tma) {
-        TmaArgs T{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col, d.tma_contig};
+        TmaArgs T{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col, d.tma_contig, d.tma_xpf};
         const int smem = d.tma_stages * d.tma_stage_bytes;
         cudaError_t e;
         switch (d.B) {
@@ -1252,6 +1321,13 @@ void device_describe(const Device* d, cme_info* f) {
     f->tma_warps = d->use_tma ? d->tma_ncw : 0;
     f->tma_stages = d->use_tma ? d->tma_stages : 0;
     f->grid = d->use_res ? d->res_grid : d->step_grid();
+    f->compact = d->cpt ? 1 : 0;
+    if (d->cpt) {   // bytes a plain step streams in the compact encoding (no inv_d)
+        const int64_t n_ell = f->n_ell, nl = d->n_own, slots = f->n_slots, sl = f->n_slices;
+        f->bytes_fmt = 10 * n_ell + (d->rearr ? nl : 0) + (d->band ? 16 * nl : 0) + 12 * sl + 16 * nl;
+        f->packed_bytes = 10 * n_ell + (d->rearr ? slots : 0) + (d->band ? 16 * slots : 0) + 8 * slots + 12 * sl + 8 +
+                          (d->use_res ? f->packed_bytes : 0);
+    }
 }
 
 cme_status device_spmv(cme_matrix_s* h, const double* x, double* y) {

@@ -90,6 +90,7 @@ void pack_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, int32_t 
     P.lo.assign((size_t)P.n_slots * nb, 0.0);
     P.up.assign((size_t)P.n_slots * nb, 0.0);
     P.inv_d.assign((size_t)P.n_slots * nb, 0.0);
+    P.dneg.assign((size_t)P.n_slots * nb, 0.0);
 #pragma omp parallel for schedule(dynamic, 256)
     for (int64_t s = 0; s < P.n_slots; ++s) {
         const int64_t q = s >> 5, lane = s & 31;
@@ -101,7 +102,10 @@ void pack_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, int32_t 
             continue;
         }
         const int64_t l = P.row_of[s], r = r0 + l;
-        for (int32_t b = 0; b < nb; ++b) P.inv_d[(size_t)s * nb + b] = 1.0 / (-A.d[(size_t)r * nb + b]);
+        for (int32_t b = 0; b < nb; ++b) {
+            P.inv_d[(size_t)s * nb + b] = 1.0 / (-A.d[(size_t)r * nb + b]);
+            P.dneg[(size_t)s * nb + b] = -A.d[(size_t)r * nb + b];
+        }
         if (band_on) {
             const int64_t pl = r > 0 ? entry(A, r, r - 1) : -1, pu = r + 1 < A.n ? entry(A, r, r + 1) : -1;
             for (int32_t b = 0; b < nb; ++b) {
@@ -119,6 +123,53 @@ void pack_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, int32_t 
         }
         for (; t < w; ++t) cq[32 * t] = (int32_t)(r - col_shift);
     }
+}
+
+bool encode_compact(const Packed& P, int64_t own_off, Compact& C) {
+    C = Compact();
+    if (P.B != 1 || P.n_slices == 0 || P.dneg.size() != (size_t)P.n_slots) return false;
+    int32_t ws = 0;
+    if (P.window > 1) {
+        if (P.window > 256 || (P.window & (P.window - 1))) return false;
+        while ((1 << ws) < P.window) ++ws;
+    }
+    const int64_t n = P.n;
+    // every stored offset j - r must fit int16 (pad entries hold their own row: 0)
+    bool ok = true;
+#pragma omp parallel for schedule(dynamic, 256) reduction(&& : ok)
+    for (int64_t s = 0; s < n; ++s) {
+        const int64_t q = s >> 5, e0 = P.slice_off[q] + (s & 31), r = own_off + P.row_of[s];
+        for (int32_t t = 0; t < P.slice_w[q]; ++t) {
+            const int64_t dlt = (int64_t)P.col[e0 + 32 * t] - r;
+            ok = ok && dlt >= INT16_MIN && dlt <= INT16_MAX;
+        }
+    }
+    if (!ok) return false;
+    C.valid = true;
+    C.win_shift = ws;
+    C.val.assign(P.n_ell, 0.0);
+    C.col16.assign(P.n_ell, 0);
+    if (P.band_on) {
+        C.lo.assign(P.n_slots, 0.0);
+        C.up.assign(P.n_slots, 0.0);
+    }
+    if (ws) C.row8.assign(P.n_slots, 0);
+#pragma omp parallel for schedule(dynamic, 256)
+    for (int64_t s = 0; s < n; ++s) {
+        const int64_t q = s >> 5, e0 = P.slice_off[q] + (s & 31), l = P.row_of[s], r = own_off + l;
+        const double dn = P.dneg[s];
+        for (int32_t t = 0; t < P.slice_w[q]; ++t) {
+            const int64_t e = e0 + 32 * t;
+            C.val[e] = P.val[e] / dn;
+            C.col16[e] = (int16_t)((int64_t)P.col[e] - r);
+        }
+        if (P.band_on) {
+            C.lo[s] = P.lo[s] / dn;
+            C.up[s] = P.up[s] / dn;
+        }
+        if (ws) C.row8[s] = (uint8_t)(l - ((s >> ws) << ws));
+    }
+    return true;
 }
 
 void pack_csr_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, Packed& P) {

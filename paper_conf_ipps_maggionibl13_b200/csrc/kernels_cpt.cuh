@@ -1,0 +1,214 @@
+// TMA-staged step kernel over the COMPACT encoding of layout v0 (B = 1;
+// DESIGN.md sec. 5b).  Same operator as sell_tma_kernel -- y = M_omega x with
+// M = |D|^-1 O (eq. 8, R1) -- but the packed matrix is stored as the
+// rows of M itself, so a plain step streams
+//   val_c  8 B / ELL slot   (a_rj / (-a_rr), one IEEE division at pack time)
+//   col16  2 B / ELL slot   (j - r: the RCM / DFS bands of the CME networks
+//                            keep every offset inside int16)
+//   row8   1 B / row        (r - window base, rearranged packs only)
+//   lo_c, up_c              (band only)
+// instead of 12 B / slot + 12 B / row: inv_d is read only by CHECK steps (the
+// paper residual needs |a_rr|, R21) and by transient steps.  The arithmetic
+// order is the plain kernel's (gathers in t order, band term first), with the
+// division moved from the row sum to the entries: per-row relative difference
+// <= (k + 2) u, inside the per-SpMV bound of DESIGN.md sec. 6.
+#pragma once
+#include "kernels_tma.cuh"
+
+namespace cme {
+
+struct CptArgs {
+    TmaArgs T;            // T.a.val / lo / up = the compact arrays, T.a.inv_d = 1/(-a_rr)
+    const int16_t* col16;
+    const uint8_t* row8;
+    int32_t win_shift;    // log2(rearrangement window), 0 = identity slot -> row
+};
+
+// Stage layout: [row8 if REARR][lo, up if BAND][val][col16] for NCW*32 slots.
+__host__ __device__ inline int cpt_fixed_bytes(int ncw, bool band, bool rearr) {
+    return ncw * 32 * ((rearr ? 1 : 0) + (band ? 16 : 0));
+}
+
+template <int NCW, bool BAND, bool REARR>
+__device__ __noinline__ void cpt_issue_call(unsigned char* st, uint64_t* bar, const int64_t* slice_off,
+                                            int64_t slice_end, const uint8_t* row8, const double* lo,
+                                            const double* up, const double* val, const int16_t* col16,
+                                            int off_val, int off_col, int64_t tile, uint64_t pol) {
+    constexpr int kSlots = NCW * 32;
+    constexpr int kOffRow = 0, kOffLo = REARR ? kSlots : 0, kOffUp = kOffLo + 8 * kSlots;
+    const int64_t q0 = tile * NCW;
+    const int64_t q1 = min(q0 + NCW, slice_end);
+    const int64_t e0 = slice_off[q0], e1 = slice_off[q1];
+    const uint32_t slots = (uint32_t)(q1 - q0) * 32u;
+    const uint32_t nval = (uint32_t)(e1 - e0);
+    uint32_t bytes = nval * 10u;
+    if (REARR) bytes += slots;
+    if (BAND) bytes += slots * 16u;
+    mbar_expect_tx(bar, bytes);
+    if (REARR) bulk_g2s(st + kOffRow, row8 + q0 * 32, slots, bar, pol);
+    if (BAND) {
+        bulk_g2s(st + kOffLo, lo + q0 * 32, slots * 8u, bar, pol);
+        bulk_g2s(st + kOffUp, up + q0 * 32, slots * 8u, bar, pol);
+    }
+    if (nval) {
+        bulk_g2s(st + off_val, val + e0, nval * 8u, bar, pol);
+        bulk_g2s(st + off_col, col16 + e0, nval * 2u, bar, pol);
+    }
+}
+
+template <int NCW, bool BAND, bool REARR>
+__device__ __forceinline__ void cpt_issue(const CptArgs& K, unsigned char* smem, uint64_t* full, int64_t tile, int s,
+                                          uint64_t pol) {
+    const StepArgs& a = K.T.a;
+    if (K.T.xpf) {
+        const int64_t r0 = tile * NCW * 32, r1 = min(r0 + NCW * 32, a.n_rows);
+        if (r1 > r0) prefetch_l2(a.x + a.own_off + r0, (uint64_t)(r1 - r0) * 8);
+    }
+    cpt_issue_call<NCW, BAND, REARR>(smem + (size_t)s * K.T.stage_bytes, &full[s], a.slice_off, a.slice_end, K.row8,
+                                     a.lo, a.up, a.val, K.col16, K.T.off_val, K.T.off_col, tile, pol);
+}
+
+// Sum over the W entries of one slot: all gathers x[r + dj] first, then the
+// FMAs in t order.
+template <int W>
+__device__ __forceinline__ void ell_row_cpt(const int16_t* scol, const double* sval, const double* xr, double& acc) {
+    double xv[W];
+#pragma unroll
+    for (int u = 0; u < W; ++u) xv[u] = __ldg(xr + scol[32 * u]);
+#pragma unroll
+    for (int u = 0; u < W; ++u) acc = fma(sval[32 * u], xv[u], acc);
+}
+
+// Row epilogue on M's rows: s = (lo_c x_{r-1} + up_c x_{r+1}) + acc = (M x)_r.
+template <bool BAND, bool CHECK>
+__device__ __forceinline__ void finish_row_cpt(const StepArgs& a, int64_t slot, int64_t r, double* yo, double acc,
+                                               double lo, double up, CheckAcc<1>& ck, const RowX<1, BAND>& X) {
+    const double s = BAND ? fma(lo, X.xl[0], up * X.xu[0]) + acc : acc;
+    const double xr = X.xr[0];
+    const bool damp = a.omega != 1.0;
+    double y = damp ? fma(1.0 - a.omega, xr, a.omega * s) : s;
+    if (a.unif_lam_inv != 0.0) {   // transient: x + (A x)_r / Lambda, (A x)_r = |a_rr| (s - x_r)
+        const double id = __ldg(a.inv_d + slot);
+        y = fma(a.unif_lam_inv, (s - xr) / id, xr);
+        double* ac = a.acc + a.own_off + r;
+        *ac = fma(a.acc_w, xr, *ac);
+    }
+    double x = (damp || CHECK) ? xr : 0.0;
+    if (a.pre_scale != nullptr) {
+        const double sc = a.pre_scale[0];
+        y *= sc;
+        x *= sc;
+    }
+    if (CHECK) ck.add(0, y, x, __ldg(a.inv_d + slot));
+    yo[r] = y;
+    for (int p = 0; p < a.npush; ++p)   // halo rows straight into the peer's buffer
+        if (r >= a.push_lo[p] && r < a.push_hi[p]) a.push_y[p][r] = y;
+}
+
+template <int NCW, bool BAND, bool REARR, bool CHECK>
+__global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBlocks)
+    sell_cpt_kernel(const CptArgs K) {
+    constexpr int kConsumers = NCW, kTileSlices = NCW, kSlots = NCW * 32;
+    constexpr int kOffRow = 0, kOffLo = REARR ? kSlots : 0, kOffUp = kOffLo + 8 * kSlots;
+    const TmaArgs& T = K.T;
+    const StepArgs& a = T.a;
+    pdl_trigger();
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ uint64_t full[8], empty[8];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int S = T.stages;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < S; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], kConsumers);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    const bool producer = warp == kConsumers && lane == 0;
+    uint64_t pol = 0;
+    int64_t t_first, my_tiles, t_stride;
+    tma_tile_range(T, &t_first, &my_tiles, &t_stride);
+    const int64_t t_end = t_first + my_tiles * t_stride;
+    const int pro = (int)(my_tiles < (int64_t)S ? my_tiles : (int64_t)S);
+    if (producer) {   // the matrix is constant: prefetch while the previous step drains
+        pol = evict_first_policy();
+        for (int i = 0; i < pro; ++i) cpt_issue<NCW, BAND, REARR>(K, smem, full, t_first + (int64_t)i * t_stride, i, pol);
+    }
+    pdl_wait();
+    if (a.stop != nullptr && *a.stop) {
+        if (producer)
+            for (int i = 0; i < pro; ++i) mbar_wait(&full[i], 0u);
+        return;
+    }
+    CheckAcc<1> ck;
+    if (warp == kConsumers) {
+        if (lane == 0 && my_tiles > pro) {
+            int s = 0;
+            uint32_t phase = 1;
+            for (int64_t tile = t_first + (int64_t)pro * t_stride; tile < t_end; tile += t_stride) {
+                mbar_wait(&empty[s], phase ^ 1u);
+                cpt_issue<NCW, BAND, REARR>(K, smem, full, tile, s, pol);
+                if (++s == S) { s = 0; phase ^= 1u; }
+            }
+        }
+    } else {
+        const double* xo = a.x + a.own_off;
+        double* yo = a.y + a.own_off;
+        int s = 0;
+        uint32_t phase = 0;
+        for (int64_t tile = t_first; tile < t_end; tile += t_stride) {
+            const int64_t q0 = tile * kTileSlices;
+            const int64_t q = q0 + warp;
+            const unsigned char* st = smem + (size_t)s * T.stage_bytes;
+            int w = 0;
+            int64_t loff = 0;
+            if (q < a.slice_end) {
+                w = __ldg(a.slice_w + q);
+                loff = __ldg(a.slice_off + q) - __ldg(a.slice_off + q0);
+            }
+            mbar_wait(&full[s], phase);
+            const int64_t slot = q * 32 + lane;
+            if (q < a.slice_end && slot < a.n_rows) {
+                const int ls = warp * 32 + lane;
+                const double* sval = reinterpret_cast<const double*>(st + T.off_val) + loff + lane;
+                const int16_t* scol = reinterpret_cast<const int16_t*>(st + T.off_col) + loff + lane;
+                const int64_t r = REARR ? ((slot >> K.win_shift) << K.win_shift) + st[kOffRow + ls] : slot;
+                RowX<1, BAND> X;
+                X.load(xo, r);
+                const double* xr = xo + r;
+                double acc = 0.0;
+                switch (w) {   // warp-uniform exact widths
+                    case 0: break;
+                    case 1: ell_row_cpt<1>(scol, sval, xr, acc); break;
+                    case 2: ell_row_cpt<2>(scol, sval, xr, acc); break;
+                    case 3: ell_row_cpt<3>(scol, sval, xr, acc); break;
+                    case 4: ell_row_cpt<4>(scol, sval, xr, acc); break;
+                    case 5: ell_row_cpt<5>(scol, sval, xr, acc); break;
+                    case 6: ell_row_cpt<6>(scol, sval, xr, acc); break;
+                    case 7: ell_row_cpt<7>(scol, sval, xr, acc); break;
+                    case 8: ell_row_cpt<8>(scol, sval, xr, acc); break;
+                    default:
+                        for (int t0 = 0; t0 < w; t0 += 8) {
+                            double xv[8];
+#pragma unroll
+                            for (int u = 0; u < 8; ++u)
+                                if (t0 + u < w) xv[u] = __ldg(xr + scol[32 * (t0 + u)]);
+#pragma unroll
+                            for (int u = 0; u < 8; ++u)
+                                if (t0 + u < w) acc = fma(sval[32 * (t0 + u)], xv[u], acc);
+                        }
+                }
+                const double lo = BAND ? reinterpret_cast<const double*>(st + kOffLo)[ls] : 0.0;
+                const double up = BAND ? reinterpret_cast<const double*>(st + kOffUp)[ls] : 0.0;
+                finish_row_cpt<BAND, CHECK>(a, slot, r, yo, acc, lo, up, ck, X);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);
+            if (++s == S) { s = 0; phase ^= 1u; }
+        }
+    }
+    if (CHECK) cta_check_partials<NCW + 1, 1>(ck, a.partials);
+}
+
+}  // namespace cme

@@ -33,6 +33,7 @@ struct TmaArgs {
     int32_t off_val;      // byte offsets inside a stage
     int32_t off_col;
     int32_t contig;       // 1: CTA b takes a contiguous run of tiles, 0: round robin (default, CME_TMA_CONTIG)
+    int32_t xpf;          // 1: L2-prefetch a tile's own x rows when its matrix tile is issued (CME_TMA_XPF)
 };
 
 // Tile sequence of one CTA: contiguous runs keep consecutive tiles -- whose x
@@ -77,6 +78,18 @@ __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
         "r"(parity)
         : "memory");
 }
+// L2 prefetch of [p, p + bytes) by the TMA engine (16-byte granules).  The
+// iterate a tile's rows will gather is first touched by the tile itself (the
+// RCM/DFS bands keep every gather within a few tiles of its row), so without
+// it those first touches are DRAM round trips on the consumers' critical
+// path.  L2 is the point of coherence: prefetching a line the previous step
+// is still writing cannot produce a stale read.
+__device__ __forceinline__ void prefetch_l2(const void* p, uint64_t bytes) {
+    const uint64_t a = reinterpret_cast<uint64_t>(p) & ~uint64_t(15);
+    const uint64_t e = (reinterpret_cast<uint64_t>(p) + bytes + 15) & ~uint64_t(15);
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a), "r"((uint32_t)(e - a)) : "memory");
+}
+
 // 1-D bulk copy global -> shared, completion counted on mbarrier `b`
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* b,
                                          uint64_t pol) {
@@ -158,6 +171,10 @@ __device__ __forceinline__ void tma_issue(const TmaArgs& T, unsigned char* smem,
                                           uint64_t pol) {
     const StepArgs& a = T.a;
     unsigned char* st = smem + (size_t)s * T.stage_bytes;
+    if (T.xpf) {
+        const int64_t r0 = tile * NCW * 32, r1 = min(r0 + NCW * 32, a.n_rows);
+        if (r1 > r0) prefetch_l2(a.x + (a.own_off + r0) * B, (uint64_t)(r1 - r0) * 8 * B);
+    }
     if (CME_TMA_PRODUCER_INLINE)
         tma_issue_body<NCW, B, BAND, REARR>(st, &full[s], a.slice_off, a.slice_end, a.inv_d, a.row_of, a.lo, a.up,
                                             a.val, a.col, T.off_val, T.off_col, tile, pol);

@@ -41,6 +41,12 @@ cudaError_t tma_occupancy(int ncw, int smem, int* blocks_per_sm);
 }  // namespace cme
 
 namespace cme {
+struct CptArgs;
+// compact-encoding TMA step kernel (step_cpt.cu, B = 1)
+cudaError_t launch_cpt(const CptArgs& K, int ncw, int grid, int smem, bool band, bool rearr, bool check, bool pdl,
+                       cudaStream_t s);
+cudaError_t cpt_prepare(int ncw, int smem);
+cudaError_t cpt_occupancy(int ncw, int smem, int* blocks_per_sm);
 struct ResArgs;
 // SMEM-resident persistent Jacobi kernel (resident.cu)
 cudaError_t resident_prepare(int smem);

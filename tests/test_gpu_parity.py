@@ -76,6 +76,59 @@ def test_spmv_wide_rates_and_ragged(cme, oracle_mod):
             assert_spmv_close(m.spmv(x), oracle_mod.jacobi_step(A, x, 1.0))
 
 
+@pytest.mark.parametrize("net", NETS, ids=lambda n: n.name)
+@pytest.mark.parametrize("layout", LAYOUTS[:5], ids=lambda l: "-".join(map(str, l)))
+def test_spmv_parity_compact_tma(cme, oracle_mod, monkeypatch, net, layout):
+    """Every SELL layout of every network through the TMA kernel on the compact
+    encoding (forced: these matrices are below the auto size), plus the
+    check partials: one solve of 2 blocks against the oracle."""
+    monkeypatch.setenv("CME_TMA", "1")
+    monkeypatch.setenv("CME_RESIDENT", "0")
+    m, A = build(cme, oracle_mod, net, *layout)
+    assert m.info().kernel == 1 and m.info().compact == 1
+    for omega in (1.0, 0.9):
+        m.set_opts(omega=omega)
+        x = W.random_start(A.n, 11)
+        assert_spmv_close(m.spmv(x), oracle_mod.jacobi_step(A, x, omega))
+    m.set_opts(omega=0.9, check_every=50, stag_tol=0.0, stop=cme.CME_STOP_PAPER_RESID)
+    p, st, it = m.solve(tol=0.0, max_iter=100)
+    ref = oracle_mod.jacobi_solve(A, omega=0.9, tol=0.0, check_every=50, max_iter=100, stag_tol=0.0)
+    assert it == ref.iters and np.abs(p - ref.p).sum() <= 1e-12
+    rep = m.report()
+    assert rep.delta == pytest.approx(ref.delta, rel=1e-9) and rep.resid == pytest.approx(ref.resid, rel=1e-9)
+
+
+@pytest.mark.parametrize("compact", ["1", "0"])
+def test_transient_on_tma_kernels(cme, oracle_mod, monkeypatch, compact):
+    """Uniformization (NEXT-3) through the TMA kernel on both encodings: the
+    compact one rebuilds (A x)_r = |a_rr| ((M x)_r - x_r) from M's rows."""
+    monkeypatch.setenv("CME_TMA", "1")
+    monkeypatch.setenv("CME_RESIDENT", "0")
+    monkeypatch.setenv("CME_COMPACT", compact)
+    states, r, c, v = oracle_mod.enumerate_network(W.toggle_switch(50))
+    A = oracle_mod.ingest(len(states), r, c, v)
+    m = cme.Matrix(A.n, r, c, v).reorder(ORD["dfs"]).pack()
+    assert m.info().compact == int(compact)
+    for t in (0.05, 0.5):
+        pt, terms = m.transient(t)
+        ref, _, _ = oracle_mod.transient(A, t)
+        assert np.abs(pt - ref).sum() <= 1e-12
+
+
+def test_compact_fallback_wide_offsets(cme, oracle_mod, monkeypatch):
+    """A transition spanning > 32767 states has no int16 offset: the TMA kernel
+    keeps layout v0 (compact = 0) and stays exact."""
+    monkeypatch.setenv("CME_TMA", "1")
+    monkeypatch.setenv("CME_RESIDENT", "0")
+    n = 70000
+    r, c, v = W.banded_markov(n, 6, 40000, True, seed=9)
+    A = oracle_mod.ingest(n, r, c, v)
+    m = cme.Matrix(n, r, c, v).pack()
+    assert m.info().kernel == 1 and m.info().compact == 0
+    x = W.random_start(n, 5)
+    assert_spmv_close(m.spmv(x), oracle_mod.jacobi_step(A, x, 1.0))
+
+
 def solve_both(cme, oracle_mod, m, A, omega, tol, C=100, max_iter=200000, p0=None, stag=1e-10):
     m.set_opts(omega=omega, check_every=C, stag_tol=stag)
     p, st, it = m.solve(p0=p0, tol=tol, max_iter=max_iter)
@@ -253,6 +306,7 @@ def test_nccl_one_rank_distributed_path(cme, oracle_mod):
 
 @pytest.mark.parametrize("knobs", [{"CME_TMA": "0", "CME_RESIDENT": "0"}, {"CME_TMA": "1", "CME_RESIDENT": "0"},
                                    {"CME_TMA": "1", "CME_TMA_WARPS": "8", "CME_RESIDENT": "0"},
+                                   {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_COMPACT": "0"},
                                    {"CME_RESIDENT": "1"}],
                          ids=lambda k: ",".join(f"{a}={b}" for a, b in k.items()))
 @pytest.mark.parametrize("net,order,omega", [(W.toggle_switch(70), "rcm", 0.9), (W.schnakenberg(120), "none", 1.0),
@@ -270,6 +324,8 @@ def test_every_step_kernel(cme, oracle_mod, monkeypatch, knobs, net, order, omeg
     f = m.info()
     expect = 3 if knobs.get("CME_RESIDENT") == "1" else 1 if knobs["CME_TMA"] == "1" else 0
     assert f.kernel == expect
+    # the TMA kernel streams the compact encoding unless CME_COMPACT=0
+    assert f.compact == (1 if expect == 1 and knobs.get("CME_COMPACT") != "0" else 0)
     m.set_opts(omega=omega, check_every=7, stag_tol=0.0)
     x = W.random_start(A.n, 21)
     assert_spmv_close(m.spmv(x), oracle_mod.jacobi_step(A, x, omega))
@@ -291,7 +347,7 @@ def test_cfg4_full_size_parity(cme, oracle_mod):
     net = W.config_network("cfg4_toggle_20m")
     m = cme.Matrix.from_network(net).reorder(cme.CME_ORDER_RCM).pack()
     info = m.info()
-    assert info.n == 20015468 and info.nnz == 120042194 and info.kernel == 1
+    assert info.n == 20015468 and info.nnz == 120042194 and info.kernel == 1 and info.compact == 1
     A = oracle_mod.network_csr(net)
     x = W.random_start(A.n, 17)
     m.set_opts(omega=1.0)

@@ -130,6 +130,18 @@ def test_pack_bit_exact(oracle_mod, net, order, window, band, fmt):
         assert got[key] == ref[key], key
     for key in ("lo", "up", "inv_d", "row_of", "slice_off", "slice_w", "val", "col"):
         assert got[key].dtype == ref[key].dtype and got[key].tobytes() == ref[key].tobytes(), key
+    # compact encoding: bit-exact too, or rejected by both
+    refc = oracle_mod.compact(oracle_mod.permute(A, perm), ref)
+    if refc is None:
+        with pytest.raises(cme.CmeError):
+            m.compact()
+    else:
+        gotc = m.compact()
+        assert gotc["win_shift"] == refc["win_shift"]
+        assert set(gotc) == set(refc)
+        for key in refc:
+            if key != "win_shift":
+                assert gotc[key].dtype == refc[key].dtype and gotc[key].tobytes() == refc[key].tobytes(), key
 
 
 def test_given_permutation_bit_exact(oracle_mod):
@@ -162,6 +174,11 @@ def test_cfg2_toggle_full_host_parity(oracle_mod):
     got = m.packed()
     for key in ("row_of", "slice_off", "slice_w", "val", "col", "inv_d", "lo", "up"):
         assert got[key].tobytes() == ref[key].tobytes(), key
+    refc = oracle_mod.compact(oracle_mod.permute(A, oracle_mod.order_rcm(A)), ref)
+    gotc = m.compact()
+    for key in refc:
+        if key != "win_shift":
+            assert gotc[key].tobytes() == refc[key].tobytes(), key
 
 
 def test_error_paths():

@@ -195,3 +195,55 @@ def test_band_rule_threshold(oracle_mod):
         cnt = int(((A.col == i - 1) | (A.col == i + 1)).sum())
         P = oracle_mod.pack(A)
         assert P["band_on"] == (3 * cnt >= 2 * (2 * n - 2))
+
+
+@pytest.mark.parametrize("order", ["none", "rcm"])
+@pytest.mark.parametrize("window,band", [(256, "auto"), (1, "never"), (64, "always")])
+def test_compact_decodes_to_jacobi_matrix(oracle_mod, order, window, band):
+    """Compact encoding pinned to the method, not to its own
+    formula: decoding (row = window base + row8, col = row + col16) must give
+    exactly the off-diagonal pattern of A; the decoded M applied to x must equal
+    the oracle's C Jacobi step (divide last, eq. 8) within (k+2)u; and
+    |d|^T M = |d|^T (the column-sum identity of the generator)."""
+    net = W.toggle_switch(30)
+    states, r, c, v = oracle_mod.enumerate_network(net)
+    A0 = oracle_mod.ingest(len(states), r, c, v)
+    A = A0 if order == "none" else oracle_mod.permute(A0, oracle_mod.order_rcm(A0))
+    P = oracle_mod.pack(A, window=window, band=band)
+    Q = oracle_mod.compact(A, P)
+    assert Q is not None and Q["win_shift"] == (window.bit_length() - 1 if window > 1 else 0)
+    n = A.n
+    rows, cols, vals = [], [], []
+    for s in range(n):
+        q, lane = divmod(s, 32)
+        rr = (s >> Q["win_shift"] << Q["win_shift"]) + int(Q["row8"][s]) if window > 1 else s
+        for t in range(P["slice_w"][q]):
+            e = P["slice_off"][q] + 32 * t + lane
+            if Q["val"][e] != 0.0:
+                rows.append(rr); cols.append(rr + int(Q["col16"][e])); vals.append(Q["val"][e])
+        if P["band_on"]:
+            for dj, key in ((-1, "lo"), (1, "up")):
+                if Q[key][s] != 0.0:
+                    rows.append(rr); cols.append(rr + dj); vals.append(Q[key][s])
+    M = sp.csr_matrix((vals, (rows, cols)), shape=(n, n))
+    ref = sp.csr_matrix((A.val, A.col, A.row_ptr), shape=(n, n))
+    assert M.nnz == A.nnz_offdiag
+    assert np.array_equal(M.indptr, ref.indptr) and np.array_equal(M.indices, ref.indices)
+    x = np.random.default_rng(3).random(n)
+    y_ref = oracle_mod.jacobi_step(A, x, omega=1.0)
+    k = np.diff(A.row_ptr)
+    assert np.all(np.abs(M @ x - y_ref) <= (k + 2) * 2.0 ** -53 * y_ref + 1e-300)
+    dabs = -A.diag
+    assert np.allclose(M.T @ dabs, dabs, rtol=1e-14, atol=0)
+
+
+def test_compact_rejects_wide_offsets_and_windows(oracle_mod):
+    """A transition spanning more than 32767 states, or a non-power-of-two
+    window, has no compact encoding."""
+    n = 40000
+    edges = [(j, j + 1) for j in range(n - 1)] + [(j + 1, j) for j in range(n - 1)] + [(0, n - 1)]
+    A = csr_from_edges(oracle_mod, n, edges)
+    assert oracle_mod.compact(A, oracle_mod.pack(A, window=256)) is None
+    B = csr_from_edges(oracle_mod, 100, [(j, j + 1) for j in range(99)] + [(j + 1, j) for j in range(99)])
+    assert oracle_mod.compact(B, oracle_mod.pack(B, window=96)) is None
+    assert oracle_mod.compact(B, oracle_mod.pack(B, window=128)) is not None
