@@ -129,6 +129,8 @@ class ClockSampler:
 
 
 def kernel_name(info):
+    if info.kernel == 1 and info.compact == 2:
+        return f"sell_vi_kernel<{info.tma_warps}>"
     if info.kernel == 1 and info.compact:
         return f"sell_cpt_kernel<{info.tma_warps}>"
     return {0: "sell_step_kernel", 1: f"sell_tma_kernel<{info.tma_warps}>", 2: "csr_step_kernel",
@@ -343,11 +345,16 @@ def main():
     t_iter = sec / iters
     achieved = info.bytes_alg / t_iter / 1e9        # algorithmic bytes per launch / launch time
     fmt_gbs = info.bytes_fmt * world / t_iter / 1e9 if world == 1 else None
-    compact_note = ("compact encoding (DESIGN.md sec. 5b): the kernel streams the rows of M = |D|^-1 O with "
-                    "int16 column and uint8 row offsets, 10 B per ELL slot + 17 B per row (format_bytes_per_launch) "
-                    "instead of the model's 12 B per non-zero + 16 B per row; frac > 1 therefore means fewer bytes "
-                    "than the SURVEY 8(d) byte model, not a faster-than-HBM kernel -- format_frac is the kernel's "
-                    "own DRAM efficiency") if info.compact else None
+    compact_note = {
+        1: "compact encoding (DESIGN.md sec. 5b): the kernel streams the rows of M = |D|^-1 O with int16 column "
+           "and uint8 row offsets, 10 B per ELL slot + 17 B per row (format_bytes_per_launch)",
+        2: "value-indexed compact encoding (DESIGN.md sec. 5c): 16-bit indices into a shared-memory dictionary of "
+           "the distinct rates + int16 column offsets (4 B per ELL slot) + inv_d and a uint8 row offset per row "
+           "(format_bytes_per_launch)"}.get(info.compact)
+    if compact_note:
+        compact_note += ("; the SURVEY 8(d) model counts 12 B per non-zero + 16 B per row, so frac > 1 means fewer "
+                         "bytes than that model, not a faster-than-HBM kernel -- format_frac is the kernel's own "
+                         "DRAM efficiency")
 
     # e2e: the public solve call with pinned host buffers, H2D + D2H inside the timed region
     p0 = torch.empty(n * B, dtype=torch.float64, pin_memory=True)
@@ -426,7 +433,8 @@ def main():
                          "format_bytes_per_launch": info.bytes_fmt,
                          "format_gbs": round(fmt_gbs, 1) if fmt_gbs else None,
                          "format_frac": round(fmt_gbs / peak, 4) if fmt_gbs else None,
-                         "encoding": "compact" if info.compact else "layout v0", "note": compact_note,
+                         "encoding": {0: "layout v0", 1: "compact", 2: "value-indexed compact"}[info.compact],
+                         "note": compact_note,
                          "launch_time_us": round(t_iter * 1e6, 3),
                          "launch_time_note": "timed-region time / step-kernel launches (includes the 2 tiny "
                                              "check kernels per 100 steps and launch gaps: conservative)"},

@@ -249,6 +249,15 @@ typedef struct cme_compact_view {
     const uint8_t* row8;     /* [n_slots], NULL when win_shift == 0          */
     const double* lo;        /* [n_slots], NULL when the band is off         */
     const double* up;        /* [n_slots], NULL when the band is off         */
+    /* Value-indexed form (CSR-VI style): dict = the distinct
+     * values of layout v0's val (all n_ell entries, pads included) and, band on,
+     * lo/up, ascending; vidx[e] / loi[s] / upi[s] = their positions in dict.
+     * n_dict = 0 and NULL pointers when there are more than 65536. */
+    int64_t n_dict;
+    const double* dict;      /* [n_dict]                                     */
+    const uint16_t* vidx;    /* [n_ell]                                      */
+    const uint16_t* loi;     /* [n_slots], NULL when the band is off         */
+    const uint16_t* upi;     /* [n_slots], NULL when the band is off         */
 } cme_compact_view;
 cme_status cme_export_compact(cme_matrix h, cme_compact_view* v);
 

@@ -259,6 +259,22 @@ def compact(A: CSR, P: dict):
     return out
 
 
+def value_index(P: dict):
+    """Value-indexed form (the CSR-VI idea) of a layout-v0
+    pack P: dict = the distinct stored values of P's val (every entry, pads
+    included) and, band on, lo/up, ascending; vidx / loi / upi = positions
+    in dict.  None when there are more than 65536 distinct values."""
+    parts = [P["val"]] + ([P["lo"], P["up"]] if P["band_on"] else [])
+    d = np.unique(np.concatenate(parts))
+    if len(d) > 65536:
+        return None
+    out = dict(dict=d, vidx=np.searchsorted(d, P["val"]).astype(np.uint16))
+    if P["band_on"]:
+        out["loi"] = np.searchsorted(d, P["lo"]).astype(np.uint16)
+        out["upi"] = np.searchsorted(d, P["up"]).astype(np.uint16)
+    return out
+
+
 def jacobi_step(A: CSR, x: np.ndarray, omega: float = 1.0) -> np.ndarray:
     x = np.ascontiguousarray(x, dtype=np.float64)
     y = np.empty(A.n)

@@ -85,7 +85,8 @@ class cme_compact_view(C.Structure):
     _fields_ = [("n", C.c_int64), ("n_slots", C.c_int64), ("n_slices", C.c_int64),
                 ("n_ell", C.c_int64), ("band_on", C.c_int32), ("win_shift", C.c_int32),
                 ("val", f64p), ("col16", C.POINTER(C.c_int16)), ("row8", C.POINTER(C.c_uint8)),
-                ("lo", f64p), ("up", f64p)]
+                ("lo", f64p), ("up", f64p), ("n_dict", C.c_int64), ("dict", f64p),
+                ("vidx", C.POINTER(C.c_uint16)), ("loi", C.POINTER(C.c_uint16)), ("upi", C.POINTER(C.c_uint16))]
 
 
 class cme_halo_view(C.Structure):
@@ -329,6 +330,12 @@ def cme_export_compact(h):
     if v.lo:
         out["lo"] = cp(v.lo, v.n_slots, np.float64)
         out["up"] = cp(v.up, v.n_slots, np.float64)
+    if v.n_dict:
+        out["dict"] = cp(v.dict, v.n_dict, np.float64)
+        out["vidx"] = cp(v.vidx, v.n_ell, np.uint16)
+        if v.loi:
+            out["loi"] = cp(v.loi, v.n_slots, np.uint16)
+            out["upi"] = cp(v.upi, v.n_slots, np.uint16)
     return out
 
 

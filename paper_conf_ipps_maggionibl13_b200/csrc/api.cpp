@@ -428,6 +428,7 @@ cme_status cme_export_compact(cme_matrix h, cme_compact_view* v) {
                 return CME_ERR_INVALID_ARG;
             }
         }
+        if (!h->Cpt.vi_valid) encode_value_index(h->P, h->Cpt);
         const Packed& P = h->P;
         const Compact& Q = h->Cpt;
         cme_compact_view o{};
@@ -437,6 +438,13 @@ cme_status cme_export_compact(cme_matrix h, cme_compact_view* v) {
         o.row8 = Q.row8.empty() ? nullptr : Q.row8.data();
         o.lo = Q.lo.empty() ? nullptr : Q.lo.data();
         o.up = Q.up.empty() ? nullptr : Q.up.data();
+        if (Q.vi_valid) {
+            o.n_dict = (int64_t)Q.dict.size();
+            o.dict = Q.dict.data();
+            o.vidx = Q.vidx.data();
+            o.loi = Q.loi.empty() ? nullptr : Q.loi.data();
+            o.upi = Q.upi.empty() ? nullptr : Q.upi.data();
+        }
         *v = o;
         return CME_OK;
     });

@@ -72,8 +72,18 @@ struct Compact {
     std::vector<double> val, lo, up;      // val: n_ell; lo/up: n_slots (band only)
     std::vector<int16_t> col16;           // n_ell
     std::vector<uint8_t> row8;            // n_slots (rearranged packs only)
+    // value-indexed variant (CSR-VI style): the distinct stored values of O
+    // (val entries incl. pads, lo/up when the band is on), ascending, and
+    // 16-bit indices into that dictionary; inv_d stays per row
+    bool vi_valid = false;
+    std::vector<double> dict;             // <= 65536 values, ascending
+    std::vector<uint16_t> vidx;           // n_ell
+    std::vector<uint16_t> loi, upi;       // n_slots (band only)
 };
 bool encode_compact(const Packed& P, int64_t own_off, Compact& C);
+// Value-index P's layout-v0 values into C (needs C.valid); false when the
+// pack holds more than 65536 distinct values.
+bool encode_value_index(const Packed& P, Compact& C);
 
 struct Device;  // device state (device.cu)
 

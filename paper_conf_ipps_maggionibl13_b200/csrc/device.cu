@@ -101,6 +101,8 @@ struct Device {
     int tma_ncw = 16;
     int tma_grid = 0, tma_stages = 0, tma_stage_bytes = 0, tma_off_val = 0, tma_off_col = 0, tma_contig = 0;
     int tma_xpf = 0;
+    int tma_occ = 0;                 // TMA CTAs per SM
+    int2* tile_meta = nullptr;       // per slice {offset inside its tile, width} for the chosen tile shape
     int64_t n_tiles = 0;
     // compact encoding (kernels_cpt.cuh): the TMA kernel streams M's rows,
     // 16-bit column offsets and 8-bit row offsets
@@ -109,6 +111,11 @@ struct Device {
     int16_t* col16 = nullptr;
     uint8_t* row8 = nullptr;
     int32_t win_shift = 0;
+    // value-indexed variant (cpt also set): dictionary + 16-bit value indices
+    bool vi = false;
+    double* dict = nullptr;
+    uint16_t *vidx = nullptr, *loi = nullptr, *upi = nullptr;
+    int dict_bytes = 0;              // shared-memory bytes of the dictionary (multiple of 128)
     // SMEM-resident persistent kernel (kernels_resident.cuh)
     bool use_res = false;
     int res_grid = 0, res_smem = 0, res_rps = 1;
@@ -367,14 +374,21 @@ static int64_t tma_stage_bytes(const Device& d, const Packed& P, int ncw, int64_
         max_nval = std::max(max_nval, P.slice_off[q1] - P.slice_off[q0]);
     }
     auto a128 = [](int64_t b) { return (b + 127) / 128 * 128; };
+    // every stage: [tile metadata (kMetaBytes)] then the data blocks, whose
+    // offsets off_val / off_col are relative to the data base
+    if (d.vi) {    // [inv_d][row8][loi, upi][vidx][col16]
+        *off_val = a128(vi_fixed_bytes(ncw, d.band, d.rearr));
+        *off_col = *off_val + a128(2 * max_nval);
+        return kMetaBytes + a128(*off_col + 2 * max_nval);
+    }
     if (d.cpt) {   // [row8][lo, up][val][col16]
         *off_val = a128(cpt_fixed_bytes(ncw, d.band, d.rearr));
         *off_col = *off_val + a128(8 * max_nval);
-        return a128(*off_col + 2 * max_nval);
+        return kMetaBytes + a128(*off_col + 2 * max_nval);
     }
     *off_val = a128(tma_fixed_bytes(ncw, d.B, d.band, d.rearr));
     *off_col = *off_val + a128(8 * d.B * max_nval);
-    return a128(*off_col + 4 * max_nval);
+    return kMetaBytes + a128(*off_col + 4 * max_nval);
 }
 
 // Choose the step kernel.  The TMA ring pays once every CTA streams >= 2
@@ -406,17 +420,24 @@ static cme_status configure_tma(Device& d, const Packed& P) {
         // largest size any handle may use (handles on several host threads --
         // an in-process rank group -- would otherwise lower it under each
         // other's launches: "invalid argument")
-        if (d.cpt) CUDA_TRY(cpt_prepare(ncw, smem_max - 1024));
-        else CUDA_TRY(tma_prepare_b(d.B, ncw, smem_max - 1024));
+        // dynamic-smem cap: the opt-in maximum minus the static shared memory
+        // (barriers, check-reduction scratch: < 2 KB for 33 warps)
+        const int cap = smem_max - (d.vi ? 4096 : 1024);
+        if (d.vi) CUDA_TRY(vi_prepare(ncw, cap));
+        else if (d.cpt) CUDA_TRY(cpt_prepare(ncw, cap));
+        else CUDA_TRY(tma_prepare_b(d.B, ncw, cap));
+        const int64_t extra = d.vi ? d.dict_bytes : 0;   // the dictionary sits in front of the stages
         auto occ_of = [&](int stages, int* occ) -> cudaError_t {
             *occ = 0;
-            if (stages * sh.stage > smem_max - 1024) return cudaSuccess;
-            return d.cpt ? cpt_occupancy(ncw, (int)(stages * sh.stage), occ)
-                         : tma_occupancy_b(d.B, ncw, (int)(stages * sh.stage), occ);
+            const int64_t bytes = extra + stages * sh.stage;
+            if (bytes > cap) return cudaSuccess;
+            return d.vi ? vi_occupancy(ncw, (int)bytes, occ)
+                        : d.cpt ? cpt_occupancy(ncw, (int)bytes, occ)
+                                : tma_occupancy_b(d.B, ncw, (int)bytes, occ);
         };
         if (stages_req > 0) {
             sh.stages = stages_req;
-            while (sh.stages > 2 && sh.stages * sh.stage > smem_max - 1024) --sh.stages;
+            while (sh.stages > 2 && extra + sh.stages * sh.stage > cap) --sh.stages;
             CUDA_TRY(occ_of(sh.stages, &sh.occ));
         } else {
             // auto: the deepest ring (<= 4 stages) that keeps the residency of
@@ -432,10 +453,13 @@ static cme_status configure_tma(Device& d, const Packed& P) {
                 sh.stages = st;
             }
         }
+        if (env_int("CME_VERBOSE", 0) > 1)
+            std::fprintf(stderr, "[cme] tma shape: ncw=%d stages=%d stage=%lld extra=%lld occ=%d\n", ncw, sh.stages,
+                         (long long)sh.stage, (long long)extra, sh.occ);
         if (sh.occ < 1) continue;   // tiles too wide for this shape
         sh.occ = std::max(1, std::min(sh.occ, env_int("CME_TMA_CTAS", sh.occ)));
         sh.grid = (int)std::min<int64_t>(sh.n_tiles, (int64_t)sms * sh.occ);
-        if (sh.ncw * sh.occ > best.ncw * best.occ) best = sh;
+        if (sh.ncw * sh.occ > best.ncw * best.occ) best = sh;   // most resident consumer warps (ties: wider tiles)
     }
     if (best.ncw == 0) return CME_OK;
     if (want < 0 && (best.ncw * best.occ < 16 || best.n_tiles < 2 * (int64_t)sms * best.occ))
@@ -447,6 +471,7 @@ static cme_status configure_tma(Device& d, const Packed& P) {
     d.tma_off_val = (int)best.off_val;
     d.tma_off_col = (int)best.off_col;
     d.tma_grid = best.grid;
+    d.tma_occ = best.occ;
     d.tma_contig = env_int("CME_TMA_CONTIG", 0) != 0;   // measured: round robin wins on cfg4 (+3%)
     // L2 prefetch of each tile's x rows: pays when the iterate does not stay
     // L2-resident across steps (measured: cfg4, 160 MB of x, 235 vs 241 us;
@@ -455,8 +480,8 @@ static cme_status configure_tma(Device& d, const Packed& P) {
     d.tma_xpf = xpf >= 0 ? xpf != 0 : (d.nx + 2) * 8 * d.B > (int64_t)48 << 20;
     d.use_tma = true;
     if (env_int("CME_VERBOSE", 0))
-        std::fprintf(stderr, "[cme] tma: B=%d compact=%d warps=%d stages=%d stage_bytes=%lld occ=%d grid=%d tiles=%lld\n",
-                     d.B, (int)d.cpt, best.ncw, best.stages, (long long)best.stage, best.occ, best.grid, (long long)best.n_tiles);
+        std::fprintf(stderr, "[cme] tma: B=%d compact=%d vi=%d dict=%d warps=%d stages=%d stage_bytes=%lld occ=%d grid=%d tiles=%lld\n",
+                     d.B, (int)d.cpt, (int)d.vi, d.dict_bytes, best.ncw, best.stages, (long long)best.stage, best.occ, best.grid, (long long)best.n_tiles);
     return CME_OK;
 }
 
@@ -565,6 +590,34 @@ static cme_status configure_resident(Device& d, const Packed& P, bool distribute
     return CME_OK;
 }
 
+// Load every kernel a solve may launch before any of them runs: with CUDA
+// lazy loading (the default) the first launch of a kernel may wait for the
+// device to drain, and a rank of an in-process group whose peer is spinning
+// in p2p_barrier_kernel would then never get its kernel loaded (observed as a
+// barrier time-out on the first run of the virtual-rank tests).
+static cme_status preload_kernels(int B) {
+    cudaFuncAttributes fa;
+    CUDA_TRY(cudaFuncGetAttributes(&fa, reduce_partials_kernel));
+    CUDA_TRY(cudaFuncGetAttributes(&fa, decide_kernel));
+    CUDA_TRY(cudaFuncGetAttributes(&fa, load_kernel<1>));
+    CUDA_TRY(cudaFuncGetAttributes(&fa, load_kernel<2>));
+    CUDA_TRY(cudaFuncGetAttributes(&fa, load_kernel<4>));
+    CUDA_TRY(cudaFuncGetAttributes(&fa, load_kernel<8>));
+    CUDA_TRY(cudaFuncGetAttributes(&fa, load_decide_kernel));
+    CUDA_TRY(cudaFuncGetAttributes(&fa, fill_kernel));
+    CUDA_TRY(cudaFuncGetAttributes(&fa, scatter_out_kernel));
+    CUDA_TRY(cudaFuncGetAttributes(&fa, scale_copy_kernel));
+    CUDA_TRY(cudaFuncGetAttributes(&fa, p2p_barrier_kernel));
+    CUDA_TRY(cudaFuncGetAttributes(&fa, multicast_copy_kernel));
+    switch (B) {
+        case 1: CUDA_TRY(sell_preload<1>()); break;
+        case 2: CUDA_TRY(sell_preload<2>()); break;
+        case 4: CUDA_TRY(sell_preload<4>()); break;
+        default: CUDA_TRY(sell_preload<8>()); break;
+    }
+    return CME_OK;
+}
+
 // Build the device state from h->P (local layout) and the partition in h.
 cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cme_comm_s* comm) {
     int dev = 0;
@@ -636,12 +689,42 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
         encode_compact(P, d->own_off, h->Cpt)) {
         d->cpt = true;
         d->win_shift = h->Cpt.win_shift;
+        // value-indexed (sec. 5c) when the dictionary fits next to a ring with
+        // as many resident consumer warps (CME_VI = -1 auto / 0 off / 1 force)
         if ((s = configure_tma(*d, P)) != CME_OK) return fail(s);   // compact stage geometry
+        const int cpt_warps = d->use_tma ? d->tma_ncw * d->tma_occ : 0;
+        const int want_vi = env_int("CME_VI", -1);
+        if (want_vi != 0 && encode_value_index(P, h->Cpt)) {
+            d->vi = true;
+            d->dict_bytes = (int)((h->Cpt.dict.size() * 8 + 127) / 128 * 128);
+            if ((s = configure_tma(*d, P)) != CME_OK) return fail(s);
+            // auto: only if the dictionary costs no resident consumer warps
+            if (!d->use_tma || (want_vi < 0 && d->tma_ncw * d->tma_occ < cpt_warps)) {
+                d->vi = false;
+                d->dict_bytes = 0;
+                if ((s = configure_tma(*d, P)) != CME_OK) return fail(s);
+            }
+        }
         if (!d->use_tma) d->cpt = false;
     }
     if ((s = configure_resident(*d, P, comm != nullptr || h->nranks > 1)) != CME_OK) return fail(s);
+    if ((s = preload_kernels(B)) != CME_OK) return fail(s);
+    if (d->use_tma) {
+        std::vector<int2> tm((size_t)d->n_tiles * d->tma_ncw, make_int2(0, 0));   // whole tiles (TMA copies)
+        for (int64_t q = 0; q < P.n_slices; ++q)
+            tm[q] = make_int2((int)(P.slice_off[q] - P.slice_off[q / d->tma_ncw * d->tma_ncw]), P.slice_w[q]);
+        if ((s = d->upload(d->tile_meta, tm)) != CME_OK) return fail(s);
+    }
     if (d->format != CME_FMT_CSR) {
-        if (d->cpt) {
+        if (d->vi) {
+            std::vector<double> dict(h->Cpt.dict);
+            dict.resize(d->dict_bytes / 8, 0.0);
+            UP(dict, dict);
+            UP(vidx, h->Cpt.vidx);
+            UP(col16, h->Cpt.col16);
+            if (d->band) { UP(loi, h->Cpt.loi); UP(upi, h->Cpt.upi); }
+            if (d->rearr) UP(row8, h->Cpt.row8);
+        } else if (d->cpt) {
             UP(cval, h->Cpt.val);
             UP(col16, h->Cpt.col16);
             if (d->band) { UP(clo, h->Cpt.lo); UP(cup, h->Cpt.up); }
@@ -901,6 +984,7 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
     a.slice_end = d.n_slices;
     a.slice_off = d.slice_off;
     a.slice_w = d.slice_w;
+    a.tile_meta = d.tile_meta;
     a.val = d.val;
     a.col = d.col;
     a.row_of = d.row_of;
@@ -923,6 +1007,13 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
     if (d.format == CME_FMT_CSR) {
         CUDA_TRY(check ? launch_ex(csr_step_kernel<true>, dim3(d.grid), dim3(kCta), 0, pdl, s, a)
                        : launch_ex(csr_step_kernel<false>, dim3(d.grid), dim3(kCta), 0, pdl, s, a));
+    } else if (d.use_tma && d.vi) {
+        ViArgs V{CptArgs{TmaArgs{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col,
+                                 d.tma_contig, d.tma_xpf},
+                         d.col16, d.row8, d.win_shift},
+                 d.dict, d.vidx, d.loi, d.upi, d.dict_bytes};
+        CUDA_TRY(launch_vi(V, d.tma_ncw, d.tma_grid, d.dict_bytes + d.tma_stages * d.tma_stage_bytes, d.band, d.rearr,
+                           check, pdl, s));
     } else if (d.use_tma && d.cpt) {
         a.val = d.cval;
         a.lo = d.clo;
@@ -1321,8 +1412,13 @@ void device_describe(const Device* d, cme_info* f) {
     f->tma_warps = d->use_tma ? d->tma_ncw : 0;
     f->tma_stages = d->use_tma ? d->tma_stages : 0;
     f->grid = d->use_res ? d->res_grid : d->step_grid();
-    f->compact = d->cpt ? 1 : 0;
-    if (d->cpt) {   // bytes a plain step streams in the compact encoding (no inv_d)
+    f->compact = d->vi ? 2 : d->cpt ? 1 : 0;
+    if (d->vi) {   // value-indexed: 4 B per ELL slot, inv_d per row
+        const int64_t n_ell = f->n_ell, nl = d->n_own, slots = f->n_slots, sl = f->n_slices;
+        f->bytes_fmt = 4 * n_ell + 8 * nl + (d->rearr ? nl : 0) + (d->band ? 4 * nl : 0) + 12 * sl + 16 * nl;
+        f->packed_bytes = 4 * n_ell + 8 * slots + (d->rearr ? slots : 0) + (d->band ? 4 * slots : 0) + 12 * sl + 8 +
+                          d->dict_bytes + (d->use_res ? f->packed_bytes : 0);
+    } else if (d->cpt) {   // bytes a plain step streams in the compact encoding (no inv_d)
         const int64_t n_ell = f->n_ell, nl = d->n_own, slots = f->n_slots, sl = f->n_slices;
         f->bytes_fmt = 10 * n_ell + (d->rearr ? nl : 0) + (d->band ? 16 * nl : 0) + 12 * sl + 16 * nl;
         f->packed_bytes = 10 * n_ell + (d->rearr ? slots : 0) + (d->band ? 16 * slots : 0) + 8 * slots + 12 * sl + 8 +

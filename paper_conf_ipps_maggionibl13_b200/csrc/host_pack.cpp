@@ -7,6 +7,9 @@
 // layout ("v0") is frozen in DESIGN.md section 5 so that the oracle packer and
 // this one agree byte for byte.
 #include <algorithm>
+#include <cstring>
+#include <unordered_map>
+#include <unordered_set>
 
 #include "cme_internal.h"
 
@@ -169,6 +172,63 @@ bool encode_compact(const Packed& P, int64_t own_off, Compact& C) {
         }
         if (ws) C.row8[s] = (uint8_t)(l - ((s >> ws) << ws));
     }
+    return true;
+}
+
+bool encode_value_index(const Packed& P, Compact& C) {
+    C.vi_valid = false;
+    C.dict.clear(); C.vidx.clear(); C.loi.clear(); C.upi.clear();
+    if (!C.valid || P.B != 1) return false;
+    constexpr size_t kMax = 65536;
+    auto bits = [](double v) { uint64_t u; std::memcpy(&u, &v, 8); return u; };
+    // distinct values (by bit pattern; stored values are finite and +0.0 or > 0)
+    std::unordered_set<uint64_t> all;
+    bool over = false;
+#pragma omp parallel
+    {
+        std::unordered_set<uint64_t> mine;
+#pragma omp for schedule(static) nowait
+        for (int64_t e = 0; e < P.n_ell; ++e) {
+            if (mine.size() > kMax) continue;
+            mine.insert(bits(P.val[e]));
+        }
+        if (P.band_on) {
+#pragma omp for schedule(static) nowait
+            for (int64_t s = 0; s < P.n_slots; ++s) {
+                if (mine.size() > kMax) continue;
+                mine.insert(bits(P.lo[s]));
+                mine.insert(bits(P.up[s]));
+            }
+        }
+#pragma omp critical
+        {
+            if (mine.size() > kMax) over = true;
+            if (!over) all.insert(mine.begin(), mine.end());
+            if (all.size() > kMax) over = true;
+        }
+    }
+    if (over) return false;
+    std::vector<double> dict;
+    dict.reserve(all.size());
+    for (uint64_t u : all) { double v; std::memcpy(&v, &u, 8); dict.push_back(v); }
+    std::sort(dict.begin(), dict.end());
+    std::unordered_map<uint64_t, uint16_t> where;
+    where.reserve(dict.size() * 2);
+    for (size_t i = 0; i < dict.size(); ++i) where[bits(dict[i])] = (uint16_t)i;
+    C.vidx.resize(P.n_ell);
+#pragma omp parallel for schedule(static)
+    for (int64_t e = 0; e < P.n_ell; ++e) C.vidx[e] = where.find(bits(P.val[e]))->second;
+    if (P.band_on) {
+        C.loi.resize(P.n_slots);
+        C.upi.resize(P.n_slots);
+#pragma omp parallel for schedule(static)
+        for (int64_t s = 0; s < P.n_slots; ++s) {
+            C.loi[s] = where.find(bits(P.lo[s]))->second;
+            C.upi[s] = where.find(bits(P.up[s]))->second;
+        }
+    }
+    C.dict = std::move(dict);
+    C.vi_valid = true;
     return true;
 }
 

@@ -52,6 +52,7 @@ struct StepArgs {
     int64_t slice_begin, slice_end;
     const int64_t* slice_off;
     const int32_t* slice_w;
+    const int2* tile_meta;  // TMA kernels: per slice {slice_off[q] - slice_off[first slice of its tile], slice_w[q]}
     const double* val;     // [n_ell][B]
     const int32_t* col;    // x-span coordinates
     const int32_t* row_of; // slot -> local row (nullptr: identity)

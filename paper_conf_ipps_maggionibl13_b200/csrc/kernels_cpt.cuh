@@ -33,7 +33,8 @@ template <int NCW, bool BAND, bool REARR>
 __device__ __noinline__ void cpt_issue_call(unsigned char* st, uint64_t* bar, const int64_t* slice_off,
                                             int64_t slice_end, const uint8_t* row8, const double* lo,
                                             const double* up, const double* val, const int16_t* col16,
-                                            int off_val, int off_col, int64_t tile, uint64_t pol) {
+                                            int off_val, int off_col, int64_t tile, uint64_t pol,
+                                            const int2* tile_meta) {
     constexpr int kSlots = NCW * 32;
     constexpr int kOffRow = 0, kOffLo = REARR ? kSlots : 0, kOffUp = kOffLo + 8 * kSlots;
     const int64_t q0 = tile * NCW;
@@ -41,10 +42,12 @@ __device__ __noinline__ void cpt_issue_call(unsigned char* st, uint64_t* bar, co
     const int64_t e0 = slice_off[q0], e1 = slice_off[q1];
     const uint32_t slots = (uint32_t)(q1 - q0) * 32u;
     const uint32_t nval = (uint32_t)(e1 - e0);
-    uint32_t bytes = nval * 10u;
+    uint32_t bytes = nval * 10u + NCW * 8u;
     if (REARR) bytes += slots;
     if (BAND) bytes += slots * 16u;
     mbar_expect_tx(bar, bytes);
+    issue_meta(st, bar, tile_meta, tile, NCW, pol);
+    st += kMetaBytes;
     if (REARR) bulk_g2s(st + kOffRow, row8 + q0 * 32, slots, bar, pol);
     if (BAND) {
         bulk_g2s(st + kOffLo, lo + q0 * 32, slots * 8u, bar, pol);
@@ -65,7 +68,7 @@ __device__ __forceinline__ void cpt_issue(const CptArgs& K, unsigned char* smem,
         if (r1 > r0) prefetch_l2(a.x + a.own_off + r0, (uint64_t)(r1 - r0) * 8);
     }
     cpt_issue_call<NCW, BAND, REARR>(smem + (size_t)s * K.T.stage_bytes, &full[s], a.slice_off, a.slice_end, K.row8,
-                                     a.lo, a.up, a.val, K.col16, K.T.off_val, K.T.off_col, tile, pol);
+                                     a.lo, a.up, a.val, K.col16, K.T.off_val, K.T.off_col, tile, pol, a.tile_meta);
 }
 
 // Sum over the W entries of one slot: all gathers x[r + dj] first, then the
@@ -160,14 +163,11 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
         for (int64_t tile = t_first; tile < t_end; tile += t_stride) {
             const int64_t q0 = tile * kTileSlices;
             const int64_t q = q0 + warp;
-            const unsigned char* st = smem + (size_t)s * T.stage_bytes;
-            int w = 0;
-            int64_t loff = 0;
-            if (q < a.slice_end) {
-                w = __ldg(a.slice_w + q);
-                loff = __ldg(a.slice_off + q) - __ldg(a.slice_off + q0);
-            }
+            const unsigned char* st = smem + (size_t)s * T.stage_bytes + kMetaBytes;
             mbar_wait(&full[s], phase);
+            const int2 meta = reinterpret_cast<const int2*>(st - kMetaBytes)[warp];   // {offset in tile, width}
+            const int w = meta.y;
+            const int64_t loff = meta.x;
             const int64_t slot = q * 32 + lane;
             if (q < a.slice_end && slot < a.n_rows) {
                 const int ls = warp * 32 + lane;
@@ -202,6 +202,199 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
                 const double lo = BAND ? reinterpret_cast<const double*>(st + kOffLo)[ls] : 0.0;
                 const double up = BAND ? reinterpret_cast<const double*>(st + kOffUp)[ls] : 0.0;
                 finish_row_cpt<BAND, CHECK>(a, slot, r, yo, acc, lo, up, ck, X);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);
+            if (++s == S) { s = 0; phase ^= 1u; }
+        }
+    }
+    if (CHECK) cta_check_partials<NCW + 1, 1>(ck, a.partials);
+}
+
+// ---------------------------------------------------------------------------
+// Value-indexed variant (the CSR-VI idea): the rates of a
+// mass-action CME take few distinct values (r_k times small binomials: 6 318
+// on the 20M-state toggle switch), so an entry is a 16-bit index into a
+// dictionary of O's distinct values held in shared memory plus the 16-bit
+// column offset -- 4 B per ELL slot -- and inv_d stays a per-row stream.  The
+// arithmetic is the layout-v0 kernel's exactly (same values, same FMA order,
+// the row sum times inv_d), so results are bit-identical to it.
+struct ViArgs {
+    CptArgs K;             // K.T.a.inv_d per row; K.col16 / row8 / win_shift as the compact encoding
+    const double* dict;    // [n_dict] ascending (padded to 16 B)
+    const uint16_t* vidx;  // [n_ell]
+    const uint16_t* loi;   // [n_slots] (band)
+    const uint16_t* upi;
+    int32_t dict_bytes;    // multiple of 128: stages start here in shared memory
+};
+
+// Stage layout: [inv_d][row8 if REARR][loi, upi if BAND][vidx][col16].
+__host__ __device__ inline int vi_fixed_bytes(int ncw, bool band, bool rearr) {
+    return ncw * 32 * (8 + (rearr ? 1 : 0) + (band ? 4 : 0));
+}
+
+template <int NCW, bool BAND, bool REARR>
+__device__ __noinline__ void vi_issue_call(unsigned char* st, uint64_t* bar, const int64_t* slice_off,
+                                           int64_t slice_end, const double* inv_d, const uint8_t* row8,
+                                           const uint16_t* loi, const uint16_t* upi, const uint16_t* vidx,
+                                           const int16_t* col16, int off_val, int off_col, int64_t tile,
+                                           uint64_t pol, const int2* tile_meta) {
+    constexpr int kSlots = NCW * 32;
+    constexpr int kOffRow = 8 * kSlots, kOffLo = kOffRow + (REARR ? kSlots : 0), kOffUp = kOffLo + 2 * kSlots;
+    const int64_t q0 = tile * NCW;
+    const int64_t q1 = min(q0 + NCW, slice_end);
+    const int64_t e0 = slice_off[q0], e1 = slice_off[q1];
+    const uint32_t slots = (uint32_t)(q1 - q0) * 32u;
+    const uint32_t nval = (uint32_t)(e1 - e0);
+    uint32_t bytes = nval * 4u + slots * 8u + NCW * 8u;
+    if (REARR) bytes += slots;
+    if (BAND) bytes += slots * 4u;
+    mbar_expect_tx(bar, bytes);
+    issue_meta(st, bar, tile_meta, tile, NCW, pol);
+    st += kMetaBytes;
+    bulk_g2s(st, inv_d + q0 * 32, slots * 8u, bar, pol);
+    if (REARR) bulk_g2s(st + kOffRow, row8 + q0 * 32, slots, bar, pol);
+    if (BAND) {
+        bulk_g2s(st + kOffLo, loi + q0 * 32, slots * 2u, bar, pol);
+        bulk_g2s(st + kOffUp, upi + q0 * 32, slots * 2u, bar, pol);
+    }
+    if (nval) {
+        bulk_g2s(st + off_val, vidx + e0, nval * 2u, bar, pol);
+        bulk_g2s(st + off_col, col16 + e0, nval * 2u, bar, pol);
+    }
+}
+
+template <int NCW, bool BAND, bool REARR>
+__device__ __forceinline__ void vi_issue(const ViArgs& V, unsigned char* stages, uint64_t* full, int64_t tile, int s,
+                                         uint64_t pol) {
+    const StepArgs& a = V.K.T.a;
+    if (V.K.T.xpf) {
+        const int64_t r0 = tile * NCW * 32, r1 = min(r0 + NCW * 32, a.n_rows);
+        if (r1 > r0) prefetch_l2(a.x + a.own_off + r0, (uint64_t)(r1 - r0) * 8);
+    }
+    vi_issue_call<NCW, BAND, REARR>(stages + (size_t)s * V.K.T.stage_bytes, &full[s], a.slice_off, a.slice_end,
+                                    a.inv_d, V.K.row8, V.loi, V.upi, V.vidx, V.K.col16, V.K.T.off_val, V.K.T.off_col,
+                                    tile, pol, a.tile_meta);
+}
+
+template <int W>
+__device__ __forceinline__ void ell_row_vi(const int16_t* scol, const uint16_t* svi, const double* sdict,
+                                           const double* xr, double& acc) {
+    double xv[W];
+#pragma unroll
+    for (int u = 0; u < W; ++u) xv[u] = __ldg(xr + scol[32 * u]);
+#pragma unroll
+    for (int u = 0; u < W; ++u) acc = fma(sdict[svi[32 * u]], xv[u], acc);
+}
+
+template <int NCW, bool BAND, bool REARR, bool CHECK>
+__global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBlocks)
+    sell_vi_kernel(const ViArgs V) {
+    constexpr int kConsumers = NCW, kTileSlices = NCW, kSlots = NCW * 32;
+    constexpr int kOffRow = 8 * kSlots, kOffLo = kOffRow + (REARR ? kSlots : 0), kOffUp = kOffLo + 2 * kSlots;
+    const CptArgs& K = V.K;
+    const TmaArgs& T = K.T;
+    const StepArgs& a = T.a;
+    pdl_trigger();
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ uint64_t full[8], empty[8], dbar;
+    const double* sdict = reinterpret_cast<const double*>(smem);
+    unsigned char* stages = smem + V.dict_bytes;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int S = T.stages;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < S; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], kConsumers);
+        }
+        mbar_init(&dbar, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    const bool producer = warp == kConsumers && lane == 0;
+    uint64_t pol = 0;
+    int64_t t_first, my_tiles, t_stride;
+    tma_tile_range(T, &t_first, &my_tiles, &t_stride);
+    const int64_t t_end = t_first + my_tiles * t_stride;
+    const int pro = (int)(my_tiles < (int64_t)S ? my_tiles : (int64_t)S);
+    if (producer) {   // dictionary and first tiles are constant: load while the previous step drains
+        pol = evict_first_policy();
+        mbar_expect_tx(&dbar, (uint32_t)V.dict_bytes);
+        uint64_t keep;   // every CTA reads the dictionary: keep it in L2
+        asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(keep));
+        bulk_g2s(smem, V.dict, (uint32_t)V.dict_bytes, &dbar, keep);
+        for (int i = 0; i < pro; ++i) vi_issue<NCW, BAND, REARR>(V, stages, full, t_first + (int64_t)i * t_stride, i, pol);
+    }
+    pdl_wait();
+    if (a.stop != nullptr && *a.stop) {
+        if (producer) {
+            mbar_wait(&dbar, 0u);
+            for (int i = 0; i < pro; ++i) mbar_wait(&full[i], 0u);
+        }
+        return;
+    }
+    CheckAcc<1> ck;
+    if (warp == kConsumers) {
+        if (lane == 0 && my_tiles > pro) {
+            int s = 0;
+            uint32_t phase = 1;
+            for (int64_t tile = t_first + (int64_t)pro * t_stride; tile < t_end; tile += t_stride) {
+                mbar_wait(&empty[s], phase ^ 1u);
+                vi_issue<NCW, BAND, REARR>(V, stages, full, tile, s, pol);
+                if (++s == S) { s = 0; phase ^= 1u; }
+            }
+        }
+        if (lane == 0 && my_tiles == 0) mbar_wait(&dbar, 0u);   // no tile ever waits on it
+    } else {
+        const double* xo = a.x + a.own_off;
+        double* yo = a.y + a.own_off;
+        mbar_wait(&dbar, 0u);
+        int s = 0;
+        uint32_t phase = 0;
+        for (int64_t tile = t_first; tile < t_end; tile += t_stride) {
+            const int64_t q0 = tile * kTileSlices;
+            const int64_t q = q0 + warp;
+            const unsigned char* st = stages + (size_t)s * T.stage_bytes + kMetaBytes;
+            mbar_wait(&full[s], phase);
+            const int2 meta = reinterpret_cast<const int2*>(st - kMetaBytes)[warp];   // {offset in tile, width}
+            const int w = meta.y;
+            const int64_t loff = meta.x;
+            const int64_t slot = q * 32 + lane;
+            if (q < a.slice_end && slot < a.n_rows) {
+                const int ls = warp * 32 + lane;
+                const uint16_t* svi = reinterpret_cast<const uint16_t*>(st + T.off_val) + loff + lane;
+                const int16_t* scol = reinterpret_cast<const int16_t*>(st + T.off_col) + loff + lane;
+                const int64_t r = REARR ? ((slot >> K.win_shift) << K.win_shift) + st[kOffRow + ls] : slot;
+                RowX<1, BAND> X;
+                X.load(xo, r);
+                const double* xr = xo + r;
+                double acc = 0.0;
+                switch (w) {   // warp-uniform exact widths
+                    case 0: break;
+                    case 1: ell_row_vi<1>(scol, svi, sdict, xr, acc); break;
+                    case 2: ell_row_vi<2>(scol, svi, sdict, xr, acc); break;
+                    case 3: ell_row_vi<3>(scol, svi, sdict, xr, acc); break;
+                    case 4: ell_row_vi<4>(scol, svi, sdict, xr, acc); break;
+                    case 5: ell_row_vi<5>(scol, svi, sdict, xr, acc); break;
+                    case 6: ell_row_vi<6>(scol, svi, sdict, xr, acc); break;
+                    case 7: ell_row_vi<7>(scol, svi, sdict, xr, acc); break;
+                    case 8: ell_row_vi<8>(scol, svi, sdict, xr, acc); break;
+                    default:
+                        for (int t0 = 0; t0 < w; t0 += 8) {
+                            double xv[8];
+#pragma unroll
+                            for (int u = 0; u < 8; ++u)
+                                if (t0 + u < w) xv[u] = __ldg(xr + scol[32 * (t0 + u)]);
+#pragma unroll
+                            for (int u = 0; u < 8; ++u)
+                                if (t0 + u < w) acc = fma(sdict[svi[32 * (t0 + u)]], xv[u], acc);
+                        }
+                }
+                const double accv[1] = {acc};
+                const double idv[1] = {reinterpret_cast<const double*>(st)[ls]};
+                const double lov[1] = {BAND ? sdict[reinterpret_cast<const uint16_t*>(st + kOffLo)[ls]] : 0.0};
+                const double upv[1] = {BAND ? sdict[reinterpret_cast<const uint16_t*>(st + kOffUp)[ls]] : 0.0};
+                finish_row_x<1, BAND, CHECK>(a, r, yo, accv, lov, upv, idv, a.pre_scale, ck, X);
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);

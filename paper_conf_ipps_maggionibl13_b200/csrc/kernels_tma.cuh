@@ -54,6 +54,14 @@ __device__ __forceinline__ void tma_tile_range(const TmaArgs& T, int64_t* first,
     }
 }
 
+// Every stage starts with the tile's slice metadata: per slice {entry offset
+// inside the tile, width} (host-built tile_meta, padded to whole tiles), moved
+// by the same TMA transaction as the tile.  Reading it from global memory put
+// two dependent L2 round trips (slice_off[q], slice_off[q0]) at the head of
+// every consumer's tile -- the top stall in the ncu source view (16.5%).
+constexpr int kMetaBytes = 128;   // >= NCW * 8 for NCW <= 16, keeps the data 128-B aligned
+
+
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
@@ -100,6 +108,11 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
         : "memory");
 }
 
+__device__ __forceinline__ void issue_meta(unsigned char* st, uint64_t* bar, const int2* tile_meta, int64_t tile,
+                                           int ncw, uint64_t pol) {
+    bulk_g2s(st, tile_meta + tile * ncw, (uint32_t)ncw * 8u, bar, pol);
+}
+
 // Stage layout: [inv_d][row_of if REARR][lo, up if BAND][val][col] for
 // NCW*32 slots and B members; the host computes the same offsets from
 // tma_fixed_bytes() and the widest tile.
@@ -133,7 +146,7 @@ __device__ __forceinline__ void tma_issue_body(unsigned char* st, uint64_t* bar,
                                                int64_t slice_end, const double* inv_d, const int32_t* row_of,
                                                const double* lo, const double* up, const double* val,
                                                const int32_t* col, int off_val, int off_col, int64_t tile,
-                                               uint64_t pol) {
+                                               uint64_t pol, const int2* tile_meta) {
     constexpr int kSlots = NCW * 32;
     constexpr int kOffInvd = 0, kOffRow = 8 * B * kSlots, kOffLo = kOffRow + (REARR ? 4 * kSlots : 0),
                   kOffUp = kOffLo + 8 * B * kSlots;
@@ -142,10 +155,12 @@ __device__ __forceinline__ void tma_issue_body(unsigned char* st, uint64_t* bar,
     const int64_t e0 = slice_off[q0], e1 = slice_off[q1];
     const uint32_t slots = (uint32_t)(q1 - q0) * 32u;
     const uint32_t nval = (uint32_t)(e1 - e0);
-    uint32_t bytes = nval * (8u * B + 4u) + slots * 8u * B;
+    uint32_t bytes = nval * (8u * B + 4u) + slots * 8u * B + NCW * 8u;
     if (REARR) bytes += slots * 4u;
     if (BAND) bytes += slots * 16u * B;
     mbar_expect_tx(bar, bytes);
+    issue_meta(st, bar, tile_meta, tile, NCW, pol);
+    st += kMetaBytes;
     bulk_g2s(st + kOffInvd, inv_d + q0 * 32 * B, slots * 8u * B, bar, pol);
     if (REARR) bulk_g2s(st + kOffRow, row_of + q0 * 32, slots * 4u, bar, pol);
     if (BAND) {
@@ -162,9 +177,9 @@ __device__ __noinline__ void tma_issue_call(unsigned char* st, uint64_t* bar, co
                                             int64_t slice_end, const double* inv_d, const int32_t* row_of,
                                             const double* lo, const double* up, const double* val,
                                             const int32_t* col, int off_val, int off_col, int64_t tile,
-                                            uint64_t pol) {
+                                            uint64_t pol, const int2* tile_meta) {
     tma_issue_body<NCW, B, BAND, REARR>(st, bar, slice_off, slice_end, inv_d, row_of, lo, up, val, col, off_val,
-                                        off_col, tile, pol);
+                                        off_col, tile, pol, tile_meta);
 }
 template <int NCW, int B, bool BAND, bool REARR>
 __device__ __forceinline__ void tma_issue(const TmaArgs& T, unsigned char* smem, uint64_t* full, int64_t tile, int s,
@@ -177,10 +192,10 @@ __device__ __forceinline__ void tma_issue(const TmaArgs& T, unsigned char* smem,
     }
     if (CME_TMA_PRODUCER_INLINE)
         tma_issue_body<NCW, B, BAND, REARR>(st, &full[s], a.slice_off, a.slice_end, a.inv_d, a.row_of, a.lo, a.up,
-                                            a.val, a.col, T.off_val, T.off_col, tile, pol);
+                                            a.val, a.col, T.off_val, T.off_col, tile, pol, a.tile_meta);
     else
         tma_issue_call<NCW, B, BAND, REARR>(st, &full[s], a.slice_off, a.slice_end, a.inv_d, a.row_of, a.lo, a.up,
-                                            a.val, a.col, T.off_val, T.off_col, tile, pol);
+                                            a.val, a.col, T.off_val, T.off_col, tile, pol, a.tile_meta);
 }
 
 #ifndef CME_TMA_EXACT_WIDTHS
@@ -255,15 +270,11 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
         for (int64_t tile = t_first; tile < t_end; tile += t_stride) {
             const int64_t q0 = tile * kTileSlices;
             const int64_t q = q0 + warp;
-            const unsigned char* st = smem + (size_t)s * T.stage_bytes;
-            // slice metadata (tiny, L1/L2 resident) before the wait
-            int w = 0;
-            int64_t loff = 0;
-            if (q < a.slice_end) {
-                w = __ldg(a.slice_w + q);
-                loff = __ldg(a.slice_off + q) - __ldg(a.slice_off + q0);
-            }
+            const unsigned char* st = smem + (size_t)s * T.stage_bytes + kMetaBytes;
             mbar_wait(&full[s], phase);
+            const int2 meta = reinterpret_cast<const int2*>(st - kMetaBytes)[warp];   // {offset in tile, width}
+            const int w = meta.y;
+            const int64_t loff = meta.x;
             const int64_t slot = q * 32 + lane;
             if (q < a.slice_end && slot < a.n_rows) {
                 const int ls = warp * 32 + lane;

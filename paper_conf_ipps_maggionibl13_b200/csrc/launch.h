@@ -37,6 +37,9 @@ template <int B>
 cudaError_t tma_prepare(int ncw, int smem);
 template <int B>
 cudaError_t tma_occupancy(int ncw, int smem, int* blocks_per_sm);
+// load every register-kernel variant of width B now (see launch_impl.cuh)
+template <int B>
+cudaError_t sell_preload();
 
 }  // namespace cme
 
@@ -47,6 +50,12 @@ cudaError_t launch_cpt(const CptArgs& K, int ncw, int grid, int smem, bool band,
                        cudaStream_t s);
 cudaError_t cpt_prepare(int ncw, int smem);
 cudaError_t cpt_occupancy(int ncw, int smem, int* blocks_per_sm);
+struct ViArgs;
+// value-indexed TMA step kernel (step_cpt.cu, B = 1)
+cudaError_t launch_vi(const ViArgs& V, int ncw, int grid, int smem, bool band, bool rearr, bool check, bool pdl,
+                      cudaStream_t s);
+cudaError_t vi_prepare(int ncw, int smem);
+cudaError_t vi_occupancy(int ncw, int smem, int* blocks_per_sm);
 struct ResArgs;
 // SMEM-resident persistent Jacobi kernel (resident.cu)
 cudaError_t resident_prepare(int smem);

@@ -63,10 +63,28 @@ cudaError_t tma_occupancy(int ncw, int smem, int* occ) {
                                                          TmaShape<8>::kThreads, smem);
 }
 
+// Force every register-kernel variant of width B (and the CSR arm) to load
+// now: under CUDA lazy loading the first launch of a kernel can wait for the
+// device to drain, which deadlocks against a peer's spinning barrier kernel
+// in an in-process rank group.
+template <int B>
+cudaError_t sell_preload() {
+    cudaFuncAttributes fa;
+    cudaError_t e = cudaSuccess;
+#define L(bd, r, c) \
+    if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, sell_step_kernel<B, bd, r, c>);
+    L(0, 0, 0) L(0, 0, 1) L(0, 1, 0) L(0, 1, 1) L(1, 0, 0) L(1, 0, 1) L(1, 1, 0) L(1, 1, 1)
+#undef L
+    if (e == cudaSuccess && B == 1) e = cudaFuncGetAttributes(&fa, csr_step_kernel<true>);
+    if (e == cudaSuccess && B == 1) e = cudaFuncGetAttributes(&fa, csr_step_kernel<false>);
+    return e;
+}
+
 #define CME_INSTANTIATE_LAUNCHERS(B)                                                                       \
     template cudaError_t launch_sell<B>(const StepArgs&, int, bool, bool, bool, bool, cudaStream_t);        \
     template cudaError_t launch_tma<B>(const TmaArgs&, int, int, int, bool, bool, bool, bool, cudaStream_t); \
     template cudaError_t tma_prepare<B>(int, int);                                                          \
-    template cudaError_t tma_occupancy<B>(int, int, int*);
+    template cudaError_t tma_occupancy<B>(int, int, int*);                                                  \
+    template cudaError_t sell_preload<B>();
 
 }  // namespace cme

@@ -78,14 +78,17 @@ def test_spmv_wide_rates_and_ragged(cme, oracle_mod):
 
 @pytest.mark.parametrize("net", NETS, ids=lambda n: n.name)
 @pytest.mark.parametrize("layout", LAYOUTS[:5], ids=lambda l: "-".join(map(str, l)))
-def test_spmv_parity_compact_tma(cme, oracle_mod, monkeypatch, net, layout):
+@pytest.mark.parametrize("vi", ["0", "1"])
+def test_spmv_parity_compact_tma(cme, oracle_mod, monkeypatch, net, layout, vi):
     """Every SELL layout of every network through the TMA kernel on the compact
-    encoding (forced: these matrices are below the auto size), plus the
-    check partials: one solve of 2 blocks against the oracle."""
+    encoding and on its value-indexed form (forced: these matrices are below
+    the auto size), plus the check partials: one solve of 2 blocks against
+    the oracle."""
     monkeypatch.setenv("CME_TMA", "1")
     monkeypatch.setenv("CME_RESIDENT", "0")
+    monkeypatch.setenv("CME_VI", vi)
     m, A = build(cme, oracle_mod, net, *layout)
-    assert m.info().kernel == 1 and m.info().compact == 1
+    assert m.info().kernel == 1 and m.info().compact == (2 if vi == "1" else 1)
     for omega in (1.0, 0.9):
         m.set_opts(omega=omega)
         x = W.random_start(A.n, 11)
@@ -98,21 +101,44 @@ def test_spmv_parity_compact_tma(cme, oracle_mod, monkeypatch, net, layout):
     assert rep.delta == pytest.approx(ref.delta, rel=1e-9) and rep.resid == pytest.approx(ref.resid, rel=1e-9)
 
 
-@pytest.mark.parametrize("compact", ["1", "0"])
-def test_transient_on_tma_kernels(cme, oracle_mod, monkeypatch, compact):
+@pytest.mark.parametrize("compact,vi", [("1", "1"), ("1", "0"), ("0", "0")])
+def test_transient_on_tma_kernels(cme, oracle_mod, monkeypatch, compact, vi):
     """Uniformization (NEXT-3) through the TMA kernel on both encodings: the
     compact one rebuilds (A x)_r = |a_rr| ((M x)_r - x_r) from M's rows."""
     monkeypatch.setenv("CME_TMA", "1")
     monkeypatch.setenv("CME_RESIDENT", "0")
     monkeypatch.setenv("CME_COMPACT", compact)
+    monkeypatch.setenv("CME_VI", vi)
     states, r, c, v = oracle_mod.enumerate_network(W.toggle_switch(50))
     A = oracle_mod.ingest(len(states), r, c, v)
     m = cme.Matrix(A.n, r, c, v).reorder(ORD["dfs"]).pack()
-    assert m.info().compact == int(compact)
+    assert m.info().compact == int(compact) + int(vi)
     for t in (0.05, 0.5):
         pt, terms = m.transient(t)
         ref, _, _ = oracle_mod.transient(A, t)
         assert np.abs(pt - ref).sum() <= 1e-12
+
+
+def test_value_index_bit_identical_to_layout_v0(cme, oracle_mod, monkeypatch):
+    """The value-indexed kernel does the layout-v0 arithmetic exactly (same
+    values from the dictionary, same FMA order, row sum times inv_d): its
+    SpMV and a fixed-iteration landscape are bit-identical to the v0 TMA
+    kernel's."""
+    monkeypatch.setenv("CME_TMA", "1")
+    monkeypatch.setenv("CME_RESIDENT", "0")
+    states, r, c, v = oracle_mod.enumerate_network(W.toggle_switch(90))
+    x = W.random_start(len(states), 8)
+    out = {}
+    for enc, env in (("v0", {"CME_COMPACT": "0"}), ("vi", {"CME_COMPACT": "1", "CME_VI": "1"})):
+        for k, val in env.items():
+            monkeypatch.setenv(k, val)
+        m = cme.Matrix(len(states), r, c, v).reorder(cme.CME_ORDER_RCM).pack()
+        m.set_opts(omega=0.9, check_every=50, stag_tol=0.0)
+        p, st, it = m.solve(tol=0.0, max_iter=300)
+        out[enc] = (m.spmv(x), p, m.info().compact)
+    assert out["v0"][2] == 0 and out["vi"][2] == 2
+    assert out["v0"][0].tobytes() == out["vi"][0].tobytes()
+    assert out["v0"][1].tobytes() == out["vi"][1].tobytes()
 
 
 def test_compact_fallback_wide_offsets(cme, oracle_mod, monkeypatch):
@@ -125,6 +151,13 @@ def test_compact_fallback_wide_offsets(cme, oracle_mod, monkeypatch):
     A = oracle_mod.ingest(n, r, c, v)
     m = cme.Matrix(n, r, c, v).pack()
     assert m.info().kernel == 1 and m.info().compact == 0
+    # rates in [1, 2) are all distinct: the compact-encodable band has no value index either
+    r2, c2, v2 = W.banded_markov(n, 6, 300, True, seed=9)
+    A2 = oracle_mod.ingest(n, r2, c2, v2)
+    m2 = cme.Matrix(n, r2, c2, v2).pack()
+    assert m2.info().kernel == 1 and m2.info().compact == 1
+    x2 = W.random_start(n, 6)
+    assert_spmv_close(m2.spmv(x2), oracle_mod.jacobi_step(A2, x2, 1.0))
     x = W.random_start(n, 5)
     assert_spmv_close(m.spmv(x), oracle_mod.jacobi_step(A, x, 1.0))
 
@@ -307,6 +340,7 @@ def test_nccl_one_rank_distributed_path(cme, oracle_mod):
 @pytest.mark.parametrize("knobs", [{"CME_TMA": "0", "CME_RESIDENT": "0"}, {"CME_TMA": "1", "CME_RESIDENT": "0"},
                                    {"CME_TMA": "1", "CME_TMA_WARPS": "8", "CME_RESIDENT": "0"},
                                    {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_COMPACT": "0"},
+                                   {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "0"},
                                    {"CME_RESIDENT": "1"}],
                          ids=lambda k: ",".join(f"{a}={b}" for a, b in k.items()))
 @pytest.mark.parametrize("net,order,omega", [(W.toggle_switch(70), "rcm", 0.9), (W.schnakenberg(120), "none", 1.0),
@@ -324,8 +358,10 @@ def test_every_step_kernel(cme, oracle_mod, monkeypatch, knobs, net, order, omeg
     f = m.info()
     expect = 3 if knobs.get("CME_RESIDENT") == "1" else 1 if knobs["CME_TMA"] == "1" else 0
     assert f.kernel == expect
-    # the TMA kernel streams the compact encoding unless CME_COMPACT=0
-    assert f.compact == (1 if expect == 1 and knobs.get("CME_COMPACT") != "0" else 0)
+    # the TMA kernel streams the value-indexed compact encoding (2) unless
+    # CME_VI=0 (compact, 1) or CME_COMPACT=0 (layout v0, 0)
+    want = 0 if expect != 1 or knobs.get("CME_COMPACT") == "0" else 1 if knobs.get("CME_VI") == "0" else 2
+    assert f.compact == want
     m.set_opts(omega=omega, check_every=7, stag_tol=0.0)
     x = W.random_start(A.n, 21)
     assert_spmv_close(m.spmv(x), oracle_mod.jacobi_step(A, x, omega))
@@ -347,7 +383,7 @@ def test_cfg4_full_size_parity(cme, oracle_mod):
     net = W.config_network("cfg4_toggle_20m")
     m = cme.Matrix.from_network(net).reorder(cme.CME_ORDER_RCM).pack()
     info = m.info()
-    assert info.n == 20015468 and info.nnz == 120042194 and info.kernel == 1 and info.compact == 1
+    assert info.n == 20015468 and info.nnz == 120042194 and info.kernel == 1 and info.compact == 2
     A = oracle_mod.network_csr(net)
     x = W.random_start(A.n, 17)
     m.set_opts(omega=1.0)

@@ -138,6 +138,9 @@ def test_pack_bit_exact(oracle_mod, net, order, window, band, fmt):
     else:
         gotc = m.compact()
         assert gotc["win_shift"] == refc["win_shift"]
+        refv = oracle_mod.value_index(ref)   # value-indexed form (sec. 5c), when <= 65536 values
+        if refv is not None:
+            refc.update(refv)
         assert set(gotc) == set(refc)
         for key in refc:
             if key != "win_shift":
@@ -175,7 +178,9 @@ def test_cfg2_toggle_full_host_parity(oracle_mod):
     for key in ("row_of", "slice_off", "slice_w", "val", "col", "inv_d", "lo", "up"):
         assert got[key].tobytes() == ref[key].tobytes(), key
     refc = oracle_mod.compact(oracle_mod.permute(A, oracle_mod.order_rcm(A)), ref)
+    refc.update(oracle_mod.value_index(ref))
     gotc = m.compact()
+    assert len(gotc["dict"]) == 447 + 1   # the toggle's distinct rates + the pad value 0
     for key in refc:
         if key != "win_shift":
             assert gotc[key].tobytes() == refc[key].tobytes(), key

@@ -247,3 +247,34 @@ def test_compact_rejects_wide_offsets_and_windows(oracle_mod):
     B = csr_from_edges(oracle_mod, 100, [(j, j + 1) for j in range(99)] + [(j + 1, j) for j in range(99)])
     assert oracle_mod.compact(B, oracle_mod.pack(B, window=96)) is None
     assert oracle_mod.compact(B, oracle_mod.pack(B, window=128)) is not None
+
+
+@pytest.mark.parametrize("net", [W.toggle_switch(40), W.schnakenberg(25), W.brusselator(30), W.birth_death(60)],
+                         ids=lambda n: n.name)
+@pytest.mark.parametrize("band", ["never", "always"])
+def test_value_index_reconstructs_layout(oracle_mod, net, band):
+    """Value-indexed form: dict[index] gives back every
+    stored value of layout v0 bit for bit (val, and lo/up when the band is on),
+    the dictionary is strictly ascending, and its size is the number of
+    distinct stored values (mass-action rates: r_k times small integers)."""
+    states, r, c, v = oracle_mod.enumerate_network(net)
+    A = oracle_mod.ingest(len(states), r, c, v)
+    P = oracle_mod.pack(A, window=256, band=band)
+    V = oracle_mod.value_index(P)
+    assert V is not None
+    d = V["dict"]
+    assert np.all(np.diff(d) > 0)
+    assert d[V["vidx"]].tobytes() == P["val"].tobytes()
+    if P["band_on"]:
+        assert d[V["loi"]].tobytes() == P["lo"].tobytes() and d[V["upi"]].tobytes() == P["up"].tobytes()
+    stored = set(P["val"].tolist()) | (set(P["lo"].tolist()) | set(P["up"].tolist()) if P["band_on"] else set())
+    assert len(d) == len(stored)
+    assert len(d) <= len(np.unique(v)) + 1       # + the pad value 0.0
+
+
+def test_value_index_limit(oracle_mod):
+    """More than 65536 distinct values: no value-indexed form."""
+    n = 70000
+    r, c, v = W.banded_markov(n, 5, 64, False, seed=2)
+    A = oracle_mod.ingest(n, r, c, v)
+    assert oracle_mod.value_index(oracle_mod.pack(A, window=256)) is None
