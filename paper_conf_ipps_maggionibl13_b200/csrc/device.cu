@@ -99,6 +99,7 @@ struct Device {
     // TMA-staged persistent kernel (kernels_tma.cuh)
     bool use_tma = false;
     int tma_ncw = 16;
+    int tma_spw = 1;                 // slices per consumer warp per tile (value-indexed kernel: 1 or 2)
     int tma_grid = 0, tma_stages = 0, tma_stage_bytes = 0, tma_off_val = 0, tma_off_col = 0, tma_contig = 0;
     int tma_xpf = 0;
     int tma_occ = 0;                 // TMA CTAs per SM
@@ -364,9 +365,10 @@ static cudaError_t tma_occupancy_b(int B, int ncw, int smem, int* occ) {
     }
 }
 
-// Stage geometry of the TMA kernel for NCW-slice tiles.
-static int64_t tma_stage_bytes(const Device& d, const Packed& P, int ncw, int64_t* off_val, int64_t* off_col,
+// Stage geometry of the TMA kernel for tiles of ts slices.
+static int64_t tma_stage_bytes(const Device& d, const Packed& P, int ts, int64_t* off_val, int64_t* off_col,
                                int64_t* n_tiles) {
+    const int ncw = ts;
     *n_tiles = (d.n_slices + ncw - 1) / ncw;
     int64_t max_nval = 0;
     for (int64_t t = 0; t < *n_tiles; ++t) {
@@ -379,7 +381,7 @@ static int64_t tma_stage_bytes(const Device& d, const Packed& P, int ncw, int64_
     if (d.vi) {    // [inv_d][row8][loi, upi][vidx][col16]
         *off_val = a128(vi_fixed_bytes(ncw, d.band, d.rearr));
         *off_col = *off_val + a128(2 * max_nval);
-        return kMetaBytes + a128(*off_col + 2 * max_nval);
+        return meta_bytes(ts) + a128(*off_col + 2 * max_nval);
     }
     if (d.cpt) {   // [row8][lo, up][val][col16]
         *off_val = a128(cpt_fixed_bytes(ncw, d.band, d.rearr));
@@ -409,13 +411,22 @@ static cme_status configure_tma(Device& d, const Packed& P) {
     const int stages_env = env_int("CME_TMA_STAGES", 0);   // 0 = auto
     const int stages_req = stages_env > 0 ? std::min(8, std::max(2, stages_env)) : 0;
     const int force_w = env_int("CME_TMA_WARPS", 0);
-    struct Shape { int ncw, stages, occ, grid; int64_t stage, off_val, off_col, n_tiles; };
+    struct Shape { int ncw, spw, stages, occ, grid; int64_t stage, off_val, off_col, n_tiles; };
+    const int force_spw = env_int("CME_TMA_SPW", 0);
+    struct Cand { int ncw, spw; };
+    // value-indexed: also 2 slices per warp on one CTA per SM (one dictionary
+    // per SM, a 5-stage ring) -- measured slower on cfg4 (210-217 vs 202 us),
+    // so it is last and wins no tie; CME_TMA_SPW=2 forces it
+    const Cand vi_cands[] = {{16, 1}, {8, 1}, {16, 2}}, std_cands[] = {{16, 1}, {8, 1}};
     Shape best{};
-    for (int ncw : {16, 8}) {
+    for (const Cand& cd : d.vi ? std::vector<Cand>(vi_cands, vi_cands + 3) : std::vector<Cand>(std_cands, std_cands + 2)) {
+        const int ncw = cd.ncw, spw = cd.spw;
         if (force_w && ncw != force_w) continue;
+        if (force_spw && d.vi && spw != force_spw) continue;
         Shape sh{};
         sh.ncw = ncw;
-        sh.stage = tma_stage_bytes(d, P, ncw, &sh.off_val, &sh.off_col, &sh.n_tiles);
+        sh.spw = spw;
+        sh.stage = tma_stage_bytes(d, P, ncw * spw, &sh.off_val, &sh.off_col, &sh.n_tiles);
         // the attribute is process-wide per kernel: always raise it to the
         // largest size any handle may use (handles on several host threads --
         // an in-process rank group -- would otherwise lower it under each
@@ -423,7 +434,7 @@ static cme_status configure_tma(Device& d, const Packed& P) {
         // dynamic-smem cap: the opt-in maximum minus the static shared memory
         // (barriers, check-reduction scratch: < 2 KB for 33 warps)
         const int cap = smem_max - (d.vi ? 4096 : 1024);
-        if (d.vi) CUDA_TRY(vi_prepare(ncw, cap));
+        if (d.vi) CUDA_TRY(vi_prepare(ncw, spw, cap));
         else if (d.cpt) CUDA_TRY(cpt_prepare(ncw, cap));
         else CUDA_TRY(tma_prepare_b(d.B, ncw, cap));
         const int64_t extra = d.vi ? d.dict_bytes : 0;   // the dictionary sits in front of the stages
@@ -431,7 +442,7 @@ static cme_status configure_tma(Device& d, const Packed& P) {
             *occ = 0;
             const int64_t bytes = extra + stages * sh.stage;
             if (bytes > cap) return cudaSuccess;
-            return d.vi ? vi_occupancy(ncw, (int)bytes, occ)
+            return d.vi ? vi_occupancy(ncw, spw, (int)bytes, occ)
                         : d.cpt ? cpt_occupancy(ncw, (int)bytes, occ)
                                 : tma_occupancy_b(d.B, ncw, (int)bytes, occ);
         };
@@ -446,7 +457,7 @@ static cme_status configure_tma(Device& d, const Packed& P) {
             // per SM loses 7% on the band-on config-5 matrices)
             sh.stages = 2;
             CUDA_TRY(occ_of(2, &sh.occ));
-            for (int st = 3; st <= 4 && sh.occ > 0; ++st) {
+            for (int st = 3; st <= (spw == 2 ? 8 : 4) && sh.occ > 0; ++st) {
                 int o = 0;
                 CUDA_TRY(occ_of(st, &o));
                 if (o < sh.occ) break;
@@ -454,17 +465,20 @@ static cme_status configure_tma(Device& d, const Packed& P) {
             }
         }
         if (env_int("CME_VERBOSE", 0) > 1)
-            std::fprintf(stderr, "[cme] tma shape: ncw=%d stages=%d stage=%lld extra=%lld occ=%d\n", ncw, sh.stages,
+            std::fprintf(stderr, "[cme] tma shape: ncw=%d spw=%d stages=%d stage=%lld extra=%lld occ=%d\n", ncw, spw, sh.stages,
                          (long long)sh.stage, (long long)extra, sh.occ);
         if (sh.occ < 1) continue;   // tiles too wide for this shape
         sh.occ = std::max(1, std::min(sh.occ, env_int("CME_TMA_CTAS", sh.occ)));
         sh.grid = (int)std::min<int64_t>(sh.n_tiles, (int64_t)sms * sh.occ);
-        if (sh.ncw * sh.occ > best.ncw * best.occ) best = sh;   // most resident consumer warps (ties: wider tiles)
+        // most slices in flight per SM (resident consumer warps x slices per
+        // warp); ties: the earlier candidate (wider tiles, fewer dictionaries)
+        if (sh.ncw * sh.spw * sh.occ > best.ncw * best.spw * best.occ) best = sh;
     }
     if (best.ncw == 0) return CME_OK;
     if (want < 0 && (best.ncw * best.occ < 16 || best.n_tiles < 2 * (int64_t)sms * best.occ))
         return CME_OK;   // too few resident consumer warps, or a small problem: register kernel
     d.tma_ncw = best.ncw;
+    d.tma_spw = best.spw;
     d.n_tiles = best.n_tiles;
     d.tma_stages = best.stages;
     d.tma_stage_bytes = (int)best.stage;
@@ -480,8 +494,8 @@ static cme_status configure_tma(Device& d, const Packed& P) {
     d.tma_xpf = xpf >= 0 ? xpf != 0 : (d.nx + 2) * 8 * d.B > (int64_t)48 << 20;
     d.use_tma = true;
     if (env_int("CME_VERBOSE", 0))
-        std::fprintf(stderr, "[cme] tma: B=%d compact=%d vi=%d dict=%d warps=%d stages=%d stage_bytes=%lld occ=%d grid=%d tiles=%lld\n",
-                     d.B, (int)d.cpt, (int)d.vi, d.dict_bytes, best.ncw, best.stages, (long long)best.stage, best.occ, best.grid, (long long)best.n_tiles);
+        std::fprintf(stderr, "[cme] tma: B=%d compact=%d vi=%d dict=%d warps=%d spw=%d stages=%d stage_bytes=%lld occ=%d grid=%d tiles=%lld\n",
+                     d.B, (int)d.cpt, (int)d.vi, d.dict_bytes, best.ncw, best.spw, best.stages, (long long)best.stage, best.occ, best.grid, (long long)best.n_tiles);
     return CME_OK;
 }
 
@@ -692,14 +706,14 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
         // value-indexed (sec. 5c) when the dictionary fits next to a ring with
         // as many resident consumer warps (CME_VI = -1 auto / 0 off / 1 force)
         if ((s = configure_tma(*d, P)) != CME_OK) return fail(s);   // compact stage geometry
-        const int cpt_warps = d->use_tma ? d->tma_ncw * d->tma_occ : 0;
+        const int cpt_warps = d->use_tma ? d->tma_ncw * d->tma_spw * d->tma_occ : 0;
         const int want_vi = env_int("CME_VI", -1);
         if (want_vi != 0 && encode_value_index(P, h->Cpt)) {
             d->vi = true;
             d->dict_bytes = (int)((h->Cpt.dict.size() * 8 + 127) / 128 * 128);
             if ((s = configure_tma(*d, P)) != CME_OK) return fail(s);
             // auto: only if the dictionary costs no resident consumer warps
-            if (!d->use_tma || (want_vi < 0 && d->tma_ncw * d->tma_occ < cpt_warps)) {
+            if (!d->use_tma || (want_vi < 0 && d->tma_ncw * d->tma_spw * d->tma_occ < cpt_warps)) {
                 d->vi = false;
                 d->dict_bytes = 0;
                 if ((s = configure_tma(*d, P)) != CME_OK) return fail(s);
@@ -710,9 +724,10 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
     if ((s = configure_resident(*d, P, comm != nullptr || h->nranks > 1)) != CME_OK) return fail(s);
     if ((s = preload_kernels(B)) != CME_OK) return fail(s);
     if (d->use_tma) {
-        std::vector<int2> tm((size_t)d->n_tiles * d->tma_ncw, make_int2(0, 0));   // whole tiles (TMA copies)
+        const int ts = d->tma_ncw * d->tma_spw;   // slices per tile
+        std::vector<int2> tm((size_t)d->n_tiles * ts, make_int2(0, 0));   // whole tiles (TMA copies)
         for (int64_t q = 0; q < P.n_slices; ++q)
-            tm[q] = make_int2((int)(P.slice_off[q] - P.slice_off[q / d->tma_ncw * d->tma_ncw]), P.slice_w[q]);
+            tm[q] = make_int2((int)(P.slice_off[q] - P.slice_off[q / ts * ts]), P.slice_w[q]);
         if ((s = d->upload(d->tile_meta, tm)) != CME_OK) return fail(s);
     }
     if (d->format != CME_FMT_CSR) {
@@ -1012,7 +1027,7 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
                                  d.tma_contig, d.tma_xpf},
                          d.col16, d.row8, d.win_shift},
                  d.dict, d.vidx, d.loi, d.upi, d.dict_bytes};
-        CUDA_TRY(launch_vi(V, d.tma_ncw, d.tma_grid, d.dict_bytes + d.tma_stages * d.tma_stage_bytes, d.band, d.rearr,
+        CUDA_TRY(launch_vi(V, d.tma_ncw, d.tma_spw, d.tma_grid, d.dict_bytes + d.tma_stages * d.tma_stage_bytes, d.band, d.rearr,
                            check, pdl, s));
     } else if (d.use_tma && d.cpt) {
         a.val = d.cval;

@@ -233,25 +233,25 @@ __host__ __device__ inline int vi_fixed_bytes(int ncw, bool band, bool rearr) {
     return ncw * 32 * (8 + (rearr ? 1 : 0) + (band ? 4 : 0));
 }
 
-template <int NCW, bool BAND, bool REARR>
+template <int TS, bool BAND, bool REARR>
 __device__ __noinline__ void vi_issue_call(unsigned char* st, uint64_t* bar, const int64_t* slice_off,
                                            int64_t slice_end, const double* inv_d, const uint8_t* row8,
                                            const uint16_t* loi, const uint16_t* upi, const uint16_t* vidx,
                                            const int16_t* col16, int off_val, int off_col, int64_t tile,
                                            uint64_t pol, const int2* tile_meta) {
-    constexpr int kSlots = NCW * 32;
+    constexpr int kSlots = TS * 32;
     constexpr int kOffRow = 8 * kSlots, kOffLo = kOffRow + (REARR ? kSlots : 0), kOffUp = kOffLo + 2 * kSlots;
-    const int64_t q0 = tile * NCW;
-    const int64_t q1 = min(q0 + NCW, slice_end);
+    const int64_t q0 = tile * TS;
+    const int64_t q1 = min(q0 + TS, slice_end);
     const int64_t e0 = slice_off[q0], e1 = slice_off[q1];
     const uint32_t slots = (uint32_t)(q1 - q0) * 32u;
     const uint32_t nval = (uint32_t)(e1 - e0);
-    uint32_t bytes = nval * 4u + slots * 8u + NCW * 8u;
+    uint32_t bytes = nval * 4u + slots * 8u + TS * 8u;
     if (REARR) bytes += slots;
     if (BAND) bytes += slots * 4u;
     mbar_expect_tx(bar, bytes);
-    issue_meta(st, bar, tile_meta, tile, NCW, pol);
-    st += kMetaBytes;
+    issue_meta(st, bar, tile_meta, tile, TS, pol);
+    st += meta_bytes(TS);
     bulk_g2s(st, inv_d + q0 * 32, slots * 8u, bar, pol);
     if (REARR) bulk_g2s(st + kOffRow, row8 + q0 * 32, slots, bar, pol);
     if (BAND) {
@@ -264,33 +264,60 @@ __device__ __noinline__ void vi_issue_call(unsigned char* st, uint64_t* bar, con
     }
 }
 
-template <int NCW, bool BAND, bool REARR>
+template <int TS, bool BAND, bool REARR>
 __device__ __forceinline__ void vi_issue(const ViArgs& V, unsigned char* stages, uint64_t* full, int64_t tile, int s,
                                          uint64_t pol) {
     const StepArgs& a = V.K.T.a;
     if (V.K.T.xpf) {
-        const int64_t r0 = tile * NCW * 32, r1 = min(r0 + NCW * 32, a.n_rows);
+        const int64_t r0 = tile * TS * 32, r1 = min(r0 + TS * 32, a.n_rows);
         if (r1 > r0) prefetch_l2(a.x + a.own_off + r0, (uint64_t)(r1 - r0) * 8);
     }
-    vi_issue_call<NCW, BAND, REARR>(stages + (size_t)s * V.K.T.stage_bytes, &full[s], a.slice_off, a.slice_end,
-                                    a.inv_d, V.K.row8, V.loi, V.upi, V.vidx, V.K.col16, V.K.T.off_val, V.K.T.off_col,
-                                    tile, pol, a.tile_meta);
+    vi_issue_call<TS, BAND, REARR>(stages + (size_t)s * V.K.T.stage_bytes, &full[s], a.slice_off, a.slice_end,
+                                   a.inv_d, V.K.row8, V.loi, V.upi, V.vidx, V.K.col16, V.K.T.off_val, V.K.T.off_col,
+                                   tile, pol, a.tile_meta);
 }
 
+// One slot's W entries: all x gathers and dictionary reads issued first, then
+// the FMAs in t order (the layout-v0 order: acc = val * x + acc).
 template <int W>
-__device__ __forceinline__ void ell_row_vi(const int16_t* scol, const uint16_t* svi, const double* sdict,
-                                           const double* xr, double& acc) {
-    double xv[W];
+__device__ __forceinline__ double vi_row(const int16_t* scol, const uint16_t* svi, const double* sdict,
+                                         const double* xr) {
+    double xv[W], vv[W];
 #pragma unroll
     for (int u = 0; u < W; ++u) xv[u] = __ldg(xr + scol[32 * u]);
 #pragma unroll
-    for (int u = 0; u < W; ++u) acc = fma(sdict[svi[32 * u]], xv[u], acc);
+    for (int u = 0; u < W; ++u) vv[u] = sdict[svi[32 * u]];
+    double acc = 0.0;
+#pragma unroll
+    for (int u = 0; u < W; ++u) acc = fma(vv[u], xv[u], acc);
+    return acc;
+}
+// Slots wider than 8: chunks of 8, same order.
+__device__ __forceinline__ double vi_row_wide(const int16_t* scol, const uint16_t* svi, const double* sdict,
+                                              const double* xr, int w) {
+    double acc = 0.0;
+    for (int t0 = 0; t0 < w; t0 += 8) {
+        double xc[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u)
+            if (t0 + u < w) xc[u] = __ldg(xr + scol[32 * (t0 + u)]);
+#pragma unroll
+        for (int u = 0; u < 8; ++u)
+            if (t0 + u < w) acc = fma(sdict[svi[32 * (t0 + u)]], xc[u], acc);
+    }
+    return acc;
 }
 
-template <int NCW, bool BAND, bool REARR, bool CHECK>
-__global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBlocks)
+// NCW consumer warps, each taking SPW slices of a tile of NCW*SPW slices:
+// with SPW = 2 the warp issues both slices' gathers before any FMA (twice the
+// memory-level parallelism per warp) and the CTA runs alone on its SM -- one
+// dictionary per SM instead of two, so the freed shared memory deepens the
+// TMA ring.
+template <int NCW, int SPW, bool BAND, bool REARR, bool CHECK>
+__global__ void __launch_bounds__(TmaShape<NCW>::kThreads, SPW == 1 ? TmaShape<NCW>::kMinBlocks : 1)
     sell_vi_kernel(const ViArgs V) {
-    constexpr int kConsumers = NCW, kTileSlices = NCW, kSlots = NCW * 32;
+    constexpr int kConsumers = NCW, kTileSlices = NCW * SPW, kSlots = kTileSlices * 32;
+    constexpr int kMeta = meta_bytes(kTileSlices);
     constexpr int kOffRow = 8 * kSlots, kOffLo = kOffRow + (REARR ? kSlots : 0), kOffUp = kOffLo + 2 * kSlots;
     const CptArgs& K = V.K;
     const TmaArgs& T = K.T;
@@ -319,11 +346,12 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
     const int pro = (int)(my_tiles < (int64_t)S ? my_tiles : (int64_t)S);
     if (producer) {   // dictionary and first tiles are constant: load while the previous step drains
         pol = evict_first_policy();
-        mbar_expect_tx(&dbar, (uint32_t)V.dict_bytes);
         uint64_t keep;   // every CTA reads the dictionary: keep it in L2
         asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(keep));
+        mbar_expect_tx(&dbar, (uint32_t)V.dict_bytes);
         bulk_g2s(smem, V.dict, (uint32_t)V.dict_bytes, &dbar, keep);
-        for (int i = 0; i < pro; ++i) vi_issue<NCW, BAND, REARR>(V, stages, full, t_first + (int64_t)i * t_stride, i, pol);
+        for (int i = 0; i < pro; ++i)
+            vi_issue<kTileSlices, BAND, REARR>(V, stages, full, t_first + (int64_t)i * t_stride, i, pol);
     }
     pdl_wait();
     if (a.stop != nullptr && *a.stop) {
@@ -340,7 +368,7 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
             uint32_t phase = 1;
             for (int64_t tile = t_first + (int64_t)pro * t_stride; tile < t_end; tile += t_stride) {
                 mbar_wait(&empty[s], phase ^ 1u);
-                vi_issue<NCW, BAND, REARR>(V, stages, full, tile, s, pol);
+                vi_issue<kTileSlices, BAND, REARR>(V, stages, full, tile, s, pol);
                 if (++s == S) { s = 0; phase ^= 1u; }
             }
         }
@@ -353,48 +381,80 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
         uint32_t phase = 0;
         for (int64_t tile = t_first; tile < t_end; tile += t_stride) {
             const int64_t q0 = tile * kTileSlices;
-            const int64_t q = q0 + warp;
-            const unsigned char* st = stages + (size_t)s * T.stage_bytes + kMetaBytes;
+            const unsigned char* st = stages + (size_t)s * T.stage_bytes + kMeta;
             mbar_wait(&full[s], phase);
-            const int2 meta = reinterpret_cast<const int2*>(st - kMetaBytes)[warp];   // {offset in tile, width}
-            const int w = meta.y;
-            const int64_t loff = meta.x;
-            const int64_t slot = q * 32 + lane;
-            if (q < a.slice_end && slot < a.n_rows) {
-                const int ls = warp * 32 + lane;
-                const uint16_t* svi = reinterpret_cast<const uint16_t*>(st + T.off_val) + loff + lane;
-                const int16_t* scol = reinterpret_cast<const int16_t*>(st + T.off_col) + loff + lane;
-                const int64_t r = REARR ? ((slot >> K.win_shift) << K.win_shift) + st[kOffRow + ls] : slot;
-                RowX<1, BAND> X;
-                X.load(xo, r);
-                const double* xr = xo + r;
-                double acc = 0.0;
-                switch (w) {   // warp-uniform exact widths
-                    case 0: break;
-                    case 1: ell_row_vi<1>(scol, svi, sdict, xr, acc); break;
-                    case 2: ell_row_vi<2>(scol, svi, sdict, xr, acc); break;
-                    case 3: ell_row_vi<3>(scol, svi, sdict, xr, acc); break;
-                    case 4: ell_row_vi<4>(scol, svi, sdict, xr, acc); break;
-                    case 5: ell_row_vi<5>(scol, svi, sdict, xr, acc); break;
-                    case 6: ell_row_vi<6>(scol, svi, sdict, xr, acc); break;
-                    case 7: ell_row_vi<7>(scol, svi, sdict, xr, acc); break;
-                    case 8: ell_row_vi<8>(scol, svi, sdict, xr, acc); break;
-                    default:
-                        for (int t0 = 0; t0 < w; t0 += 8) {
-                            double xv[8];
+            int w[SPW], ls[SPW];
+            int64_t r[SPW];
+            bool live[SPW];
+            RowX<1, BAND> X[SPW];
+            double acc[SPW];
+            const int16_t* scol[SPW];
+            const uint16_t* svi[SPW];
 #pragma unroll
-                            for (int u = 0; u < 8; ++u)
-                                if (t0 + u < w) xv[u] = __ldg(xr + scol[32 * (t0 + u)]);
-#pragma unroll
-                            for (int u = 0; u < 8; ++u)
-                                if (t0 + u < w) acc = fma(sdict[svi[32 * (t0 + u)]], xv[u], acc);
-                        }
+            for (int j = 0; j < SPW; ++j) {   // the warp's slices: rows, own/band x loads
+                const int sl = warp + j * NCW;
+                const int2 meta = reinterpret_cast<const int2*>(st - kMeta)[sl];   // {offset in tile, width}
+                const int64_t q = q0 + sl, slot = q * 32 + lane;
+                w[j] = meta.y;
+                ls[j] = sl * 32 + lane;
+                live[j] = q < a.slice_end && slot < a.n_rows;
+                acc[j] = 0.0;
+                r[j] = live[j] ? (REARR ? ((slot >> K.win_shift) << K.win_shift) + st[kOffRow + ls[j]] : slot) : 0;
+                svi[j] = reinterpret_cast<const uint16_t*>(st + T.off_val) + meta.x + lane;
+                scol[j] = reinterpret_cast<const int16_t*>(st + T.off_col) + meta.x + lane;
+                if (live[j]) X[j].load(xo, r[j]);
+            }
+            if constexpr (SPW == 1) {
+                if (live[0]) {
+                    const double* xr = xo + r[0];
+                    switch (w[0]) {   // warp-uniform exact widths: gathers + dictionary reads, then FMAs
+                        case 0: break;
+                        case 1: acc[0] = vi_row<1>(scol[0], svi[0], sdict, xr); break;
+                        case 2: acc[0] = vi_row<2>(scol[0], svi[0], sdict, xr); break;
+                        case 3: acc[0] = vi_row<3>(scol[0], svi[0], sdict, xr); break;
+                        case 4: acc[0] = vi_row<4>(scol[0], svi[0], sdict, xr); break;
+                        case 5: acc[0] = vi_row<5>(scol[0], svi[0], sdict, xr); break;
+                        case 6: acc[0] = vi_row<6>(scol[0], svi[0], sdict, xr); break;
+                        case 7: acc[0] = vi_row<7>(scol[0], svi[0], sdict, xr); break;
+                        case 8: acc[0] = vi_row<8>(scol[0], svi[0], sdict, xr); break;
+                        default: acc[0] = vi_row_wide(scol[0], svi[0], sdict, xr, w[0]);
+                    }
                 }
-                const double accv[1] = {acc};
-                const double idv[1] = {reinterpret_cast<const double*>(st)[ls]};
-                const double lov[1] = {BAND ? sdict[reinterpret_cast<const uint16_t*>(st + kOffLo)[ls]] : 0.0};
-                const double upv[1] = {BAND ? sdict[reinterpret_cast<const uint16_t*>(st + kOffUp)[ls]] : 0.0};
-                finish_row_x<1, BAND, CHECK>(a, r, yo, accv, lov, upv, idv, a.pre_scale, ck, X);
+            } else {
+                // both slices' loads in flight before any FMA; widths <= 8
+                // predicated (static register indices), wider slices chunked
+                // (dictionary values are read at FMA time: 96 registers per
+                // thread at 17 warps per SM do not hold them too)
+                double xv[SPW][8];
+#pragma unroll
+                for (int j = 0; j < SPW; ++j) {
+                    const double* xr = xo + r[j];
+                    if (live[j] && w[j] <= 8) {
+#pragma unroll
+                        for (int u = 0; u < 8; ++u)
+                            if (u < w[j]) xv[j][u] = __ldg(xr + scol[j][32 * u]);
+                    }
+                }
+#pragma unroll
+                for (int j = 0; j < SPW; ++j) {
+                    if (!live[j]) continue;
+                    if (w[j] <= 8) {
+#pragma unroll
+                        for (int u = 0; u < 8; ++u)
+                            if (u < w[j]) acc[j] = fma(sdict[svi[j][32 * u]], xv[j][u], acc[j]);
+                    } else {
+                        acc[j] = vi_row_wide(scol[j], svi[j], sdict, xo + r[j], w[j]);
+                    }
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < SPW; ++j) {   // epilogue
+                if (!live[j]) continue;
+                const double accv[1] = {acc[j]};
+                const double idv[1] = {reinterpret_cast<const double*>(st)[ls[j]]};
+                const double lov[1] = {BAND ? sdict[reinterpret_cast<const uint16_t*>(st + kOffLo)[ls[j]]] : 0.0};
+                const double upv[1] = {BAND ? sdict[reinterpret_cast<const uint16_t*>(st + kOffUp)[ls[j]]] : 0.0};
+                finish_row_x<1, BAND, CHECK>(a, r[j], yo, accv, lov, upv, idv, a.pre_scale, ck, X[j]);
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);

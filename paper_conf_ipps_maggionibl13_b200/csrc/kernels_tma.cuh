@@ -59,7 +59,9 @@ __device__ __forceinline__ void tma_tile_range(const TmaArgs& T, int64_t* first,
 // by the same TMA transaction as the tile.  Reading it from global memory put
 // two dependent L2 round trips (slice_off[q], slice_off[q0]) at the head of
 // every consumer's tile -- the top stall in the ncu source view (16.5%).
-constexpr int kMetaBytes = 128;   // >= NCW * 8 for NCW <= 16, keeps the data 128-B aligned
+// bytes of the metadata block of a tile of ts slices (keeps the data 128-B aligned)
+__host__ __device__ constexpr int meta_bytes(int ts) { return (ts * 8 + 127) / 128 * 128; }
+constexpr int kMetaBytes = 128;   // = meta_bytes(NCW) for the NCW <= 16 one-slice-per-warp tiles
 
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
