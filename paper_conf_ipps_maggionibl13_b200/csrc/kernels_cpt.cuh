@@ -228,9 +228,12 @@ struct ViArgs {
     int32_t dict_bytes;    // multiple of 128: stages start here in shared memory
 };
 
-// Stage layout: [inv_d][row8 if REARR][loi, upi if BAND][vidx][col16].
+// Stage layout: [row8 if REARR][loi, upi if BAND][vidx][col16].  inv_d is not
+// staged: each lane streams its own 8 bytes from global memory next to its x
+// loads, which keeps the stages small enough for a 4-deep ring next to the
+// two dictionaries of an SM (measured: 3 stages 178 us vs 2 stages 206 us).
 __host__ __device__ inline int vi_fixed_bytes(int ncw, bool band, bool rearr) {
-    return ncw * 32 * (8 + (rearr ? 1 : 0) + (band ? 4 : 0));
+    return ncw * 32 * ((rearr ? 1 : 0) + (band ? 4 : 0));
 }
 
 template <int TS, bool BAND, bool REARR>
@@ -240,19 +243,18 @@ __device__ __noinline__ void vi_issue_call(unsigned char* st, uint64_t* bar, con
                                            const int16_t* col16, int off_val, int off_col, int64_t tile,
                                            uint64_t pol, const int2* tile_meta) {
     constexpr int kSlots = TS * 32;
-    constexpr int kOffRow = 8 * kSlots, kOffLo = kOffRow + (REARR ? kSlots : 0), kOffUp = kOffLo + 2 * kSlots;
+    constexpr int kOffRow = 0, kOffLo = kOffRow + (REARR ? kSlots : 0), kOffUp = kOffLo + 2 * kSlots;
     const int64_t q0 = tile * TS;
     const int64_t q1 = min(q0 + TS, slice_end);
     const int64_t e0 = slice_off[q0], e1 = slice_off[q1];
     const uint32_t slots = (uint32_t)(q1 - q0) * 32u;
     const uint32_t nval = (uint32_t)(e1 - e0);
-    uint32_t bytes = nval * 4u + slots * 8u + TS * 8u;
+    uint32_t bytes = nval * 4u + TS * 8u;
     if (REARR) bytes += slots;
     if (BAND) bytes += slots * 4u;
     mbar_expect_tx(bar, bytes);
     issue_meta(st, bar, tile_meta, tile, TS, pol);
     st += meta_bytes(TS);
-    bulk_g2s(st, inv_d + q0 * 32, slots * 8u, bar, pol);
     if (REARR) bulk_g2s(st + kOffRow, row8 + q0 * 32, slots, bar, pol);
     if (BAND) {
         bulk_g2s(st + kOffLo, loi + q0 * 32, slots * 2u, bar, pol);
@@ -318,7 +320,7 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, SPW == 1 ? TmaShape<N
     sell_vi_kernel(const ViArgs V) {
     constexpr int kConsumers = NCW, kTileSlices = NCW * SPW, kSlots = kTileSlices * 32;
     constexpr int kMeta = meta_bytes(kTileSlices);
-    constexpr int kOffRow = 8 * kSlots, kOffLo = kOffRow + (REARR ? kSlots : 0), kOffUp = kOffLo + 2 * kSlots;
+    constexpr int kOffRow = 0, kOffLo = kOffRow + (REARR ? kSlots : 0), kOffUp = kOffLo + 2 * kSlots;
     const CptArgs& K = V.K;
     const TmaArgs& T = K.T;
     const StepArgs& a = T.a;
@@ -373,6 +375,72 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, SPW == 1 ? TmaShape<N
             }
         }
         if (lane == 0 && my_tiles == 0) mbar_wait(&dbar, 0u);   // no tile ever waits on it
+    } else if constexpr (SPW == 1) {
+        // one slice per warp: loop invariants hoisted (the ncu instruction
+        // census found ~120 per-slice instructions, mostly kernel-parameter
+        // reloads and 64-bit index arithmetic); 32-bit slot/row indices
+        // (n < 2^31); the epilogue is finish_row_x's arithmetic, with the
+        // pending scale (constant for this launch) read once
+        const double* xo = a.x + a.own_off;
+        double* yo = a.y + a.own_off;
+        const int n_rows = (int)a.n_rows, slice_end = (int)a.slice_end, ws = K.win_shift;
+        const int stage_bytes = T.stage_bytes, off_val = T.off_val, off_col = T.off_col;
+        const double om = a.omega, om1 = 1.0 - a.omega;
+        const bool damp = om != 1.0, unif = a.unif_lam_inv != 0.0;
+        const double sc = a.pre_scale != nullptr ? a.pre_scale[0] : 1.0;
+        const int npush = a.npush;
+        const uint64_t pol_s = evict_first_policy();
+        mbar_wait(&dbar, 0u);
+        int s = 0;
+        uint32_t phase = 0;
+        for (int64_t tile = t_first; tile < t_end; tile += t_stride) {
+            const unsigned char* st = stages + s * stage_bytes + kMeta;
+            mbar_wait(&full[s], phase);
+            const int2 meta = reinterpret_cast<const int2*>(st - kMeta)[warp];   // {offset in tile, width}
+            const int q = (int)tile * kTileSlices + warp;
+            const int slot = q * 32 + lane;
+            if (q < slice_end && slot < n_rows) {
+                const int ls = warp * 32 + lane;
+                const int r = REARR ? ((slot >> ws) << ws) + st[kOffRow + ls] : slot;
+                const double id = ld_stream(a.inv_d + slot, pol_s);   // with the x loads, before the gathers
+                RowX<1, BAND> X;
+                X.load(xo, r);
+                const double* xr = xo + r;
+                const uint16_t* svi = reinterpret_cast<const uint16_t*>(st + off_val) + meta.x + lane;
+                const int16_t* scol = reinterpret_cast<const int16_t*>(st + off_col) + meta.x + lane;
+                double acc = 0.0;
+                switch (meta.y) {   // warp-uniform exact widths
+                    case 0: break;
+                    case 1: acc = vi_row<1>(scol, svi, sdict, xr); break;
+                    case 2: acc = vi_row<2>(scol, svi, sdict, xr); break;
+                    case 3: acc = vi_row<3>(scol, svi, sdict, xr); break;
+                    case 4: acc = vi_row<4>(scol, svi, sdict, xr); break;
+                    case 5: acc = vi_row<5>(scol, svi, sdict, xr); break;
+                    case 6: acc = vi_row<6>(scol, svi, sdict, xr); break;
+                    case 7: acc = vi_row<7>(scol, svi, sdict, xr); break;
+                    case 8: acc = vi_row<8>(scol, svi, sdict, xr); break;
+                    default: acc = vi_row_wide(scol, svi, sdict, xr, meta.y);
+                }
+                const double sum = BAND ? fma(sdict[reinterpret_cast<const uint16_t*>(st + kOffLo)[ls]], X.xl[0],
+                                              sdict[reinterpret_cast<const uint16_t*>(st + kOffUp)[ls]] * X.xu[0]) + acc
+                                        : acc;
+                const double x_r = X.xr[0];
+                double y = damp ? fma(om1, x_r, om * (id * sum)) : id * sum;
+                if (unif) {   // transient: (I + A/Lambda) x with a_rr = -1/id
+                    y = fma(a.unif_lam_inv, sum - x_r / id, x_r);
+                    double* ac = a.acc + a.own_off + r;
+                    *ac = fma(a.acc_w, x_r, *ac);
+                }
+                y *= sc;   // = finish_row_x's pending-scale multiply (exact when sc = 1)
+                yo[r] = y;
+                if (CHECK) ck.add(0, y, ((damp || CHECK) ? x_r : 0.0) * sc, id);
+                for (int p = 0; p < npush; ++p)   // halo rows straight into the peer's buffer
+                    if (r >= a.push_lo[p] && r < a.push_hi[p]) a.push_y[p][r] = y;
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);
+            if (++s == S) { s = 0; phase ^= 1u; }
+        }
     } else {
         const double* xo = a.x + a.own_off;
         double* yo = a.y + a.own_off;
@@ -451,7 +519,7 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, SPW == 1 ? TmaShape<N
             for (int j = 0; j < SPW; ++j) {   // epilogue
                 if (!live[j]) continue;
                 const double accv[1] = {acc[j]};
-                const double idv[1] = {reinterpret_cast<const double*>(st)[ls[j]]};
+                const double idv[1] = {__ldg(a.inv_d + (q0 + warp + j * NCW) * 32 + lane)};
                 const double lov[1] = {BAND ? sdict[reinterpret_cast<const uint16_t*>(st + kOffLo)[ls[j]]] : 0.0};
                 const double upv[1] = {BAND ? sdict[reinterpret_cast<const uint16_t*>(st + kOffUp)[ls[j]]] : 0.0};
                 finish_row_x<1, BAND, CHECK>(a, r[j], yo, accv, lov, upv, idv, a.pre_scale, ck, X[j]);
