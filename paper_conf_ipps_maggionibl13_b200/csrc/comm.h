@@ -35,6 +35,7 @@ struct P2PRank {
     double* io = nullptr;       // [n_global * B] reordered staging
     int64_t span_lo = 0;        // first global row of the x-span
     int device = 0;
+    unsigned char uuid[16] = {};  // physical GPU (cudaDeviceProp::uuid)
 };
 
 int comm_transport(const cme_comm_s* c);

@@ -93,6 +93,7 @@ struct Device {
     int64_t push_lo[kMaxPushPeers] = {}, push_hi[kMaxPushPeers] = {};   // local rows
     double* push_y[2][kMaxPushPeers] = {};   // peer buffer (parity b) shifted to my local rows
     bool peers_ready = false;        // IPC transport: attach done
+    bool bar_pdl = false;            // step barrier launched with PDL (peers on other GPUs only)
     std::vector<void*> ipc_opened;   // peer allocations mapped into this process
     HaloPlan halo;                   // counts/offsets in doubles (rows x B)
     std::vector<int64_t> cuts;       // in doubles (rows x B) for the output broadcast
@@ -259,8 +260,16 @@ struct BarrierArgs {
     int npeer, rank;
     const int32_t* stop;   // nullable: skip when the solve has stopped (all ranks agree)
     Ctrl* ctrl;
+    int32_t early;   // 1: let the next step launch early (peers on other GPUs only)
 };
 __global__ void p2p_barrier_kernel(const BarrierArgs a) {
+    // launched with programmatic dependent launch after a step: wait for the
+    // step's grid (its stores, peer pushes included, are then complete), then
+    // let the next step's CTAs launch and run their prologue (TMA prefetch of
+    // their first tiles, dictionary load) while this thread publishes/spins;
+    // the next step's griddepcontrol.wait still waits for this kernel
+    pdl_wait();
+    if (a.early) pdl_trigger();   // (the trigger, not the launch attribute, releases the dependent)
     if (threadIdx.x != 0) return;
     if (a.stop != nullptr && *a.stop) return;
     const int64_t e = *a.epoch + 1;
@@ -803,8 +812,8 @@ static cme_status p2p_barrier(Device& d, cudaStream_t s, bool respect_stop) {
     b.rank = d.rank;
     b.stop = respect_stop ? &d.ctrl->stop : nullptr;
     b.ctrl = d.ctrl;
-    p2p_barrier_kernel<<<1, 32, 0, s>>>(b);
-    CUDA_TRY(cudaGetLastError());
+    b.early = d.bar_pdl ? 1 : 0;
+    CUDA_TRY(launch_ex(p2p_barrier_kernel, dim3(1), dim3(32), 0, d.bar_pdl, s, b));
     return CME_OK;
 }
 
@@ -891,6 +900,12 @@ static void p2p_wire(cme_matrix_s* h, const std::vector<P2PRank>& all) {
         for (int b = 0; b < 2; ++b) d.push_y[b][d.npush] = all[sp].xb[b] + shift;
         ++d.npush;
     }
+    // the step barrier may let the next step's CTAs launch early (PDL) only
+    // when no peer shares this GPU: early-resident persistent CTAs would keep
+    // a same-GPU peer's step off the SMs while the barrier waits for it
+    d.bar_pdl = env_int("CME_PDL", 1) != 0;
+    for (int r = 0; r < d.nranks; ++r)
+        if (r != d.rank && std::memcmp(all[r].uuid, all[d.rank].uuid, 16) == 0) d.bar_pdl = false;
     d.peers_ready = true;
 }
 
@@ -904,6 +919,8 @@ static P2PRank p2p_mine(cme_matrix_s* h) {
     mine.io = d.io;
     mine.span_lo = h->span[2 * h->rank];
     mine.device = d.dev;
+    cudaDeviceProp pr;
+    if (cudaGetDeviceProperties(&pr, d.dev) == cudaSuccess) std::memcpy(mine.uuid, &pr.uuid, 16);
     return mine;
 }
 
@@ -926,6 +943,7 @@ struct IpcBlob {
     int64_t span_lo;
     cudaIpcMemHandle_t h[5];   // xb[0] base, xb[1] base, flags, gather, io
     int64_t off[5];            // byte offset of the published pointer in its allocation
+    unsigned char uuid[16];    // the exporting process's physical GPU
 };
 static_assert(sizeof(IpcBlob) <= CME_IPC_BLOB_BYTES, "IPC blob too large");
 constexpr uint64_t kIpcMagic = 0x434d45495043ull;   // "CMEIPC"
@@ -939,6 +957,10 @@ cme_status device_ipc_export(cme_matrix_s* h, uint8_t* out) {
     b.rank = d.rank;
     b.device = d.dev;
     b.span_lo = h->span[2 * h->rank];
+    {
+        const P2PRank me = p2p_mine(h);
+        std::memcpy(b.uuid, me.uuid, 16);
+    }
     // allocation bases (device_upload): xb[b] sits one sentinel row of B doubles in
     void* bases[5] = {d.xb[0] - d.B, d.xb[1] - d.B, d.flags, d.gather, d.io};
     const int64_t offs[5] = {(int64_t)(d.B * sizeof(double)), (int64_t)(d.B * sizeof(double)), 0, 0, 0};
@@ -974,6 +996,7 @@ cme_status device_ipc_attach(cme_matrix_s* h, const uint8_t* blobs) {
         all[r].io = (double*)mapped[4];
         all[r].span_lo = b.span_lo;
         all[r].device = b.device;
+        std::memcpy(all[r].uuid, b.uuid, 16);
     }
     p2p_wire(h, all);
     return CME_OK;
@@ -1130,8 +1153,10 @@ static cme_status enqueue_block(Device& d, cudaStream_t s, int start, int64_t C,
     return launch_finalize(d, s, (int32_t)C, final_partial ? 1 : 0);
 }
 
-static cme_status ensure_graphs(Device& d, int64_t C, double omega) {
+static cme_status ensure_graphs(Device& d, int64_t C, double omega, bool* built = nullptr) {
+    if (built) *built = false;
     if (d.gC == C && d.gomega == omega && d.gexec[0]) return CME_OK;
+    if (built) *built = true;
     if (d.comm && !d.p2p) {
         // NCCL sets up peer connections lazily on first use: do that outside
         // the capture (one throw-away exchange + gather on the private stream)
@@ -1155,6 +1180,19 @@ static cme_status ensure_graphs(Device& d, int64_t C, double omega) {
     }
     d.gC = C;
     d.gomega = omega;
+    return CME_OK;
+}
+
+// Build the check-block graphs before any exchange of this call, and in an
+// in-process rank group let every rank finish building before any rank
+// launches a spinning barrier: graph instantiation/destruction in one rank's
+// thread can wait on the device, i.e. on a peer's barrier kernel that waits
+// for this rank (observed as sporadic barrier time-outs of the virtual-rank
+// tests).  All ranks rebuild at the same calls (same C and omega).
+static cme_status prepare_graphs(Device& d, int64_t C, double omega) {
+    bool built = false;
+    CME_TRY(ensure_graphs(d, C, omega, &built));
+    if (built && d.comm && comm_transport(d.comm) == kTransportP2P) comm_p2p_host_barrier(d.comm);
     return CME_OK;
 }
 
@@ -1307,6 +1345,7 @@ cme_status device_solve(cme_matrix_s* h, const double* p0, double tol, int64_t m
     cudaStream_t s = stream_of(h);
     const int64_t C = h->sopts.check_every;
     const double omega = effective_omega(h);
+    if (!d.use_res) CME_TRY(prepare_graphs(d, C, omega));
     CME_TRY(load_iterate(h, p0, true, s));
     // solve parameters (inv_s / mass / bad_input from the load are kept: they
     // live after `bad_input` in Ctrl)
@@ -1329,7 +1368,6 @@ cme_status device_solve(cme_matrix_s* h, const double* p0, double tol, int64_t m
         CME_TRY(launch_res(d, s, 0, max_iter, true, C, omega));
         return solve_epilogue(h, s, omega, max_iter, p_out, iters_out);
     }
-    CME_TRY(ensure_graphs(d, C, omega));
     const int64_t nfull = max_iter / C, rem = max_iter % C;
     CUDA_TRY(cudaEventRecord(d.t0, s));
     int64_t launched = 0, done = 0;
@@ -1460,6 +1498,10 @@ cme_status device_load(cme_matrix_s* h, const double* p0) {
     CME_TRY(peers_check(d));
     CUDA_TRY(cudaSetDevice(d.dev));
     cudaStream_t s = stream_of(h);
+    // free-run control: omega/C for the graphs, never stop
+    const double omega = effective_omega(h);
+    const int64_t C = h->sopts.check_every;
+    if (!d.use_res) CME_TRY(prepare_graphs(d, C, omega));
     CME_TRY(load_iterate(h, p0, true, s));
     CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
@@ -1467,13 +1509,10 @@ cme_status device_load(cme_matrix_s* h, const double* p0) {
         set_error("p0 has a negative/NaN entry or no positive mass");
         return CME_ERR_INVALID_ARG;
     }
-    // free-run control: omega/C for the graphs, never stop
-    const double omega = effective_omega(h);
-    const int64_t C = h->sopts.check_every;
     CUDA_TRY(cudaMemcpyAsync(&d.ctrl->omega, &omega, sizeof(double), cudaMemcpyHostToDevice, s));
     CUDA_TRY(cudaMemcpyAsync(&d.ctrl->C, &C, sizeof(int64_t), cudaMemcpyHostToDevice, s));
     CUDA_TRY(cudaStreamSynchronize(s));
-    return d.use_res ? CME_OK : ensure_graphs(d, C, omega);
+    return CME_OK;
 }
 
 cme_status device_run(cme_matrix_s* h, int64_t blocks) {
@@ -1487,7 +1526,7 @@ cme_status device_run(cme_matrix_s* h, int64_t blocks) {
         d.cur = (int)((d.cur + blocks * C) & 1);
         return CME_OK;
     }
-    CME_TRY(ensure_graphs(d, C, effective_omega(h)));
+    CME_TRY(prepare_graphs(d, C, effective_omega(h)));
     for (int64_t b = 0; b < blocks; ++b) {
         CUDA_TRY(cudaGraphLaunch(d.gexec[d.cur], s));
         d.cur = (int)((d.cur + C) & 1);

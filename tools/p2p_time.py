@@ -43,6 +43,9 @@ def worker(k):
     cme.cme_solver_run(mm.h, blocks)
     torch.cuda.synchronize()
     times[k] = (time.perf_counter() - t0) / (blocks * 100)
+    p, st, it = mm.solve(tol=0.0, max_iter=100)   # a barrier time-out would surface here
+    if st != "NOT_CONVERGED":
+        print(f"rank {k}: status {st} after the timed blocks", flush=True)
     mm.close()
 
 
