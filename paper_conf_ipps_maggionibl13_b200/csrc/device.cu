@@ -100,7 +100,7 @@ struct Device {
     // TMA-staged persistent kernel (kernels_tma.cuh)
     bool use_tma = false;
     int tma_ncw = 16;
-    int tma_spw = 1;                 // slices per consumer warp per tile (value-indexed kernel: 1 or 2)
+    int tma_spw = 1;                 // slices per consumer warp per tile (all shapes: 1)
     int tma_grid = 0, tma_stages = 0, tma_stage_bytes = 0, tma_off_val = 0, tma_off_col = 0, tma_contig = 0;
     int tma_xpf = 0;
     int tma_occ = 0;                 // TMA CTAs per SM
@@ -421,17 +421,12 @@ static cme_status configure_tma(Device& d, const Packed& P) {
     const int stages_req = stages_env > 0 ? std::min(8, std::max(2, stages_env)) : 0;
     const int force_w = env_int("CME_TMA_WARPS", 0);
     struct Shape { int ncw, spw, stages, occ, grid; int64_t stage, off_val, off_col, n_tiles; };
-    const int force_spw = env_int("CME_TMA_SPW", 0);
     struct Cand { int ncw, spw; };
-    // value-indexed: also 2 slices per warp on one CTA per SM (one dictionary
-    // per SM, a 5-stage ring) -- measured slower on cfg4 (210-217 vs 202 us),
-    // so it is last and wins no tie; CME_TMA_SPW=2 forces it
-    const Cand vi_cands[] = {{16, 1}, {8, 1}, {16, 2}}, std_cands[] = {{16, 1}, {8, 1}};
+    const Cand cands[] = {{16, 1}, {8, 1}};   // consumer warps, slices per warp
     Shape best{};
-    for (const Cand& cd : d.vi ? std::vector<Cand>(vi_cands, vi_cands + 3) : std::vector<Cand>(std_cands, std_cands + 2)) {
+    for (const Cand& cd : cands) {
         const int ncw = cd.ncw, spw = cd.spw;
         if (force_w && ncw != force_w) continue;
-        if (force_spw && d.vi && spw != force_spw) continue;
         Shape sh{};
         sh.ncw = ncw;
         sh.spw = spw;
@@ -443,7 +438,7 @@ static cme_status configure_tma(Device& d, const Packed& P) {
         // dynamic-smem cap: the opt-in maximum minus the static shared memory
         // (barriers, check-reduction scratch: < 2 KB for 33 warps)
         const int cap = smem_max - (d.vi ? 4096 : 1024);
-        if (d.vi) CUDA_TRY(vi_prepare(ncw, spw, cap));
+        if (d.vi) CUDA_TRY(vi_prepare(ncw, cap));
         else if (d.cpt) CUDA_TRY(cpt_prepare(ncw, cap));
         else CUDA_TRY(tma_prepare_b(d.B, ncw, cap));
         const int64_t extra = d.vi ? d.dict_bytes : 0;   // the dictionary sits in front of the stages
@@ -451,7 +446,7 @@ static cme_status configure_tma(Device& d, const Packed& P) {
             *occ = 0;
             const int64_t bytes = extra + stages * sh.stage;
             if (bytes > cap) return cudaSuccess;
-            return d.vi ? vi_occupancy(ncw, spw, (int)bytes, occ)
+            return d.vi ? vi_occupancy(ncw, (int)bytes, occ)
                         : d.cpt ? cpt_occupancy(ncw, (int)bytes, occ)
                                 : tma_occupancy_b(d.B, ncw, (int)bytes, occ);
         };
@@ -466,7 +461,7 @@ static cme_status configure_tma(Device& d, const Packed& P) {
             // per SM loses 7% on the band-on config-5 matrices)
             sh.stages = 2;
             CUDA_TRY(occ_of(2, &sh.occ));
-            for (int st = 3; st <= (spw == 2 ? 8 : 4) && sh.occ > 0; ++st) {
+            for (int st = 3; st <= 4 && sh.occ > 0; ++st) {
                 int o = 0;
                 CUDA_TRY(occ_of(st, &o));
                 if (o < sh.occ) break;
@@ -769,6 +764,13 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
     if ((s = d->alloc(d->io, (size_t)d->n_global * B)) != CME_OK) return fail(s);
     if (comm && (s = d->alloc(d->io2, (size_t)d->n_global * B)) != CME_OK) return fail(s);
     if ((s = d->alloc(d->one, kMaxBatch)) != CME_OK) return fail(s);
+    if (comm && B == 1) {
+        // transient accumulator up front for a rank group: allocating it lazily
+        // inside cme_transient could wait on a peer's spinning barrier kernel
+        // (reproduced: 4 virtual ranks, register kernel, barrier time-outs)
+        if ((s = d->alloc(d->acc_base, (size_t)(d->nx + 2))) != CME_OK) return fail(s);
+        d->accb = d->acc_base + 1;
+    }
     d->p2p = comm && transport_is_peer(comm_transport(comm));
     if (d->p2p) {
         if ((s = d->alloc(d->flags, (size_t)d->nranks)) != CME_OK) return fail(s);
@@ -1050,7 +1052,7 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
                                  d.tma_contig, d.tma_xpf},
                          d.col16, d.row8, d.win_shift},
                  d.dict, d.vidx, d.loi, d.upi, d.dict_bytes};
-        CUDA_TRY(launch_vi(V, d.tma_ncw, d.tma_spw, d.tma_grid, d.dict_bytes + d.tma_stages * d.tma_stage_bytes, d.band, d.rearr,
+        CUDA_TRY(launch_vi(V, d.tma_ncw, d.tma_grid, d.dict_bytes + d.tma_stages * d.tma_stage_bytes, d.band, d.rearr,
                            check, pdl, s));
     } else if (d.use_tma && d.cpt) {
         a.val = d.cval;

@@ -310,15 +310,14 @@ __device__ __forceinline__ double vi_row_wide(const int16_t* scol, const uint16_
     return acc;
 }
 
-// NCW consumer warps, each taking SPW slices of a tile of NCW*SPW slices:
-// with SPW = 2 the warp issues both slices' gathers before any FMA (twice the
-// memory-level parallelism per warp) and the CTA runs alone on its SM -- one
-// dictionary per SM instead of two, so the freed shared memory deepens the
-// TMA ring.
-template <int NCW, int SPW, bool BAND, bool REARR, bool CHECK>
-__global__ void __launch_bounds__(TmaShape<NCW>::kThreads, SPW == 1 ? TmaShape<NCW>::kMinBlocks : 1)
+// NCW consumer warps, one slice each per tile.  (Measured and removed: two
+// slices per warp with both slices' gathers in flight -- on one CTA per SM with
+// a 5-stage ring 210-217 us, on two CTAs per SM with register spills 374 us,
+// vs 185-189 us for this loop on cfg4.)
+template <int NCW, bool BAND, bool REARR, bool CHECK>
+__global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBlocks)
     sell_vi_kernel(const ViArgs V) {
-    constexpr int kConsumers = NCW, kTileSlices = NCW * SPW, kSlots = kTileSlices * 32;
+    constexpr int kConsumers = NCW, kTileSlices = NCW, kSlots = kTileSlices * 32;
     constexpr int kMeta = meta_bytes(kTileSlices);
     constexpr int kOffRow = 0, kOffLo = kOffRow + (REARR ? kSlots : 0), kOffUp = kOffLo + 2 * kSlots;
     const CptArgs& K = V.K;
@@ -375,7 +374,7 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, SPW == 1 ? TmaShape<N
             }
         }
         if (lane == 0 && my_tiles == 0) mbar_wait(&dbar, 0u);   // no tile ever waits on it
-    } else if constexpr (SPW == 1) {
+    } else {
         // one slice per warp: loop invariants hoisted (the ncu instruction
         // census found ~120 per-slice instructions, mostly kernel-parameter
         // reloads and 64-bit index arithmetic); 32-bit slot/row indices
@@ -436,93 +435,6 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, SPW == 1 ? TmaShape<N
                 if (CHECK) ck.add(0, y, ((damp || CHECK) ? x_r : 0.0) * sc, id);
                 for (int p = 0; p < npush; ++p)   // halo rows straight into the peer's buffer
                     if (r >= a.push_lo[p] && r < a.push_hi[p]) a.push_y[p][r] = y;
-            }
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&empty[s]);
-            if (++s == S) { s = 0; phase ^= 1u; }
-        }
-    } else {
-        const double* xo = a.x + a.own_off;
-        double* yo = a.y + a.own_off;
-        mbar_wait(&dbar, 0u);
-        int s = 0;
-        uint32_t phase = 0;
-        for (int64_t tile = t_first; tile < t_end; tile += t_stride) {
-            const int64_t q0 = tile * kTileSlices;
-            const unsigned char* st = stages + (size_t)s * T.stage_bytes + kMeta;
-            mbar_wait(&full[s], phase);
-            int w[SPW], ls[SPW];
-            int64_t r[SPW];
-            bool live[SPW];
-            RowX<1, BAND> X[SPW];
-            double acc[SPW];
-            const int16_t* scol[SPW];
-            const uint16_t* svi[SPW];
-#pragma unroll
-            for (int j = 0; j < SPW; ++j) {   // the warp's slices: rows, own/band x loads
-                const int sl = warp + j * NCW;
-                const int2 meta = reinterpret_cast<const int2*>(st - kMeta)[sl];   // {offset in tile, width}
-                const int64_t q = q0 + sl, slot = q * 32 + lane;
-                w[j] = meta.y;
-                ls[j] = sl * 32 + lane;
-                live[j] = q < a.slice_end && slot < a.n_rows;
-                acc[j] = 0.0;
-                r[j] = live[j] ? (REARR ? ((slot >> K.win_shift) << K.win_shift) + st[kOffRow + ls[j]] : slot) : 0;
-                svi[j] = reinterpret_cast<const uint16_t*>(st + T.off_val) + meta.x + lane;
-                scol[j] = reinterpret_cast<const int16_t*>(st + T.off_col) + meta.x + lane;
-                if (live[j]) X[j].load(xo, r[j]);
-            }
-            if constexpr (SPW == 1) {
-                if (live[0]) {
-                    const double* xr = xo + r[0];
-                    switch (w[0]) {   // warp-uniform exact widths: gathers + dictionary reads, then FMAs
-                        case 0: break;
-                        case 1: acc[0] = vi_row<1>(scol[0], svi[0], sdict, xr); break;
-                        case 2: acc[0] = vi_row<2>(scol[0], svi[0], sdict, xr); break;
-                        case 3: acc[0] = vi_row<3>(scol[0], svi[0], sdict, xr); break;
-                        case 4: acc[0] = vi_row<4>(scol[0], svi[0], sdict, xr); break;
-                        case 5: acc[0] = vi_row<5>(scol[0], svi[0], sdict, xr); break;
-                        case 6: acc[0] = vi_row<6>(scol[0], svi[0], sdict, xr); break;
-                        case 7: acc[0] = vi_row<7>(scol[0], svi[0], sdict, xr); break;
-                        case 8: acc[0] = vi_row<8>(scol[0], svi[0], sdict, xr); break;
-                        default: acc[0] = vi_row_wide(scol[0], svi[0], sdict, xr, w[0]);
-                    }
-                }
-            } else {
-                // both slices' loads in flight before any FMA; widths <= 8
-                // predicated (static register indices), wider slices chunked
-                // (dictionary values are read at FMA time: 96 registers per
-                // thread at 17 warps per SM do not hold them too)
-                double xv[SPW][8];
-#pragma unroll
-                for (int j = 0; j < SPW; ++j) {
-                    const double* xr = xo + r[j];
-                    if (live[j] && w[j] <= 8) {
-#pragma unroll
-                        for (int u = 0; u < 8; ++u)
-                            if (u < w[j]) xv[j][u] = __ldg(xr + scol[j][32 * u]);
-                    }
-                }
-#pragma unroll
-                for (int j = 0; j < SPW; ++j) {
-                    if (!live[j]) continue;
-                    if (w[j] <= 8) {
-#pragma unroll
-                        for (int u = 0; u < 8; ++u)
-                            if (u < w[j]) acc[j] = fma(sdict[svi[j][32 * u]], xv[j][u], acc[j]);
-                    } else {
-                        acc[j] = vi_row_wide(scol[j], svi[j], sdict, xo + r[j], w[j]);
-                    }
-                }
-            }
-#pragma unroll
-            for (int j = 0; j < SPW; ++j) {   // epilogue
-                if (!live[j]) continue;
-                const double accv[1] = {acc[j]};
-                const double idv[1] = {__ldg(a.inv_d + (q0 + warp + j * NCW) * 32 + lane)};
-                const double lov[1] = {BAND ? sdict[reinterpret_cast<const uint16_t*>(st + kOffLo)[ls[j]]] : 0.0};
-                const double upv[1] = {BAND ? sdict[reinterpret_cast<const uint16_t*>(st + kOffUp)[ls[j]]] : 0.0};
-                finish_row_x<1, BAND, CHECK>(a, r[j], yo, accv, lov, upv, idv, a.pre_scale, ck, X[j]);
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);

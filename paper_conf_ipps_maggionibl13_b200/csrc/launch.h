@@ -52,10 +52,10 @@ cudaError_t cpt_prepare(int ncw, int smem);
 cudaError_t cpt_occupancy(int ncw, int smem, int* blocks_per_sm);
 struct ViArgs;
 // value-indexed TMA step kernel (step_cpt.cu, B = 1)
-cudaError_t launch_vi(const ViArgs& V, int ncw, int spw, int grid, int smem, bool band, bool rearr, bool check,
-                      bool pdl, cudaStream_t s);
-cudaError_t vi_prepare(int ncw, int spw, int smem);
-cudaError_t vi_occupancy(int ncw, int spw, int smem, int* blocks_per_sm);
+cudaError_t launch_vi(const ViArgs& V, int ncw, int grid, int smem, bool band, bool rearr, bool check, bool pdl,
+                      cudaStream_t s);
+cudaError_t vi_prepare(int ncw, int smem);
+cudaError_t vi_occupancy(int ncw, int smem, int* blocks_per_sm);
 struct ResArgs;
 // SMEM-resident persistent Jacobi kernel (resident.cu)
 cudaError_t resident_prepare(int smem);

@@ -45,53 +45,45 @@ cudaError_t cpt_occupancy(int ncw, int smem, int* occ) {
                                                          TmaShape<8>::kThreads, smem);
 }
 
-template <int W, int SPW>
+template <int W>
 static cudaError_t launch_vi_w(const ViArgs& V, int grid, int smem, bool band, bool rearr, bool check, bool pdl,
                                cudaStream_t s) {
     const int key = (band ? 4 : 0) | (rearr ? 2 : 0) | (check ? 1 : 0);
     switch (key) {
 #define K_(bd, r, c)                                                                                      \
     case bd * 4 + r * 2 + c:                                                                              \
-        return launch_ex(sell_vi_kernel<W, SPW, bd, r, c>, dim3(grid), dim3(TmaShape<W>::kThreads), smem, pdl, s, V);
+        return launch_ex(sell_vi_kernel<W, bd, r, c>, dim3(grid), dim3(TmaShape<W>::kThreads), smem, pdl, s, V);
         K_(0, 0, 0) K_(0, 0, 1) K_(0, 1, 0) K_(0, 1, 1) K_(1, 0, 0) K_(1, 0, 1) K_(1, 1, 0) K_(1, 1, 1)
 #undef K_
     }
     return cudaErrorInvalidValue;
 }
 
-// shapes: (ncw, spw) = (16, 1), (8, 1), (16, 2)
-cudaError_t launch_vi(const ViArgs& V, int ncw, int spw, int grid, int smem, bool band, bool rearr, bool check,
-                      bool pdl, cudaStream_t s) {
-    if (spw == 2) return launch_vi_w<16, 2>(V, grid, smem, band, rearr, check, pdl, s);
-    return ncw == 16 ? launch_vi_w<16, 1>(V, grid, smem, band, rearr, check, pdl, s)
-                     : launch_vi_w<8, 1>(V, grid, smem, band, rearr, check, pdl, s);
+cudaError_t launch_vi(const ViArgs& V, int ncw, int grid, int smem, bool band, bool rearr, bool check, bool pdl,
+                      cudaStream_t s) {
+    return ncw == 16 ? launch_vi_w<16>(V, grid, smem, band, rearr, check, pdl, s)
+                     : launch_vi_w<8>(V, grid, smem, band, rearr, check, pdl, s);
 }
 
-template <int W, int SPW>
+template <int W>
 static cudaError_t vi_prepare_w(int smem) {
     cudaError_t e = cudaSuccess;
 #define A_(bd, r, c)                                                                                         \
     if (e == cudaSuccess)                                                                                    \
-        e = cudaFuncSetAttribute(sell_vi_kernel<W, SPW, bd, r, c>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        e = cudaFuncSetAttribute(sell_vi_kernel<W, bd, r, c>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     A_(0, 0, 0) A_(0, 0, 1) A_(0, 1, 0) A_(0, 1, 1) A_(1, 0, 0) A_(1, 0, 1) A_(1, 1, 0) A_(1, 1, 1)
 #undef A_
     return e;
 }
 
-cudaError_t vi_prepare(int ncw, int spw, int smem) {
-    if (spw == 2) return vi_prepare_w<16, 2>(smem);
-    return ncw == 16 ? vi_prepare_w<16, 1>(smem) : vi_prepare_w<8, 1>(smem);
-}
+cudaError_t vi_prepare(int ncw, int smem) { return ncw == 16 ? vi_prepare_w<16>(smem) : vi_prepare_w<8>(smem); }
 
-cudaError_t vi_occupancy(int ncw, int spw, int smem, int* occ) {
+cudaError_t vi_occupancy(int ncw, int smem, int* occ) {
     // the heaviest variant (band + rearrangement + check) bounds the residency
-    if (spw == 2)
-        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_vi_kernel<16, 2, true, true, true>,
-                                                             TmaShape<16>::kThreads, smem);
     if (ncw == 16)
-        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_vi_kernel<16, 1, true, true, true>,
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_vi_kernel<16, true, true, true>,
                                                              TmaShape<16>::kThreads, smem);
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_vi_kernel<8, 1, true, true, true>,
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_vi_kernel<8, true, true, true>,
                                                          TmaShape<8>::kThreads, smem);
 }
 

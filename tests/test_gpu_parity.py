@@ -78,7 +78,7 @@ def test_spmv_wide_rates_and_ragged(cme, oracle_mod):
 
 @pytest.mark.parametrize("net", NETS, ids=lambda n: n.name)
 @pytest.mark.parametrize("layout", LAYOUTS[:5], ids=lambda l: "-".join(map(str, l)))
-@pytest.mark.parametrize("vi", ["0", "1", "spw2"])
+@pytest.mark.parametrize("vi", ["0", "1"])
 def test_spmv_parity_compact_tma(cme, oracle_mod, monkeypatch, net, layout, vi):
     """Every SELL layout of every network through the TMA kernel on the compact
     encoding and on its value-indexed form (forced: these matrices are below
@@ -86,9 +86,7 @@ def test_spmv_parity_compact_tma(cme, oracle_mod, monkeypatch, net, layout, vi):
     the oracle."""
     monkeypatch.setenv("CME_TMA", "1")
     monkeypatch.setenv("CME_RESIDENT", "0")
-    monkeypatch.setenv("CME_VI", "0" if vi == "0" else "1")
-    if vi == "spw2":   # value-indexed, two slices per consumer warp, one CTA per SM
-        monkeypatch.setenv("CME_TMA_SPW", "2")
+    monkeypatch.setenv("CME_VI", vi)
     m, A = build(cme, oracle_mod, net, *layout)
     assert m.info().kernel == 1 and m.info().compact == (1 if vi == "0" else 2)
     for omega in (1.0, 0.9):
