@@ -37,6 +37,12 @@ import numpy as np
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
+# one process per GPU: split the host cores between the ranks for the host
+# setup (enumeration, ingest, RCM, pack use OpenMP) before any library loads
+if int(os.environ.get("WORLD_SIZE", "1")) > 1 and "OMP_NUM_THREADS" not in os.environ:
+    _lw = max(1, int(os.environ.get("LOCAL_WORLD_SIZE", os.environ["WORLD_SIZE"])))
+    os.environ["OMP_NUM_THREADS"] = str(max(1, len(os.sched_getaffinity(0)) // _lw))
+
 import workloads as W  # noqa: E402
 
 C_BLOCK = 100
