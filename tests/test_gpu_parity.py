@@ -141,6 +141,31 @@ def test_value_index_bit_identical_to_layout_v0(cme, oracle_mod, monkeypatch):
     assert out["v0"][1].tobytes() == out["vi"][1].tobytes()
 
 
+@pytest.mark.parametrize("vi", ["0", "1"])
+def test_wide_slices_compact_and_value_index(cme, oracle_mod, monkeypatch, vi):
+    """ELL widths above 8 (the chunked wide-row path of both compact kernels):
+    config-5 pattern with mu = 15 and irregular degrees (rows of up to ~25
+    entries), rates quantised to 8 distinct values so the value index applies."""
+    monkeypatch.setenv("CME_TMA", "1")
+    monkeypatch.setenv("CME_RESIDENT", "0")
+    monkeypatch.setenv("CME_VI", vi)
+    n = 9000
+    r, c, v = W.banded_markov(n, 15, 300, True, seed=4)
+    v = 1.0 + np.floor((v - 1.0) * 8.0) / 8.0          # 8 distinct rates in [1, 2)
+    A = oracle_mod.ingest(n, r, c, v)
+    m = cme.Matrix(n, r, c, v).pack()
+    f = m.info()
+    assert f.kernel == 1 and f.compact == (2 if vi == "1" else 1)
+    assert m.packed()["slice_w"].max() > 8
+    for omega in (1.0, 0.7):
+        m.set_opts(omega=omega, check_every=20, stag_tol=0.0)
+        x = W.random_start(n, 13)
+        assert_spmv_close(m.spmv(x), oracle_mod.jacobi_step(A, x, omega))
+    p, st, it = m.solve(tol=0.0, max_iter=60)
+    ref = oracle_mod.jacobi_solve(A, omega=0.7, tol=0.0, check_every=20, max_iter=60, stag_tol=0.0)
+    assert it == ref.iters and np.abs(p - ref.p).sum() <= 1e-12
+
+
 def test_compact_fallback_wide_offsets(cme, oracle_mod, monkeypatch):
     """A transition spanning > 32767 states has no int16 offset: the TMA kernel
     keeps layout v0 (compact = 0) and stays exact."""
