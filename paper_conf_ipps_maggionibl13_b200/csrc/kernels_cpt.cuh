@@ -82,32 +82,6 @@ __device__ __forceinline__ void ell_row_cpt(const int16_t* scol, const double* s
     for (int u = 0; u < W; ++u) acc = fma(sval[32 * u], xv[u], acc);
 }
 
-// Row epilogue on M's rows: s = (lo_c x_{r-1} + up_c x_{r+1}) + acc = (M x)_r.
-template <bool BAND, bool CHECK>
-__device__ __forceinline__ void finish_row_cpt(const StepArgs& a, int64_t slot, int64_t r, double* yo, double acc,
-                                               double lo, double up, CheckAcc<1>& ck, const RowX<1, BAND>& X) {
-    const double s = BAND ? fma(lo, X.xl[0], up * X.xu[0]) + acc : acc;
-    const double xr = X.xr[0];
-    const bool damp = a.omega != 1.0;
-    double y = damp ? fma(1.0 - a.omega, xr, a.omega * s) : s;
-    if (a.unif_lam_inv != 0.0) {   // transient: x + (A x)_r / Lambda, (A x)_r = |a_rr| (s - x_r)
-        const double id = __ldg(a.inv_d + slot);
-        y = fma(a.unif_lam_inv, (s - xr) / id, xr);
-        double* ac = a.acc + a.own_off + r;
-        *ac = fma(a.acc_w, xr, *ac);
-    }
-    double x = (damp || CHECK) ? xr : 0.0;
-    if (a.pre_scale != nullptr) {
-        const double sc = a.pre_scale[0];
-        y *= sc;
-        x *= sc;
-    }
-    if (CHECK) ck.add(0, y, x, __ldg(a.inv_d + slot));
-    yo[r] = y;
-    for (int p = 0; p < a.npush; ++p)   // halo rows straight into the peer's buffer
-        if (r >= a.push_lo[p] && r < a.push_hi[p]) a.push_y[p][r] = y;
-}
-
 template <int NCW, bool BAND, bool REARR, bool CHECK>
 __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBlocks)
     sell_cpt_kernel(const CptArgs K) {
@@ -156,29 +130,34 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
             }
         }
     } else {
+        // loop invariants hoisted and 32-bit slot/row indices, as in
+        // sell_vi_kernel; the epilogue: y = (1-omega) x_r + omega (M x)_r, pending scale, check terms
         const double* xo = a.x + a.own_off;
         double* yo = a.y + a.own_off;
+        const int n_rows = (int)a.n_rows, slice_end = (int)a.slice_end, ws = K.win_shift;
+        const int stage_bytes = T.stage_bytes, off_val = T.off_val, off_col = T.off_col;
+        const double om = a.omega, om1 = 1.0 - a.omega;
+        const bool damp = om != 1.0, unif = a.unif_lam_inv != 0.0;
+        const double sc = a.pre_scale != nullptr ? a.pre_scale[0] : 1.0;
+        const int npush = a.npush;
         int s = 0;
         uint32_t phase = 0;
         for (int64_t tile = t_first; tile < t_end; tile += t_stride) {
-            const int64_t q0 = tile * kTileSlices;
-            const int64_t q = q0 + warp;
-            const unsigned char* st = smem + (size_t)s * T.stage_bytes + kMetaBytes;
+            const unsigned char* st = smem + s * stage_bytes + kMetaBytes;
             mbar_wait(&full[s], phase);
             const int2 meta = reinterpret_cast<const int2*>(st - kMetaBytes)[warp];   // {offset in tile, width}
-            const int w = meta.y;
-            const int64_t loff = meta.x;
-            const int64_t slot = q * 32 + lane;
-            if (q < a.slice_end && slot < a.n_rows) {
+            const int q = (int)tile * kTileSlices + warp;
+            const int slot = q * 32 + lane;
+            if (q < slice_end && slot < n_rows) {
                 const int ls = warp * 32 + lane;
-                const double* sval = reinterpret_cast<const double*>(st + T.off_val) + loff + lane;
-                const int16_t* scol = reinterpret_cast<const int16_t*>(st + T.off_col) + loff + lane;
-                const int64_t r = REARR ? ((slot >> K.win_shift) << K.win_shift) + st[kOffRow + ls] : slot;
+                const double* sval = reinterpret_cast<const double*>(st + off_val) + meta.x + lane;
+                const int16_t* scol = reinterpret_cast<const int16_t*>(st + off_col) + meta.x + lane;
+                const int r = REARR ? ((slot >> ws) << ws) + st[kOffRow + ls] : slot;
                 RowX<1, BAND> X;
                 X.load(xo, r);
                 const double* xr = xo + r;
                 double acc = 0.0;
-                switch (w) {   // warp-uniform exact widths
+                switch (meta.y) {   // warp-uniform exact widths
                     case 0: break;
                     case 1: ell_row_cpt<1>(scol, sval, xr, acc); break;
                     case 2: ell_row_cpt<2>(scol, sval, xr, acc); break;
@@ -189,19 +168,32 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
                     case 7: ell_row_cpt<7>(scol, sval, xr, acc); break;
                     case 8: ell_row_cpt<8>(scol, sval, xr, acc); break;
                     default:
-                        for (int t0 = 0; t0 < w; t0 += 8) {
+                        for (int t0 = 0; t0 < meta.y; t0 += 8) {
                             double xv[8];
 #pragma unroll
                             for (int u = 0; u < 8; ++u)
-                                if (t0 + u < w) xv[u] = __ldg(xr + scol[32 * (t0 + u)]);
+                                if (t0 + u < meta.y) xv[u] = __ldg(xr + scol[32 * (t0 + u)]);
 #pragma unroll
                             for (int u = 0; u < 8; ++u)
-                                if (t0 + u < w) acc = fma(sval[32 * (t0 + u)], xv[u], acc);
+                                if (t0 + u < meta.y) acc = fma(sval[32 * (t0 + u)], xv[u], acc);
                         }
                 }
-                const double lo = BAND ? reinterpret_cast<const double*>(st + kOffLo)[ls] : 0.0;
-                const double up = BAND ? reinterpret_cast<const double*>(st + kOffUp)[ls] : 0.0;
-                finish_row_cpt<BAND, CHECK>(a, slot, r, yo, acc, lo, up, ck, X);
+                const double sum = BAND ? fma(reinterpret_cast<const double*>(st + kOffLo)[ls], X.xl[0],
+                                              reinterpret_cast<const double*>(st + kOffUp)[ls] * X.xu[0]) + acc
+                                        : acc;
+                const double x_r = X.xr[0];
+                double y = damp ? fma(om1, x_r, om * sum) : sum;
+                if (unif) {   // transient: x + (A x)_r / Lambda, (A x)_r = |a_rr| (s - x_r)
+                    const double id = __ldg(a.inv_d + slot);
+                    y = fma(a.unif_lam_inv, (sum - x_r) / id, x_r);
+                    double* ac = a.acc + a.own_off + r;
+                    *ac = fma(a.acc_w, x_r, *ac);
+                }
+                y *= sc;
+                yo[r] = y;
+                if (CHECK) ck.add(0, y, x_r * sc, __ldg(a.inv_d + slot));
+                for (int p = 0; p < npush; ++p)   // halo rows straight into the peer's buffer
+                    if (r >= a.push_lo[p] && r < a.push_hi[p]) a.push_y[p][r] = y;
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);

@@ -77,6 +77,7 @@ def run_point(n, mu, w, irr, blocks, C=100):
     torch.cuda.synchronize()
     ti = e0.elapsed_time(e1) * 1e-3 / (blocks * C)
     out = dict(n=n, mu=mu, width=w, irregular=irr, nnz=int(f.nnz), kernel=int(f.kernel), band_on=int(f.band_on),
+               encoding=int(f.compact),
                us_per_iter=ti * 1e6, gflops=2 * f.nnz / ti / 1e9, alg_gbs=f.bytes_alg / ti / 1e9,
                fmt_gbs=f.bytes_fmt / ti / 1e9, bytes_alg=int(f.bytes_alg), bytes_fmt=int(f.bytes_fmt),
                mass_invariant_rel=float(inv), gen_s=round(t_gen, 2), ingest_pack_s=round(t_pack, 2))
@@ -111,15 +112,17 @@ def main():
     with open(a.out + ".json", "w") as f:
         json.dump(dict(peak_gbs=peak, peak_source=src, points=rows), f, indent=1)
     kn = {0: "register", 1: "tma", 2: "csr"}
+    enc = {0: " (v0)", 1: " (compact)", 2: " (value-indexed)"}
     with open(a.out + ".md", "w") as f:
         f.write(f"# Config 5 sweep: synthetic banded Markov generator, fused Jacobi step on one B200\n\n"
                 f"Peak {peak:.1f} GB/s ({src}). `alg` = B_alg = 12 nnz + 16 n per iteration; `fmt` = the "
-                f"packed layout's compulsory bytes. Natural order, DIAG+SELL, auto band, omega = 1.\n\n"
+                f"packed layout's compulsory bytes (of the encoding the kernel streams). Natural order, DIAG+SELL, "
+                f"auto band, omega = 1.\n\n"
                 "| n | mu | width | irregular | nnz | kernel | us/iter | GFLOPS | alg GB/s | % peak (alg) | "
                 "fmt GB/s | % peak (fmt) |\n|---|---|---|---|---|---|---|---|---|---|---|---|\n")
         for o in rows:
             f.write(f"| {o['n']:,} | {o['mu']} | {o['width']:,} | {int(o['irregular'])} | {o['nnz']:,} | "
-                    f"{kn.get(o['kernel'], o['kernel'])} | {o['us_per_iter']:.1f} | {o['gflops']:.0f} | "
+                    f"{kn.get(o['kernel'], o['kernel'])}{enc.get(o.get('encoding', 0), '')} | {o['us_per_iter']:.1f} | {o['gflops']:.0f} | "
                     f"{o['alg_gbs']:.0f} | {100 * o['frac_alg']:.1f} | {o['fmt_gbs']:.0f} | "
                     f"{100 * o['frac_fmt']:.1f} |\n")
 
