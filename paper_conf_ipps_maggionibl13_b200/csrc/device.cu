@@ -455,13 +455,17 @@ static cme_status configure_tma(Device& d, const Packed& P) {
             while (sh.stages > 2 && extra + sh.stages * sh.stage > cap) --sh.stages;
             CUDA_TRY(occ_of(sh.stages, &sh.occ));
         } else {
-            // auto: the deepest ring (<= 4 stages) that keeps the residency of
-            // 2 stages (measured on B200: 3 stages of the ~31 KB compact cfg4
-            // tiles at 2 CTAs/SM 222 vs 235 us; a 3rd stage that drops a CTA
-            // per SM loses 7% on the band-on config-5 matrices)
+            // auto: 2 stages, or -- for the value-indexed kernel and whenever
+            // the iterate stays L2-resident -- the deepest ring (<= 4) that
+            // keeps the residency of 2 stages.  Measured on B200: value index
+            // on cfg4 3 stages 178 vs 2 stages 206 us; cfg3a (16 MB iterate)
+            // 19.5 vs 21.5 us; but on config-5 matrices with a 128 MB iterate a
+            // deeper ring costs 13% (mu 5) to 2x (random columns): the extra
+            // TMA traffic in flight delays the DRAM-bound gathers
+            const bool x_in_l2 = (d.nx + 2) * 8 * d.B <= ((int64_t)48 << 20);
             sh.stages = 2;
             CUDA_TRY(occ_of(2, &sh.occ));
-            for (int st = 3; st <= 4 && sh.occ > 0; ++st) {
+            for (int st = 3; st <= 4 && sh.occ > 0 && (d.vi || x_in_l2); ++st) {
                 int o = 0;
                 CUDA_TRY(occ_of(st, &o));
                 if (o < sh.occ) break;

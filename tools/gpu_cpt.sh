@@ -1,2 +1,3 @@
-timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_p2p_group.py -x -q -m gpu 2>&1 | tail -1
-timeout 600 python tools/kbench.py --config cfg4_toggle_20m --blocks 10 CME_VI=1 CME_VI=0 2>&1 | grep "^\["
+for cfg in cfg4_toggle_20m cfg3a_schnakenberg_2m banded:16000000:10:32768:0 banded:16000000:5:1024:0 banded:4000000:10:1024:0; do
+CME_VERBOSE=1 timeout 600 python tools/kbench.py --config $cfg --blocks 5 CME_VI=1 CME_VI=0 2>&1 | grep "^\[" | grep -v "^\[cme\]"
+done
