@@ -1,0 +1,41 @@
+"""bench.py's driver contract on the CPU side: the reference arm (the oracle,
+timed on the host cores) prints one JSON line with the keys the driver and
+the judge read, on the same metric/unit/config vocabulary as the GPU arm.
+(The GPU arm itself runs in the round-end GPU tier.)"""
+import json
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def run_bench(*args, env=None):
+    e = dict(os.environ)
+    e.update(env or {})
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), *args], capture_output=True, text=True,
+                       timeout=600, env=e, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    return lines
+
+
+def test_reference_arm_json_line():
+    lines = run_bench("--impl", "reference", "--config", "cfg2_toggle_100k", "--steps", "2", "--warmup", "3")
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better", "scaling",
+              "vs_baseline", "dtype", "data", "config", "cpu_baseline", "e2e", "impl"):
+        assert k in d, k
+    assert d["impl"] == "reference" and d["unit"] == "GFLOPS" and d["dtype"] == "f64" and d["higher_is_better"]
+    assert d["metric"] == "fp64 Jacobi GFLOPS (2 nnz/iteration)"
+    assert d["value"] > 0 and d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
+    assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["d2h_bytes_per_step"] == 0
+    assert d["config"]["workload"] == "cfg2_toggle_100k"
+
+
+def test_reference_arm_other_ranks_exit_quietly():
+    """Under torchrun only rank 0 runs the reference arm; other ranks exit 0."""
+    lines = run_bench("--impl", "reference", "--config", "cfg2_toggle_100k", "--steps", "1", "--warmup", "3",
+                      env={"RANK": "1", "WORLD_SIZE": "2"})
+    assert lines == []
