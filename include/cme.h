@@ -235,12 +235,13 @@ cme_status cme_export_packed(cme_matrix h, cme_packed_view* v);
  * indices.  val[e] = a_rj / (-a_rr) (one IEEE division), lo/up likewise;
  * col16[e] = j - r (x-span column minus the entry's own row, int16); row8[s]
  * = r - (s >> win_shift << win_shift) (row inside its rearrangement window).
- * Pad entries: val 0, col16 0; pad slots: all 0.  Library-owned host arrays,
+ * Pad entries: val 0, col16 0; pad slots: all 0.  A batch (B rate sets on one
+ * pattern) has the offsets and the value index of its entries' B-tuples only.  Library-owned host arrays,
  * valid until destroy or the next pack/distribute; computed on demand when
  * the device does not use it (so host-only packs can be checked too).
  * Errors: BAD_STATE before cme_pack; INVALID_ARG when the pack does not
- * qualify (batch > 1, CSR format, window not a power of two <= 256, or an
- * offset outside int16). */
+ * qualify (CSR format, window not a power of two <= 256, or an offset outside
+ * int16). */
 typedef struct cme_compact_view {
     int64_t n, n_slots, n_slices, n_ell;
     int32_t band_on, win_shift;
@@ -254,10 +255,12 @@ typedef struct cme_compact_view {
      * lo/up, ascending; vidx[e] / loi[s] / upi[s] = their positions in dict.
      * n_dict = 0 and NULL pointers when there are more than 65536. */
     int64_t n_dict;
-    const double* dict;      /* [n_dict]                                     */
+    const double* dict;      /* [n_dict * batch]: tuples, member-minor         */
     const uint16_t* vidx;    /* [n_ell]                                      */
     const uint16_t* loi;     /* [n_slots], NULL when the band is off         */
     const uint16_t* upi;     /* [n_slots], NULL when the band is off         */
+    int32_t batch, pad_;     /* rate sets B; for B > 1 `val`/`lo`/`up` are NULL (only the
+                                offsets and the value index of the B-tuples are built)     */
 } cme_compact_view;
 cme_status cme_export_compact(cme_matrix h, cme_compact_view* v);
 

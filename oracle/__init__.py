@@ -263,15 +263,32 @@ def value_index(P: dict):
     """Value-indexed form (the CSR-VI idea) of a layout-v0
     pack P: dict = the distinct stored values of P's val (every entry, pads
     included) and, band on, lo/up, ascending; vidx / loi / upi = positions
-    in dict.  None when there are more than 65536 distinct values."""
-    parts = [P["val"]] + ([P["lo"], P["up"]] if P["band_on"] else [])
-    d = np.unique(np.concatenate(parts))
+    in dict.  For a batch (P["batch"] = B > 1, member-minor values) the
+    distinct B-tuples in lexicographic order, flattened member-minor.  None
+    when there are more than 65536 distinct values (tuples)."""
+    B = P.get("batch", 1)
+    if B == 1:
+        parts = [P["val"]] + ([P["lo"], P["up"]] if P["band_on"] else [])
+        d = np.unique(np.concatenate(parts))
+        if len(d) > 65536:
+            return None
+        out = dict(dict=d, vidx=np.searchsorted(d, P["val"]).astype(np.uint16))
+        if P["band_on"]:
+            out["loi"] = np.searchsorted(d, P["lo"]).astype(np.uint16)
+            out["upi"] = np.searchsorted(d, P["up"]).astype(np.uint16)
+        return out
+    # a batch (B rate sets on one pattern, member-minor values): the distinct
+    # B-tuples, lexicographically ascending, and each entry's tuple index
+    parts = [P["val"].reshape(-1, B)] + ([P["lo"].reshape(-1, B), P["up"].reshape(-1, B)] if P["band_on"] else [])
+    d, inv = np.unique(np.concatenate(parts), axis=0, return_inverse=True)
     if len(d) > 65536:
         return None
-    out = dict(dict=d, vidx=np.searchsorted(d, P["val"]).astype(np.uint16))
+    inv = inv.reshape(-1).astype(np.uint16)
+    ne = len(parts[0])
+    out = dict(dict=d.reshape(-1), vidx=inv[:ne])
     if P["band_on"]:
-        out["loi"] = np.searchsorted(d, P["lo"]).astype(np.uint16)
-        out["upi"] = np.searchsorted(d, P["up"]).astype(np.uint16)
+        ns = len(parts[1])
+        out["loi"], out["upi"] = inv[ne:ne + ns], inv[ne + ns:]
     return out
 
 

@@ -86,7 +86,8 @@ class cme_compact_view(C.Structure):
                 ("n_ell", C.c_int64), ("band_on", C.c_int32), ("win_shift", C.c_int32),
                 ("val", f64p), ("col16", C.POINTER(C.c_int16)), ("row8", C.POINTER(C.c_uint8)),
                 ("lo", f64p), ("up", f64p), ("n_dict", C.c_int64), ("dict", f64p),
-                ("vidx", C.POINTER(C.c_uint16)), ("loi", C.POINTER(C.c_uint16)), ("upi", C.POINTER(C.c_uint16))]
+                ("vidx", C.POINTER(C.c_uint16)), ("loi", C.POINTER(C.c_uint16)), ("upi", C.POINTER(C.c_uint16)),
+                ("batch", C.c_int32), ("pad_", C.c_int32)]
 
 
 class cme_halo_view(C.Structure):
@@ -323,15 +324,16 @@ def cme_export_compact(h):
     def cp(ptr, k, dt):
         return np.ctypeslib.as_array(ptr, shape=(k,)).astype(dt, copy=True) if k and ptr else np.zeros(0, dt)
 
-    out = dict(val=cp(v.val, v.n_ell, np.float64), col16=cp(v.col16, v.n_ell, np.int16),
-               win_shift=v.win_shift)
+    out = dict(col16=cp(v.col16, v.n_ell, np.int16), win_shift=v.win_shift)
+    if v.batch <= 1:   # (a batch has only the offsets and the tuple index)
+        out["val"] = cp(v.val, v.n_ell, np.float64)
     if v.row8:
         out["row8"] = cp(v.row8, v.n_slots, np.uint8)
     if v.lo:
         out["lo"] = cp(v.lo, v.n_slots, np.float64)
         out["up"] = cp(v.up, v.n_slots, np.float64)
     if v.n_dict:
-        out["dict"] = cp(v.dict, v.n_dict, np.float64)
+        out["dict"] = cp(v.dict, v.n_dict * max(1, v.batch), np.float64)
         out["vidx"] = cp(v.vidx, v.n_ell, np.uint16)
         if v.loi:
             out["loi"] = cp(v.loi, v.n_slots, np.uint16)

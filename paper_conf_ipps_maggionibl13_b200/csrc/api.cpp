@@ -424,7 +424,7 @@ cme_status cme_export_compact(cme_matrix h, cme_compact_view* v) {
         if (!h->Cpt.valid) {
             const int64_t own_off = h->nranks > 1 ? h->cuts[h->rank] - h->span[2 * h->rank] : 0;
             if (!encode_compact(h->P, own_off, h->Cpt)) {
-                set_error("compact encoding: batch, window or column offsets do not qualify");
+                set_error("compact encoding: window or column offsets do not qualify");
                 return CME_ERR_INVALID_ARG;
             }
         }
@@ -434,12 +434,14 @@ cme_status cme_export_compact(cme_matrix h, cme_compact_view* v) {
         cme_compact_view o{};
         o.n = P.n; o.n_slots = P.n_slots; o.n_slices = P.n_slices; o.n_ell = P.n_ell;
         o.band_on = P.band_on; o.win_shift = Q.win_shift;
-        o.val = Q.val.data(); o.col16 = Q.col16.data();
+        o.batch = P.B;
+        o.val = Q.val.empty() ? nullptr : Q.val.data();
+        o.col16 = Q.col16.data();
         o.row8 = Q.row8.empty() ? nullptr : Q.row8.data();
         o.lo = Q.lo.empty() ? nullptr : Q.lo.data();
         o.up = Q.up.empty() ? nullptr : Q.up.data();
         if (Q.vi_valid) {
-            o.n_dict = (int64_t)Q.dict.size();
+            o.n_dict = (int64_t)Q.dict.size() / std::max<int64_t>(1, P.B);   // tuples
             o.dict = Q.dict.data();
             o.vidx = Q.vidx.data();
             o.loi = Q.loi.empty() ? nullptr : Q.loi.data();

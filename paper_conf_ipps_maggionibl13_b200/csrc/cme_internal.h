@@ -73,10 +73,12 @@ struct Compact {
     std::vector<int16_t> col16;           // n_ell
     std::vector<uint8_t> row8;            // n_slots (rearranged packs only)
     // value-indexed variant (CSR-VI style): the distinct stored values of O
-    // (val entries incl. pads, lo/up when the band is on), ascending, and
-    // 16-bit indices into that dictionary; inv_d stays per row
+    // (val entries incl. pads, lo/up when the band is on) -- for a batch the
+    // distinct B-tuples, shared indices -- ascending, and 16-bit indices into
+    // that dictionary; inv_d stays per row (and member).  A batch's Compact
+    // holds only the offsets (col16, row8) besides the value index.
     bool vi_valid = false;
-    std::vector<double> dict;             // <= 65536 values, ascending
+    std::vector<double> dict;             // <= 65536 tuples x B, ascending (lexicographic), member-minor
     std::vector<uint16_t> vidx;           // n_ell
     std::vector<uint16_t> loi, upi;       // n_slots (band only)
 };

@@ -438,7 +438,8 @@ static cme_status configure_tma(Device& d, const Packed& P) {
         // dynamic-smem cap: the opt-in maximum minus the static shared memory
         // (barriers, check-reduction scratch: < 2 KB for 33 warps)
         const int cap = smem_max - (d.vi ? 4096 : 1024);
-        if (d.vi) CUDA_TRY(vi_prepare(ncw, cap));
+        if (d.vi && d.B > 1) CUDA_TRY(vib_prepare(d.B, ncw, cap));
+        else if (d.vi) CUDA_TRY(vi_prepare(ncw, cap));
         else if (d.cpt) CUDA_TRY(cpt_prepare(ncw, cap));
         else CUDA_TRY(tma_prepare_b(d.B, ncw, cap));
         const int64_t extra = d.vi ? d.dict_bytes : 0;   // the dictionary sits in front of the stages
@@ -446,7 +447,8 @@ static cme_status configure_tma(Device& d, const Packed& P) {
             *occ = 0;
             const int64_t bytes = extra + stages * sh.stage;
             if (bytes > cap) return cudaSuccess;
-            return d.vi ? vi_occupancy(ncw, (int)bytes, occ)
+            return d.vi && d.B > 1 ? vib_occupancy(d.B, ncw, (int)bytes, occ)
+                   : d.vi ? vi_occupancy(ncw, (int)bytes, occ)
                         : d.cpt ? cpt_occupancy(ncw, (int)bytes, occ)
                                 : tma_occupancy_b(d.B, ncw, (int)bytes, occ);
         };
@@ -729,6 +731,21 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
         }
         if (!d->use_tma) d->cpt = false;
     }
+    if (d->B > 1 && d->format == CME_FMT_DIAG_SELL && env_int("CME_COMPACT", 1) != 0 && env_int("CME_VI", -1) != 0 &&
+        env_int("CME_TMA", -1) != 0 && encode_compact(P, d->own_off, h->Cpt) && encode_value_index(P, h->Cpt)) {
+        // a batch whose entries' rate tuples have a value index: the batched
+        // value-indexed kernel (shared indices, tuple dictionary in L2)
+        const bool was_tma = d->use_tma;
+        d->cpt = d->vi = true;
+        d->win_shift = h->Cpt.win_shift;
+        d->dict_bytes = 0;   // read from global memory, not staged in shared memory
+        if ((s = configure_tma(*d, P)) != CME_OK) return fail(s);
+        if (!d->use_tma) {   // no TMA shape: back to layout v0
+            d->cpt = d->vi = false;
+            h->Cpt = Compact();
+            if (was_tma && (s = configure_tma(*d, P)) != CME_OK) return fail(s);
+        }
+    }
     if ((s = configure_resident(*d, P, comm != nullptr || h->nranks > 1)) != CME_OK) return fail(s);
     if ((s = preload_kernels(B)) != CME_OK) return fail(s);
     if (d->use_tma) {
@@ -741,7 +758,7 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
     if (d->format != CME_FMT_CSR) {
         if (d->vi) {
             std::vector<double> dict(h->Cpt.dict);
-            dict.resize(d->dict_bytes / 8, 0.0);
+            if (d->B == 1) dict.resize(d->dict_bytes / 8, 0.0);   // (B = 1: staged in shared memory, 128-B padded)
             UP(dict, dict);
             UP(vidx, h->Cpt.vidx);
             UP(col16, h->Cpt.col16);
@@ -1051,6 +1068,13 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
     if (d.format == CME_FMT_CSR) {
         CUDA_TRY(check ? launch_ex(csr_step_kernel<true>, dim3(d.grid), dim3(kCta), 0, pdl, s, a)
                        : launch_ex(csr_step_kernel<false>, dim3(d.grid), dim3(kCta), 0, pdl, s, a));
+    } else if (d.use_tma && d.vi && d.B > 1) {
+        ViArgs V{CptArgs{TmaArgs{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col,
+                                 d.tma_contig, d.tma_xpf},
+                         d.col16, d.row8, d.win_shift},
+                 d.dict, d.vidx, d.loi, d.upi, 0};
+        CUDA_TRY(launch_vib(V, d.B, d.tma_ncw, d.tma_grid, d.tma_stages * d.tma_stage_bytes, d.band, d.rearr, check, pdl,
+                            s));
     } else if (d.use_tma && d.vi) {
         ViArgs V{CptArgs{TmaArgs{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col,
                                  d.tma_contig, d.tma_xpf},
@@ -1472,10 +1496,10 @@ void device_describe(const Device* d, cme_info* f) {
     f->tma_stages = d->use_tma ? d->tma_stages : 0;
     f->grid = d->use_res ? d->res_grid : d->step_grid();
     f->compact = d->vi ? 2 : d->cpt ? 1 : 0;
-    if (d->vi) {   // value-indexed: 4 B per ELL slot, inv_d per row
-        const int64_t n_ell = f->n_ell, nl = d->n_own, slots = f->n_slots, sl = f->n_slices;
-        f->bytes_fmt = 4 * n_ell + 8 * nl + (d->rearr ? nl : 0) + (d->band ? 4 * nl : 0) + 12 * sl + 16 * nl;
-        f->packed_bytes = 4 * n_ell + 8 * slots + (d->rearr ? slots : 0) + (d->band ? 4 * slots : 0) + 12 * sl + 8 +
+    if (d->vi) {   // value-indexed: 4 B per ELL slot (shared by a batch), inv_d per row and member
+        const int64_t n_ell = f->n_ell, nl = d->n_own, slots = f->n_slots, sl = f->n_slices, nb = d->B;
+        f->bytes_fmt = 4 * n_ell + 8 * nb * nl + (d->rearr ? nl : 0) + (d->band ? 4 * nl : 0) + 12 * sl + 16 * nb * nl;
+        f->packed_bytes = 4 * n_ell + 8 * nb * slots + (d->rearr ? slots : 0) + (d->band ? 4 * slots : 0) + 12 * sl + 8 +
                           d->dict_bytes + (d->use_res ? f->packed_bytes : 0);
     } else if (d->cpt) {   // bytes a plain step streams in the compact encoding (no inv_d)
         const int64_t n_ell = f->n_ell, nl = d->n_own, slots = f->n_slots, sl = f->n_slices;

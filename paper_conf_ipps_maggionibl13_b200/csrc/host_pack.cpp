@@ -130,7 +130,7 @@ void pack_rows(const Csr& A, int64_t r0, int64_t r1, int64_t col_shift, int32_t 
 
 bool encode_compact(const Packed& P, int64_t own_off, Compact& C) {
     C = Compact();
-    if (P.B != 1 || P.n_slices == 0 || P.dneg.size() != (size_t)P.n_slots) return false;
+    if (P.n_slices == 0 || P.dneg.size() != (size_t)P.n_slots * P.B) return false;
     int32_t ws = 0;
     if (P.window > 1) {
         if (P.window > 256 || (P.window & (P.window - 1))) return false;
@@ -150,13 +150,23 @@ bool encode_compact(const Packed& P, int64_t own_off, Compact& C) {
     if (!ok) return false;
     C.valid = true;
     C.win_shift = ws;
-    C.val.assign(P.n_ell, 0.0);
     C.col16.assign(P.n_ell, 0);
+    if (ws) C.row8.assign(P.n_slots, 0);
+    if (P.B != 1) {   // a batch: the (shared) offsets only -- its values go through the value index
+#pragma omp parallel for schedule(dynamic, 256)
+        for (int64_t s = 0; s < n; ++s) {
+            const int64_t q = s >> 5, e0 = P.slice_off[q] + (s & 31), l = P.row_of[s], r = own_off + l;
+            for (int32_t t = 0; t < P.slice_w[q]; ++t)
+                C.col16[e0 + 32 * t] = (int16_t)((int64_t)P.col[e0 + 32 * t] - r);
+            if (ws) C.row8[s] = (uint8_t)(l - ((s >> ws) << ws));
+        }
+        return true;
+    }
+    C.val.assign(P.n_ell, 0.0);
     if (P.band_on) {
         C.lo.assign(P.n_slots, 0.0);
         C.up.assign(P.n_slots, 0.0);
     }
-    if (ws) C.row8.assign(P.n_slots, 0);
 #pragma omp parallel for schedule(dynamic, 256)
     for (int64_t s = 0; s < n; ++s) {
         const int64_t q = s >> 5, e0 = P.slice_off[q] + (s & 31), l = P.row_of[s], r = own_off + l;
@@ -175,29 +185,50 @@ bool encode_compact(const Packed& P, int64_t own_off, Compact& C) {
     return true;
 }
 
+namespace {
+// a stored entry's B-tuple of values (batch member b at w[b]), by bit pattern
+struct VKey {
+    uint64_t w[8];
+    bool operator==(const VKey& o) const { return std::memcmp(w, o.w, sizeof(w)) == 0; }
+};
+struct VKeyHash {
+    size_t operator()(const VKey& k) const {
+        uint64_t h = 0x9E3779B97F4A7C15ull;
+        for (uint64_t v : k.w) { h ^= v + 0x9E3779B97F4A7C15ull + (h << 6) + (h >> 2); }
+        return (size_t)h;
+    }
+};
+inline VKey vkey(const double* v, int B) {
+    VKey k{};
+    std::memcpy(k.w, v, sizeof(double) * B);
+    return k;
+}
+}  // namespace
+
 bool encode_value_index(const Packed& P, Compact& C) {
     C.vi_valid = false;
     C.dict.clear(); C.vidx.clear(); C.loi.clear(); C.upi.clear();
-    if (!C.valid || P.B != 1) return false;
+    const int B = P.B;
+    if (!C.valid || B < 1 || B > 8) return false;
     constexpr size_t kMax = 65536;
-    auto bits = [](double v) { uint64_t u; std::memcpy(&u, &v, 8); return u; };
-    // distinct values (by bit pattern; stored values are finite and +0.0 or > 0)
-    std::unordered_set<uint64_t> all;
+    // distinct B-tuples (B = 1: distinct values) of the stored entries; all
+    // stored values are finite and +0.0 or > 0
+    std::unordered_set<VKey, VKeyHash> all;
     bool over = false;
 #pragma omp parallel
     {
-        std::unordered_set<uint64_t> mine;
+        std::unordered_set<VKey, VKeyHash> mine;
 #pragma omp for schedule(static) nowait
         for (int64_t e = 0; e < P.n_ell; ++e) {
             if (mine.size() > kMax) continue;
-            mine.insert(bits(P.val[e]));
+            mine.insert(vkey(P.val.data() + (size_t)e * B, B));
         }
         if (P.band_on) {
 #pragma omp for schedule(static) nowait
             for (int64_t s = 0; s < P.n_slots; ++s) {
                 if (mine.size() > kMax) continue;
-                mine.insert(bits(P.lo[s]));
-                mine.insert(bits(P.up[s]));
+                mine.insert(vkey(P.lo.data() + (size_t)s * B, B));
+                mine.insert(vkey(P.up.data() + (size_t)s * B, B));
             }
         }
 #pragma omp critical
@@ -208,23 +239,33 @@ bool encode_value_index(const Packed& P, Compact& C) {
         }
     }
     if (over) return false;
-    std::vector<double> dict;
-    dict.reserve(all.size());
-    for (uint64_t u : all) { double v; std::memcpy(&v, &u, 8); dict.push_back(v); }
-    std::sort(dict.begin(), dict.end());
-    std::unordered_map<uint64_t, uint16_t> where;
-    where.reserve(dict.size() * 2);
-    for (size_t i = 0; i < dict.size(); ++i) where[bits(dict[i])] = (uint16_t)i;
+    // ascending lexicographic order of the tuples (member 0 first)
+    std::vector<VKey> keys(all.begin(), all.end());
+    auto as_d = [](const VKey& k, int b) { double v; std::memcpy(&v, &k.w[b], 8); return v; };
+    std::sort(keys.begin(), keys.end(), [&](const VKey& a, const VKey& b) {
+        for (int m = 0; m < B; ++m) {
+            const double x = as_d(a, m), y = as_d(b, m);
+            if (x != y) return x < y;
+        }
+        return false;
+    });
+    std::unordered_map<VKey, uint16_t, VKeyHash> where;
+    where.reserve(keys.size() * 2);
+    std::vector<double> dict((size_t)keys.size() * B);
+    for (size_t i = 0; i < keys.size(); ++i) {
+        where[keys[i]] = (uint16_t)i;
+        for (int m = 0; m < B; ++m) dict[i * B + m] = as_d(keys[i], m);
+    }
     C.vidx.resize(P.n_ell);
 #pragma omp parallel for schedule(static)
-    for (int64_t e = 0; e < P.n_ell; ++e) C.vidx[e] = where.find(bits(P.val[e]))->second;
+    for (int64_t e = 0; e < P.n_ell; ++e) C.vidx[e] = where.find(vkey(P.val.data() + (size_t)e * B, B))->second;
     if (P.band_on) {
         C.loi.resize(P.n_slots);
         C.upi.resize(P.n_slots);
 #pragma omp parallel for schedule(static)
         for (int64_t s = 0; s < P.n_slots; ++s) {
-            C.loi[s] = where.find(bits(P.lo[s]))->second;
-            C.upi[s] = where.find(bits(P.up[s]))->second;
+            C.loi[s] = where.find(vkey(P.lo.data() + (size_t)s * B, B))->second;
+            C.upi[s] = where.find(vkey(P.up.data() + (size_t)s * B, B))->second;
         }
     }
     C.dict = std::move(dict);

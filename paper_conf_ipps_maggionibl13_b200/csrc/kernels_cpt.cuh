@@ -258,13 +258,13 @@ __device__ __noinline__ void vi_issue_call(unsigned char* st, uint64_t* bar, con
     }
 }
 
-template <int TS, bool BAND, bool REARR>
+template <int TS, bool BAND, bool REARR, int B = 1>
 __device__ __forceinline__ void vi_issue(const ViArgs& V, unsigned char* stages, uint64_t* full, int64_t tile, int s,
                                          uint64_t pol) {
     const StepArgs& a = V.K.T.a;
-    if (V.K.T.xpf) {
+    if (V.K.T.xpf) {   // the tile's own x rows (B members each, member-minor)
         const int64_t r0 = tile * TS * 32, r1 = min(r0 + TS * 32, a.n_rows);
-        if (r1 > r0) prefetch_l2(a.x + a.own_off + r0, (uint64_t)(r1 - r0) * 8);
+        if (r1 > r0) prefetch_l2(a.x + (a.own_off + r0) * B, (uint64_t)(r1 - r0) * 8 * B);
     }
     vi_issue_call<TS, BAND, REARR>(stages + (size_t)s * V.K.T.stage_bytes, &full[s], a.slice_off, a.slice_end,
                                    a.inv_d, V.K.row8, V.loi, V.upi, V.vidx, V.K.col16, V.K.T.off_val, V.K.T.off_col,
@@ -434,6 +434,121 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
         }
     }
     if (CHECK) cta_check_partials<NCW + 1, 1>(ck, a.partials);
+}
+
+// ---------------------------------------------------------------------------
+// Batched value-indexed kernel (B = 2, 4, 8 rate sets on one pattern; DESIGN.md
+// sec. 5c): every stored entry's B-tuple of rates is one dictionary tuple, so
+// the members share the 16-bit index and the 16-bit column offset -- 4/B bytes
+// per entry per member.  The tuples (n_dict x B doubles, member-minor) are read
+// from global memory (L1/L2) with one B-wide vector load, next to the B-wide x
+// gather; inv_d is a per-lane B-wide stream.  Arithmetic = the layout-v0
+// batched kernels' (same values, FMAs in t order per member, row sum x inv_d).
+template <int NCW, int B, bool BAND, bool REARR, bool CHECK>
+__global__ void __launch_bounds__(TmaShape<NCW>::kThreads, 1) sell_vib_kernel(const ViArgs V) {
+    constexpr int kConsumers = NCW, kTileSlices = NCW, kSlots = kTileSlices * 32;
+    constexpr int kMeta = meta_bytes(kTileSlices);
+    constexpr int kOffRow = 0, kOffLo = kOffRow + (REARR ? kSlots : 0), kOffUp = kOffLo + 2 * kSlots;
+    constexpr int U = Chunk<B>::U;   // entries whose loads are in flight together
+    const CptArgs& K = V.K;
+    const TmaArgs& T = K.T;
+    const StepArgs& a = T.a;
+    pdl_trigger();
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ uint64_t full[8], empty[8];
+    unsigned char* stages = smem;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int S = T.stages;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < S; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], kConsumers);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    const bool producer = warp == kConsumers && lane == 0;
+    uint64_t pol = 0;
+    int64_t t_first, my_tiles, t_stride;
+    tma_tile_range(T, &t_first, &my_tiles, &t_stride);
+    const int64_t t_end = t_first + my_tiles * t_stride;
+    const int pro = (int)(my_tiles < (int64_t)S ? my_tiles : (int64_t)S);
+    if (producer) {
+        pol = evict_first_policy();
+        for (int i = 0; i < pro; ++i)
+            vi_issue<kTileSlices, BAND, REARR, B>(V, stages, full, t_first + (int64_t)i * t_stride, i, pol);
+    }
+    pdl_wait();
+    if (a.stop != nullptr && *a.stop) {
+        if (producer)
+            for (int i = 0; i < pro; ++i) mbar_wait(&full[i], 0u);
+        return;
+    }
+    CheckAcc<B> ck;
+    if (warp == kConsumers) {
+        if (lane == 0 && my_tiles > pro) {
+            int s = 0;
+            uint32_t phase = 1;
+            for (int64_t tile = t_first + (int64_t)pro * t_stride; tile < t_end; tile += t_stride) {
+                mbar_wait(&empty[s], phase ^ 1u);
+                vi_issue<kTileSlices, BAND, REARR, B>(V, stages, full, tile, s, pol);
+                if (++s == S) { s = 0; phase ^= 1u; }
+            }
+        }
+    } else {
+        const double* xo = a.x + a.own_off * B;
+        double* yo = a.y + a.own_off * B;
+        const int n_rows = (int)a.n_rows, slice_end = (int)a.slice_end, ws = K.win_shift;
+        const int stage_bytes = T.stage_bytes, off_val = T.off_val, off_col = T.off_col;
+        const uint64_t pol_s = evict_first_policy();
+        const double* dict = V.dict;
+        int s = 0;
+        uint32_t phase = 0;
+        for (int64_t tile = t_first; tile < t_end; tile += t_stride) {
+            const unsigned char* st = stages + s * stage_bytes + kMeta;
+            mbar_wait(&full[s], phase);
+            const int2 meta = reinterpret_cast<const int2*>(st - kMeta)[warp];   // {offset in tile, width}
+            const int q = (int)tile * kTileSlices + warp;
+            const int slot = q * 32 + lane;
+            if (q < slice_end && slot < n_rows) {
+                const int ls = warp * 32 + lane;
+                const int r = REARR ? ((slot >> ws) << ws) + st[kOffRow + ls] : slot;
+                double id[B];
+                ld_stream_vec<B>(a.inv_d + (int64_t)slot * B, pol_s, id);
+                RowX<B, BAND> X;
+                X.load(xo, r);
+                const uint16_t* svi = reinterpret_cast<const uint16_t*>(st + off_val) + meta.x + lane;
+                const int16_t* scol = reinterpret_cast<const int16_t*>(st + off_col) + meta.x + lane;
+                double acc[B];
+#pragma unroll
+                for (int b = 0; b < B; ++b) acc[b] = 0.0;
+                for (int t0 = 0; t0 < meta.y; t0 += U) {
+                    double xv[U][B], vv[U][B];
+#pragma unroll
+                    for (int u = 0; u < U; ++u)
+                        if (t0 + u < meta.y) {
+                            ld_vec<B>(xo + (int64_t)(r + scol[32 * (t0 + u)]) * B, xv[u]);
+                            ld_vec<B>(dict + (int64_t)svi[32 * (t0 + u)] * B, vv[u]);
+                        }
+#pragma unroll
+                    for (int u = 0; u < U; ++u)
+                        if (t0 + u < meta.y)
+#pragma unroll
+                            for (int b = 0; b < B; ++b) acc[b] = fma(vv[u][b], xv[u][b], acc[b]);
+                }
+                double lo[B], up[B];
+                if (BAND) {
+                    ld_vec<B>(dict + (int64_t)reinterpret_cast<const uint16_t*>(st + kOffLo)[ls] * B, lo);
+                    ld_vec<B>(dict + (int64_t)reinterpret_cast<const uint16_t*>(st + kOffUp)[ls] * B, up);
+                }
+                finish_row_x<B, BAND, CHECK>(a, r, yo, acc, lo, up, id, a.pre_scale, ck, X);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);
+            if (++s == S) { s = 0; phase ^= 1u; }
+        }
+    }
+    if (CHECK) cta_check_partials<NCW + 1, B>(ck, a.partials);
 }
 
 }  // namespace cme

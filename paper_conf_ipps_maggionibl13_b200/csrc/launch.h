@@ -56,6 +56,11 @@ cudaError_t launch_vi(const ViArgs& V, int ncw, int grid, int smem, bool band, b
                       cudaStream_t s);
 cudaError_t vi_prepare(int ncw, int smem);
 cudaError_t vi_occupancy(int ncw, int smem, int* blocks_per_sm);
+// batched value-indexed TMA step kernel (step_cpt.cu, B = 2, 4, 8)
+cudaError_t launch_vib(const ViArgs& V, int B, int ncw, int grid, int smem, bool band, bool rearr, bool check,
+                       bool pdl, cudaStream_t s);
+cudaError_t vib_prepare(int B, int ncw, int smem);
+cudaError_t vib_occupancy(int B, int ncw, int smem, int* blocks_per_sm);
 struct ResArgs;
 // SMEM-resident persistent Jacobi kernel (resident.cu)
 cudaError_t resident_prepare(int smem);

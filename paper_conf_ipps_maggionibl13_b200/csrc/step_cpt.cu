@@ -87,4 +87,65 @@ cudaError_t vi_occupancy(int ncw, int smem, int* occ) {
                                                          TmaShape<8>::kThreads, smem);
 }
 
+template <int W, int B>
+static cudaError_t launch_vib_w(const ViArgs& V, int grid, int smem, bool band, bool rearr, bool check, bool pdl,
+                                cudaStream_t s) {
+    const int key = (band ? 4 : 0) | (rearr ? 2 : 0) | (check ? 1 : 0);
+    switch (key) {
+#define K_(bd, r, c)                                                                                           \
+    case bd * 4 + r * 2 + c:                                                                                   \
+        return launch_ex(sell_vib_kernel<W, B, bd, r, c>, dim3(grid), dim3(TmaShape<W>::kThreads), smem, pdl, s, V);
+        K_(0, 0, 0) K_(0, 0, 1) K_(0, 1, 0) K_(0, 1, 1) K_(1, 0, 0) K_(1, 0, 1) K_(1, 1, 0) K_(1, 1, 1)
+#undef K_
+    }
+    return cudaErrorInvalidValue;
+}
+template <int B>
+static cudaError_t launch_vib_b(const ViArgs& V, int ncw, int grid, int smem, bool band, bool rearr, bool check,
+                                bool pdl, cudaStream_t s) {
+    return ncw == 16 ? launch_vib_w<16, B>(V, grid, smem, band, rearr, check, pdl, s)
+                     : launch_vib_w<8, B>(V, grid, smem, band, rearr, check, pdl, s);
+}
+cudaError_t launch_vib(const ViArgs& V, int B, int ncw, int grid, int smem, bool band, bool rearr, bool check,
+                       bool pdl, cudaStream_t s) {
+    switch (B) {
+        case 2: return launch_vib_b<2>(V, ncw, grid, smem, band, rearr, check, pdl, s);
+        case 4: return launch_vib_b<4>(V, ncw, grid, smem, band, rearr, check, pdl, s);
+        case 8: return launch_vib_b<8>(V, ncw, grid, smem, band, rearr, check, pdl, s);
+    }
+    return cudaErrorInvalidValue;
+}
+
+template <int W, int B>
+static cudaError_t vib_prepare_w(int smem) {
+    cudaError_t e = cudaSuccess;
+#define A_(bd, r, c)                                                                                          \
+    if (e == cudaSuccess)                                                                                     \
+        e = cudaFuncSetAttribute(sell_vib_kernel<W, B, bd, r, c>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    A_(0, 0, 0) A_(0, 0, 1) A_(0, 1, 0) A_(0, 1, 1) A_(1, 0, 0) A_(1, 0, 1) A_(1, 1, 0) A_(1, 1, 1)
+#undef A_
+    return e;
+}
+cudaError_t vib_prepare(int B, int ncw, int smem) {
+    switch (B) {
+        case 2: return ncw == 16 ? vib_prepare_w<16, 2>(smem) : vib_prepare_w<8, 2>(smem);
+        case 4: return ncw == 16 ? vib_prepare_w<16, 4>(smem) : vib_prepare_w<8, 4>(smem);
+        case 8: return ncw == 16 ? vib_prepare_w<16, 8>(smem) : vib_prepare_w<8, 8>(smem);
+    }
+    return cudaErrorInvalidValue;
+}
+template <int W, int B>
+static cudaError_t vib_occ_w(int smem, int* occ) {
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_vib_kernel<W, B, true, true, true>,
+                                                         TmaShape<W>::kThreads, smem);
+}
+cudaError_t vib_occupancy(int B, int ncw, int smem, int* occ) {
+    switch (B) {
+        case 2: return ncw == 16 ? vib_occ_w<16, 2>(smem, occ) : vib_occ_w<8, 2>(smem, occ);
+        case 4: return ncw == 16 ? vib_occ_w<16, 4>(smem, occ) : vib_occ_w<8, 4>(smem, occ);
+        case 8: return ncw == 16 ? vib_occ_w<16, 8>(smem, occ) : vib_occ_w<8, 8>(smem, occ);
+    }
+    return cudaErrorInvalidValue;
+}
+
 }  // namespace cme

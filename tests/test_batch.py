@@ -49,6 +49,25 @@ def test_batch_pack_bit_exact(oracle_mod, B, order, window, band):
             assert got[key].tobytes() == ref[key].tobytes(), key
         for key in ("val", "inv_d", "lo", "up"):
             assert got[key][b::B].tobytes() == ref[key].tobytes(), (key, b)
+    # shared offsets + value index of the members' B-tuples,
+    # bit-exact against the oracle's definition applied to the oracle packs
+    refs = [oracle_mod.pack(oracle_mod.permute(As[b], perm), window=window, band=band) for b in range(B)]
+    Pb = dict(refs[0])
+    Pb["batch"] = B
+    for key in ("val", "lo", "up"):
+        Pb[key] = np.stack([rf[key] for rf in refs], axis=1).reshape(-1)
+    gotc = m.compact()
+    refc = oracle_mod.compact(oracle_mod.permute(As[0], perm), refs[0])   # offsets: member-independent
+    for key in ("col16", "row8"):
+        if key in refc:
+            assert gotc[key].tobytes() == refc[key].tobytes(), key
+    refv = oracle_mod.value_index(Pb)
+    assert refv is not None and "val" not in gotc
+    for key, v in refv.items():
+        assert gotc[key].dtype == v.dtype and gotc[key].tobytes() == v.tobytes(), key
+    # each entry's tuple reproduces every member's stored value
+    d = gotc["dict"].reshape(-1, B)
+    assert d[gotc["vidx"]].reshape(-1).tobytes() == got["val"].tobytes()
 
 
 def test_batch_union_pattern_with_member_zeros(oracle_mod):
@@ -97,7 +116,8 @@ def test_batch_errors():
 
 # ------------------------------------------------------------------ GPU -------
 
-KNOBS = [{"CME_TMA": "0"}, {"CME_TMA": "1"}, {"CME_TMA": "1", "CME_TMA_WARPS": "8"}]
+KNOBS = [{"CME_TMA": "0"}, {"CME_TMA": "1", "CME_VI": "0"}, {"CME_TMA": "1", "CME_TMA_WARPS": "8", "CME_VI": "0"},
+         {"CME_TMA": "1"}, {"CME_TMA": "1", "CME_TMA_WARPS": "8"}]   # the last two: batched value index
 
 
 @pytest.mark.gpu
@@ -109,6 +129,7 @@ def test_batch_spmv_and_landscape_parity(oracle_mod, monkeypatch, B, knobs):
     n, r, c, rates, As = batch_inputs(oracle_mod, toggle_members(26, B))
     m = cme.Matrix(n, r, c, rates).reorder(cme.CME_ORDER_RCM).pack()
     assert m.info().kernel == (1 if knobs["CME_TMA"] == "1" else 0)
+    assert m.info().compact == (2 if knobs["CME_TMA"] == "1" and knobs.get("CME_VI") != "0" else 0)
     m.set_opts(omega=0.9, check_every=7, stag_tol=0.0)
     x = np.concatenate([W.random_start(n, 30 + b) for b in range(B)])
     y = m.spmv(x)
