@@ -419,14 +419,25 @@ static cme_status configure_tma(Device& d, const Packed& P) {
     CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
     const int stages_env = env_int("CME_TMA_STAGES", 0);   // 0 = auto
     const int stages_req = stages_env > 0 ? std::min(8, std::max(2, stages_env)) : 0;
-    const int force_w = env_int("CME_TMA_WARPS", 0);
+    int force_w = env_int("CME_TMA_WARPS", 0);
+    if (force_w == 31 && !(d.vi && d.B == 1)) force_w = 16;   // the 31-warp shape exists for sell_vi_kernel only
+    if (force_w == 15 && !(d.vi && d.B > 1)) force_w = 16;    // and the 15-warp one for sell_vib_kernel
     struct Shape { int ncw, spw, stages, occ, grid; int64_t stage, off_val, off_col, n_tiles; };
     struct Cand { int ncw, spw; };
-    const Cand cands[] = {{16, 1}, {8, 1}};   // consumer warps, slices per warp
+    // consumer warps, slices per warp; 31 warps (one 1024-thread CTA per SM,
+    // one dictionary per SM) only for the value-indexed kernel at B = 1, 15
+    // (a 512-thread CTA: 128 registers) only for the batched one
+    const Cand cands[] = {{16, 1}, {8, 1}, {31, 1}, {15, 1}};
     Shape best{};
     for (const Cand& cd : cands) {
         const int ncw = cd.ncw, spw = cd.spw;
         if (force_w && ncw != force_w) continue;
+        if (ncw == 31 && !(d.vi && d.B == 1)) continue;
+        if (ncw == 15 && !(d.vi && d.B > 1)) continue;
+        // auto at B = 8: the 15-warp shape (128 registers, 24-byte spill) beats
+        // 16 warps (96 registers, 48-200 byte spills): cfg4 1 437 vs 1 523 us
+        // per iteration; at B = 2 / 4 the 16-warp shape stays ahead by 1-2%
+        if (ncw == 16 && d.vi && d.B == 8 && !force_w) continue;
         Shape sh{};
         sh.ncw = ncw;
         sh.spw = spw;
@@ -485,8 +496,8 @@ static cme_status configure_tma(Device& d, const Packed& P) {
         if (sh.ncw * sh.spw * sh.occ > best.ncw * best.spw * best.occ) best = sh;
     }
     if (best.ncw == 0) return CME_OK;
-    if (want < 0 && (best.ncw * best.occ < 16 || best.n_tiles < 2 * (int64_t)sms * best.occ))
-        return CME_OK;   // too few resident consumer warps, or a small problem: register kernel
+    if (want < 0 && (best.ncw * best.occ < 15 || best.n_tiles < 2 * (int64_t)sms * best.occ))
+        return CME_OK;   // too few resident consumer warps (< 15: the batched 15-warp shape passes), or a small problem: register kernel
     d.tma_ncw = best.ncw;
     d.tma_spw = best.spw;
     d.n_tiles = best.n_tiles;
@@ -750,9 +761,10 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
     if ((s = preload_kernels(B)) != CME_OK) return fail(s);
     if (d->use_tma) {
         const int ts = d->tma_ncw * d->tma_spw;   // slices per tile
-        std::vector<int2> tm((size_t)d->n_tiles * ts, make_int2(0, 0));   // whole tiles (TMA copies)
+        const int ms = meta_stride(ts);   // per-tile records, 16-byte aligned
+        std::vector<int2> tm((size_t)d->n_tiles * ms, make_int2(0, 0));   // whole tiles (TMA copies)
         for (int64_t q = 0; q < P.n_slices; ++q)
-            tm[q] = make_int2((int)(P.slice_off[q] - P.slice_off[q / ts * ts]), P.slice_w[q]);
+            tm[q / ts * ms + q % ts] = make_int2((int)(P.slice_off[q] - P.slice_off[q / ts * ts]), P.slice_w[q]);
         if ((s = d->upload(d->tile_meta, tm)) != CME_OK) return fail(s);
     }
     if (d->format != CME_FMT_CSR) {

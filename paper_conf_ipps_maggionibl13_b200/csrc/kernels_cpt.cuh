@@ -42,7 +42,7 @@ __device__ __noinline__ void cpt_issue_call(unsigned char* st, uint64_t* bar, co
     const int64_t e0 = slice_off[q0], e1 = slice_off[q1];
     const uint32_t slots = (uint32_t)(q1 - q0) * 32u;
     const uint32_t nval = (uint32_t)(e1 - e0);
-    uint32_t bytes = nval * 10u + NCW * 8u;
+    uint32_t bytes = nval * 10u + meta_stride(NCW) * 8u;
     if (REARR) bytes += slots;
     if (BAND) bytes += slots * 16u;
     mbar_expect_tx(bar, bytes);
@@ -241,7 +241,7 @@ __device__ __noinline__ void vi_issue_call(unsigned char* st, uint64_t* bar, con
     const int64_t e0 = slice_off[q0], e1 = slice_off[q1];
     const uint32_t slots = (uint32_t)(q1 - q0) * 32u;
     const uint32_t nval = (uint32_t)(e1 - e0);
-    uint32_t bytes = nval * 4u + TS * 8u;
+    uint32_t bytes = nval * 4u + meta_stride(TS) * 8u;
     if (REARR) bytes += slots;
     if (BAND) bytes += slots * 4u;
     mbar_expect_tx(bar, bytes);

@@ -22,7 +22,8 @@ namespace cme {
 template <int NCW>
 struct TmaShape {
     static constexpr int kThreads = 32 * (NCW + 1);
-    static constexpr int kMinBlocks = NCW == 8 ? 3 : 2;   // register cap: 75 / 60 regs
+    // register cap: 75 / 60 regs; 31 consumer warps = one 1024-thread CTA per SM (64 regs)
+    static constexpr int kMinBlocks = NCW == 8 ? 3 : NCW == 31 ? 1 : 2;
 };
 
 struct TmaArgs {
@@ -116,9 +117,14 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
         : "memory");
 }
 
+// Per-tile metadata stride in int2 entries: an even count keeps every tile's
+// record 16-byte aligned and sized for the bulk copy (odd tile shapes: 31).
+__host__ __device__ constexpr int meta_stride(int ts) { return (ts + 1) & ~1; }
+
 __device__ __forceinline__ void issue_meta(unsigned char* st, uint64_t* bar, const int2* tile_meta, int64_t tile,
                                            int ncw, uint64_t pol) {
-    bulk_g2s(st, tile_meta + tile * ncw, (uint32_t)ncw * 8u, bar, pol);
+    const int ms = meta_stride(ncw);
+    bulk_g2s(st, tile_meta + tile * ms, (uint32_t)ms * 8u, bar, pol);
 }
 
 // Stage layout: [inv_d][row_of if REARR][lo, up if BAND][val][col] for
@@ -163,7 +169,7 @@ __device__ __forceinline__ void tma_issue_body(unsigned char* st, uint64_t* bar,
     const int64_t e0 = slice_off[q0], e1 = slice_off[q1];
     const uint32_t slots = (uint32_t)(q1 - q0) * 32u;
     const uint32_t nval = (uint32_t)(e1 - e0);
-    uint32_t bytes = nval * (8u * B + 4u) + slots * 8u * B + NCW * 8u;
+    uint32_t bytes = nval * (8u * B + 4u) + slots * 8u * B + meta_stride(NCW) * 8u;
     if (REARR) bytes += slots * 4u;
     if (BAND) bytes += slots * 16u * B;
     mbar_expect_tx(bar, bytes);

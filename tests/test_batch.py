@@ -117,7 +117,8 @@ def test_batch_errors():
 # ------------------------------------------------------------------ GPU -------
 
 KNOBS = [{"CME_TMA": "0"}, {"CME_TMA": "1", "CME_VI": "0"}, {"CME_TMA": "1", "CME_TMA_WARPS": "8", "CME_VI": "0"},
-         {"CME_TMA": "1"}, {"CME_TMA": "1", "CME_TMA_WARPS": "8"}]   # the last two: batched value index
+         {"CME_TMA": "1"}, {"CME_TMA": "1", "CME_TMA_WARPS": "8"},
+         {"CME_TMA": "1", "CME_TMA_WARPS": "15"}]   # the last three: batched value index
 
 
 @pytest.mark.gpu
@@ -130,6 +131,8 @@ def test_batch_spmv_and_landscape_parity(oracle_mod, monkeypatch, B, knobs):
     m = cme.Matrix(n, r, c, rates).reorder(cme.CME_ORDER_RCM).pack()
     assert m.info().kernel == (1 if knobs["CME_TMA"] == "1" else 0)
     assert m.info().compact == (2 if knobs["CME_TMA"] == "1" and knobs.get("CME_VI") != "0" else 0)
+    if "CME_TMA_WARPS" in knobs:
+        assert m.info().tma_warps == int(knobs["CME_TMA_WARPS"])
     m.set_opts(omega=0.9, check_every=7, stag_tol=0.0)
     x = np.concatenate([W.random_start(n, 30 + b) for b in range(B)])
     y = m.spmv(x)
