@@ -293,14 +293,25 @@ def main():
     dist_path = "RANK" in os.environ
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # more ranks than GPUs (a one-GPU test box only): ranks share the GPUs over
+    # the peer-memory transport (CUDA IPC works within one GPU), and the host-side
+    # collectives (barrier, max over ranks, IPC blob exchange) go over gloo,
+    # because NCCL refuses two ranks on one device
+    ndev = max(1, torch.cuda.device_count())
+    shared_gpus = dist_path and world > ndev
+    local %= ndev
     torch.cuda.set_device(local)
+    coll_dev = "cpu" if shared_gpus else "cuda"
     import __graft_entry__
     __graft_entry__.build()
     import paper_conf_ipps_maggionibl13_b200 as cme
 
     comm = None
     if dist_path:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if shared_gpus:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         if args.transport == "nccl":
             obj = [cme.cme_comm_unique_id() if rank == 0 else None]
             dist.broadcast_object_list(obj, src=0)
@@ -341,7 +352,7 @@ def main():
         barrier()
     ms = e0.elapsed_time(e1)
     if world > 1:
-        t = torch.tensor([ms], device="cuda", dtype=torch.float64)
+        t = torch.tensor([ms], device=coll_dev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
     iters = args.steps * C_BLOCK
@@ -375,7 +386,7 @@ def main():
     barrier()
     e2e_s = time.perf_counter() - t
     if world > 1:
-        tt = torch.tensor([e2e_s], device="cuda", dtype=torch.float64)
+        tt = torch.tensor([e2e_s], device=coll_dev, dtype=torch.float64)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         e2e_s = float(tt.item())
     e2e_gflops = 2.0 * nnz * B * C_BLOCK * e2e_steps / e2e_s / 1e9
@@ -391,7 +402,7 @@ def main():
         rep_c = m.report()
         dev_s = rep_c.seconds
         if world > 1:
-            tt = torch.tensor([dev_s], device="cuda", dtype=torch.float64)
+            tt = torch.tensor([dev_s], device=coll_dev, dtype=torch.float64)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             dev_s = float(tt.item())
         conv_main = {"workload": name, "tol": 1e-12, "omega": cfg["omega"], "status": st_c, "iters": it_c,
