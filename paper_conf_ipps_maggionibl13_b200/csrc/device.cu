@@ -733,8 +733,12 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
             d->vi = true;
             d->dict_bytes = (int)((h->Cpt.dict.size() * 8 + 127) / 128 * 128);
             if ((s = configure_tma(*d, P)) != CME_OK) return fail(s);
-            // auto: only if the dictionary costs no resident consumer warps
-            if (!d->use_tma || (want_vi < 0 && d->tma_ncw * d->tma_spw * d->tma_occ < cpt_warps)) {
+            // auto: only if the dictionary costs at most one resident consumer
+            // warp -- a dictionary too large for two copies per SM runs on the
+            // 31-warp single-dictionary CTA (100M-state toggle, 14.1K distinct
+            // rates, 113 KB: 949 us per iteration vs 1 242 us on the compact
+            // encoding with 2 x 16 warps)
+            if (!d->use_tma || (want_vi < 0 && d->tma_ncw * d->tma_spw * d->tma_occ < cpt_warps - 1)) {
                 d->vi = false;
                 d->dict_bytes = 0;
                 if ((s = configure_tma(*d, P)) != CME_OK) return fail(s);

@@ -171,6 +171,28 @@ def test_wide_slices_compact_and_value_index(cme, oracle_mod, monkeypatch, vi):
     assert it == ref.iters and np.abs(p - ref.p).sum() <= 1e-12
 
 
+def test_large_dictionary_single_dictionary_cta(cme, oracle_mod, monkeypatch):
+    """A dictionary too large for two copies per SM (~14 000 distinct rates, 112 KB)
+    runs the value-indexed kernel on the 31-warp single-dictionary CTA in auto
+    mode (the 100M-state toggle's case: 14.1K distinct rates), with oracle parity."""
+    monkeypatch.setenv("CME_TMA", "1")
+    monkeypatch.setenv("CME_RESIDENT", "0")
+    n = 60000
+    r, c, v = W.banded_markov(n, 6, 200, True, seed=9)
+    v = 1.0 + np.floor((v - 1.0) * 14000.0) / 14000.0    # ~14 000 distinct rates in [1, 2)
+    A = oracle_mod.ingest(n, r, c, v)
+    m = cme.Matrix(n, r, c, v).pack()
+    f = m.info()
+    assert f.kernel == 1 and f.compact == 2 and f.tma_warps == 31
+    for omega in (1.0, 0.8):
+        m.set_opts(omega=omega, check_every=20, stag_tol=0.0)
+        x = W.random_start(n, 17)
+        assert_spmv_close(m.spmv(x), oracle_mod.jacobi_step(A, x, omega))
+    p, st, it = m.solve(tol=0.0, max_iter=60)
+    ref = oracle_mod.jacobi_solve(A, omega=0.8, tol=0.0, check_every=20, max_iter=60, stag_tol=0.0)
+    assert it == ref.iters and np.abs(p - ref.p).sum() <= 1e-12
+
+
 def test_compact_fallback_wide_offsets(cme, oracle_mod, monkeypatch):
     """A transition spanning > 32767 states has no int16 offset: the TMA kernel
     keeps layout v0 (compact = 0) and stays exact."""
