@@ -73,15 +73,19 @@ def hbm_peak():
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def ncu_traffic(workload):
-    """dram bytes/launch of the step kernel from the committed ncu --set full capture."""
+def ncu_traffic(workload, kernel):
+    """dram bytes/launch of the step kernel from the committed ncu --set full
+    capture (profiles/ncu_summary.json), only if it was taken of this kernel;
+    returns (bytes, "committed ncu capture @ <commit>: <kernel>")."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
     try:
         with open(p) as f:
-            d = json.load(f)
-        return d.get(workload, {}).get("dram_bytes_per_launch")
+            d = json.load(f).get(workload, {})
     except (OSError, ValueError):
-        return None
+        return None, None
+    if not d.get("dram_bytes_per_launch") or d.get("kernel_short") != kernel:
+        return None, "no committed ncu capture of this kernel"
+    return d["dram_bytes_per_launch"], f"committed ncu capture @ {d.get('commit', '?')}: {d.get('kernel')}"
 
 
 class ClockSampler:
@@ -168,51 +172,92 @@ def build_matrix(cme, name, dev_mode, batch=1):
     return m, cfg, setup
 
 
-def cpu_oracle_timing(name, budget_s=20.0, steps=1, warmup=0, omega=0.9):
-    """Time the oracle (plain C CSR Jacobi, OpenMP over all host cores) on a
-    bounded sample of the workload: a few iterations of the full matrix."""
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def oracle_run(oracle, A, iters, omega, nthreads):
+    """One oracle call of `iters` Jacobi iterations (one check block of `iters`)."""
+    t = time.perf_counter()
+    oracle.jacobi_solve(A, omega=omega, tol=0.0, check_every=iters, max_iter=iters, stag_tol=0.0, nthreads=nthreads)
+    return time.perf_counter() - t
+
+
+def cpu_oracle_timing(name, budget_s=20.0, omega=0.9, budget_1t_s=10.0):
+    """Time the oracle (plain C CSR Jacobi, as it stands) on a bounded sample of
+    the workload -- one call of up to C = 100 iterations of the full matrix on
+    all host cores, and a shorter one on 1 thread (both thread
+    counts and the CPU model).  The calls include the oracle's own per-call
+    setup (norm, iterate allocation), amortised over the sample."""
     import oracle
     net = W.config_network(name)
     t0 = time.perf_counter()
     A = oracle.network_csr(net)
     t_setup = time.perf_counter() - t0
     cores = len(os.sched_getaffinity(0))
-    # calibrate: one iteration
-    t = time.perf_counter()
-    oracle.jacobi_solve(A, omega=omega, tol=0.0, check_every=C_BLOCK, max_iter=1, stag_tol=0.0, nthreads=cores)
-    one = max(time.perf_counter() - t, 1e-6)
-    iters = int(max(1, min(C_BLOCK, budget_s / one / max(1, steps + warmup))))  # per step
-    for _ in range(warmup):
-        oracle.jacobi_solve(A, omega=omega, tol=0.0, check_every=C_BLOCK, max_iter=iters, stag_tol=0.0, nthreads=cores)
-    times = []
-    for _ in range(steps):
-        t = time.perf_counter()
-        oracle.jacobi_solve(A, omega=omega, tol=0.0, check_every=C_BLOCK, max_iter=iters, stag_tol=0.0, nthreads=cores)
-        times.append(time.perf_counter() - t)
-    tt = float(np.mean(times))
+    one = max(oracle_run(oracle, A, 2, omega, cores) / 2, 1e-6)            # calibrate
+    iters = int(max(2, min(C_BLOCK, budget_s / one)))
+    tt = oracle_run(oracle, A, iters, omega, cores)
+    one1 = max(oracle_run(oracle, A, 1, omega, 1), 1e-6)
+    iters1 = int(max(1, min(C_BLOCK, budget_1t_s / one1)))
+    tt1 = oracle_run(oracle, A, iters1, omega, 1)
     gflops = 2.0 * A.nnz * iters / tt / 1e9
     return dict(value=round(gflops, 4), unit="GFLOPS", cores=cores, kind="oracle",
-                sample=f"{iters} Jacobi iterations of the full {name} matrix (n={A.n}, nnz={A.nnz}), "
-                       f"oracle CSR, OpenMP {cores} threads, mean of {steps} run(s)",
-                iters_per_s=round(iters / tt, 3), seconds_per_iter=tt / iters,
+                sample=f"{iters} Jacobi iterations of the full {name} matrix (n={A.n}, nnz={A.nnz}) in one oracle "
+                       f"call (plain C CSR, OpenMP {cores} threads); 1-thread: {iters1} iterations",
+                cpu_model=cpu_model(), iters_per_s=round(iters / tt, 3), seconds_per_iter=tt / iters,
+                value_1thread=round(2.0 * A.nnz * iters1 / tt1 / 1e9, 4), iters_per_s_1thread=round(iters1 / tt1, 3),
                 oracle_setup_s=round(t_setup, 1))
 
 
 def run_reference(args):
+    """The reference arm of this paper-only tier: the oracle (plain C, CPU, all
+    host cores) timed as it stands on the same workload and metric.  A step is
+    one check block of C = 100 iterations (fewer only if 100 would not fit the
+    few-minute budget -- then iters_per_step says how many); warm-up and timed
+    steps each run as ONE oracle call of W (K) blocks with its check every
+    block, so ms_per_step is measured, not extrapolated, and the call's setup
+    (||A||_inf, allocations) is amortised over the K steps."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
+    import oracle
     name = args.config
-    cb = cpu_oracle_timing(name, budget_s=90.0, steps=args.steps, warmup=args.warmup,
-                           omega=DEFAULTS[name]["omega"])
-    line = {"metric": "fp64 Jacobi GFLOPS (2 nnz/iteration)", "value": cb["value"], "unit": "GFLOPS",
+    omega = DEFAULTS[name]["omega"]
+    A = oracle.network_csr(W.config_network(name))   # setup: not timed
+    cores = len(os.sched_getaffinity(0))
+    one = max(oracle_run(oracle, A, 2, omega, cores) / 2, 1e-6)
+    budget = float(os.environ.get("CME_REF_BUDGET_S", "240"))
+    per_step = int(max(1, min(C_BLOCK, budget / one / (args.steps + args.warmup))))
+
+    def blocks(k):
+        t = time.perf_counter()
+        oracle.jacobi_solve(A, omega=omega, tol=0.0, check_every=per_step, max_iter=k * per_step, stag_tol=0.0,
+                            nthreads=cores)
+        return time.perf_counter() - t
+
+    blocks(args.warmup)
+    sec = blocks(args.steps)
+    iters = args.steps * per_step
+    gflops = 2.0 * A.nnz * iters / sec / 1e9
+    line = {"metric": "fp64 Jacobi GFLOPS (2 nnz/iteration)", "value": round(gflops, 4), "unit": "GFLOPS",
             "impl": "reference", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": round(cb["seconds_per_iter"] * C_BLOCK * 1e3, 3), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": name, "iters_per_step": C_BLOCK, "reference": "oracle/ (plain C, CPU)"},
-            "cpu_baseline": {k: cb[k] for k in ("value", "unit", "cores", "kind", "sample")},
-            "e2e": {"value": cb["value"], "unit": "GFLOPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
-            "iters_per_s": cb["iters_per_s"]}
+            "ms_per_step": round(sec / args.steps * 1e3, 3), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": name, "iters_per_step": per_step, "check_every": per_step,
+                       "reference": "oracle/ (plain C CSR Jacobi, CPU)"},
+            "cpu_baseline": {"value": round(gflops, 4), "unit": "GFLOPS", "cores": cores, "kind": "oracle",
+                             "sample": f"{args.steps} steps x {per_step} Jacobi iterations of the full {name} matrix "
+                                       f"(n={A.n}, nnz={A.nnz}) in one oracle call, OpenMP {cores} threads",
+                             "cpu_model": cpu_model()},
+            "e2e": {"value": round(gflops, 4), "unit": "GFLOPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+            "iters_per_s": round(iters / sec, 3)}
     print(json.dumps(line), flush=True)
     return 0
 
@@ -265,6 +310,20 @@ def converge_closed_form(cme, name="cfg3a_schnakenberg_2m", tol=1e-12):
     return out
 
 
+def self_launch(nproc):
+    """`bench.py --gpus N` outside torchrun: launch the N ranks ourselves (one
+    process per GPU, the launcher the driver uses, rendezvous on 127.0.0.1)
+    instead of silently measuring one GPU.  Rank 0 prints the JSON line."""
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={nproc}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    log("[bench] --gpus", nproc, "without torchrun: launching", " ".join(cmd[2:6]))
+    return subprocess.call(cmd)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -282,6 +341,8 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
+    if args.gpus > 1 and "RANK" not in os.environ:
+        return self_launch(args.gpus)
     if args.impl == "reference":
         return run_reference(args)
 
@@ -361,17 +422,23 @@ def main():
     peak, peak_src = hbm_peak()
     t_iter = sec / iters
     achieved = info.bytes_alg / t_iter / 1e9        # algorithmic bytes per launch / launch time
-    fmt_gbs = info.bytes_fmt * world / t_iter / 1e9 if world == 1 else None
-    compact_note = {
-        1: "compact encoding (DESIGN.md sec. 5b): the kernel streams the rows of M = |D|^-1 O with int16 column "
-           "and uint8 row offsets, 10 B per ELL slot + 17 B per row (format_bytes_per_launch)",
+    # kernel bytes per iteration: this rank's packed encoding (bytes_fmt is per
+    # rank; the whole job moves the sum over ranks in the same time)
+    fmt_tot = float(info.bytes_fmt)
+    if world > 1:
+        tb = torch.tensor([fmt_tot], device=coll_dev, dtype=torch.float64)
+        dist.all_reduce(tb, op=dist.ReduceOp.SUM)
+        fmt_tot = float(tb.item())
+    fmt_gbs = fmt_tot / t_iter / 1e9
+    fmt_frac = fmt_gbs / (peak * world)
+    enc_bytes = {
+        0: "layout v0, 12 B per ELL slot (8 B value + 4 B column) + 8 B inv_d, 4 B row map, 16 B x/y per row",
+        1: "compact encoding (DESIGN.md sec. 5b): the rows of M = |D|^-1 O with int16 column and uint8 row "
+           "offsets, 10 B per ELL slot + 17 B per row",
         2: "value-indexed compact encoding (DESIGN.md sec. 5c): 16-bit indices into a shared-memory dictionary of "
-           "the distinct rates + int16 column offsets (4 B per ELL slot) + inv_d and a uint8 row offset per row "
-           "(format_bytes_per_launch)"}.get(info.compact)
-    if compact_note:
-        compact_note += ("; the SURVEY 8(d) model counts 12 B per non-zero + 16 B per row, so frac > 1 means fewer "
-                         "bytes than that model, not a faster-than-HBM kernel -- format_frac is the kernel's own "
-                         "DRAM efficiency")
+           "the distinct rates + int16 column offsets (4 B per ELL slot) + inv_d, a uint8 row offset and x/y "
+           "(25 B per row)"}[info.compact]
+    traffic, traffic_src = ncu_traffic(name, kernel_name(info)) if world == 1 else (None, None)
 
     # e2e: the public solve call with pinned host buffers, H2D + D2H inside the timed region
     p0 = torch.empty(n * B, dtype=torch.float64, pin_memory=True)
@@ -425,7 +492,7 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and B == 1 and not args.no_cpu_baseline:
         cb = cpu_oracle_timing(name, budget_s=20.0, omega=cfg["omega"])
-        cpu = {k: cb[k] for k in ("value", "unit", "cores", "kind", "sample")}
+        cpu = {k: cb[k] for k in ("value", "unit", "cores", "kind", "sample", "cpu_model", "value_1thread")}
 
     if rank == 0:
         line = {
@@ -441,20 +508,27 @@ def main():
                        "parallelism": f"rows{world}", "setup": setup,
                        "transport": args.transport if dist_path else None},
             "iters_per_s": round(iters / sec, 2),
-            "pct_hbm_roofline": round(100.0 * achieved / (peak * world), 2),
-            "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak * world, "unit": "GB/s",
-                         "frac": round(achieved / (peak * world), 4),
-                         "traffic": ncu_traffic(name) if world == 1 else None,
+            "pct_hbm_roofline": round(100.0 * fmt_frac, 2) if fmt_frac is not None else None,
+            "roofline": {"bound": "hbm", "achieved": round(fmt_gbs, 1) if fmt_gbs else None,
+                         "peak": peak * world, "unit": "GB/s",
+                         "frac": round(fmt_frac, 4) if fmt_frac is not None else None,
+                         "traffic": traffic, "traffic_source": traffic_src,
                          "peak_source": peak_src, "kernel": kernel_name(info),
-                         "bytes_per_launch": info.bytes_alg, "bytes_model": "12 nnz + 16 n per member (SURVEY 8(d))" if B == 1 else f"(12 nnz + 16 n) x {B} members: each member counted as if solved alone",
-                         "format_bytes_per_launch": info.bytes_fmt,
-                         "format_gbs": round(fmt_gbs, 1) if fmt_gbs else None,
-                         "format_frac": round(fmt_gbs / peak, 4) if fmt_gbs else None,
+                         "bytes_per_launch": info.bytes_fmt,
+                         "bytes_note": "the bytes the step kernel must move per iteration for the packed "
+                                       "encoding it streams (DESIGN.md sec. 7): " + enc_bytes,
                          "encoding": {0: "layout v0", 1: "compact", 2: "value-indexed compact"}[info.compact],
-                         "note": compact_note,
+                         "model_bytes_per_launch": info.bytes_alg,
+                         "model_bytes": "12 nnz + 16 n per member (SURVEY 8(d))" if B == 1 else
+                                        f"(12 nnz + 16 n) x {B} members: each member counted as if solved alone",
+                         "model_gbs": round(achieved, 1),
+                         "model_bytes_ratio": round(achieved / (peak * world), 4),
+                         "model_note": "SURVEY 8(d) byte model / launch time / peak: > 1 means the encoding moves "
+                                       "fewer bytes than the 12 nnz + 16 n model, not a faster-than-HBM kernel",
                          "launch_time_us": round(t_iter * 1e6, 3),
-                         "launch_time_note": "timed-region time / step-kernel launches (includes the 2 tiny "
-                                             "check kernels per 100 steps and launch gaps: conservative)"},
+                         "launch_time_note": "timed-region time / step-kernel launches, CUDA events on the "
+                                             "solver's stream (includes the 2 tiny check kernels per 100 steps "
+                                             "and launch gaps: conservative)"},
             "clocks": clocks,
             "e2e": {"value": round(e2e_gflops, 3), "unit": "GFLOPS", "h2d_bytes_per_step": 8 * n * B,
                     "d2h_bytes_per_step": 8 * n * B, "steps": e2e_steps,

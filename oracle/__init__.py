@@ -34,14 +34,28 @@ class OracleError(RuntimeError):
         self.code = code
 
 
+def _src_hash() -> str:
+    """sha256 of the oracle's C source and header (rebuild on any change; mtimes
+    are not trusted)."""
+    import hashlib
+    h = hashlib.sha256()
+    for p in (_SRC, os.path.join(_HERE, "cme_oracle.h")):
+        with open(p, "rb") as f:
+            h.update(f.read())
+    return h.hexdigest()
+
+
 def build(force: bool = False) -> str:
     """Compile liboracle.so with gcc (no CUDA)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < max(
-            os.path.getmtime(_SRC), os.path.getmtime(os.path.join(_HERE, "cme_oracle.h"))):
+    digest = _src_hash()
+    stamp = _LIB + ".sha256"
+    if force or not os.path.exists(_LIB) or not os.path.exists(stamp) or open(stamp).read().strip() != digest:
         tmp = _LIB + f".tmp{os.getpid()}"
         subprocess.check_call(["gcc", "-O2", "-std=c99", "-fopenmp", "-fPIC", "-shared",
                                "-Wall", "-o", tmp, _SRC, "-lm"])
         os.replace(tmp, _LIB)
+        with open(stamp, "w") as f:
+            f.write(digest + "\n")
     return _LIB
 
 

@@ -777,8 +777,11 @@ int oracle_jacobi_solve(int64_t n, const int64_t* rp, const int32_t* col, const 
     double* x = (double*)malloc(sizeof(double) * n);
     double* y = (double*)malloc(sizeof(double) * n);
     if (!x || !y) { free(x); free(y); return ORACLE_OOM; }
-    /* ||A||_inf: max row sum of |a_ij| including the diagonal */
+    /* ||A||_inf: max row sum of |a_ij| including the diagonal.  Each
+     * row sum is the same serial sum in every thread count; the max of them
+     * does not depend on the order, so the threads only change the time. */
     double normA = 0.0;
+#pragma omp parallel for schedule(static) reduction(max : normA) num_threads(g_threads) if (g_threads > 1)
     for (int64_t i = 0; i < n; i++) {
         double s = fabs(diag[i]);
         for (int64_t p = rp[i]; p < rp[i + 1]; p++) s += fabs(val[p]);

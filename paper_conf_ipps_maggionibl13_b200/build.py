@@ -7,6 +7,7 @@
 from __future__ import annotations
 
 import glob
+import hashlib
 import os
 import shutil
 import subprocess
@@ -49,23 +50,49 @@ def _deps():
         [os.path.join(ROOT, "include", "cme.h")]
 
 
-def up_to_date() -> bool:
-    if not os.path.exists(LIB):
+def _common_flags(defines=()):
+    return ["-std=c++17", "-O3", "-lineinfo", "-I", os.path.join(ROOT, "include"), "-I", CSRC,
+            "-I", nccl_include(), "-Xcompiler", "-fPIC,-fopenmp,-ffp-contract=off,-Wall"] + [f"-D{d}" for d in defines]
+
+
+def source_hash(defines=()) -> str:
+    """sha256 over every source/header byte, the compiler flags and the nvcc
+    version: the library is rebuilt whenever any of them differs from the hash
+    recorded beside it (file mtimes are not trusted: a shipped libcme.so newer
+    than its sources would otherwise be reused unbuilt)."""
+    h = hashlib.sha256()
+    for p in sorted(_deps()):
+        h.update(os.path.relpath(p, ROOT).encode())
+        with open(p, "rb") as f:
+            h.update(f.read())
+    h.update(" ".join(ARCH + _common_flags(defines)).replace(ROOT, "<root>").encode())
+    try:
+        h.update(subprocess.run([nvcc(), "--version"], capture_output=True, text=True).stdout.encode())
+    except (OSError, RuntimeError):
+        pass
+    return h.hexdigest()
+
+
+def _stamp(lib: str) -> str:
+    return lib + ".sha256"
+
+
+def up_to_date(lib: str = LIB, defines=()) -> bool:
+    if not os.path.exists(lib) or not os.path.exists(_stamp(lib)):
         return False
-    t = os.path.getmtime(LIB)
-    return all(os.path.getmtime(p) <= t for p in _deps())
+    with open(_stamp(lib)) as f:
+        return f.read().strip() == source_hash(defines)
 
 
 def build(force: bool = False, verbose: bool = False, out: str | None = None, defines=()) -> str:
     """Compile libcme.so (or `out` with extra -D`defines`, for kernel A/B builds)."""
     lib = out or LIB
-    if not force and out is None and up_to_date():
-        return LIB
+    digest = source_hash(defines)
+    if not force and up_to_date(lib, defines):
+        return lib
     obj_dir = OBJ if out is None else OBJ + "_" + os.path.basename(out).replace(".so", "")
     os.makedirs(obj_dir, exist_ok=True)
-    common = ["-std=c++17", "-O3", "-lineinfo", "-I", os.path.join(ROOT, "include"), "-I", CSRC,
-              "-I", nccl_include(), "-Xcompiler", "-fPIC,-fopenmp,-ffp-contract=off,-Wall"]
-    common += [f"-D{d}" for d in defines]
+    common = _common_flags(defines)
 
     def compile_one(src):
         obj = os.path.join(obj_dir, os.path.basename(src) + ".o")
@@ -89,6 +116,8 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None, de
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stderr}")
     os.replace(tmp, lib)
+    with open(_stamp(lib), "w") as f:
+        f.write(digest + "\n")
     return lib
 
 

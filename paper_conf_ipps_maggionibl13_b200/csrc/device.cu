@@ -89,6 +89,8 @@ struct Device {
     int64_t* peer_flags[kMaxPushPeers] = {};
     double* peer_gather[kMaxPushPeers] = {};
     double* peer_io[kMaxPushPeers] = {};
+    bool peer_nbr[kMaxPushPeers] = {};   // a halo neighbour (send or receive side)
+    bool nbr_barrier = true;         // per-step barrier over the halo neighbours only
     int npush = 0;                   // peers that need some of my rows
     int64_t push_lo[kMaxPushPeers] = {}, push_hi[kMaxPushPeers] = {};   // local rows
     double* push_y[2][kMaxPushPeers] = {};   // peer buffer (parity b) shifted to my local rows
@@ -118,6 +120,7 @@ struct Device {
     double* dict = nullptr;
     uint16_t *vidx = nullptr, *loi = nullptr, *upi = nullptr;
     int dict_bytes = 0;              // shared-memory bytes of the dictionary (multiple of 128)
+    int vi_idpf = 1;                 // L2 prefetch of the tile's inv_d by the producer (CME_VI_IDPF)
     // SMEM-resident persistent kernel (kernels_resident.cuh)
     bool use_res = false;
     int res_grid = 0, res_smem = 0, res_rps = 1;
@@ -513,6 +516,10 @@ static cme_status configure_tma(Device& d, const Packed& P) {
     // cfg3a, 16 MB, 21.5 vs 20.5 us).  CME_TMA_XPF = -1 auto / 0 / 1.
     const int xpf = env_int("CME_TMA_XPF", -1);
     d.tma_xpf = xpf >= 0 ? xpf != 0 : (d.nx + 2) * 8 * d.B > (int64_t)48 << 20;
+    // inv_d prefetch (value-indexed kernels): auto = with the x prefetch (the
+    // streams that leave L2 between steps); CME_VI_IDPF = -1 auto / 0 / 1
+    const int idpf = env_int("CME_VI_IDPF", -1);
+    d.vi_idpf = idpf >= 0 ? idpf != 0 : d.tma_xpf;
     d.use_tma = true;
     if (env_int("CME_VERBOSE", 0))
         std::fprintf(stderr, "[cme] tma: B=%d compact=%d vi=%d dict=%d warps=%d spw=%d stages=%d stage_bytes=%lld occ=%d grid=%d tiles=%lld\n",
@@ -720,14 +727,19 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
     // compact encoding when the TMA kernel streams a single matrix
     // (CME_COMPACT = 0 keeps layout v0 on the TMA kernel too)
     h->Cpt = Compact();
-    if (d->use_tma && d->B == 1 && d->format == CME_FMT_DIAG_SELL && env_int("CME_COMPACT", 1) != 0 &&
+    // (tried even when layout v0's stages were too wide for a TMA shape: the
+    // compact and value-indexed stages are 2.5-3x smaller)
+    const bool v0_tma = d->use_tma;
+    const int v0_warps = v0_tma ? d->tma_ncw * d->tma_spw * d->tma_occ : 0;
+    if (d->B == 1 && d->format == CME_FMT_DIAG_SELL && env_int("CME_COMPACT", 1) != 0 && env_int("CME_TMA", -1) != 0 &&
         encode_compact(P, d->own_off, h->Cpt)) {
         d->cpt = true;
         d->win_shift = h->Cpt.win_shift;
         // value-indexed (sec. 5c) when the dictionary fits next to a ring with
         // as many resident consumer warps (CME_VI = -1 auto / 0 off / 1 force)
         if ((s = configure_tma(*d, P)) != CME_OK) return fail(s);   // compact stage geometry
-        const int cpt_warps = d->use_tma ? d->tma_ncw * d->tma_spw * d->tma_occ : 0;
+        // the warps the value index must match: the compact shape's, else layout v0's
+        const int cpt_warps = d->use_tma ? d->tma_ncw * d->tma_spw * d->tma_occ : v0_warps;
         const int want_vi = env_int("CME_VI", -1);
         if (want_vi != 0 && encode_value_index(P, h->Cpt)) {
             d->vi = true;
@@ -744,7 +756,12 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
                 if ((s = configure_tma(*d, P)) != CME_OK) return fail(s);
             }
         }
-        if (!d->use_tma) d->cpt = false;
+        if (!d->use_tma) {   // no TMA shape for the compact encoding: back to layout v0
+            d->cpt = d->vi = false;
+            d->dict_bytes = 0;
+            h->Cpt = Compact();
+            if (v0_tma && (s = configure_tma(*d, P)) != CME_OK) return fail(s);
+        }
     }
     if (d->B > 1 && d->format == CME_FMT_DIAG_SELL && env_int("CME_COMPACT", 1) != 0 && env_int("CME_VI", -1) != 0 &&
         env_int("CME_TMA", -1) != 0 && encode_compact(P, d->own_off, h->Cpt) && encode_value_index(P, h->Cpt)) {
@@ -838,16 +855,26 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
 // exchanges of the row-sharded solve: NCCL (grouped send/recv, allgather,
 // broadcast) or the peer-memory transport (direct stores + flag barriers)
 // ------------------------------------------------------------------------------
-static cme_status p2p_barrier(Device& d, cudaStream_t s, bool respect_stop) {
+// neighbours_only: the per-step barrier, which only has to order the halo
+// stores -- RAW with the ranks that push rows to me, WAR with the ranks I push
+// rows to -- so it publishes to and waits for those ranks only (under RCM the
+// two row-range neighbours).  Every other exchange (check records, load, output
+// segments) is a barrier over all ranks.  One epoch counter serves both: every
+// rank runs the same sequence of barriers, so at a full barrier every rank
+// publishes the same epoch to everyone, and a flag left behind by skipped
+// step barriers only ever lags (the waits compare with >=).
+static cme_status p2p_barrier(Device& d, cudaStream_t s, bool respect_stop, bool neighbours_only = false) {
     if (d.npeer == 0) return CME_OK;   // a group of one
     BarrierArgs b{};
     b.flags = d.flags;
     b.epoch = d.epoch;
+    b.npeer = 0;
     for (int p = 0; p < d.npeer; ++p) {
-        b.peer_flags[p] = d.peer_flags[p];
-        b.peer_rank[p] = d.peer_rank[p];
+        if (neighbours_only && !d.peer_nbr[p]) continue;
+        b.peer_flags[b.npeer] = d.peer_flags[p];
+        b.peer_rank[b.npeer] = d.peer_rank[p];
+        ++b.npeer;
     }
-    b.npeer = d.npeer;
     b.rank = d.rank;
     b.stop = respect_stop ? &d.ctrl->stop : nullptr;
     b.ctrl = d.ctrl;
@@ -860,7 +887,7 @@ static cme_status p2p_barrier(Device& d, cudaStream_t s, bool respect_stop) {
 // the halo rows were already stored into the peers by the step kernel)
 static cme_status exch_after_step(Device& d, int dst, cudaStream_t s) {
     if (!d.comm) return CME_OK;
-    if (d.p2p) return p2p_barrier(d, s, true);
+    if (d.p2p) return p2p_barrier(d, s, true, d.nbr_barrier);
     return comm_halo(d.comm, d.halo, d.xb[dst], s);
 }
 
@@ -926,8 +953,13 @@ static void p2p_wire(cme_matrix_s* h, const std::vector<P2PRank>& all) {
         d.peer_flags[d.npeer] = all[r].flags;
         d.peer_gather[d.npeer] = all[r].gather;
         d.peer_io[d.npeer] = all[r].io;
+        const HaloPlan& hp = h->halo;   // halo neighbours: I push rows to r, or r pushes rows to me
+        d.peer_nbr[d.npeer] = std::find(hp.send_peer.begin(), hp.send_peer.end(), r) != hp.send_peer.end() ||
+                              std::find(hp.recv_peer.begin(), hp.recv_peer.end(), r) != hp.recv_peer.end();
         ++d.npeer;
     }
+    // CME_P2P_NBR = 0 restores the all-rank step barrier (A/B, tests)
+    d.nbr_barrier = env_int("CME_P2P_NBR", 1) != 0;
     const HaloPlan& hp = h->halo;   // rows (not scaled by B)
     d.npush = 0;
     for (size_t i = 0; i < hp.send_peer.size(); ++i) {
@@ -1088,14 +1120,14 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
         ViArgs V{CptArgs{TmaArgs{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col,
                                  d.tma_contig, d.tma_xpf},
                          d.col16, d.row8, d.win_shift},
-                 d.dict, d.vidx, d.loi, d.upi, 0};
+                 d.dict, d.vidx, d.loi, d.upi, 0, d.vi_idpf};
         CUDA_TRY(launch_vib(V, d.B, d.tma_ncw, d.tma_grid, d.tma_stages * d.tma_stage_bytes, d.band, d.rearr, check, pdl,
                             s));
     } else if (d.use_tma && d.vi) {
         ViArgs V{CptArgs{TmaArgs{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col,
                                  d.tma_contig, d.tma_xpf},
                          d.col16, d.row8, d.win_shift},
-                 d.dict, d.vidx, d.loi, d.upi, d.dict_bytes};
+                 d.dict, d.vidx, d.loi, d.upi, d.dict_bytes, d.vi_idpf};
         CUDA_TRY(launch_vi(V, d.tma_ncw, d.tma_grid, d.dict_bytes + d.tma_stages * d.tma_stage_bytes, d.band, d.rearr,
                            check, pdl, s));
     } else if (d.use_tma && d.cpt) {
@@ -1531,10 +1563,10 @@ cme_status device_spmv(cme_matrix_s* h, const double* x, double* y) {
     CUDA_TRY(cudaSetDevice(d.dev));
     cudaStream_t s = stream_of(h);
     CME_TRY(load_iterate(h, x, false, s));
-    if (d.use_res)   // one resident step (C beyond reach: no check)
-        CME_TRY(launch_res(d, s, 0, 1, false, INT64_MAX / 4, effective_omega(h)));
-    else
-        CME_TRY(launch_step(d, s, 0, 1, false, nullptr, effective_omega(h)));
+    // always a plain step kernel: the SMEM-resident kernel carries its epoch in
+    // the iterate's sign bit and so needs x >= +0, while y = M_omega x is
+    // defined for any x (layout v0 is uploaded whenever the resident kernel is)
+    CME_TRY(launch_step(d, s, 0, 1, false, nullptr, effective_omega(h)));
     d.cur = 1;
     return write_out(h, y, d.one, s);
 }

@@ -108,16 +108,20 @@ struct Table {
     uint64_t mask;
 };
 
-// insert; true if this call inserted the key
+// insert; true if this call inserted the key.  Slot ownership is decided by
+// the 128-bit atomicCAS alone: a plain 128-bit load is not single-copy atomic
+// in the PTX memory model, so a load racing another thread's insert could tear
+// into a value that is neither empty nor k.  The plain load only short-cuts
+// the common case "already here": a slot changes once, empty -> key, so a
+// torn load mixes one half of a key with one all-ones half of the empty key,
+// and no valid key has an all-ones half (counts <= kMaxCount < 0xFFFF).
 __device__ __forceinline__ bool table_insert(const Table& T, u128 k) {
     for (uint64_t p = hash_key(k) & T.mask;; p = (p + 1) & T.mask) {
-        const u128 cur = T.key[p];
-        if (cur == k) return false;
-        if (cur == empty_key()) {
-            const u128 old = atomicCAS(&T.key[p], empty_key(), k);
-            if (old == empty_key()) return true;
-            if (old == k) return false;
-        }
+        if (T.key[p] == k) return false;
+        const u128 old = atomicCAS(&T.key[p], empty_key(), k);
+        if (old == empty_key()) return true;
+        if (old == k) return false;
+        // another key owns the slot (single-copy atomic CAS result): probe on
     }
 }
 __device__ __forceinline__ int64_t table_find(const Table& T, u128 k) {

@@ -218,6 +218,7 @@ struct ViArgs {
     const uint16_t* loi;   // [n_slots] (band)
     const uint16_t* upi;
     int32_t dict_bytes;    // multiple of 128: stages start here in shared memory
+    int32_t idpf;          // L2 prefetch of each tile's inv_d rows with the tile (CME_VI_IDPF)
 };
 
 // Stage layout: [row8 if REARR][loi, upi if BAND][vidx][col16].  inv_d is not
@@ -262,9 +263,14 @@ template <int TS, bool BAND, bool REARR, int B = 1>
 __device__ __forceinline__ void vi_issue(const ViArgs& V, unsigned char* stages, uint64_t* full, int64_t tile, int s,
                                          uint64_t pol) {
     const StepArgs& a = V.K.T.a;
-    if (V.K.T.xpf) {   // the tile's own x rows (B members each, member-minor)
+    if (V.K.T.xpf || V.idpf) {
         const int64_t r0 = tile * TS * 32, r1 = min(r0 + TS * 32, a.n_rows);
-        if (r1 > r0) prefetch_l2(a.x + (a.own_off + r0) * B, (uint64_t)(r1 - r0) * 8 * B);
+        // the tile's own x rows (B members each, member-minor)
+        if (V.K.T.xpf && r1 > r0) prefetch_l2(a.x + (a.own_off + r0) * B, (uint64_t)(r1 - r0) * 8 * B);
+        // and its inv_d slots: each consumer lane loads its own inv_d next to
+        // its x loads, and without the prefetch that load is a DRAM round trip
+        // on every slice's critical path (ablation on cfg4)
+        if (V.idpf && r1 > r0) prefetch_l2(a.inv_d + r0 * B, (uint64_t)(r1 - r0) * 8 * B);
     }
     vi_issue_call<TS, BAND, REARR>(stages + (size_t)s * V.K.T.stage_bytes, &full[s], a.slice_off, a.slice_end,
                                    a.inv_d, V.K.row8, V.loi, V.upi, V.vidx, V.K.col16, V.K.T.off_val, V.K.T.off_col,
@@ -277,10 +283,20 @@ template <int W>
 __device__ __forceinline__ double vi_row(const int16_t* scol, const uint16_t* svi, const double* sdict,
                                          const double* xr) {
     double xv[W], vv[W];
+#if defined(CME_ABL_NOGATHER)
+#pragma unroll
+    for (int u = 0; u < W; ++u) xv[u] = __ldg(xr + (scol[32 * u] & 1));
+#else
 #pragma unroll
     for (int u = 0; u < W; ++u) xv[u] = __ldg(xr + scol[32 * u]);
+#endif
+#if defined(CME_ABL_NODICT)
+#pragma unroll
+    for (int u = 0; u < W; ++u) vv[u] = (double)svi[32 * u];
+#else
 #pragma unroll
     for (int u = 0; u < W; ++u) vv[u] = sdict[svi[32 * u]];
+#endif
     double acc = 0.0;
 #pragma unroll
     for (int u = 0; u < W; ++u) acc = fma(vv[u], xv[u], acc);
@@ -390,10 +406,18 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
             const int2 meta = reinterpret_cast<const int2*>(st - kMeta)[warp];   // {offset in tile, width}
             const int q = (int)tile * kTileSlices + warp;
             const int slot = q * 32 + lane;
+#if defined(CME_ABL_NOCOMPUTE)
+            if (q < slice_end && slot < n_rows && meta.y == 12345) {
+#else
             if (q < slice_end && slot < n_rows) {
+#endif
                 const int ls = warp * 32 + lane;
                 const int r = REARR ? ((slot >> ws) << ws) + st[kOffRow + ls] : slot;
+#if defined(CME_ABL_NOINVD)
+                const double id = 0.5;
+#else
                 const double id = ld_stream(a.inv_d + slot, pol_s);   // with the x loads, before the gathers
+#endif
                 RowX<1, BAND> X;
                 X.load(xo, r);
                 const double* xr = xo + r;

@@ -39,3 +39,29 @@ def test_reference_arm_other_ranks_exit_quietly():
     lines = run_bench("--impl", "reference", "--config", "cfg2_toggle_100k", "--steps", "1", "--warmup", "3",
                       env={"RANK": "1", "WORLD_SIZE": "2"})
     assert lines == []
+
+
+def test_reference_arm_times_whole_steps():
+    """ms_per_step is measured over the K timed steps (one oracle call of K check
+    blocks), not extrapolated from a shorter sample: value x ms_per_step agrees."""
+    lines = run_bench("--impl", "reference", "--config", "cfg2_toggle_100k", "--steps", "3", "--warmup", "3")
+    d = json.loads(lines[0])
+    it = d["config"]["iters_per_step"]
+    assert 1 <= it <= 100 and d["config"]["check_every"] == it
+    nnz = 595874
+    gflops_from_ms = 2.0 * nnz * it / (d["ms_per_step"] * 1e-3) / 1e9
+    assert abs(gflops_from_ms - d["value"]) <= 0.01 * d["value"] + 1e-3
+
+
+def test_gpus_flag_self_launches_ranks():
+    """--gpus N outside torchrun launches N ranks itself (never a silent 1-GPU
+    run): with the reference arm, exactly one line from rank 0 with n_gpus N."""
+    env = {k: v for k, v in os.environ.items() if k not in ("RANK", "WORLD_SIZE", "LOCAL_RANK")}
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--gpus", "2",
+                        "--config", "cfg2_toggle_100k", "--steps", "1", "--warmup", "3"],
+                       capture_output=True, text=True, timeout=600, env=env, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1
+    assert json.loads(lines[0])["n_gpus"] == 2
+    assert "launching" in r.stderr

@@ -65,6 +65,26 @@ def test_spmv_parity(cme, oracle_mod, net, layout, omega):
     assert_spmv_close(y, oracle_mod.jacobi_step(A, x, omega))
 
 
+@pytest.mark.parametrize("resident", ["-1", "1"])
+def test_spmv_signed_input(cme, oracle_mod, monkeypatch, resident):
+    """cme_spmv is y = M_omega x for ANY x (include/cme.h), including negative
+    entries and -0.0, also on a matrix whose solves run the SMEM-resident
+    kernel (which tags epochs in the sign bit and so needs x >= +0)."""
+    monkeypatch.setenv("CME_RESIDENT", resident)
+    m, A = build(cme, oracle_mod, W.toggle_switch(40), "rcm")
+    x = W.random_start(A.n, 4) - 0.5 / A.n
+    x[::7] = -0.0
+    for omega in (1.0, 0.9):
+        m.set_opts(omega=omega)
+        y = m.spmv(x)
+        ref = oracle_mod.jacobi_step(A, x, omega)
+        scale = np.abs(oracle_mod.jacobi_step(A, np.abs(x), omega))   # no-cancellation magnitude
+        assert np.all(np.abs(y - ref) <= 1e-13 * scale + 1e-300)
+    p, st, it = m.solve(tol=1e-10, max_iter=5000)   # a solve after the signed SpMV
+    assert st == "CONVERGED"
+    m.close()
+
+
 def test_spmv_wide_rates_and_ragged(cme, oracle_mod):
     """Config-5 generator: irregular widths, rates in [1,2), ragged last slice."""
     for n, mu, width, irr in [(1000, 10, 64, True), (777, 5, 2, False), (5000, 15, 5000, True), (33, 6, 8, True)]:

@@ -104,6 +104,16 @@ def test_orderings_bit_exact(oracle_mod, net, order):
     assert np.array_equal(m.permutation(), ref)
 
 
+def test_rcm_hand_worked_library():
+    """cme_reorder(RCM) on the hand-worked graph of test_oracle_order_pack.py (R12)."""
+    from test_oracle_order_pack import RCM_HAND_EDGES, RCM_HAND_PERM
+    r = np.array([i for j, i in RCM_HAND_EDGES], np.int32)
+    c = np.array([j for j, i in RCM_HAND_EDGES], np.int32)
+    m = cme.Matrix(12, r, c, np.ones(len(r)))
+    m.reorder(cme.CME_ORDER_RCM)
+    assert m.permutation().tolist() == RCM_HAND_PERM
+
+
 PACK_CASES = [("none", 256, "auto", cme.CME_FMT_DIAG_SELL), ("dfs", 256, "auto", cme.CME_FMT_DIAG_SELL),
               ("none", 1, "auto", cme.CME_FMT_SELL256), ("rcm", 1, "never", cme.CME_FMT_SELL256),
               ("rcm", 1 << 30, "never", cme.CME_FMT_DIAG_SELL),

@@ -43,6 +43,31 @@ def test_dfs_restarts_at_smallest_unvisited(oracle_mod):
     assert oracle_mod.order_dfs(A, 3).tolist() == [3, 2, 0, 1]
 
 
+# RCM hand-worked case (R12: George-Liu start, Cuthill-McKee by (degree, index),
+# reverse).  Transitions j -> i; some edges one-way to exercise the A + A^T
+# symmetrisation.  Undirected pattern and degrees:
+#   0:{5,7} 2   1:{3,4} 2   2:{5,7} 2   3:{1,6,7,8} 4   4:{1,6} 2   5:{0,2} 2
+#   6:{3,4} 2   7:{0,2,3} 3 8:{3} 1     9:{10} 1   10:{9,11} 2   11:{10} 1
+# Component of 0 = {0..8}.  Start = min (degree, index) = 8.  BFS(8) levels
+#   {8} {3} {1,6,7} {0,2,4} {5}: eccentricity 4; the last level's min is 5.
+#   BFS(5): {5} {0,2} {7} {3} {1,6,8} {4}: eccentricity 5 > 4, so move to 5;
+#   last level {4}; BFS(4): {4} {1,6} {3} {7,8} {0,2} {5}: 5, not > 5: stop.
+# Cuthill-McKee from 5: 5 | nbrs 0,2 (deg 2, 2 -> by index) | from 0: 7 |
+#   from 2: - | from 7: 3 | from 3: 8 (deg 1), 1, 6 (deg 2) | from 8: - |
+#   from 1: 4 | -> [5,0,2,7,3,8,1,6,4].
+# Component of 9 = {9,10,11}: start 9 (deg 1); BFS(9) eccentricity 2, last
+#   level {11}, BFS(11) also 2: stay at 9 -> [9,10,11].
+# Reverse of the concatenation: [11,10,9,4,6,1,8,3,7,2,0,5].
+RCM_HAND_EDGES = [(5, 2), (2, 5), (0, 5), (2, 7), (7, 0), (7, 3), (3, 7), (1, 3), (3, 6), (6, 3), (4, 1),
+                  (6, 4), (4, 6), (8, 3), (3, 8), (9, 10), (10, 11), (11, 10)]
+RCM_HAND_PERM = [11, 10, 9, 4, 6, 1, 8, 3, 7, 2, 0, 5]
+
+
+def test_rcm_hand_worked(oracle_mod):
+    A = csr_from_edges(oracle_mod, 12, RCM_HAND_EDGES)
+    assert oracle_mod.order_rcm(A).tolist() == RCM_HAND_PERM
+
+
 def test_rcm_path_and_grid(oracle_mod):
     rng = np.random.default_rng(0)
     n = 200

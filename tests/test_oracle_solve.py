@@ -9,6 +9,7 @@ Closed forms (textbook, not the oracle's formulas):
 plus numpy.linalg.solve (LAPACK dgesv), dense numpy products, and invariants.
 """
 import math
+import os
 
 import numpy as np
 import pytest
@@ -53,6 +54,42 @@ def test_jacobi_birth_death_damped(oracle_mod, bd):
     r = oracle_mod.jacobi_solve(bd, omega=0.9, tol=1e-14, max_iter=200000)
     assert r.status == "CONVERGED" and r.iters % 100 == 0
     assert np.abs(r.p - poisson_trunc(10.0, 100)).sum() < 1e-11
+
+
+@pytest.mark.parametrize("omega", [0.9, 0.3, 1.0])
+def test_damping_on_the_minus_one_eigenvector(oracle_mod, bd, omega):
+    """Where omega sits in the damped step (R1), pinned by the spectrum, not by
+    restating the formula.  A u = 0 <=> O u = |D| u <=> M u = u for
+    M = |D|^-1 O, and u = the truncated Poisson law (closed form).  The
+    birth-death chain is bipartite: O only links x to x +- 1, so with
+    S = diag((-1)^x), O S = -S O and M (S u) = -S u.  Hence
+    M_omega (S u) = (1 - 2 omega) S u; a swapped omega <-> 1 - omega would
+    give 2 omega - 1 instead (+0.8 vs -0.8 at omega = 0.9)."""
+    u = poisson_trunc(10.0, 100)             # A u = 0  <=>  M u = u (M = |D|^-1 O)
+    S = np.where(np.arange(101) % 2 == 0, 1.0, -1.0)
+    v = S * u
+    y = oracle_mod.jacobi_step(bd, v, omega)
+    ref = (1.0 - 2.0 * omega) * v
+    big = np.abs(v) > 1e-200
+    assert np.max(np.abs(y[big] - ref[big]) / np.abs(v[big])) < 1e-12
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("omega,status,iters", [(0.9, "CONVERGED", 3400), (0.5, "CONVERGED", 5900),
+                                                (1.0, "STAGNATED", None)])
+def test_survey_c3_toggle_iteration_counts(oracle_mod, omega, status, iters):
+    """SURVEY C3 / F2 (an independent computation, recorded at survey time):
+    config 2 (toggle switch N = 224, 99 908 states), uniform p0, C = 100,
+    tol 1e-12: omega = 0.9 stops at 3 400 iterations, omega = 0.5 at 5 900, and
+    pure Jacobi (omega = 1) stalls with delta = 1.404e-5 (period 2)."""
+    A = oracle_mod.network_csr(W.toggle_switch(224))
+    assert A.n == 99908
+    r = oracle_mod.jacobi_solve(A, omega=omega, tol=1e-12, max_iter=20000, nthreads=os.cpu_count() or 1)
+    assert r.status == status
+    if iters is not None:
+        assert r.iters == iters and r.delta <= 1e-12
+    else:
+        assert r.delta == pytest.approx(1.404e-5, rel=1e-3)
 
 
 def test_pure_jacobi_stagnates_on_period_two(oracle_mod, bd):

@@ -320,10 +320,16 @@ _gen = None
 
 def build_generator(force: bool = False) -> str:
     """Compile libwl_gen.so (gcc, OpenMP; input generation only)."""
-    if force or not _os.path.exists(_GEN_LIB) or _os.path.getmtime(_GEN_LIB) < _os.path.getmtime(_GEN_SRC):
+    import hashlib
+    with open(_GEN_SRC, "rb") as f:
+        digest = hashlib.sha256(f.read()).hexdigest()   # rebuild on any source change (not mtimes)
+    stamp = _GEN_LIB + ".sha256"
+    if force or not _os.path.exists(_GEN_LIB) or not _os.path.exists(stamp) or open(stamp).read().strip() != digest:
         tmp = _GEN_LIB + f".tmp{_os.getpid()}"
         _sp.check_call(["gcc", "-O2", "-std=c99", "-fopenmp", "-fPIC", "-shared", "-Wall", "-o", tmp, _GEN_SRC])
         _os.replace(tmp, _GEN_LIB)
+        with open(stamp, "w") as f:
+            f.write(digest + "\n")
     return _GEN_LIB
 
 
