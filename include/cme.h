@@ -50,7 +50,10 @@ typedef enum cme_status {
     CME_NOT_CONVERGED = 8,     /* solve hit max_iter (p_out still written, normalised) */
     CME_STAGNATED = 9,         /* delta stopped changing (R3), p_out written */
     CME_ERR_NUMERIC = 10,      /* NaN/Inf or zero mass in the iterate */
-    CME_ERR_NO_DEVICE = 11     /* no CUDA device visible */
+    CME_ERR_NO_DEVICE = 11,    /* no CUDA device visible */
+    CME_ERR_TIMEOUT = 12       /* a bounded device-side wait expired: a peer rank's flag barrier
+                                  (peer-memory transport) or a resident-kernel dependency
+                                  (CME_RES_TIMEOUT_MS); the solve stopped instead of hanging */
 } cme_status;
 
 typedef struct cme_matrix_s* cme_matrix; /* opaque */

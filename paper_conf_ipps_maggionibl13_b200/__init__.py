@@ -30,6 +30,7 @@ _lib = C.CDLL(LIB_PATH, mode=C.RTLD_GLOBAL)
 CME_OK, CME_ERR_INVALID_ARG, CME_ERR_NEGATIVE_RATE, CME_ERR_ZERO_OUTFLOW = 0, 1, 2, 3
 CME_ERR_BAD_STATE, CME_ERR_OOM, CME_ERR_CUDA, CME_ERR_NCCL = 4, 5, 6, 7
 CME_NOT_CONVERGED, CME_STAGNATED, CME_ERR_NUMERIC, CME_ERR_NO_DEVICE = 8, 9, 10, 11
+CME_ERR_TIMEOUT = 12
 CME_DIAG_FROM_COLSUMS, CME_DIAG_GIVEN = 0, 1
 CME_ORDER_NONE, CME_ORDER_DFS, CME_ORDER_RCM = 0, 1, 2
 CME_FMT_DIAG_SELL, CME_FMT_ELL, CME_FMT_CSR, CME_FMT_SELL256 = 0, 1, 2, 3

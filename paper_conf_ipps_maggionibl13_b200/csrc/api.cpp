@@ -539,6 +539,7 @@ const char* cme_status_string(cme_status s) {
         case CME_STAGNATED: return "CME_STAGNATED";
         case CME_ERR_NUMERIC: return "CME_ERR_NUMERIC";
         case CME_ERR_NO_DEVICE: return "CME_ERR_NO_DEVICE";
+        case CME_ERR_TIMEOUT: return "CME_ERR_TIMEOUT";
     }
     return "CME_UNKNOWN";
 }

@@ -254,7 +254,7 @@ __global__ void scale_copy_kernel(const double* x, int64_t n, int B, const doubl
 // it into every peer's flag slot (release, system scope: the step's halo
 // stores into that peer are ordered before it) and waits (acquire) until every
 // peer has published the same epoch.  Bounded spin: a peer that never arrives
-// turns the solve into CME_ERR_NCCL instead of a hung GPU.
+// turns the solve into CME_ERR_TIMEOUT instead of a hung GPU.
 struct BarrierArgs {
     int64_t* flags;
     int64_t* epoch;
@@ -288,7 +288,7 @@ __global__ void p2p_barrier_kernel(const BarrierArgs a) {
             asm volatile("ld.acquire.sys.global.s64 %0, [%1];" : "=l"(v) : "l"(f) : "memory");
             if (v >= e) break;
             if (++spins > (1LL << 28)) {   // ~ tens of seconds: a peer is gone
-                a.ctrl->status = CME_ERR_NCCL;
+                a.ctrl->status = CME_ERR_TIMEOUT;
                 a.ctrl->stop = 1;
                 return;
             }
@@ -1403,10 +1403,11 @@ static cme_status solve_epilogue(cme_matrix_s* h, cudaStream_t s, double omega, 
     d.cur = (int)(f.iter & 1);
     float ms = 0.f;
     cudaEventElapsedTime(&ms, d.t0, d.t1);
-    if (f.status == CME_ERR_CUDA && d.use_res) {
-        set_error("resident kernel: a dependency wait timed out (CME_RES_TIMEOUT_MS)");
+    if (f.status == CME_ERR_TIMEOUT) {
+        set_error(d.use_res ? "resident kernel: a dependency wait timed out (CME_RES_TIMEOUT_MS)"
+                            : "peer-memory transport: a peer rank never reached the flag barrier");
         if (iters_out) *iters_out = f.iter;
-        return CME_ERR_CUDA;
+        return CME_ERR_TIMEOUT;
     }
     const int32_t overall = max_iter == 0 ? CME_NOT_CONVERGED : f.status;
     fill_reports(h, f, omega, ms * 1e-3, overall);

@@ -15,6 +15,10 @@
 #pragma once
 #include "kernels_tma.cuh"
 
+#ifndef CME_ABL   // kernel ablation level for dev A/B builds only (tools/gpu_abl.sh); 0 = the product kernel
+#define CME_ABL 0
+#endif
+
 namespace cme {
 
 struct CptArgs {
@@ -283,17 +287,24 @@ template <int W>
 __device__ __forceinline__ double vi_row(const int16_t* scol, const uint16_t* svi, const double* sdict,
                                          const double* xr) {
     double xv[W], vv[W];
-#if defined(CME_ABL_NOGATHER)
+#if CME_ABL == 3
 #pragma unroll
-    for (int u = 0; u < W; ++u) xv[u] = __ldg(xr + (scol[32 * u] & 1));
+    for (int u = 0; u < W; ++u) xv[u] = (double)scol[32 * u];   // (ablation: no gathers, no dictionary)
+#pragma unroll
+    for (int u = 0; u < W; ++u) vv[u] = (double)svi[32 * u];
+#elif CME_ABL == 4
+#pragma unroll
+    for (int u = 0; u < W; ++u) xv[u] = __ldg(xr + (scol[32 * u] & 1));   // (ablation: no gathers, no dictionary)
+#pragma unroll
+    for (int u = 0; u < W; ++u) vv[u] = (double)svi[32 * u];
+#elif CME_ABL == 5
+#pragma unroll
+    for (int u = 0; u < W; ++u) xv[u] = __ldg(xr + (scol[32 * u] & 1));   // (ablation: no gathers)
+#pragma unroll
+    for (int u = 0; u < W; ++u) vv[u] = sdict[svi[32 * u]];
 #else
 #pragma unroll
     for (int u = 0; u < W; ++u) xv[u] = __ldg(xr + scol[32 * u]);
-#endif
-#if defined(CME_ABL_NODICT)
-#pragma unroll
-    for (int u = 0; u < W; ++u) vv[u] = (double)svi[32 * u];
-#else
 #pragma unroll
     for (int u = 0; u < W; ++u) vv[u] = sdict[svi[32 * u]];
 #endif
@@ -363,7 +374,7 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
             vi_issue<kTileSlices, BAND, REARR>(V, stages, full, t_first + (int64_t)i * t_stride, i, pol);
     }
     pdl_wait();
-    if (a.stop != nullptr && *a.stop) {
+    if (!CME_ABL && a.stop != nullptr && *a.stop) {   // (ablation builds run every launch)
         if (producer) {
             mbar_wait(&dbar, 0u);
             for (int i = 0; i < pro; ++i) mbar_wait(&full[i], 0u);
@@ -406,24 +417,23 @@ __global__ void __launch_bounds__(TmaShape<NCW>::kThreads, TmaShape<NCW>::kMinBl
             const int2 meta = reinterpret_cast<const int2*>(st - kMeta)[warp];   // {offset in tile, width}
             const int q = (int)tile * kTileSlices + warp;
             const int slot = q * 32 + lane;
-#if defined(CME_ABL_NOCOMPUTE)
+#if CME_ABL == 1   // (ablation: the ring alone)
             if (q < slice_end && slot < n_rows && meta.y == 12345) {
 #else
             if (q < slice_end && slot < n_rows) {
 #endif
                 const int ls = warp * 32 + lane;
                 const int r = REARR ? ((slot >> ws) << ws) + st[kOffRow + ls] : slot;
-#if defined(CME_ABL_NOINVD)
-                const double id = 0.5;
-#else
                 const double id = ld_stream(a.inv_d + slot, pol_s);   // with the x loads, before the gathers
-#endif
                 RowX<1, BAND> X;
                 X.load(xo, r);
                 const double* xr = xo + r;
                 const uint16_t* svi = reinterpret_cast<const uint16_t*>(st + off_val) + meta.x + lane;
                 const int16_t* scol = reinterpret_cast<const int16_t*>(st + off_col) + meta.x + lane;
                 double acc = 0.0;
+#if CME_ABL == 2   // (ablation: the row stream without the entries)
+                if (meta.y != 12345) {} else
+#endif
                 switch (meta.y) {   // warp-uniform exact widths
                     case 0: break;
                     case 1: acc = vi_row<1>(scol, svi, sdict, xr); break;

@@ -32,7 +32,7 @@
 //   state the next launch (or write_out) expects.
 //
 // Every spin is bounded by a %globaltimer deadline: a lost CTA turns the solve
-// into CME_ERR_CUDA ("resident kernel timed out"), never a hung GPU.
+// into CME_ERR_TIMEOUT ("resident kernel timed out"), never a hung GPU.
 #pragma once
 #include "kernels.cuh"
 
@@ -382,7 +382,7 @@ __global__ void __launch_bounds__(kResThreads, 1) sell_resident_kernel(const Res
         }
     }
     if (timed_out && tid == 0) {
-        a.ctrl->status = CME_ERR_CUDA;
+        a.ctrl->status = CME_ERR_TIMEOUT;
         a.ctrl->stop = 1;
     }
 }

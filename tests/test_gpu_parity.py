@@ -446,18 +446,27 @@ def test_every_step_kernel(cme, oracle_mod, monkeypatch, knobs, net, order, omeg
     assert st == ref.status and abs(it - ref.iters) <= 7
 
 
+@pytest.fixture(scope="module")
+def cfg4(cme, oracle_mod):
+    """The bench workload (configs[3]: toggle N=3164, n = 20,015,468), packed
+    exactly as bench.py packs it, and the oracle's own enumeration + CSR."""
+    net = W.config_network("cfg4_toggle_20m")
+    m = cme.Matrix.from_network(net).reorder(cme.CME_ORDER_RCM).pack()
+    A = oracle_mod.network_csr(net)
+    yield m, A
+    m.close()
+
+
 @pytest.mark.slow
-def test_cfg4_full_size_parity(cme, oracle_mod):
+def test_cfg4_full_size_parity(cme, oracle_mod, cfg4):
     """The bench workload itself (configs[3]: toggle N=3164, n = 20,015,468, RCM,
     the kernel bench.py times): one SpMV on every row, the |d|-weighted mass
     invariant, and 300 iterations of the landscape against the
     oracle's own enumeration + CSR Jacobi (16 host threads)."""
     import os
-    net = W.config_network("cfg4_toggle_20m")
-    m = cme.Matrix.from_network(net).reorder(cme.CME_ORDER_RCM).pack()
+    m, A = cfg4
     info = m.info()
     assert info.n == 20015468 and info.nnz == 120042194 and info.kernel == 1 and info.compact == 2
-    A = oracle_mod.network_csr(net)
     x = W.random_start(A.n, 17)
     m.set_opts(omega=1.0)
     y = m.spmv(x)
@@ -470,6 +479,32 @@ def test_cfg4_full_size_parity(cme, oracle_mod):
                                   nthreads=len(os.sched_getaffinity(0)))
     assert it == ref.iters == 300
     assert np.abs(p - ref.p).sum() <= 1e-10
+
+
+@pytest.mark.slow
+def test_cfg4_converged_landscape(cme, oracle_mod, cfg4):
+    """North-star landscape parity at the headline scale (SURVEY 8(c5)(iii),
+    P:L111-125): cfg4 solved to tol 1e-12 from uniform p0 with C = 100 by the
+    kernel bench.py times (value-indexed TMA kernel, info.compact == 2) and by
+    the oracle (plain C CSR Jacobi, all host cores).  Same stop iteration
+    within +-C; if the counts differ the oracle is re-run for exactly the GPU's
+    count; then ||p_gpu - p_oracle||_1 <= 1e-10."""
+    import os
+    m, A = cfg4
+    info = m.info()
+    assert info.kernel == 1 and info.compact == 2
+    m.set_opts(omega=0.9, check_every=100, stag_tol=1e-10, stop=cme.CME_STOP_DELTA_L1)
+    p, st, it = m.solve(tol=1e-12, max_iter=200000)
+    nt = len(os.sched_getaffinity(0))
+    ref = oracle_mod.jacobi_solve(A, omega=0.9, tol=1e-12, check_every=100, max_iter=200000, nthreads=nt)
+    assert st == ref.status == "CONVERGED", (st, ref.status)
+    assert abs(it - ref.iters) <= 100, (it, ref.iters)
+    if it != ref.iters:
+        ref = oracle_mod.jacobi_solve(A, omega=0.9, tol=0.0, check_every=100, max_iter=it, stag_tol=0.0,
+                                      nthreads=nt)
+    err = float(np.abs(p - ref.p).sum())
+    assert err <= 1e-10, err
+    assert abs(p.sum() - 1.0) <= 1e-12 and np.all(p >= 0)
 
 
 def directed_ring(n, hops=(1, 5), rates=(1.0, 0.5)):
@@ -523,3 +558,42 @@ def test_resident_dependency_ranges(cme, oracle_mod, monkeypatch, width):
     cme.cme_solver_fetch(m.h, n, q)
     ref = oracle_mod.jacobi_solve(A, p0=x, omega=0.8, tol=0.0, check_every=10, max_iter=70, stag_tol=0.0)
     assert np.abs(q - ref.p).sum() <= 1e-12
+
+
+ABLATION_ARMS = [("sell256", dict(fmt=3, window=1)), ("random-order", dict(perm=True)),
+                 ("global-window", dict(window=1 << 30)), ("ell", dict(fmt=1, window=1)),
+                 ("csr", dict(fmt=2, window=1))]
+
+
+@pytest.mark.parametrize("arm,kw", ABLATION_ARMS, ids=[a for a, _ in ABLATION_ARMS])
+@pytest.mark.parametrize("net", [W.toggle_switch(60), W.schnakenberg(35), W.brusselator(40)], ids=lambda n: n.name)
+@pytest.mark.parametrize("tma", ["0", "1"])
+def test_ablation_arms_on_gpu(cme, oracle_mod, monkeypatch, arm, kw, net, tma):
+    """NEXT-2 format/ordering arms of Tables II-III and sec. VII-C
+    through the GPU path, against the oracle: 256-row block-sliced ELL ([5],
+    P:L159), a seeded random ordering (the locality stress of P:L225), the
+    global rearrangement window (pJDS-like, window >= n), plain ELL and CSR.
+    SpMV per step, a fixed-iteration landscape and a solve to convergence."""
+    assert cme.CME_FMT_SELL256 == 3 and cme.CME_FMT_ELL == 1 and cme.CME_FMT_CSR == 2
+    monkeypatch.setenv("CME_TMA", tma)
+    monkeypatch.setenv("CME_RESIDENT", "0")
+    states, r, c, v = oracle_mod.enumerate_network(net)
+    A = oracle_mod.ingest(len(states), r, c, v)
+    m = cme.Matrix(A.n, r, c, v)
+    if kw.get("perm"):
+        m.set_permutation(np.random.default_rng(9).permutation(A.n).astype(np.int32))
+    m.pack(kw.get("fmt", 0), kw.get("window", 256), 0)
+    omega = 0.9 if oracle_mod.period(A) != 1 else 1.0
+    m.set_opts(omega=omega, check_every=40, stag_tol=0.0)
+    x = W.random_start(A.n, 6)
+    assert_spmv_close(m.spmv(x), oracle_mod.jacobi_step(A, x, omega))
+    p, st, it = m.solve(tol=0.0, max_iter=200)
+    ref = oracle_mod.jacobi_solve(A, omega=omega, tol=0.0, check_every=40, max_iter=200, stag_tol=0.0)
+    assert it == ref.iters == 200 and np.abs(p - ref.p).sum() <= 1e-12
+    p, st, it = m.solve(tol=1e-11, max_iter=30000)   # toggle converges; the others stop at max_iter
+    ref = oracle_mod.jacobi_solve(A, omega=omega, tol=1e-11, check_every=40, max_iter=30000, stag_tol=0.0)
+    assert st == ref.status and abs(it - ref.iters) <= 40
+    if it != ref.iters:
+        ref = oracle_mod.jacobi_solve(A, omega=omega, tol=0.0, check_every=40, max_iter=it, stag_tol=0.0)
+    assert np.abs(p - ref.p).sum() <= 1e-10
+    m.close()

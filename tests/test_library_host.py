@@ -34,6 +34,7 @@ def test_abi_exports_every_declared_symbol():
     assert sorted(declared) == cme.ABI_SYMBOLS
     assert cme.cme_abi_version() == 1
     assert cme.cme_status_string(cme.CME_STAGNATED) == "CME_STAGNATED"
+    assert cme.cme_status_string(cme.CME_ERR_TIMEOUT) == "CME_ERR_TIMEOUT"
 
 
 @pytest.mark.parametrize("net", NETS, ids=lambda n: n.name)

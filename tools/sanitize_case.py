@@ -1,4 +1,13 @@
-"""Small end-to-end run of every step kernel for compute-sanitizer (tools/gpu_sanitize.sh)."""
+"""Small end-to-end run of every step kernel for compute-sanitizer (tools/gpu_sanitize.sh).
+
+Covers: the register SELL kernel, the TMA kernel on layout v0, the compact
+encoding, the value-indexed kernel (16-, 8- and 31-warp tiles: the hot kernel
+and its single-dictionary shape), the SMEM-resident kernel, the batched
+value-indexed kernel (B = 2 and B = 8 on 15-warp tiles) and the GPU
+enumerator.  (Not the in-process peer-memory rank group: its ranks' step
+kernels wait on each other's flag barriers, and the sanitizer serialises
+kernels, so they would wait out the barrier time-out.)
+"""
 import os
 import sys
 
@@ -9,25 +18,49 @@ import numpy as np  # noqa: E402
 import paper_conf_ipps_maggionibl13_b200 as cme  # noqa: E402
 import workloads as W  # noqa: E402
 
-for knobs in ({"CME_TMA": "0", "CME_RESIDENT": "0"}, {"CME_TMA": "1", "CME_RESIDENT": "0"},
-              {"CME_TMA": "1", "CME_TMA_WARPS": "8", "CME_RESIDENT": "0"}, {"CME_TMA": "-1", "CME_RESIDENT": "1"}):
-    os.environ.update(knobs)
+KNOBS = [
+    ("register", {"CME_TMA": "0", "CME_RESIDENT": "0"}),
+    ("tma-v0", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_COMPACT": "0"}),
+    ("compact", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "0"}),
+    ("vi16", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_TMA_WARPS": "16"}),
+    ("vi8", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_TMA_WARPS": "8"}),
+    ("vi31", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_TMA_WARPS": "31"}),
+    ("resident", {"CME_TMA": "-1", "CME_RESIDENT": "1"}),
+]
+ALL_KEYS = sorted({k for _, kn in KNOBS for k in kn} | {"CME_TMA_WARPS"})
+
+
+def set_knobs(kn):
+    for k in ALL_KEYS:
+        os.environ.pop(k, None)
+    os.environ.update(kn)
+
+
+for label, knobs in KNOBS:
+    set_knobs(knobs)
     for net, order in ((W.toggle_switch(30), cme.CME_ORDER_RCM), (W.schnakenberg(40), cme.CME_ORDER_NONE)):
         m = cme.Matrix.from_network(net).reorder(order).pack()
         m.set_opts(omega=0.9, check_every=7)
         p, st, it = m.solve(tol=1e-9, max_iter=300)
         y = m.spmv(W.random_start(m.n, 1))
         pt, terms = m.transient(0.05)
-        print(knobs, net.name, m.info().kernel, st, it, float(p.sum()), terms, flush=True)
+        f = m.info()
+        print(label, net.name, "kernel", f.kernel, "compact", f.compact, "warps", f.tma_warps, st, it,
+              float(p.sum()), terms, flush=True)
         m.close()
-    states, r, c, v = cme.cme_network_enumerate(W.toggle_switch(20))
-    vs = np.stack([v * f for f in (1.0, 1.5)])
-    os.environ["CME_RESIDENT"] = "-1"   # batches have no resident kernel
+
+# batches: the batched value-indexed kernel (B = 2 default shape, B = 8 on 15-warp tiles)
+states, r, c, v = cme.cme_network_enumerate(W.toggle_switch(20))
+for B, warps in ((2, None), (8, "15")):
+    set_knobs({"CME_TMA": "1", "CME_RESIDENT": "-1"} | ({"CME_TMA_WARPS": warps} if warps else {}))
+    vs = np.stack([v * (1.0 + 0.1 * b) for b in range(B)])
     m = cme.Matrix(len(states), r, c, vs).reorder(cme.CME_ORDER_RCM).pack()
     m.set_opts(omega=0.9, check_every=10)
     p, st, it = m.solve(tol=1e-9, max_iter=200)
-    print(knobs, "batch2", m.info().kernel, st, it, flush=True)
+    f = m.info()
+    print("batch", B, "kernel", f.kernel, "compact", f.compact, "warps", f.tma_warps, st, it, flush=True)
     m.close()
+
 # GPU state enumerator
 for net in (W.toggle_switch(25), W.brusselator(30)):
     states, r, c, v = cme.cme_network_enumerate_gpu(net)
