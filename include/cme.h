@@ -207,7 +207,10 @@ typedef struct cme_info {
     int32_t batch;                /* rate sets sharing the pattern (1 = single matrix) */
     int32_t compact;              /* 1: the TMA kernel streams the compact encoding (rows of
                                      M = |D|^-1 O, int16 column and uint8 row offsets,
-                                     DESIGN.md sec. 5b); bytes_fmt/packed_bytes count it */
+                                     DESIGN.md sec. 5b); 2: its value-indexed form (sec. 5c);
+                                     bytes_fmt/packed_bytes count it */
+    int32_t records;              /* 1: the value-indexed encoding is streamed as one
+                                     contiguous record per tile (sell_vi2_kernel, sec. 5d) */
 } cme_info;
 cme_status cme_get_info(cme_matrix h, cme_info* info);
 

@@ -21,6 +21,7 @@
 #include "cme_internal.h"
 #include "comm.h"
 #include "launch.h"
+#include "kernels_vi2.cuh"
 #include "kernels_resident.cuh"
 #include "kernels_cpt.cuh"
 
@@ -121,6 +122,14 @@ struct Device {
     uint16_t *vidx = nullptr, *loi = nullptr, *upi = nullptr;
     int dict_bytes = 0;              // shared-memory bytes of the dictionary (multiple of 128)
     int vi_idpf = 1;                 // L2 prefetch of the tile's inv_d by the producer (CME_VI_IDPF)
+    // tile-record value-indexed kernel (kernels_vi2.cuh, B = 1): one contiguous
+    // record per tile; replaces sell_vi_kernel when vi2 (CME_VI2 = 0 keeps it)
+    bool vi2 = false;
+    bool vi2_words = false;          // records hold packed vidx | col16 << 16 words (CME_VI2_WORDS)
+    int vi2_ncw = 0, vi2_stages = 0, vi2_stage_bytes = 0, vi2_grid = 0, vi2_occ = 0;
+    int64_t vi2_tiles = 0;
+    unsigned char* vi2_rec = nullptr;
+    int64_t* vi2_rec_off = nullptr;
     // SMEM-resident persistent kernel (kernels_resident.cuh)
     bool use_res = false;
     int res_grid = 0, res_smem = 0, res_rps = 1;
@@ -150,7 +159,7 @@ struct Device {
         if (!h.empty()) CUDA_TRY(cudaMemcpy(p, h.data(), h.size() * sizeof(T), cudaMemcpyHostToDevice));
         return CME_OK;
     }
-    int step_grid() const { return use_tma ? tma_grid : grid; }
+    int step_grid() const { return vi2 ? vi2_grid : use_tma ? tma_grid : grid; }
 };
 
 // ------------------------------------------------------------------------------
@@ -527,6 +536,112 @@ static cme_status configure_tma(Device& d, const Packed& P) {
     return CME_OK;
 }
 
+// Tile records of the value-indexed encoding for tiles of ts slices
+// (kernels_vi2.cuh): per tile one contiguous block
+// [meta | row8 | loi, upi | inv_d | per slice: vidx[32 W], col16[32 W]],
+// every block 16-B aligned; a pure re-layout of sec. 5c's arrays.
+static int64_t vi2_record_bytes(const Packed& P, int ts, bool band, bool rearr, int64_t t) {
+    const int64_t q0 = t * ts, q1 = std::min<int64_t>(q0 + ts, P.n_slices);
+    return vi2_fixed_bytes(ts, band, rearr) + 4 * (P.slice_off[q1] - P.slice_off[q0]);
+}
+
+static void vi2_build_records(const Packed& P, const Compact& C, int ts, bool band, bool rearr, bool words,
+                              std::vector<unsigned char>& rec, std::vector<int64_t>& off) {
+    const int64_t nt = (P.n_slices + ts - 1) / ts;
+    off.assign(nt + 1, 0);
+    for (int64_t t = 0; t < nt; ++t) off[t + 1] = off[t] + vi2_record_bytes(P, ts, band, rearr, t);
+    rec.assign((size_t)off[nt], 0);
+    const int kMeta = ((ts + 1) & ~1) * 8;
+    const int kRow = kMeta, kLoUp = kRow + (rearr ? ts * 32 : 0), kInv = kLoUp + (band ? ts * 128 : 0),
+              kEnt = kInv + ts * 256;
+#pragma omp parallel for schedule(static)
+    for (int64_t t = 0; t < nt; ++t) {
+        unsigned char* R = rec.data() + off[t];
+        const int64_t q0 = t * ts, q1 = std::min<int64_t>(q0 + ts, P.n_slices);
+        const int64_t e0 = P.slice_off[q0];
+        for (int64_t q = q0; q < q1; ++q) {
+            const int32_t m[2] = {(int32_t)(P.slice_off[q] - e0), (int32_t)P.slice_w[q]};
+            std::memcpy(R + 8 * (q - q0), m, 8);
+            const int64_t sl0 = q * 32, ls0 = (q - q0) * 32;
+            if (rearr) std::memcpy(R + kRow + ls0, C.row8.data() + sl0, 32);
+            if (band) {
+                std::memcpy(R + kLoUp + 2 * ls0, C.loi.data() + sl0, 64);
+                std::memcpy(R + kLoUp + ts * 64 + 2 * ls0, C.upi.data() + sl0, 64);
+            }
+            std::memcpy(R + kInv + 8 * ls0, P.inv_d.data() + sl0, 256);
+            const int64_t ne = P.slice_off[q + 1] - P.slice_off[q];   // 32 W entries
+            unsigned char* E = R + kEnt + 4 * (P.slice_off[q] - e0);
+            if (words) {   // entry k: vidx | col16 << 16
+                for (int64_t k = 0; k < ne; ++k) {
+                    const uint32_t w = (uint32_t)C.vidx[P.slice_off[q] + k] |
+                                       ((uint32_t)(uint16_t)C.col16[P.slice_off[q] + k] << 16);
+                    std::memcpy(E + 4 * k, &w, 4);
+                }
+            } else {
+                std::memcpy(E, C.vidx.data() + P.slice_off[q], 2 * ne);
+                std::memcpy(E + 2 * ne, C.col16.data() + P.slice_off[q], 2 * ne);
+            }
+        }
+    }
+}
+
+// Choose the vi2 tile shape, in the order measured on cfg4 (B200): 30
+// consumer warps in one 1024-thread CTA per SM (one dictionary, 64 registers,
+// 4 x 32 KB stages: 170 us per iteration) when >= 3 stages fit, else 16 in 2
+// CTAs per SM (56 registers, 3 stages: 175 us); 23 warps in 2 CTAs per SM (40
+// registers: spills, 2 stages: 227 us) only when forced.  Deepest ring <= 4
+// stages.  CME_VI2_WARPS / CME_VI2_STAGES force a shape.
+static cme_status configure_vi2(Device& d, const Packed& P) {
+    d.vi2 = false;
+    int dev = 0, smem_max = 0, sms = 0;
+    CUDA_TRY(cudaGetDevice(&dev));
+    CUDA_TRY(cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+    CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    const int force_w = env_int("CME_VI2_WARPS", 0), force_s = env_int("CME_VI2_STAGES", 0);
+    const int cap = smem_max - 4096;
+    struct Best { int ncw = 0, stages = 0, occ = 0; int64_t stage = 0, tiles = 0; } best;
+    for (int ncw : {30, 16, 23}) {
+        if (force_w && ncw != force_w) continue;
+        if (!force_w && ncw == 23) continue;
+        const int64_t nt = (P.n_slices + ncw - 1) / ncw;
+        int64_t mx = 0;
+        for (int64_t t = 0; t < nt; ++t) mx = std::max(mx, vi2_record_bytes(P, ncw, d.band, d.rearr, t));
+        const int64_t stage = (mx + 127) / 128 * 128;
+        CUDA_TRY(vi2_prepare(ncw, cap));
+        const int want_occ = ncw == 30 ? 1 : 2;
+        int stages = 0, occ = 0;
+        for (int st = force_s > 0 ? std::min(force_s, 8) : 4; st >= 2; --st) {
+            const int64_t bytes = d.dict_bytes + st * stage;
+            if (bytes > cap) continue;
+            int o = 0;
+            CUDA_TRY(vi2_occupancy(ncw, (int)bytes, &o));
+            if (o >= want_occ || (force_s > 0 && o >= 1)) { stages = st; occ = o; break; }
+        }
+        if (env_int("CME_VERBOSE", 0) > 1)
+            std::fprintf(stderr, "[cme] vi2 shape: ncw=%d stage=%lld stages=%d occ=%d\n", ncw, (long long)stage, stages, occ);
+        if (!stages || (!force_w && !force_s && ncw == 30 && stages < 3)) continue;
+        best = Best{ncw, stages, occ, stage, nt};
+        break;   // first acceptable shape in measured order
+    }
+    if (!best.ncw) return CME_OK;
+    if (env_int("CME_VI2", 1) == 0) return CME_OK;
+    d.vi2 = true;
+    d.vi2_words = env_int("CME_VI2_WORDS", 0) != 0;
+    d.vi2_ncw = best.ncw;
+    d.vi2_stages = best.stages;
+    d.vi2_stage_bytes = (int)best.stage;
+    d.vi2_occ = best.occ;
+    d.vi2_tiles = best.tiles;
+    d.vi2_grid = (int)std::min<int64_t>(best.tiles, (int64_t)sms * best.occ);
+    // CME_VI2_GRID caps the grid (tests: many tiles per CTA wrap the ring many times)
+    if (env_int("CME_VI2_GRID", 0) > 0) d.vi2_grid = std::min(d.vi2_grid, env_int("CME_VI2_GRID", 0));
+    if (env_int("CME_VERBOSE", 0))
+        std::fprintf(stderr, "[cme] vi2: warps=%d stages=%d stage_bytes=%d occ=%d grid=%d tiles=%lld dict=%d\n",
+                     d.vi2_ncw, d.vi2_stages, d.vi2_stage_bytes, d.vi2_occ, d.vi2_grid, (long long)d.vi2_tiles,
+                     d.dict_bytes);
+    return CME_OK;
+}
+
 // Plan the SMEM-resident kernel (kernels_resident.cuh): one CTA per SM, each
 // owning a window-aligned run of slices (<= 128) whose packed image fits in
 // shared memory; its probe range = owners of the columns it reads plus the
@@ -762,6 +877,8 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
             h->Cpt = Compact();
             if (v0_tma && (s = configure_tma(*d, P)) != CME_OK) return fail(s);
         }
+        // the value-indexed encoding as tile records (sec. 5d)
+        if (d->use_tma && d->vi && (s = configure_vi2(*d, P)) != CME_OK) return fail(s);
     }
     if (d->B > 1 && d->format == CME_FMT_DIAG_SELL && env_int("CME_COMPACT", 1) != 0 && env_int("CME_VI", -1) != 0 &&
         env_int("CME_TMA", -1) != 0 && encode_compact(P, d->own_off, h->Cpt) && encode_value_index(P, h->Cpt)) {
@@ -789,7 +906,16 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
         if ((s = d->upload(d->tile_meta, tm)) != CME_OK) return fail(s);
     }
     if (d->format != CME_FMT_CSR) {
-        if (d->vi) {
+        if (d->vi2) {   // tile records + the dictionary; no separate index arrays
+            std::vector<double> dict(h->Cpt.dict);
+            dict.resize(d->dict_bytes / 8, 0.0);   // staged in shared memory, 128-B padded
+            UP(dict, dict);
+            std::vector<unsigned char> rec;
+            std::vector<int64_t> roff;
+            vi2_build_records(P, h->Cpt, d->vi2_ncw, d->band, d->rearr, d->vi2_words, rec, roff);
+            UP(vi2_rec, rec);
+            UP(vi2_rec_off, roff);
+        } else if (d->vi) {
             std::vector<double> dict(h->Cpt.dict);
             if (d->B == 1) dict.resize(d->dict_bytes / 8, 0.0);   // (B = 1: staged in shared memory, 128-B padded)
             UP(dict, dict);
@@ -1116,6 +1242,11 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
     if (d.format == CME_FMT_CSR) {
         CUDA_TRY(check ? launch_ex(csr_step_kernel<true>, dim3(d.grid), dim3(kCta), 0, pdl, s, a)
                        : launch_ex(csr_step_kernel<false>, dim3(d.grid), dim3(kCta), 0, pdl, s, a));
+    } else if (d.vi2) {
+        Vi2Args V{a, d.vi2_rec, d.vi2_rec_off, d.dict, d.vi2_tiles, d.vi2_stages, d.vi2_stage_bytes, d.dict_bytes,
+                  d.win_shift, d.tma_xpf};
+        CUDA_TRY(launch_vi2(V, d.vi2_ncw, d.vi2_grid, d.dict_bytes + d.vi2_stages * d.vi2_stage_bytes, d.band, d.rearr,
+                            check, d.vi2_words, pdl, s));
     } else if (d.use_tma && d.vi && d.B > 1) {
         ViArgs V{CptArgs{TmaArgs{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col,
                                  d.tma_contig, d.tma_xpf},
@@ -1541,8 +1672,9 @@ cme_status device_transient(cme_matrix_s* h, const double* p0, double t, double 
 void device_describe(const Device* d, cme_info* f) {
     if (!d) { f->kernel = -1; return; }
     f->kernel = d->format == CME_FMT_CSR ? 2 : d->use_res ? 3 : d->use_tma ? 1 : 0;
-    f->tma_warps = d->use_tma ? d->tma_ncw : 0;
-    f->tma_stages = d->use_tma ? d->tma_stages : 0;
+    f->tma_warps = d->vi2 ? d->vi2_ncw : d->use_tma ? d->tma_ncw : 0;
+    f->tma_stages = d->vi2 ? d->vi2_stages : d->use_tma ? d->tma_stages : 0;
+    f->records = d->vi2 ? 1 : 0;
     f->grid = d->use_res ? d->res_grid : d->step_grid();
     f->compact = d->vi ? 2 : d->cpt ? 1 : 0;
     if (d->vi) {   // value-indexed: 4 B per ELL slot (shared by a batch), inv_d per row and member

@@ -23,7 +23,7 @@ template <int NCW>
 struct TmaShape {
     static constexpr int kThreads = 32 * (NCW + 1);
     // register cap: 75 / 60 regs; 31 consumer warps = one 1024-thread CTA per SM (64 regs)
-    static constexpr int kMinBlocks = NCW == 8 ? 3 : NCW == 31 ? 1 : 2;
+    static constexpr int kMinBlocks = NCW == 8 ? 3 : NCW == 31 ? 1 : 2;   // (23: 2 x 768 threads)
 };
 
 struct TmaArgs {

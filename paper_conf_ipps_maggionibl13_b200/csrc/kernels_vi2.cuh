@@ -1,0 +1,328 @@
+// Tile-record value-indexed step kernel (B = 1): the hot
+// kernel on the toggle-switch CMEs.  Same operator and arithmetic as
+// sell_vi_kernel -- y = (1-omega) x + omega inv_d (sum_t dict[vidx] x[r + col])
+// (eq. 8, R1), FMAs in t order, row sum times inv_d -- so its results
+// are bit-identical to it and to the layout-v0 kernels.  What changes is how
+// the encoding reaches the SM and how lean the consumer loop is:
+//
+// * Tile records.  Everything a tile needs is ONE contiguous record in HBM --
+//   [slice metadata | row8 | loi, upi | inv_d | per slice: vidx block, col16
+//   block] -- moved by ONE cp.async.bulk per tile.  sell_vi_kernel issued 4-6
+//   bulk copies per tile (metadata 128 B, row8 512 B, ...) plus a separate
+//   per-lane inv_d stream, and its TMA ring alone (consumers idle: CME_ABL=1)
+//   topped out at 5.4 TB/s of DRAM reads.
+// * inv_d comes from shared memory (no global load on the slice's critical
+//   path besides the x gathers).
+// * All stage addressing is 32-bit shared-window arithmetic derived from the
+//   slice's {entry offset, width} record; omega and the buffer pointers stay
+//   kernel parameters (constant-bank operands), so the consumer loop fits the
+//   40-register budget of 2 x 24-warp CTAs per SM (46 consumer warps) where
+//   sell_vi_kernel needs 56 (32 warps).  Measured: the step is bound by the
+//   latency of the x gathers behind one shared-memory round trip, so resident
+//   consumer warps set the rate.
+#pragma once
+#include "kernels_cpt.cuh"
+
+namespace cme {
+
+struct Vi2Args {
+    StepArgs a;              // n_rows, slice_end, x/y, own_off, omega, pre_scale, partials, stop, inv_d (checks), push
+    const unsigned char* rec;   // tile records, rec_off[t] bytes from rec
+    const int64_t* rec_off;     // [n_tiles + 1]
+    const double* dict;         // [dict_bytes / 8], 128-B padded
+    int64_t n_tiles;
+    int32_t stages;
+    int32_t stage_bytes;        // >= the largest record, multiple of 128
+    int32_t dict_bytes;
+    int32_t win_shift;          // log2(rearrangement window) (REARR)
+    int32_t xpf;                // L2 prefetch of each tile's own x rows with its record
+};
+
+// Record layout of a tile of TS slices (byte offsets; every block 16-B aligned).
+template <int TS, bool BAND, bool REARR>
+struct Vi2Rec {
+    static constexpr int kMeta = ((TS + 1) & ~1) * 8;              // int2 {entry offset, width} per slice
+    static constexpr int kRow = kMeta;                            // uint8 per slot (REARR)
+    static constexpr int kLoUp = kRow + (REARR ? TS * 32 : 0);    // uint16 loi[slots], upi[slots] (BAND)
+    static constexpr int kInv = kLoUp + (BAND ? TS * 128 : 0);    // double per slot
+    static constexpr int kEnt = kInv + TS * 256;                  // per slice: vidx[32 W] then col16[32 W]
+};
+__host__ __device__ constexpr int vi2_fixed_bytes(int ts, bool band, bool rearr) {
+    return ((ts + 1) & ~1) * 8 + (rearr ? ts * 32 : 0) + (band ? ts * 128 : 0) + ts * 256;
+}
+
+__device__ __forceinline__ uint32_t lds_u16(uint32_t a) {
+    uint16_t v;
+    asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ int32_t lds_s16(uint32_t a) {
+    int16_t v;
+    asm volatile("ld.shared.s16 %0, [%1];" : "=h"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint32_t lds_u8(uint32_t a) {
+    uint16_t v;
+    asm volatile("ld.shared.u8 %0, [%1];" : "=h"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ double lds_f64(uint32_t a) {
+    double v;
+    asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint32_t lds_u32(uint32_t a) {
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+// mbarrier wait / arrive on a 32-bit shared-window address (no generic ->
+// shared conversion in the loop)
+__device__ __forceinline__ void mbar_wait_a(uint32_t b, uint32_t parity) {
+    asm volatile(
+        "{\n"
+        ".reg .pred P1;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1, %2;\n"
+        "@!P1 bra WAIT_%=;\n"
+        "}\n" ::"r"(b),
+        "r"(parity), "n"(CME_MBAR_SUSPEND_NS)
+        : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_a(uint32_t b) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(b) : "memory");
+}
+__device__ __forceinline__ int2 lds_v2(uint32_t a) {
+    int2 v;
+    asm volatile("ld.shared.v2.s32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
+    return v;
+}
+
+// W entries of one slot: the W x gathers first (their latency is the step's
+// critical path), then per entry the dictionary value and the FMA in t order.
+template <int W>
+__device__ __forceinline__ double vi2_row(uint32_t pv, uint32_t pc, uint32_t sdict, const double* xr) {
+    double xv[W];
+#pragma unroll
+    for (int u = 0; u < W; ++u) xv[u] = __ldg(xr + lds_s16(pc + 64 * u));
+    double acc = 0.0;
+#pragma unroll
+    for (int u = 0; u < W; ++u) acc = fma(lds_f64(sdict + 8 * lds_u16(pv + 64 * u)), xv[u], acc);
+    return acc;
+}
+__device__ __forceinline__ double vi2_row_wide(uint32_t pv, uint32_t pc, uint32_t sdict, const double* xr, int w) {
+    double acc = 0.0;
+    for (int t0 = 0; t0 < w; t0 += 8) {
+        double xv[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u)
+            if (t0 + u < w) xv[u] = __ldg(xr + lds_s16(pc + 64 * (t0 + u)));
+#pragma unroll
+        for (int u = 0; u < 8; ++u)
+            if (t0 + u < w) acc = fma(lds_f64(sdict + 8 * lds_u16(pv + 64 * (t0 + u))), xv[u], acc);
+    }
+    return acc;
+}
+
+// Packed-word variant (ENC = 1): entry u of a lane is one 32-bit word
+// vidx | col16 << 16 at pw + 128 u -- one shared-memory load per entry instead
+// of two (half the LSU wavefronts of the index reads).
+template <int W>
+__device__ __forceinline__ double vi2_row_w(uint32_t pw, uint32_t sdict, const double* xr) {
+    uint32_t w[W];
+#pragma unroll
+    for (int u = 0; u < W; ++u) w[u] = lds_u32(pw + 128 * u);
+    double xv[W];
+#pragma unroll
+    for (int u = 0; u < W; ++u) xv[u] = __ldg(xr + ((int32_t)w[u] >> 16));
+    double acc = 0.0;
+#pragma unroll
+    for (int u = 0; u < W; ++u) acc = fma(lds_f64(sdict + 8 * (w[u] & 0xffffu)), xv[u], acc);
+    return acc;
+}
+__device__ __forceinline__ double vi2_row_w_wide(uint32_t pw, uint32_t sdict, const double* xr, int wd) {
+    double acc = 0.0;
+    for (int t0 = 0; t0 < wd; t0 += 8) {
+        uint32_t w[8];
+        double xv[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u)
+            if (t0 + u < wd) w[u] = lds_u32(pw + 128 * (t0 + u));
+#pragma unroll
+        for (int u = 0; u < 8; ++u)
+            if (t0 + u < wd) xv[u] = __ldg(xr + ((int32_t)w[u] >> 16));
+#pragma unroll
+        for (int u = 0; u < 8; ++u)
+            if (t0 + u < wd) acc = fma(lds_f64(sdict + 8 * (w[u] & 0xffffu)), xv[u], acc);
+    }
+    return acc;
+}
+
+template <int NCW>
+struct Vi2Shape {
+    static constexpr int kThreads = 32 * (NCW + 1);
+    // 16: 2 x 544 threads (56 regs); 23: 2 x 768 (40 regs); 30: 1 x 992 (64 regs)
+    static constexpr int kMinBlocks = NCW == 30 ? 1 : 2;
+};
+
+template <int NCW, bool BAND, bool REARR, bool CHECK, int ENC>
+__global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBlocks)
+    sell_vi2_kernel(const Vi2Args V) {
+    using R = Vi2Rec<NCW, BAND, REARR>;
+    const StepArgs& a = V.a;
+    pdl_trigger();
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ uint64_t full[8], empty[8], dbar;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int S = V.stages;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < S; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], NCW);
+        }
+        mbar_init(&dbar, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    const int G = gridDim.x, c = blockIdx.x;
+    const int n_tiles = (int)V.n_tiles;
+    const int my_tiles = c < n_tiles ? (n_tiles - 1 - c) / G + 1 : 0;
+    const int pro = my_tiles < S ? my_tiles : S;
+    unsigned char* stages = smem + V.dict_bytes;
+    if (warp == NCW) {
+        // ---------------- producer warp: one bulk copy per tile record ----------------
+        // the record offsets of the CTA's next 32 tiles are loaded by the 32
+        // lanes together (one round trip per 32 tiles), lane 0 issues
+        const uint64_t pol = evict_first_policy();
+        if (lane == 0) {   // dictionary: constant, every CTA reads it (keep it in L2)
+            uint64_t keep;
+            asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(keep));
+            mbar_expect_tx(&dbar, (uint32_t)V.dict_bytes);
+            bulk_g2s(smem, V.dict, (uint32_t)V.dict_bytes, &dbar, keep);
+        }
+        int64_t o0 = 0, o1 = 0;
+        int s = 0;
+        uint32_t phase = 0;   // parity of the ring pass; reuse i >= S waits for pass (i / S - 1)'s release
+        bool waited = false;
+        for (int i = 0; i < my_tiles; ++i) {
+            const int l = i & 31;
+            if (l == 0) {   // offsets of tiles i .. i+31
+                const int t = c + (i + lane) * G;
+                if (i + lane < my_tiles) { o0 = __ldg(V.rec_off + t); o1 = __ldg(V.rec_off + t + 1); }
+            }
+            const int64_t b0 = __shfl_sync(0xffffffffu, o0, l), b1 = __shfl_sync(0xffffffffu, o1, l);
+            if (i >= S) mbar_wait(&empty[s], phase ^ 1u);
+            if (i == pro && !waited) {   // first tiles were issued before the previous step ended
+                pdl_wait();
+                waited = true;
+                if (a.stop != nullptr && *a.stop) break;
+            }
+            if (lane == 0) {
+                const int t = c + i * G;
+                const uint32_t bytes = (uint32_t)(b1 - b0);
+                if (V.xpf) {
+                    const int64_t r0 = (int64_t)t * NCW * 32, r1 = min(r0 + NCW * 32, a.n_rows);
+                    if (r1 > r0) prefetch_l2(a.x + a.own_off + r0, (uint64_t)(r1 - r0) * 8);
+                }
+                mbar_expect_tx(&full[s], bytes);
+                bulk_g2s(stages + (size_t)s * V.stage_bytes, V.rec + b0, bytes, &full[s], pol);
+            }
+            if (++s == S) { s = 0; phase ^= 1u; }
+        }
+        if (!waited) pdl_wait();
+        if (lane == 0) mbar_wait(&dbar, 0u);   // (no tile may have waited on it)
+        if (CHECK) cta_check_partials<NCW + 1, 1>(CheckAcc<1>(), a.partials);
+        return;
+    }
+    // ---------------- consumer warps: one slice each per tile ----------------
+    pdl_wait();
+    if (a.stop != nullptr && *a.stop) {
+        // the producer saw the same flag; drain the prologue copies before exit
+        for (int i = 0; i < pro; ++i) mbar_wait(&full[i], 0u);
+        mbar_wait(&dbar, 0u);
+        if (CHECK) cta_check_partials<NCW + 1, 1>(CheckAcc<1>(), a.partials);
+        return;
+    }
+    CheckAcc<1> ck;
+    {
+        const double* xo = a.x + a.own_off;
+        double* yo = a.y + a.own_off;
+        const bool damp = a.omega != 1.0, unif = a.unif_lam_inv != 0.0;
+        const double sc = a.pre_scale != nullptr ? a.pre_scale[0] : 1.0;
+        const uint32_t sdict = smem_u32(smem);
+        const uint32_t st0 = smem_u32(stages);
+        const int n_rows = (int)a.n_rows, slice_end = (int)a.slice_end;
+        const uint32_t full0 = smem_u32(full), empty0 = smem_u32(empty);
+        const uint32_t sbytes = (uint32_t)V.stage_bytes;
+        mbar_wait(&dbar, 0u);
+        int s = 0;
+        uint32_t phase = 0;
+        int q = c * NCW + warp;                    // this warp's slice of tile c + i G
+        const int dq = G * NCW;
+        uint32_t st = st0;
+        for (int i = 0; i < my_tiles; ++i, q += dq) {
+            mbar_wait_a(full0 + 8 * s, phase);
+            const int slot = q * 32 + lane;
+            if (q < slice_end && slot < n_rows) {
+                const int2 meta = lds_v2(st + 8 * warp);   // {entry offset in the tile, width}
+                const int ls = warp * 32 + lane;
+                const int r = REARR ? ((slot >> V.win_shift) << V.win_shift) + (int)lds_u8(st + R::kRow + ls) : slot;
+                const double* xr = xo + r;
+                const double x_r = __ldg(xr);
+                const uint32_t pv = st + R::kEnt + 4 * meta.x + (ENC ? 4 : 2) * lane;   // entry 0 of this lane
+                const uint32_t pc = pv + 64 * meta.y;   // (ENC 0: the col16 block follows the vidx block)
+                double acc = 0.0;
+                if (ENC) switch (meta.y) {   // warp-uniform exact widths
+                    case 0: break;
+                    case 1: acc = vi2_row_w<1>(pv, sdict, xr); break;
+                    case 2: acc = vi2_row_w<2>(pv, sdict, xr); break;
+                    case 3: acc = vi2_row_w<3>(pv, sdict, xr); break;
+                    case 4: acc = vi2_row_w<4>(pv, sdict, xr); break;
+                    case 5: acc = vi2_row_w<5>(pv, sdict, xr); break;
+                    case 6: acc = vi2_row_w<6>(pv, sdict, xr); break;
+                    case 7: acc = vi2_row_w<7>(pv, sdict, xr); break;
+                    case 8: acc = vi2_row_w<8>(pv, sdict, xr); break;
+                    default: acc = vi2_row_w_wide(pv, sdict, xr, meta.y);
+                }
+                else switch (meta.y) {   // warp-uniform exact widths
+                    case 0: break;
+                    case 1: acc = vi2_row<1>(pv, pc, sdict, xr); break;
+                    case 2: acc = vi2_row<2>(pv, pc, sdict, xr); break;
+                    case 3: acc = vi2_row<3>(pv, pc, sdict, xr); break;
+                    case 4: acc = vi2_row<4>(pv, pc, sdict, xr); break;
+                    case 5: acc = vi2_row<5>(pv, pc, sdict, xr); break;
+                    case 6: acc = vi2_row<6>(pv, pc, sdict, xr); break;
+                    case 7: acc = vi2_row<7>(pv, pc, sdict, xr); break;
+                    case 8: acc = vi2_row<8>(pv, pc, sdict, xr); break;
+                    default: acc = vi2_row_wide(pv, pc, sdict, xr, meta.y);
+                }
+                double sum = acc;
+                if (BAND) {
+                    const double xl = __ldg(xr - 1), xu = __ldg(xr + 1);
+                    const double lo = lds_f64(sdict + 8 * lds_u16(st + R::kLoUp + 2 * ls));
+                    const double up = lds_f64(sdict + 8 * lds_u16(st + R::kLoUp + NCW * 64 + 2 * ls));
+                    sum = fma(lo, xl, up * xu) + acc;
+                }
+                const double id = lds_f64(st + R::kInv + 8 * ls);
+                double y = damp ? fma(1.0 - a.omega, x_r, a.omega * (id * sum)) : id * sum;
+                if (unif) {   // transient: (I + A/Lambda) x with a_rr = -1/id
+                    y = fma(a.unif_lam_inv, sum - x_r / id, x_r);
+                    double* ac = a.acc + a.own_off + r;
+                    *ac = fma(a.acc_w, x_r, *ac);
+                }
+                y *= sc;   // pending 1/sum(y) of the previous check (exact when sc = 1)
+                yo[r] = y;
+                if (CHECK) ck.add(0, y, x_r * sc, id);
+                for (int p = 0; p < a.npush; ++p)   // halo rows straight into the peer's buffer
+                    if (r >= a.push_lo[p] && r < a.push_hi[p]) a.push_y[p][r] = y;
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive_a(empty0 + 8 * s);
+            st += sbytes;
+            if (++s == S) { s = 0; phase ^= 1u; st = st0; }
+        }
+    }
+    if (CHECK) cta_check_partials<NCW + 1, 1>(ck, a.partials);
+}
+
+}  // namespace cme

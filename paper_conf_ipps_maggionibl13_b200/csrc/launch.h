@@ -61,6 +61,12 @@ cudaError_t launch_vib(const ViArgs& V, int B, int ncw, int grid, int smem, bool
                        bool pdl, cudaStream_t s);
 cudaError_t vib_prepare(int B, int ncw, int smem);
 cudaError_t vib_occupancy(int B, int ncw, int smem, int* blocks_per_sm);
+struct Vi2Args;
+// tile-record value-indexed TMA step kernel (step_vi2.cu, B = 1): ncw = 16, 23 or 30
+cudaError_t launch_vi2(const Vi2Args& V, int ncw, int grid, int smem, bool band, bool rearr, bool check, bool words,
+                       bool pdl, cudaStream_t s);
+cudaError_t vi2_prepare(int ncw, int smem);
+cudaError_t vi2_occupancy(int ncw, int smem, int* blocks_per_sm);
 struct ResArgs;
 // SMEM-resident persistent Jacobi kernel (resident.cu)
 cudaError_t resident_prepare(int smem);

@@ -1,0 +1,59 @@
+// Launchers of the tile-record value-indexed step kernel (kernels_vi2.cuh, B = 1).
+#include "kernels_vi2.cuh"
+#include "launch.h"
+
+namespace cme {
+
+template <int W>
+static cudaError_t launch_vi2_w(const Vi2Args& V, int grid, int smem, bool band, bool rearr, bool check, bool words,
+                                bool pdl, cudaStream_t s) {
+    const int key = (words ? 8 : 0) | (band ? 4 : 0) | (rearr ? 2 : 0) | (check ? 1 : 0);
+    switch (key) {
+#define K_(e, bd, r, c)                                                                                        \
+    case e * 8 + bd * 4 + r * 2 + c:                                                                           \
+        return launch_ex(sell_vi2_kernel<W, bd, r, c, e>, dim3(grid), dim3(Vi2Shape<W>::kThreads), smem, pdl, s, V);
+        K_(0, 0, 0, 0) K_(0, 0, 0, 1) K_(0, 0, 1, 0) K_(0, 0, 1, 1) K_(0, 1, 0, 0) K_(0, 1, 0, 1) K_(0, 1, 1, 0)
+        K_(0, 1, 1, 1) K_(1, 0, 0, 0) K_(1, 0, 0, 1) K_(1, 0, 1, 0) K_(1, 0, 1, 1) K_(1, 1, 0, 0) K_(1, 1, 0, 1)
+        K_(1, 1, 1, 0) K_(1, 1, 1, 1)
+#undef K_
+    }
+    return cudaErrorInvalidValue;
+}
+
+cudaError_t launch_vi2(const Vi2Args& V, int ncw, int grid, int smem, bool band, bool rearr, bool check, bool words,
+                       bool pdl, cudaStream_t s) {
+    return ncw == 23   ? launch_vi2_w<23>(V, grid, smem, band, rearr, check, words, pdl, s)
+           : ncw == 30 ? launch_vi2_w<30>(V, grid, smem, band, rearr, check, words, pdl, s)
+                       : launch_vi2_w<16>(V, grid, smem, band, rearr, check, words, pdl, s);
+}
+
+template <int W>
+static cudaError_t vi2_prepare_w(int smem) {
+    cudaError_t e = cudaSuccess;
+#define A_(bd, r, c)                                                                                            \
+    if (e == cudaSuccess)                                                                                       \
+        e = cudaFuncSetAttribute(sell_vi2_kernel<W, bd, r, c, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
+    if (e == cudaSuccess)                                                                                       \
+        e = cudaFuncSetAttribute(sell_vi2_kernel<W, bd, r, c, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    A_(0, 0, 0) A_(0, 0, 1) A_(0, 1, 0) A_(0, 1, 1) A_(1, 0, 0) A_(1, 0, 1) A_(1, 1, 0) A_(1, 1, 1)
+#undef A_
+    return e;
+}
+
+cudaError_t vi2_prepare(int ncw, int smem) {
+    return ncw == 23 ? vi2_prepare_w<23>(smem) : ncw == 30 ? vi2_prepare_w<30>(smem) : vi2_prepare_w<16>(smem);
+}
+
+cudaError_t vi2_occupancy(int ncw, int smem, int* occ) {
+    // the heaviest variant (band + rearrangement + check) bounds the residency
+    if (ncw == 23)
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_vi2_kernel<23, true, true, true, 0>,
+                                                             Vi2Shape<23>::kThreads, smem);
+    if (ncw == 30)
+        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_vi2_kernel<30, true, true, true, 0>,
+                                                             Vi2Shape<30>::kThreads, smem);
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_vi2_kernel<16, true, true, true, 0>,
+                                                         Vi2Shape<16>::kThreads, smem);
+}
+
+}  // namespace cme

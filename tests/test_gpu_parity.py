@@ -149,18 +149,26 @@ def test_value_index_bit_identical_to_layout_v0(cme, oracle_mod, monkeypatch):
     states, r, c, v = oracle_mod.enumerate_network(W.toggle_switch(90))
     x = W.random_start(len(states), 8)
     out = {}
-    for enc, env in (("v0", {"CME_COMPACT": "0"}), ("vi", {"CME_COMPACT": "1", "CME_VI": "1"}),
-                     ("vi31", {"CME_TMA_WARPS": "31"})):   # one 1024-thread CTA per SM, 31-slice tiles
+    for enc, env in (("v0", {"CME_COMPACT": "0"}), ("vi", {"CME_COMPACT": "1", "CME_VI": "1", "CME_VI2": "0"}),
+                     ("vi31", {"CME_TMA_WARPS": "31"}),   # one 1024-thread CTA per SM, 31-slice tiles
+                     ("vi2", {"CME_TMA_WARPS": "16", "CME_VI2": "1", "CME_VI2_WARPS": "16"}),   # tile records
+                     ("vi2w23", {"CME_VI2_WARPS": "23"}), ("vi2w30", {"CME_VI2_WARPS": "30"}),
+                     ("vi2words", {"CME_VI2_WORDS": "1"})):
         for k, val in env.items():
             monkeypatch.setenv(k, val)
         m = cme.Matrix(len(states), r, c, v).reorder(cme.CME_ORDER_RCM).pack()
         m.set_opts(omega=0.9, check_every=50, stag_tol=0.0)
         p, st, it = m.solve(tol=0.0, max_iter=300)
-        out[enc] = (m.spmv(x), p, m.info().compact, m.info().tma_warps)
-    assert out["v0"][2] == 0 and out["vi"][2] == 2 and out["vi31"][2:] == (2, 31)
-    for enc in ("vi", "vi31"):
-        assert out["v0"][0].tobytes() == out[enc][0].tobytes()
+        f = m.info()
+        out[enc] = (m.spmv(x), p, f.compact, f.tma_warps, f.records)
+    assert out["v0"][2] == 0 and out["vi"][2:] == (2, 16, 0) and out["vi31"][2:] == (2, 31, 0)
+    assert out["vi2"][2:] == (2, 16, 1) and out["vi2w23"][2:] == (2, 23, 1) and out["vi2w30"][2:] == (2, 30, 1)
+    assert out["vi2words"][2:] == (2, 30, 1)
+    for enc in ("vi", "vi31", "vi2", "vi2w23", "vi2w30", "vi2words"):
+        assert out["v0"][0].tobytes() == out[enc][0].tobytes(), enc
     assert out["v0"][1].tobytes() == out["vi"][1].tobytes()
+    for enc in ("vi2", "vi2w23", "vi2w30", "vi2words"):   # (other grids group the check partials differently)
+        assert np.abs(out["v0"][1] - out[enc][1]).sum() <= 1e-14, enc
     # 31-slice tiles group the check partials (sum y, sum |y - x|) differently,
     # so the normalising sum can differ in its last bit: same landscape to rounding
     assert np.abs(out["v0"][1] - out["vi31"][1]).sum() <= 1e-14
@@ -596,4 +604,30 @@ def test_ablation_arms_on_gpu(cme, oracle_mod, monkeypatch, arm, kw, net, tma):
     if it != ref.iters:
         ref = oracle_mod.jacobi_solve(A, omega=omega, tol=0.0, check_every=40, max_iter=it, stag_tol=0.0)
     assert np.abs(p - ref.p).sum() <= 1e-10
+    m.close()
+
+
+@pytest.mark.parametrize("words", ["0", "1"])
+@pytest.mark.parametrize("warps,stages,grid", [(16, 2, 3), (23, 2, 5), (30, 3, 2), (23, 4, 7)])
+@pytest.mark.parametrize("net,order,omega", [(W.toggle_switch(120), "rcm", 0.9), (W.toggle_switch(90), "dfs", 0.9)],
+                         ids=lambda x: getattr(x, "name", str(x)))
+def test_vi2_ring_wraps(cme, oracle_mod, monkeypatch, warps, stages, grid, net, order, omega, words):
+    """Tile-record kernel (sell_vi2_kernel) with its grid capped to a few CTAs,
+    so every CTA streams dozens of tiles through its 2-4 stage ring (the ring
+    reuse and mbarrier parity logic that a full grid never exercises on a
+    small matrix): SpMV and a fixed-iteration landscape vs the oracle."""
+    for k, v_ in {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI2_WARPS": str(warps), "CME_VI2_STAGES": str(stages),
+                  "CME_VI2_GRID": str(grid), "CME_VI2_WORDS": words}.items():
+        monkeypatch.setenv(k, v_)
+    states, r, c, v = oracle_mod.enumerate_network(net)
+    A = oracle_mod.ingest(len(states), r, c, v)
+    m = cme.Matrix(A.n, r, c, v).reorder(ORD[order]).pack()
+    f = m.info()
+    assert f.records == 1 and f.tma_warps == warps and f.grid == grid
+    m.set_opts(omega=omega, check_every=30, stag_tol=0.0)
+    x = W.random_start(A.n, 12)
+    assert_spmv_close(m.spmv(x), oracle_mod.jacobi_step(A, x, omega))
+    p, st, it = m.solve(tol=0.0, max_iter=90)
+    ref = oracle_mod.jacobi_solve(A, omega=omega, tol=0.0, check_every=30, max_iter=90, stag_tol=0.0)
+    assert it == ref.iters == 90 and np.abs(p - ref.p).sum() <= 1e-12
     m.close()
