@@ -54,8 +54,11 @@ DEFAULTS = {
 }
 
 
+_T0 = time.time()
+
+
 def log(*a):
-    print(*a, file=sys.stderr, flush=True)
+    print(f"[{time.time() - _T0:7.1f}s]", *a, file=sys.stderr, flush=True)
 
 
 def measured_peaks():
@@ -288,9 +291,10 @@ def solve_paper_mode(cme, m, name, omega, eps=1e-8):
     iterations, from uniform p0 -- the Table IV convention."""
     m.set_opts(omega=omega, check_every=C_BLOCK, stop=cme.CME_STOP_PAPER_RESID)
     t = time.perf_counter()
-    p, st, it = m.solve(tol=eps, max_iter=2_000_000)
+    p, st, it = m.solve(tol=eps, max_iter=200_000)
     wall = time.perf_counter() - t
     rep = m.report()
+    log(f"[bench] paper mode {name}: {st} after {it} iterations, {wall:.1f}s")
     m.set_opts(omega=omega, check_every=C_BLOCK, stop=cme.CME_STOP_DELTA_L1)
     return {"workload": name, "stop": "paper residual ||Ap||_inf/(||A||_inf ||p||_inf) (P:L117)", "eps": eps,
             "check_every": C_BLOCK, "omega": omega, "status": st, "iters": it, "resid": rep.resid,
@@ -309,6 +313,7 @@ def converge_closed_form(cme, name="cfg3a_schnakenberg_2m", tol=1e-12):
     t = time.perf_counter()
     p, st, it = m.solve(tol=tol, max_iter=2_000_000)
     wall = time.perf_counter() - t
+    log(f"[bench] {name}: {st} after {it} iterations, {wall:.1f}s")
     rep = m.report()
     info = m.info()
     meta = W.config_network(name).meta
@@ -400,7 +405,9 @@ def main():
 
     name = args.config
     B = args.batch
+    log("[bench] building", args.config)
     m, cfg, setup = build_matrix(cme, name, cme.CME_DEVICE_HOST_ONLY if dist_path else local, B)
+    log("[bench] built", setup)
     if comm is not None:
         cme.cme_matrix_distribute(m.h, comm)
         if args.transport == "p2p":
@@ -458,6 +465,7 @@ def main():
            "(25 B per row)"}[info.compact]
     traffic, traffic_src = ncu_traffic(name, kernel_name(info)) if world == 1 else (None, None)
 
+    log(f"[bench] timed region: {ms / args.steps:.3f} ms/step")
     # e2e: the public solve call with pinned host buffers, H2D + D2H inside the timed region
     p0 = torch.empty(n * B, dtype=torch.float64, pin_memory=True)
     p0.copy_(torch.from_numpy(np.tile(W.uniform_start(n), B)))
@@ -482,7 +490,9 @@ def main():
     conv_main = None
     if B == 1 and not args.no_converge:
         t = time.perf_counter()
+        log("[bench] e2e done; converging", name)
         p_c, st_c, it_c = m.solve(tol=1e-12, max_iter=200000)
+        log("[bench] converged", st_c, it_c, "; paper mode")
         wall_c = time.perf_counter() - t
         rep_c = m.report()
         dev_s = rep_c.seconds
@@ -504,18 +514,22 @@ def main():
     conv = None
     if rank == 0 and world == 1 and B == 1 and not args.no_converge:
         try:
+            log("[bench] converge_line cfg2")
             conv = converge_line(cme)
         except Exception as ex:  # report, do not hide
             conv = {"error": repr(ex)}
     conv3 = None
     if rank == 0 and world == 1 and B == 1 and not args.no_converge:
         try:
+            log("[bench] converge_closed_form cfg3a")
             conv3 = converge_closed_form(cme)
         except Exception as ex:  # report, do not hide
             conv3 = {"error": repr(ex)}
     cpu = None
     if rank == 0 and world == 1 and B == 1 and not args.no_cpu_baseline:
+        log("[bench] cpu baseline")
         cb = cpu_oracle_timing(name, budget_s=20.0, omega=cfg["omega"])
+        log("[bench] cpu baseline done")
         cpu = {k: cb[k] for k in ("value", "unit", "cores", "kind", "sample", "cpu_model", "value_1thread")}
 
     if rank == 0:

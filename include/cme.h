@@ -211,6 +211,10 @@ typedef struct cme_info {
                                      bytes_fmt/packed_bytes count it */
     int32_t records;              /* 1: the value-indexed encoding is streamed as one
                                      contiguous record per tile (sell_vi2_kernel, sec. 5d) */
+    int32_t wf_steps;             /* s > 1: check blocks run as wavefront passes of s steps
+                                     (sell_wf_kernel, sec. 5e; the records re-read from L2);
+                                     0: one launch per step */
+    int32_t wf_lag;               /* wavefront lag L in tiles (0 when wf_steps = 0)     */
 } cme_info;
 cme_status cme_get_info(cme_matrix h, cme_info* info);
 

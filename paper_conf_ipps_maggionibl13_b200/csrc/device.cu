@@ -21,7 +21,7 @@
 #include "cme_internal.h"
 #include "comm.h"
 #include "launch.h"
-#include "kernels_vi2.cuh"
+#include "kernels_wf.cuh"
 #include "kernels_resident.cuh"
 #include "kernels_cpt.cuh"
 
@@ -126,10 +126,21 @@ struct Device {
     // record per tile; replaces sell_vi_kernel when vi2 (CME_VI2 = 0 keeps it)
     bool vi2 = false;
     bool vi2_words = false;          // records hold packed vidx | col16 << 16 words (CME_VI2_WORDS)
+    bool vi2_f64 = false;            // records of the f64 compact encoding (no value index; CME_REC)
     int vi2_ncw = 0, vi2_stages = 0, vi2_stage_bytes = 0, vi2_grid = 0, vi2_occ = 0;
     int64_t vi2_tiles = 0;
     unsigned char* vi2_rec = nullptr;
     int64_t* vi2_rec_off = nullptr;
+    // wavefront s-step kernel over the tile records (kernels_wf.cuh): one
+    // launch per s steps of a check block (single GPU, vi2 shapes)
+    bool wf = false;
+    int wf_s = 0;                    // steps per pass (CME_WF; 0/1 = off)
+    int wf_lag = 0;                  // L: tiles between step j-1 and step j of a wave
+    int wf_keep = 1;                 // records of non-final steps evict_normal in L2 (CME_WF_KEEP)
+    uint32_t* wf_items = nullptr;    // [s * tiles] (j << 24) | t in wave order
+    int2* wf_dep = nullptr;          // [tiles] dependency tile range
+    uint32_t* wf_cnt = nullptr;      // [tiles] completion counters
+    uint32_t* wf_sync = nullptr;     // [2] passes done, CTAs finished
     // SMEM-resident persistent kernel (kernels_resident.cuh)
     bool use_res = false;
     int res_grid = 0, res_smem = 0, res_rps = 1;
@@ -540,20 +551,20 @@ static cme_status configure_tma(Device& d, const Packed& P) {
 // (kernels_vi2.cuh): per tile one contiguous block
 // [meta | row8 | loi, upi | inv_d | per slice: vidx[32 W], col16[32 W]],
 // every block 16-B aligned; a pure re-layout of sec. 5c's arrays.
-static int64_t vi2_record_bytes(const Packed& P, int ts, bool band, bool rearr, int64_t t) {
+static int64_t vi2_record_bytes(const Packed& P, int ts, bool band, bool rearr, int64_t t, bool f64 = false) {
     const int64_t q0 = t * ts, q1 = std::min<int64_t>(q0 + ts, P.n_slices);
-    return vi2_fixed_bytes(ts, band, rearr) + 4 * (P.slice_off[q1] - P.slice_off[q0]);
+    return vi2_fixed_bytes(ts, band, rearr, f64) + (f64 ? 10 : 4) * (P.slice_off[q1] - P.slice_off[q0]);
 }
 
 static void vi2_build_records(const Packed& P, const Compact& C, int ts, bool band, bool rearr, bool words,
-                              std::vector<unsigned char>& rec, std::vector<int64_t>& off) {
+                              std::vector<unsigned char>& rec, std::vector<int64_t>& off, bool f64 = false) {
     const int64_t nt = (P.n_slices + ts - 1) / ts;
     off.assign(nt + 1, 0);
-    for (int64_t t = 0; t < nt; ++t) off[t + 1] = off[t] + vi2_record_bytes(P, ts, band, rearr, t);
+    for (int64_t t = 0; t < nt; ++t) off[t + 1] = off[t] + vi2_record_bytes(P, ts, band, rearr, t, f64);
     rec.assign((size_t)off[nt], 0);
     const int kMeta = ((ts + 1) & ~1) * 8;
-    const int kRow = kMeta, kLoUp = kRow + (rearr ? ts * 32 : 0), kInv = kLoUp + (band ? ts * 128 : 0),
-              kEnt = kInv + ts * 256;
+    const int kRow = kMeta, kLoUp = kRow + (rearr ? ts * 32 : 0), kInv = kLoUp + (band ? ts * (f64 ? 512 : 128) : 0),
+              kEnt = kInv + (f64 ? 0 : ts * 256);
 #pragma omp parallel for schedule(static)
     for (int64_t t = 0; t < nt; ++t) {
         unsigned char* R = rec.data() + off[t];
@@ -564,6 +575,17 @@ static void vi2_build_records(const Packed& P, const Compact& C, int ts, bool ba
             std::memcpy(R + 8 * (q - q0), m, 8);
             const int64_t sl0 = q * 32, ls0 = (q - q0) * 32;
             if (rearr) std::memcpy(R + kRow + ls0, C.row8.data() + sl0, 32);
+            if (f64) {   // [lo_c, up_c (band)] | per slice: val_c[32 W] then col16[32 W]
+                if (band) {
+                    std::memcpy(R + kLoUp + 8 * ls0, C.lo.data() + sl0, 256);
+                    std::memcpy(R + kLoUp + ts * 256 + 8 * ls0, C.up.data() + sl0, 256);
+                }
+                const int64_t ne = P.slice_off[q + 1] - P.slice_off[q];
+                unsigned char* E = R + kEnt + 10 * (P.slice_off[q] - e0);
+                std::memcpy(E, C.val.data() + P.slice_off[q], 8 * ne);
+                std::memcpy(E + 8 * ne, C.col16.data() + P.slice_off[q], 2 * ne);
+                continue;
+            }
             if (band) {
                 std::memcpy(R + kLoUp + 2 * ls0, C.loi.data() + sl0, 64);
                 std::memcpy(R + kLoUp + ts * 64 + 2 * ls0, C.upi.data() + sl0, 64);
@@ -591,8 +613,9 @@ static void vi2_build_records(const Packed& P, const Compact& C, int ts, bool ba
 // CTAs per SM (56 registers, 3 stages: 175 us); 23 warps in 2 CTAs per SM (40
 // registers: spills, 2 stages: 227 us) only when forced.  Deepest ring <= 4
 // stages.  CME_VI2_WARPS / CME_VI2_STAGES force a shape.
-static cme_status configure_vi2(Device& d, const Packed& P) {
+static cme_status configure_vi2(Device& d, const Packed& P, bool f64 = false) {
     d.vi2 = false;
+    d.vi2_f64 = false;
     int dev = 0, smem_max = 0, sms = 0;
     CUDA_TRY(cudaGetDevice(&dev));
     CUDA_TRY(cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
@@ -605,7 +628,7 @@ static cme_status configure_vi2(Device& d, const Packed& P) {
         if (!force_w && ncw == 23) continue;
         const int64_t nt = (P.n_slices + ncw - 1) / ncw;
         int64_t mx = 0;
-        for (int64_t t = 0; t < nt; ++t) mx = std::max(mx, vi2_record_bytes(P, ncw, d.band, d.rearr, t));
+        for (int64_t t = 0; t < nt; ++t) mx = std::max(mx, vi2_record_bytes(P, ncw, d.band, d.rearr, t, f64));
         const int64_t stage = (mx + 127) / 128 * 128;
         CUDA_TRY(vi2_prepare(ncw, cap));
         const int want_occ = ncw == 30 ? 1 : 2;
@@ -614,7 +637,7 @@ static cme_status configure_vi2(Device& d, const Packed& P) {
             const int64_t bytes = d.dict_bytes + st * stage;
             if (bytes > cap) continue;
             int o = 0;
-            CUDA_TRY(vi2_occupancy(ncw, (int)bytes, &o));
+            CUDA_TRY(vi2_occupancy(ncw, (int)bytes, &o, f64 ? 2 : 0));
             if (o >= want_occ || (force_s > 0 && o >= 1)) { stages = st; occ = o; break; }
         }
         if (env_int("CME_VERBOSE", 0) > 1)
@@ -626,7 +649,8 @@ static cme_status configure_vi2(Device& d, const Packed& P) {
     if (!best.ncw) return CME_OK;
     if (env_int("CME_VI2", 1) == 0) return CME_OK;
     d.vi2 = true;
-    d.vi2_words = env_int("CME_VI2_WORDS", 0) != 0;
+    d.vi2_words = !f64 && env_int("CME_VI2_WORDS", 0) != 0;
+    d.vi2_f64 = f64;
     d.vi2_ncw = best.ncw;
     d.vi2_stages = best.stages;
     d.vi2_stage_bytes = (int)best.stage;
@@ -640,6 +664,59 @@ static cme_status configure_vi2(Device& d, const Packed& P) {
                      d.vi2_ncw, d.vi2_stages, d.vi2_stage_bytes, d.vi2_occ, d.vi2_grid, (long long)d.vi2_tiles,
                      d.dict_bytes);
     return CME_OK;
+}
+
+// Wavefront plan (kernels_wf.cuh): per tile of ncw slices, the union of the
+// tiles holding the rows it gathers (RAW) and the tiles gathering its rows
+// (WAR), as one [first, last] range; then the (step, tile) items in wave
+// order with lag L = max |dep - t| + 1 + extra (extra: tiles the G CTAs keep
+// in flight, so a dependency is normally complete when it is polled).
+static int wf_plan(const Packed& P, int ncw, bool band, int s, int extra, std::vector<int2>& dep,
+                   std::vector<uint32_t>& items) {
+    const int64_t n = P.n, ts = (int64_t)ncw * 32;
+    const int64_t T = (P.n_slices + ncw - 1) / ncw;
+    std::vector<int32_t> tile_of(n);
+    for (int64_t slot = 0; slot < std::min(P.n_slots, n); ++slot) tile_of[P.row_of[slot]] = (int32_t)(slot / ts);
+    dep.assign(T, make_int2(INT32_MAX, -1));
+    std::vector<int2> war(T, make_int2(INT32_MAX, -1));
+    for (int64_t u = 0; u < T; ++u) {
+        int2 raw = make_int2(INT32_MAX, -1);
+        auto see = [&](int64_t col) {
+            if (col < 0 || col >= n) return;   // zero sentinels
+            const int32_t t = tile_of[col];
+            raw.x = std::min(raw.x, t);
+            raw.y = std::max(raw.y, t);
+            war[t].x = std::min(war[t].x, (int32_t)u);
+            war[t].y = std::max(war[t].y, (int32_t)u);
+        };
+        for (int64_t q = u * ncw; q < std::min((u + 1) * ncw, P.n_slices); ++q)
+            for (int lane = 0; lane < 32; ++lane) {
+                const int64_t slot = q * 32 + lane;
+                if (slot >= n) continue;
+                const int64_t r = P.row_of[slot];
+                see(r);
+                if (band) { see(r - 1); see(r + 1); }
+                for (int w = 0; w < P.slice_w[q]; ++w) see(P.col[P.slice_off[q] + lane + 32 * w]);
+            }
+        dep[u] = raw;
+    }
+    int dd = 0;
+    for (int64_t t = 0; t < T; ++t) {
+        int2& d = dep[t];
+        d.x = std::min(d.x, war[t].x);
+        d.y = std::max(d.y, war[t].y);
+        if (d.y < 0) d = make_int2((int)t, (int)t);
+        dd = std::max(dd, (int)std::max(d.y - t, t - d.x));
+    }
+    const int L = dd + 1 + std::max(extra, 0);
+    items.clear();
+    items.reserve((size_t)s * T);
+    for (int64_t w = 0; w < T + (int64_t)(s - 1) * L; ++w)
+        for (int j = 0; j < s; ++j) {
+            const int64_t t = w - (int64_t)j * L;
+            if (t >= 0 && t < T) items.push_back(((uint32_t)j << 24) | (uint32_t)t);
+        }
+    return L;
 }
 
 // Plan the SMEM-resident kernel (kernels_resident.cuh): one CTA per SM, each
@@ -879,6 +956,9 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
         }
         // the value-indexed encoding as tile records (sec. 5d)
         if (d->use_tma && d->vi && (s = configure_vi2(*d, P)) != CME_OK) return fail(s);
+        // the f64 compact encoding as tile records too (CME_REC = 0 keeps sell_cpt_kernel)
+        if (d->use_tma && d->cpt && !d->vi && env_int("CME_REC", 1) != 0 && (s = configure_vi2(*d, P, true)) != CME_OK)
+            return fail(s);
     }
     if (d->B > 1 && d->format == CME_FMT_DIAG_SELL && env_int("CME_COMPACT", 1) != 0 && env_int("CME_VI", -1) != 0 &&
         env_int("CME_TMA", -1) != 0 && encode_compact(P, d->own_off, h->Cpt) && encode_value_index(P, h->Cpt)) {
@@ -907,14 +987,44 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
     }
     if (d->format != CME_FMT_CSR) {
         if (d->vi2) {   // tile records + the dictionary; no separate index arrays
-            std::vector<double> dict(h->Cpt.dict);
-            dict.resize(d->dict_bytes / 8, 0.0);   // staged in shared memory, 128-B padded
-            UP(dict, dict);
+            if (!d->vi2_f64) {
+                std::vector<double> dict(h->Cpt.dict);
+                dict.resize(d->dict_bytes / 8, 0.0);   // staged in shared memory, 128-B padded
+                UP(dict, dict);
+            }
             std::vector<unsigned char> rec;
             std::vector<int64_t> roff;
-            vi2_build_records(P, h->Cpt, d->vi2_ncw, d->band, d->rearr, d->vi2_words, rec, roff);
+            vi2_build_records(P, h->Cpt, d->vi2_ncw, d->band, d->rearr, d->vi2_words, rec, roff, d->vi2_f64);
             UP(vi2_rec, rec);
             UP(vi2_rec_off, roff);
+            // wavefront s-step passes (CME_WF = s; single GPU, same grid as
+            // the vi2 kernel so the check partials keep their layout)
+            const int wf_s = env_int("CME_WF", 0);
+            if (wf_s >= 2 && wf_s <= 8 && !comm && h->nranks == 1 && (d->vi2_ncw == 30 || d->vi2_ncw == 16) &&
+                !d->vi2_words && !d->vi2_f64 && d->vi2_tiles < (1 << 24)) {
+                const int smem = d->dict_bytes + d->vi2_stages * d->vi2_stage_bytes;
+                int occ = 0;
+                if (wf_prepare(d->vi2_ncw, smem) == cudaSuccess &&
+                    wf_occupancy(d->vi2_ncw, smem, &occ) == cudaSuccess && occ >= d->vi2_occ) {
+                    std::vector<int2> dep;
+                    std::vector<uint32_t> items;
+                    const int extra = env_int("CME_WF_LAG", (d->vi2_stages + 2) * d->vi2_grid / wf_s);
+                    d->wf_lag = wf_plan(P, d->vi2_ncw, d->band, wf_s, extra, dep, items);
+                    UP(wf_dep, dep);
+                    UP(wf_items, items);
+                    if ((s = d->alloc(d->wf_cnt, (size_t)d->vi2_tiles)) != CME_OK) return fail(s);
+                    if ((s = d->alloc(d->wf_sync, 2)) != CME_OK) return fail(s);
+                    if (cudaMemset(d->wf_cnt, 0, d->vi2_tiles * 4) != cudaSuccess ||
+                        cudaMemset(d->wf_sync, 0, 8) != cudaSuccess)
+                        return fail(CME_ERR_CUDA);
+                    d->wf = true;
+                    d->wf_s = wf_s;
+                    d->wf_keep = env_int("CME_WF_KEEP", 1);
+                    if (env_int("CME_VERBOSE", 0))
+                        std::fprintf(stderr, "[cme] wavefront: s=%d lag=%d tiles=%lld items=%zu\n", wf_s, d->wf_lag,
+                                     (long long)d->vi2_tiles, items.size());
+                }
+            }
         } else if (d->vi) {
             std::vector<double> dict(h->Cpt.dict);
             if (d->B == 1) dict.resize(d->dict_bytes / 8, 0.0);   // (B = 1: staged in shared memory, 128-B padded)
@@ -1246,7 +1356,7 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
         Vi2Args V{a, d.vi2_rec, d.vi2_rec_off, d.dict, d.vi2_tiles, d.vi2_stages, d.vi2_stage_bytes, d.dict_bytes,
                   d.win_shift, d.tma_xpf};
         CUDA_TRY(launch_vi2(V, d.vi2_ncw, d.vi2_grid, d.dict_bytes + d.vi2_stages * d.vi2_stage_bytes, d.band, d.rearr,
-                            check, d.vi2_words, pdl, s));
+                            check, d.vi2_f64 ? 2 : d.vi2_words ? 1 : 0, pdl, s));
     } else if (d.use_tma && d.vi && d.B > 1) {
         ViArgs V{CptArgs{TmaArgs{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col,
                                  d.tma_contig, d.tma_xpf},
@@ -1341,6 +1451,30 @@ static cme_status launch_res(Device& d, cudaStream_t s, int start, int64_t nstep
     return CME_OK;
 }
 
+// s = d.wf_s consecutive steps from buffer src in one wavefront launch; the
+// result lands in buffer (src + s) & 1 like s single steps.
+static cme_status launch_wf_pass(Device& d, cudaStream_t s, int src, bool check, const double* pre, double omega) {
+    StepArgs a{};
+    a.n_rows = d.n_own;
+    a.slice_begin = 0;
+    a.slice_end = d.n_slices;
+    a.x = d.xb[src];
+    a.y = d.xb[1 - src];
+    a.own_off = d.own_off;
+    a.omega = omega;
+    a.pre_scale = pre;
+    a.partials = d.partials;
+    a.stop = &d.ctrl->stop;
+    WfArgs A{Vi2Args{a, d.vi2_rec, d.vi2_rec_off, d.dict, d.vi2_tiles, d.vi2_stages, d.vi2_stage_bytes, d.dict_bytes,
+                     d.win_shift, d.tma_xpf},
+             d.wf_items, d.wf_dep, d.wf_cnt, d.wf_sync, d.ctrl, d.wf_s, d.wf_keep,
+             (int64_t)std::max(1, env_int("CME_RES_TIMEOUT_MS", 2000)) * 1000000};
+    const bool pdl = env_int("CME_PDL", 1) != 0;
+    CUDA_TRY(launch_wf(A, d.vi2_ncw, d.vi2_grid, d.dict_bytes + d.vi2_stages * d.vi2_stage_bytes, d.band, d.rearr,
+                       check, pdl, s));
+    return CME_OK;
+}
+
 // reduce partials of the last CHECK step and decide
 static cme_status launch_finalize(Device& d, cudaStream_t s, int32_t len, int32_t final_partial) {
     const bool pdl = (!d.comm || d.p2p) && env_int("CME_PDL", 1) != 0;
@@ -1355,7 +1489,12 @@ static cme_status launch_finalize(Device& d, cudaStream_t s, int32_t len, int32_
 // One check block of C steps starting from buffer `start`: steps 0..C-2 plain,
 // step C-1 CHECK; the first step applies the pending 1/||y_b||_1 (R5).
 static cme_status enqueue_block(Device& d, cudaStream_t s, int start, int64_t C, double omega, bool final_partial) {
-    for (int64_t t = 0; t < C; ++t) {
+    int64_t t0 = 0;
+    if (d.wf)   // wavefront passes of s steps, single steps for the remainder
+        for (; t0 + d.wf_s <= C; t0 += d.wf_s)
+            CME_TRY(launch_wf_pass(d, s, (int)((start + t0) & 1), t0 + d.wf_s == C, t0 == 0 ? d.ctrl->inv_s : nullptr,
+                                   omega));
+    for (int64_t t = t0; t < C; ++t) {
         const int src = (int)((start + t) & 1);
         CME_TRY(launch_step(d, s, src, 1 - src, t == C - 1, t == 0 ? d.ctrl->inv_s : nullptr, omega));
     }
@@ -1439,6 +1578,10 @@ static cme_status load_iterate(cme_matrix_s* h, const double* p0, bool normalise
     double* x = d.xb[0] + d.own_off * B;
     const Ctrl c = fresh_ctrl(h, d);
     CUDA_TRY(cudaMemcpyAsync(d.ctrl, &c, sizeof(Ctrl), cudaMemcpyHostToDevice, s));
+    if (d.wf) {   // wavefront completion counters restart with the solve
+        CUDA_TRY(cudaMemsetAsync(d.wf_cnt, 0, (size_t)d.vi2_tiles * 4, s));
+        CUDA_TRY(cudaMemsetAsync(d.wf_sync, 0, 8, s));
+    }
     if (!p0) {
         fill_kernel<<<grid_for(d.n_own * B), kCta, 0, s>>>(x, d.n_own * B, 1.0 / (double)d.n_global);
         CUDA_TRY(cudaGetLastError());
@@ -1536,6 +1679,7 @@ static cme_status solve_epilogue(cme_matrix_s* h, cudaStream_t s, double omega, 
     cudaEventElapsedTime(&ms, d.t0, d.t1);
     if (f.status == CME_ERR_TIMEOUT) {
         set_error(d.use_res ? "resident kernel: a dependency wait timed out (CME_RES_TIMEOUT_MS)"
+                  : d.wf    ? "wavefront kernel: a tile dependency wait timed out (CME_RES_TIMEOUT_MS)"
                             : "peer-memory transport: a peer rank never reached the flag barrier");
         if (iters_out) *iters_out = f.iter;
         return CME_ERR_TIMEOUT;
@@ -1675,6 +1819,8 @@ void device_describe(const Device* d, cme_info* f) {
     f->tma_warps = d->vi2 ? d->vi2_ncw : d->use_tma ? d->tma_ncw : 0;
     f->tma_stages = d->vi2 ? d->vi2_stages : d->use_tma ? d->tma_stages : 0;
     f->records = d->vi2 ? 1 : 0;
+    f->wf_steps = d->wf ? d->wf_s : 0;
+    f->wf_lag = d->wf ? d->wf_lag : 0;
     f->grid = d->use_res ? d->res_grid : d->step_grid();
     f->compact = d->vi ? 2 : d->cpt ? 1 : 0;
     if (d->vi) {   // value-indexed: 4 B per ELL slot (shared by a batch), inv_d per row and member

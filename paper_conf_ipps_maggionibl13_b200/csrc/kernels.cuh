@@ -173,6 +173,7 @@ __device__ __forceinline__ void cta_check_partials(const CheckAcc<B>& c, double*
         const double sy = warp_sum(c.sy[b]), sx = warp_sum(c.sx[b]), sd = warp_sum(c.sd[b]);
         const double md = warp_max(c.md[b]), mx = warp_max(c.mx[b]);
         if (lane == 0) { red[w][0] = sy; red[w][1] = sx; red[w][2] = sd; red[w][3] = md; red[w][4] = mx; }
+        __syncwarp();      // converged warps at the aligned CTA barrier (compute-sanitizer synccheck)
         __syncthreads();
         if (threadIdx.x == 0) {
             double a = 0, bb = 0, cc = 0, d = 0, e = 0;
@@ -183,6 +184,7 @@ __device__ __forceinline__ void cta_check_partials(const CheckAcc<B>& c, double*
             double* o = partials + ((size_t)blockIdx.x * B + b) * kPartials;
             o[0] = a; o[1] = bb; o[2] = cc; o[3] = d; o[4] = e; o[5] = 0; o[6] = 0; o[7] = 0;
         }
+        __syncwarp();
         __syncthreads();
     }
 }

@@ -39,16 +39,21 @@ struct Vi2Args {
 };
 
 // Record layout of a tile of TS slices (byte offsets; every block 16-B aligned).
-template <int TS, bool BAND, bool REARR>
+// F64 (ENC = 2, the compact encoding of sec. 5b, no value index): lo/up are
+// M's band values (double), no inv_d block (only CHECK/transient steps read
+// inv_d, from global memory), and a slice's entries are val_c[32 W] (double)
+// then col16[32 W].
+template <int TS, bool BAND, bool REARR, bool F64 = false>
 struct Vi2Rec {
     static constexpr int kMeta = ((TS + 1) & ~1) * 8;              // int2 {entry offset, width} per slice
     static constexpr int kRow = kMeta;                            // uint8 per slot (REARR)
-    static constexpr int kLoUp = kRow + (REARR ? TS * 32 : 0);    // uint16 loi[slots], upi[slots] (BAND)
-    static constexpr int kInv = kLoUp + (BAND ? TS * 128 : 0);    // double per slot
-    static constexpr int kEnt = kInv + TS * 256;                  // per slice: vidx[32 W] then col16[32 W]
+    static constexpr int kLoUp = kRow + (REARR ? TS * 32 : 0);    // uint16 loi, upi (F64: double lo, up) per slot (BAND)
+    static constexpr int kInv = kLoUp + (BAND ? TS * (F64 ? 512 : 128) : 0);   // double per slot (not F64)
+    static constexpr int kEnt = kInv + (F64 ? 0 : TS * 256);      // per slice: vidx (F64: val_c) [32 W] then col16[32 W]
+    static constexpr int kEntBytes = F64 ? 10 : 4;                // bytes per entry
 };
-__host__ __device__ constexpr int vi2_fixed_bytes(int ts, bool band, bool rearr) {
-    return ((ts + 1) & ~1) * 8 + (rearr ? ts * 32 : 0) + (band ? ts * 128 : 0) + ts * 256;
+__host__ __device__ constexpr int vi2_fixed_bytes(int ts, bool band, bool rearr, bool f64 = false) {
+    return ((ts + 1) & ~1) * 8 + (rearr ? ts * 32 : 0) + (band ? ts * (f64 ? 512 : 128) : 0) + (f64 ? 0 : ts * 256);
 }
 
 __device__ __forceinline__ uint32_t lds_u16(uint32_t a) {
@@ -158,6 +163,32 @@ __device__ __forceinline__ double vi2_row_w_wide(uint32_t pw, uint32_t sdict, co
     return acc;
 }
 
+// F64 records (ENC = 2): entry u of a lane has its value at pv + 256 u and
+// its col16 at pc + 64 u; FMAs in t order (sell_cpt_kernel's arithmetic).
+template <int W>
+__device__ __forceinline__ double vi2_row_f(uint32_t pv, uint32_t pc, const double* xr) {
+    double xv[W];
+#pragma unroll
+    for (int u = 0; u < W; ++u) xv[u] = __ldg(xr + lds_s16(pc + 64 * u));
+    double acc = 0.0;
+#pragma unroll
+    for (int u = 0; u < W; ++u) acc = fma(lds_f64(pv + 256 * u), xv[u], acc);
+    return acc;
+}
+__device__ __forceinline__ double vi2_row_f_wide(uint32_t pv, uint32_t pc, const double* xr, int w) {
+    double acc = 0.0;
+    for (int t0 = 0; t0 < w; t0 += 8) {
+        double xv[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u)
+            if (t0 + u < w) xv[u] = __ldg(xr + lds_s16(pc + 64 * (t0 + u)));
+#pragma unroll
+        for (int u = 0; u < 8; ++u)
+            if (t0 + u < w) acc = fma(lds_f64(pv + 256 * (t0 + u)), xv[u], acc);
+    }
+    return acc;
+}
+
 template <int NCW>
 struct Vi2Shape {
     static constexpr int kThreads = 32 * (NCW + 1);
@@ -168,7 +199,8 @@ struct Vi2Shape {
 template <int NCW, bool BAND, bool REARR, bool CHECK, int ENC>
 __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBlocks)
     sell_vi2_kernel(const Vi2Args V) {
-    using R = Vi2Rec<NCW, BAND, REARR>;
+    constexpr bool F64 = ENC == 2;
+    using R = Vi2Rec<NCW, BAND, REARR, F64>;
     const StepArgs& a = V.a;
     pdl_trigger();
     extern __shared__ __align__(128) unsigned char smem[];
@@ -194,11 +226,13 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
         // the record offsets of the CTA's next 32 tiles are loaded by the 32
         // lanes together (one round trip per 32 tiles), lane 0 issues
         const uint64_t pol = evict_first_policy();
-        if (lane == 0) {   // dictionary: constant, every CTA reads it (keep it in L2)
+        if (lane == 0 && V.dict_bytes > 0) {   // dictionary: constant, every CTA reads it (keep it in L2)
             uint64_t keep;
             asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(keep));
             mbar_expect_tx(&dbar, (uint32_t)V.dict_bytes);
             bulk_g2s(smem, V.dict, (uint32_t)V.dict_bytes, &dbar, keep);
+        } else if (lane == 0) {
+            mbar_arrive(&dbar);   // (F64 records: no dictionary)
         }
         int64_t o0 = 0, o1 = 0;
         int s = 0;
@@ -211,12 +245,15 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
                 if (i + lane < my_tiles) { o0 = __ldg(V.rec_off + t); o1 = __ldg(V.rec_off + t + 1); }
             }
             const int64_t b0 = __shfl_sync(0xffffffffu, o0, l), b1 = __shfl_sync(0xffffffffu, o1, l);
-            if (i >= S) mbar_wait(&empty[s], phase ^ 1u);
-            if (i == pro && !waited) {   // first tiles were issued before the previous step ended
+            // first tiles were issued before the previous step ended; the stop
+            // test comes before any ring reuse: on a stopped launch the
+            // consumers release no stage, so waiting on empty[] would hang
+            if (i == pro && !waited) {
                 pdl_wait();
                 waited = true;
                 if (a.stop != nullptr && *a.stop) break;
             }
+            if (i >= S) mbar_wait(&empty[s], phase ^ 1u);
             if (lane == 0) {
                 const int t = c + i * G;
                 const uint32_t bytes = (uint32_t)(b1 - b0);
@@ -269,10 +306,23 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
                 const int r = REARR ? ((slot >> V.win_shift) << V.win_shift) + (int)lds_u8(st + R::kRow + ls) : slot;
                 const double* xr = xo + r;
                 const double x_r = __ldg(xr);
-                const uint32_t pv = st + R::kEnt + 4 * meta.x + (ENC ? 4 : 2) * lane;   // entry 0 of this lane
-                const uint32_t pc = pv + 64 * meta.y;   // (ENC 0: the col16 block follows the vidx block)
+                const uint32_t pv = st + R::kEnt + R::kEntBytes * meta.x + (ENC == 1 ? 4 : ENC == 2 ? 8 : 2) * lane;
+                // (ENC 0: the col16 block follows the vidx block; ENC 2: it follows the val_c block)
+                const uint32_t pc = F64 ? st + R::kEnt + 10 * meta.x + 256 * meta.y + 2 * lane : pv + 64 * meta.y;
                 double acc = 0.0;
-                if (ENC) switch (meta.y) {   // warp-uniform exact widths
+                if (F64) switch (meta.y) {   // warp-uniform exact widths
+                    case 0: break;
+                    case 1: acc = vi2_row_f<1>(pv, pc, xr); break;
+                    case 2: acc = vi2_row_f<2>(pv, pc, xr); break;
+                    case 3: acc = vi2_row_f<3>(pv, pc, xr); break;
+                    case 4: acc = vi2_row_f<4>(pv, pc, xr); break;
+                    case 5: acc = vi2_row_f<5>(pv, pc, xr); break;
+                    case 6: acc = vi2_row_f<6>(pv, pc, xr); break;
+                    case 7: acc = vi2_row_f<7>(pv, pc, xr); break;
+                    case 8: acc = vi2_row_f<8>(pv, pc, xr); break;
+                    default: acc = vi2_row_f_wide(pv, pc, xr, meta.y);
+                }
+                else if (ENC) switch (meta.y) {   // warp-uniform exact widths
                     case 0: break;
                     case 1: acc = vi2_row_w<1>(pv, sdict, xr); break;
                     case 2: acc = vi2_row_w<2>(pv, sdict, xr); break;
@@ -299,14 +349,18 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
                 double sum = acc;
                 if (BAND) {
                     const double xl = __ldg(xr - 1), xu = __ldg(xr + 1);
-                    const double lo = lds_f64(sdict + 8 * lds_u16(st + R::kLoUp + 2 * ls));
-                    const double up = lds_f64(sdict + 8 * lds_u16(st + R::kLoUp + NCW * 64 + 2 * ls));
+                    const double lo = F64 ? lds_f64(st + R::kLoUp + 8 * ls)
+                                          : lds_f64(sdict + 8 * lds_u16(st + R::kLoUp + 2 * ls));
+                    const double up = F64 ? lds_f64(st + R::kLoUp + NCW * 256 + 8 * ls)
+                                          : lds_f64(sdict + 8 * lds_u16(st + R::kLoUp + NCW * 64 + 2 * ls));
                     sum = fma(lo, xl, up * xu) + acc;
                 }
-                const double id = lds_f64(st + R::kInv + 8 * ls);
-                double y = damp ? fma(1.0 - a.omega, x_r, a.omega * (id * sum)) : id * sum;
+                // F64: the rows are M's (sum = (M x)_r already); inv_d only for checks / transient
+                const double id = F64 ? ((CHECK || unif) ? __ldg(a.inv_d + slot) : 1.0) : lds_f64(st + R::kInv + 8 * ls);
+                double y = F64 ? (damp ? fma(1.0 - a.omega, x_r, a.omega * sum) : sum)
+                               : (damp ? fma(1.0 - a.omega, x_r, a.omega * (id * sum)) : id * sum);
                 if (unif) {   // transient: (I + A/Lambda) x with a_rr = -1/id
-                    y = fma(a.unif_lam_inv, sum - x_r / id, x_r);
+                    y = F64 ? fma(a.unif_lam_inv, (sum - x_r) / id, x_r) : fma(a.unif_lam_inv, sum - x_r / id, x_r);
                     double* ac = a.acc + a.own_off + r;
                     *ac = fma(a.acc_w, x_r, *ac);
                 }

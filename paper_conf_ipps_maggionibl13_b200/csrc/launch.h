@@ -62,14 +62,23 @@ cudaError_t launch_vib(const ViArgs& V, int B, int ncw, int grid, int smem, bool
 cudaError_t vib_prepare(int B, int ncw, int smem);
 cudaError_t vib_occupancy(int B, int ncw, int smem, int* blocks_per_sm);
 struct Vi2Args;
-// tile-record value-indexed TMA step kernel (step_vi2.cu, B = 1): ncw = 16, 23 or 30
-cudaError_t launch_vi2(const Vi2Args& V, int ncw, int grid, int smem, bool band, bool rearr, bool check, bool words,
+// tile-record TMA step kernel (step_vi2.cu, B = 1): ncw = 16, 23 or 30; enc 0 value
+// index, 1 value index as packed words, 2 f64 compact values (no dictionary)
+cudaError_t launch_vi2(const Vi2Args& V, int ncw, int grid, int smem, bool band, bool rearr, bool check, int enc,
                        bool pdl, cudaStream_t s);
 cudaError_t vi2_prepare(int ncw, int smem);
-cudaError_t vi2_occupancy(int ncw, int smem, int* blocks_per_sm);
+cudaError_t vi2_occupancy(int ncw, int smem, int* blocks_per_sm, int enc = 0);
 struct ResArgs;
 // SMEM-resident persistent Jacobi kernel (resident.cu)
 cudaError_t resident_prepare(int smem);
 cudaError_t resident_occupancy(int smem, int* blocks_per_sm);
 cudaError_t launch_resident(const ResArgs& a, int grid, int smem, bool band, bool rearr, int rps, cudaStream_t s);
+}  // namespace cme
+namespace cme {
+struct WfArgs;
+// wavefront s-step kernel over the tile records (step_wf.cu, B = 1, one GPU): ncw = 16 or 30
+cudaError_t launch_wf(const WfArgs& A, int ncw, int grid, int smem, bool band, bool rearr, bool check, bool pdl,
+                      cudaStream_t s);
+cudaError_t wf_prepare(int ncw, int smem);
+cudaError_t wf_occupancy(int ncw, int smem, int* blocks_per_sm);
 }  // namespace cme

@@ -5,26 +5,27 @@
 namespace cme {
 
 template <int W>
-static cudaError_t launch_vi2_w(const Vi2Args& V, int grid, int smem, bool band, bool rearr, bool check, bool words,
+static cudaError_t launch_vi2_w(const Vi2Args& V, int grid, int smem, bool band, bool rearr, bool check, int enc,
                                 bool pdl, cudaStream_t s) {
-    const int key = (words ? 8 : 0) | (band ? 4 : 0) | (rearr ? 2 : 0) | (check ? 1 : 0);
+    const int key = enc * 8 | (band ? 4 : 0) | (rearr ? 2 : 0) | (check ? 1 : 0);
     switch (key) {
 #define K_(e, bd, r, c)                                                                                        \
     case e * 8 + bd * 4 + r * 2 + c:                                                                           \
         return launch_ex(sell_vi2_kernel<W, bd, r, c, e>, dim3(grid), dim3(Vi2Shape<W>::kThreads), smem, pdl, s, V);
         K_(0, 0, 0, 0) K_(0, 0, 0, 1) K_(0, 0, 1, 0) K_(0, 0, 1, 1) K_(0, 1, 0, 0) K_(0, 1, 0, 1) K_(0, 1, 1, 0)
         K_(0, 1, 1, 1) K_(1, 0, 0, 0) K_(1, 0, 0, 1) K_(1, 0, 1, 0) K_(1, 0, 1, 1) K_(1, 1, 0, 0) K_(1, 1, 0, 1)
-        K_(1, 1, 1, 0) K_(1, 1, 1, 1)
+        K_(1, 1, 1, 0) K_(1, 1, 1, 1) K_(2, 0, 0, 0) K_(2, 0, 0, 1) K_(2, 0, 1, 0) K_(2, 0, 1, 1) K_(2, 1, 0, 0)
+        K_(2, 1, 0, 1) K_(2, 1, 1, 0) K_(2, 1, 1, 1)
 #undef K_
     }
     return cudaErrorInvalidValue;
 }
 
-cudaError_t launch_vi2(const Vi2Args& V, int ncw, int grid, int smem, bool band, bool rearr, bool check, bool words,
+cudaError_t launch_vi2(const Vi2Args& V, int ncw, int grid, int smem, bool band, bool rearr, bool check, int enc,
                        bool pdl, cudaStream_t s) {
-    return ncw == 23   ? launch_vi2_w<23>(V, grid, smem, band, rearr, check, words, pdl, s)
-           : ncw == 30 ? launch_vi2_w<30>(V, grid, smem, band, rearr, check, words, pdl, s)
-                       : launch_vi2_w<16>(V, grid, smem, band, rearr, check, words, pdl, s);
+    return ncw == 23   ? launch_vi2_w<23>(V, grid, smem, band, rearr, check, enc, pdl, s)
+           : ncw == 30 ? launch_vi2_w<30>(V, grid, smem, band, rearr, check, enc, pdl, s)
+                       : launch_vi2_w<16>(V, grid, smem, band, rearr, check, enc, pdl, s);
 }
 
 template <int W>
@@ -34,7 +35,9 @@ static cudaError_t vi2_prepare_w(int smem) {
     if (e == cudaSuccess)                                                                                       \
         e = cudaFuncSetAttribute(sell_vi2_kernel<W, bd, r, c, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
     if (e == cudaSuccess)                                                                                       \
-        e = cudaFuncSetAttribute(sell_vi2_kernel<W, bd, r, c, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        e = cudaFuncSetAttribute(sell_vi2_kernel<W, bd, r, c, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
+    if (e == cudaSuccess)                                                                                       \
+        e = cudaFuncSetAttribute(sell_vi2_kernel<W, bd, r, c, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     A_(0, 0, 0) A_(0, 0, 1) A_(0, 1, 0) A_(0, 1, 1) A_(1, 0, 0) A_(1, 0, 1) A_(1, 1, 0) A_(1, 1, 1)
 #undef A_
     return e;
@@ -44,16 +47,18 @@ cudaError_t vi2_prepare(int ncw, int smem) {
     return ncw == 23 ? vi2_prepare_w<23>(smem) : ncw == 30 ? vi2_prepare_w<30>(smem) : vi2_prepare_w<16>(smem);
 }
 
-cudaError_t vi2_occupancy(int ncw, int smem, int* occ) {
+template <int W>
+static cudaError_t vi2_occupancy_w(int enc, int smem, int* occ) {
     // the heaviest variant (band + rearrangement + check) bounds the residency
-    if (ncw == 23)
-        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_vi2_kernel<23, true, true, true, 0>,
-                                                             Vi2Shape<23>::kThreads, smem);
-    if (ncw == 30)
-        return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_vi2_kernel<30, true, true, true, 0>,
-                                                             Vi2Shape<30>::kThreads, smem);
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_vi2_kernel<16, true, true, true, 0>,
-                                                         Vi2Shape<16>::kThreads, smem);
+    return enc == 2 ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_vi2_kernel<W, true, true, true, 2>,
+                                                                     Vi2Shape<W>::kThreads, smem)
+                    : cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, sell_vi2_kernel<W, true, true, true, 0>,
+                                                                     Vi2Shape<W>::kThreads, smem);
+}
+
+cudaError_t vi2_occupancy(int ncw, int smem, int* occ, int enc) {
+    return ncw == 23 ? vi2_occupancy_w<23>(enc, smem, occ)
+           : ncw == 30 ? vi2_occupancy_w<30>(enc, smem, occ) : vi2_occupancy_w<16>(enc, smem, occ);
 }
 
 }  // namespace cme

@@ -211,7 +211,9 @@ def test_large_dictionary_single_dictionary_cta(cme, oracle_mod, monkeypatch):
     A = oracle_mod.ingest(n, r, c, v)
     m = cme.Matrix(n, r, c, v).pack()
     f = m.info()
-    assert f.kernel == 1 and f.compact == 2 and f.tma_warps == 31
+    # single-dictionary CTA: the tile-record kernel's 30 consumer warps (or
+    # sell_vi_kernel's 31 when the records are off)
+    assert f.kernel == 1 and f.compact == 2 and (f.tma_warps, f.records) in ((30, 1), (31, 0))
     for omega in (1.0, 0.8):
         m.set_opts(omega=omega, check_every=20, stag_tol=0.0)
         x = W.random_start(n, 17)
@@ -631,3 +633,111 @@ def test_vi2_ring_wraps(cme, oracle_mod, monkeypatch, warps, stages, grid, net, 
     ref = oracle_mod.jacobi_solve(A, omega=omega, tol=0.0, check_every=30, max_iter=90, stag_tol=0.0)
     assert it == ref.iters == 90 and np.abs(p - ref.p).sum() <= 1e-12
     m.close()
+
+
+@pytest.mark.parametrize("steps", [2, 3])
+@pytest.mark.parametrize("warps,grid,lag", [(30, 0, -1), (16, 3, 0)])
+@pytest.mark.parametrize("net,order,omega", [(W.toggle_switch(120), "rcm", 0.9), (W.toggle_switch(90), "dfs", 0.9)],
+                         ids=lambda x: getattr(x, "name", str(x)))
+def test_wavefront_passes(cme, oracle_mod, monkeypatch, steps, warps, grid, lag, net, order, omega):
+    """Wavefront s-step kernel (sell_wf_kernel): check
+    blocks run as passes of s Jacobi steps whose later steps wait on per-tile
+    completion counters.  Capped grids (3 or 5 CTAs) and a minimal lag make
+    the dependency waits and the ring reuse happen on every item; C = 40 with
+    s = 3 leaves a 1-step remainder per block on the single-step kernel, and
+    max_iter = 95 a partial last block.  Fixed-iteration landscapes and a
+    converged solve vs the oracle."""
+    env = {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI2_WARPS": str(warps), "CME_WF": str(steps)}
+    if grid:
+        env["CME_VI2_GRID"] = str(grid)
+    if lag >= 0:
+        env["CME_WF_LAG"] = str(lag)
+    for k, v_ in env.items():
+        monkeypatch.setenv(k, v_)
+    states, r, c, v = oracle_mod.enumerate_network(net)
+    A = oracle_mod.ingest(len(states), r, c, v)
+    m = cme.Matrix(A.n, r, c, v).reorder(ORD[order]).pack()
+    f = m.info()
+    assert f.records == 1 and f.wf_steps == steps and f.tma_warps == warps and f.wf_lag > 0
+    if grid:
+        assert f.grid == grid
+    m.set_opts(omega=omega, check_every=30, stag_tol=0.0)
+    for max_iter in (90, 95):
+        p, st, it = m.solve(tol=0.0, max_iter=max_iter)
+        ref = oracle_mod.jacobi_solve(A, omega=omega, tol=0.0, check_every=30, max_iter=max_iter, stag_tol=0.0)
+        assert it == ref.iters == max_iter and np.abs(p - ref.p).sum() <= 1e-12, (max_iter, np.abs(p - ref.p).sum())
+    m.set_opts(omega=omega, check_every=40, stag_tol=0.0)
+    p, st, it = m.solve(tol=1e-9, max_iter=20000)
+    ref = oracle_mod.jacobi_solve(A, omega=omega, tol=1e-9, check_every=40, max_iter=20000, stag_tol=0.0)
+    assert st == ref.status and abs(it - ref.iters) <= 40
+    if it != ref.iters:
+        ref = oracle_mod.jacobi_solve(A, omega=omega, tol=0.0, check_every=40, max_iter=it, stag_tol=0.0)
+    assert np.abs(p - ref.p).sum() <= 1e-10
+    m.close()
+
+
+def test_wavefront_bit_identical_steps(cme, monkeypatch):
+    """Between checks the wavefront passes apply the same per-row arithmetic
+    as the single-step kernel: with no check inside the run (C larger than
+    max_iter) and the same final normalisation, 24 iterations as 12 passes of
+    2 / 8 passes of 3 / 6 of 4 give the single-step result to the last bit up
+    to the final 1/sum scale (whose summation order differs)."""
+    net = W.toggle_switch(150)
+    states, r, c, v = cme.cme_network_enumerate(net)
+    outs = {}
+    for s in ("0", "2", "3", "4"):
+        for k, v_ in {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_WF": s}.items():
+            monkeypatch.setenv(k, v_)
+        m = cme.Matrix(len(states), r, c, v).reorder(2).pack()
+        assert m.info().wf_steps == (int(s) if s != "0" else 0)
+        m.set_opts(omega=0.9, check_every=24, stag_tol=0.0)
+        p, st, it = m.solve(tol=0.0, max_iter=24, p0=W.random_start(len(states), 5))
+        assert it == 24
+        outs[s] = p
+        m.close()
+    for s in ("2", "3", "4"):
+        ratio = outs[s] / outs["0"]      # one common scale: x_24 itself is identical
+        assert np.abs(ratio / ratio[0] - 1.0).max() <= 1e-15, (s, np.abs(ratio / ratio[0] - 1.0).max())
+        assert abs(ratio[0] - 1.0) <= 1e-13
+
+
+@pytest.mark.parametrize("warps,grid", [(30, 0), (16, 3), (30, 2)])
+@pytest.mark.parametrize("net,order,omega", [(W.schnakenberg(60), "none", 1.0), (W.brusselator(70), "dfs", 0.9),
+                                             (W.schlogl(300), "rcm", 0.9)],
+                         ids=lambda x: getattr(x, "name", str(x)))
+def test_f64_records_bit_identical_to_compact(cme, oracle_mod, monkeypatch, warps, grid, net, order, omega):
+    """Tile records of the f64 compact encoding (sell_vi2_kernel ENC = 2:
+    networks without a value index, e.g. Schnakenberg / Brusselator with ~10^6
+    distinct rates at scale) run sell_cpt_kernel's arithmetic: SpMV and a
+    fixed-iteration landscape bit-identical to CME_REC = 0 (the compact
+    kernel) with the same check grid, and vs the oracle; capped grids wrap the
+    ring many times."""
+    states, r, c, v = oracle_mod.enumerate_network(net)
+    A = oracle_mod.ingest(len(states), r, c, v)
+    x = W.random_start(A.n, 21)
+    outs = {}
+    for rec in ("0", "1"):
+        env = {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "0", "CME_REC": rec}
+        if rec == "1":
+            env["CME_VI2_WARPS"] = str(warps)
+            if grid:
+                env["CME_VI2_GRID"] = str(grid)
+        for k, v_ in env.items():
+            monkeypatch.setenv(k, v_)
+        for k in ("CME_VI2_WARPS", "CME_VI2_GRID"):
+            if k not in env:
+                monkeypatch.delenv(k, raising=False)
+        m = cme.Matrix(A.n, r, c, v).reorder(ORD[order]).pack()
+        f = m.info()
+        assert f.compact == 1 and f.records == int(rec), (f.compact, f.records)
+        if rec == "1":
+            assert f.tma_warps == warps and (not grid or f.grid == grid)
+        m.set_opts(omega=omega, check_every=25, stag_tol=0.0)
+        y = m.spmv(x)
+        assert_spmv_close(y, oracle_mod.jacobi_step(A, x, omega))
+        p, st, it = m.solve(tol=0.0, max_iter=75)
+        ref = oracle_mod.jacobi_solve(A, omega=omega, tol=0.0, check_every=25, max_iter=75, stag_tol=0.0)
+        assert it == ref.iters == 75 and np.abs(p - ref.p).sum() <= 1e-12
+        outs[rec] = (y, p)
+        m.close()
+    assert np.array_equal(outs["0"][0], outs["1"][0])   # same per-row arithmetic

@@ -87,6 +87,6 @@ for var in a.variants:
     it = a.blocks * a.C
     ti = ms * 1e-3 / it
     print(f"[{var or 'default'}] {a.config} B={a.batch} kernel={f.kernel} order={order} n={f.n} nnz={f.nnz} "
-          f"band={f.band_on} rec={f.records} warps={f.tma_warps} st={f.tma_stages} t/iter={ti * 1e6:.1f}us GFLOPS={2 * f.nnz * a.batch / ti / 1e9:.1f} "
+          f"band={f.band_on} rec={f.records} wf={f.wf_steps}/{f.wf_lag} warps={f.tma_warps} st={f.tma_stages} t/iter={ti * 1e6:.1f}us GFLOPS={2 * f.nnz * a.batch / ti / 1e9:.1f} "
           f"alg={f.bytes_alg / ti / 1e9:.0f}GB/s ({100 * f.bytes_alg / ti / 1e9 / peak:.1f}%) "
           f"fmt={f.bytes_fmt / ti / 1e9:.0f}GB/s", flush=True)

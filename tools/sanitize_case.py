@@ -22,12 +22,18 @@ KNOBS = [
     ("register", {"CME_TMA": "0", "CME_RESIDENT": "0"}),
     ("tma-v0", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_COMPACT": "0"}),
     ("compact", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "0"}),
-    ("vi16", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_TMA_WARPS": "16"}),
-    ("vi8", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_TMA_WARPS": "8"}),
-    ("vi31", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_TMA_WARPS": "31"}),
+    ("vi16", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_VI2": "0", "CME_TMA_WARPS": "16"}),
+    ("vi8", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_VI2": "0", "CME_TMA_WARPS": "8"}),
+    ("vi31", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_VI2": "0", "CME_TMA_WARPS": "31"}),
+    # tile-record kernel (sell_vi2_kernel, the cfg4 hot kernel): 30- and 16-warp
+    # shapes, packed-word entries, and a capped grid that wraps the ring
+    ("vi2-30", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_VI2_WARPS": "30"}),
+    ("vi2-16", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_VI2_WARPS": "16"}),
+    ("vi2-words", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_VI2_WORDS": "1"}),
+    ("vi2-grid2", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_VI2_GRID": "2"}),
     ("resident", {"CME_TMA": "-1", "CME_RESIDENT": "1"}),
 ]
-ALL_KEYS = sorted({k for _, kn in KNOBS for k in kn} | {"CME_TMA_WARPS"})
+ALL_KEYS = sorted({k for _, kn in KNOBS for k in kn} | {"CME_TMA_WARPS", "CME_VI2_WARPS"})
 
 
 def set_knobs(kn):
@@ -45,7 +51,7 @@ for label, knobs in KNOBS:
         y = m.spmv(W.random_start(m.n, 1))
         pt, terms = m.transient(0.05)
         f = m.info()
-        print(label, net.name, "kernel", f.kernel, "compact", f.compact, "warps", f.tma_warps, st, it,
+        print(label, net.name, "kernel", f.kernel, "compact", f.compact, "records", f.records, "warps", f.tma_warps, st, it,
               float(p.sum()), terms, flush=True)
         m.close()
 
