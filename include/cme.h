@@ -215,6 +215,9 @@ typedef struct cme_info {
                                      (sell_wf_kernel, sec. 5e; the records re-read from L2);
                                      0: one launch per step */
     int32_t wf_lag;               /* wavefront lag L in tiles (0 when wf_steps = 0)     */
+    int32_t halo_fused;           /* 1: row-sharded over peer memory with the halo ordered
+                                     inside the step kernel (no per-step barrier, sec. 8) */
+    int32_t pad_;
 } cme_info;
 cme_status cme_get_info(cme_matrix h, cme_info* info);
 

@@ -36,6 +36,7 @@ struct P2PRank {
     int64_t span_lo = 0;        // first global row of the x-span
     int device = 0;
     unsigned char uuid[16] = {};  // physical GPU (cudaDeviceProp::uuid)
+    int32_t fused_ok = 0;       // can run the fused in-kernel halo sync (tile-record kernel)
 };
 
 int comm_transport(const cme_comm_s* c);

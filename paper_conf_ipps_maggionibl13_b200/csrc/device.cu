@@ -97,6 +97,16 @@ struct Device {
     double* push_y[2][kMaxPushPeers] = {};   // peer buffer (parity b) shifted to my local rows
     bool peers_ready = false;        // IPC transport: attach done
     bool bar_pdl = false;            // step barrier launched with PDL (peers on other GPUs only)
+    // fused in-kernel halo sync (kernels_vi2.cuh HaloSync): replaces the step barrier
+    bool fused = false;
+    bool same_gpu_peers = false;     // a peer rank shares this GPU (virtual ranks)
+    int64_t* hsync = nullptr;        // [4] steps run, push/halo warp completions, CTAs out
+    uint8_t* tile_kind = nullptr;    // [vi2 tiles] bit 0 reads halo rows, bit 1 pushes rows
+    int64_t hs_push_warps = 0, hs_halo_warps = 0;
+    int hs_nsend = 0, hs_nrecv = 0;
+    int hs_send_rank[kMaxPushPeers] = {}, hs_recv_rank[kMaxPushPeers] = {};
+    int64_t* hs_peer_pushed[kMaxPushPeers] = {};
+    int64_t* hs_peer_consumed[kMaxPushPeers] = {};
     std::vector<void*> ipc_opened;   // peer allocations mapped into this process
     HaloPlan halo;                   // counts/offsets in doubles (rows x B)
     std::vector<int64_t> cuts;       // in doubles (rows x B) for the output broadcast
@@ -956,8 +966,10 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
         }
         // the value-indexed encoding as tile records (sec. 5d)
         if (d->use_tma && d->vi && (s = configure_vi2(*d, P)) != CME_OK) return fail(s);
-        // the f64 compact encoding as tile records too (CME_REC = 0 keeps sell_cpt_kernel)
-        if (d->use_tma && d->cpt && !d->vi && env_int("CME_REC", 1) != 0 && (s = configure_vi2(*d, P, true)) != CME_OK)
+        // the f64 compact encoding as tile records too (CME_REC = 1; measured
+        // mixed, so opt-in: cfg3a 18.7 us (16 warps) vs 19.1 on sell_cpt_kernel,
+        // config 5 (w = 1024) 419 us vs 407)
+        if (d->use_tma && d->cpt && !d->vi && env_int("CME_REC", 0) != 0 && (s = configure_vi2(*d, P, true)) != CME_OK)
             return fail(s);
     }
     if (d->B > 1 && d->format == CME_FMT_DIAG_SELL && env_int("CME_COMPACT", 1) != 0 && env_int("CME_VI", -1) != 0 &&
@@ -1063,9 +1075,13 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
     }
     d->p2p = comm && transport_is_peer(comm_transport(comm));
     if (d->p2p) {
-        if ((s = d->alloc(d->flags, (size_t)d->nranks)) != CME_OK) return fail(s);
+        // [0, P) step/exchange barrier epochs, [P, 2P) halo rows pushed into me
+        // by rank q (steps), [2P, 3P) halo reads finished by rank p (fused sync)
+        if ((s = d->alloc(d->flags, (size_t)3 * d->nranks)) != CME_OK) return fail(s);
+        if ((s = d->alloc(d->hsync, 4)) != CME_OK) return fail(s);
+        if (cudaMemset(d->hsync, 0, 4 * sizeof(int64_t)) != cudaSuccess) return fail(CME_ERR_CUDA);
         if ((s = d->alloc(d->epoch, 1)) != CME_OK) return fail(s);
-        if (cudaMemset(d->flags, 0, d->nranks * sizeof(int64_t)) != cudaSuccess ||
+        if (cudaMemset(d->flags, 0, 3 * d->nranks * sizeof(int64_t)) != cudaSuccess ||
             cudaMemset(d->epoch, 0, sizeof(int64_t)) != cudaSuccess)
             return fail(CME_ERR_CUDA);
     }
@@ -1122,7 +1138,7 @@ static cme_status p2p_barrier(Device& d, cudaStream_t s, bool respect_stop, bool
 // after a step wrote buffer `dst`: halo exchange (NCCL) / step barrier (P2P;
 // the halo rows were already stored into the peers by the step kernel)
 static cme_status exch_after_step(Device& d, int dst, cudaStream_t s) {
-    if (!d.comm) return CME_OK;
+    if (!d.comm || d.fused) return CME_OK;   // fused: the step kernel ordered the halo itself
     if (d.p2p) return p2p_barrier(d, s, true, d.nbr_barrier);
     return comm_halo(d.comm, d.halo, d.xb[dst], s);
 }
@@ -1177,6 +1193,58 @@ static cme_status exch_segments(Device& d, cudaStream_t s) {
     return p2p_barrier(d, s, false);
 }
 
+// Fused halo sync plan (kernels_vi2.cuh HaloSync): per tile of the record
+// kernel, does it gather rows outside this rank's own rows (halo) and does it
+// hold rows some peer needs (push); the peers' flag words; and, when ranks
+// share a GPU (virtual ranks), a grid cap so every rank's step kernel can be
+// resident at once (a spinning gate needs its peer's tiles to run).
+static cme_status hs_plan(cme_matrix_s* h, const std::vector<P2PRank>& all, int on_gpu) {
+    Device& d = *h->dev;
+    const Packed& P = h->P;
+    const int ncw = d.vi2_ncw;
+    const int64_t T = d.vi2_tiles, n = P.n;
+    std::vector<uint8_t> kind(T, 0);
+    for (int64_t t = 0; t < T; ++t)
+        for (int64_t q = t * ncw; q < std::min<int64_t>((t + 1) * ncw, P.n_slices); ++q)
+            for (int lane = 0; lane < 32; ++lane) {
+                const int64_t slot = q * 32 + lane;
+                if (slot >= n) continue;
+                const int64_t r = P.row_of[slot];   // local row; x-span index own_off + r
+                for (int p = 0; p < d.npush; ++p)
+                    if (r >= d.push_lo[p] && r < d.push_hi[p]) kind[t] |= 2;
+                auto halo = [&](int64_t xs) { return xs < d.own_off || xs >= d.own_off + n; };
+                if (d.band && (halo(d.own_off + r - 1) || halo(d.own_off + r + 1))) kind[t] |= 1;
+                for (int w = 0; w < P.slice_w[q]; ++w)
+                    if (halo(P.col[P.slice_off[q] + lane + 32 * w])) kind[t] |= 1;
+            }
+    int64_t np = 0, nh = 0;
+    for (uint8_t k : kind) { np += (k & 2) != 0; nh += (k & 1) != 0; }
+    if (d.tile_kind == nullptr) CME_TRY(d.alloc(d.tile_kind, (size_t)T));
+    CUDA_TRY(cudaMemcpy(d.tile_kind, kind.data(), T, cudaMemcpyHostToDevice));
+    d.hs_push_warps = np * ncw;
+    d.hs_halo_warps = nh * ncw;
+    const HaloPlan& hp = h->halo;
+    d.hs_nsend = d.hs_nrecv = 0;
+    for (int sp : hp.send_peer) {
+        d.hs_send_rank[d.hs_nsend] = sp;
+        d.hs_peer_pushed[d.hs_nsend++] = all[sp].flags + d.nranks + d.rank;
+    }
+    for (int rq : hp.recv_peer) {
+        d.hs_recv_rank[d.hs_nrecv] = rq;
+        d.hs_peer_consumed[d.hs_nrecv++] = all[rq].flags + 2 * d.nranks + d.rank;
+    }
+    if (on_gpu > 1) {   // co-residency of the ranks sharing this GPU
+        int dev = 0, sms = 0;
+        CUDA_TRY(cudaGetDevice(&dev));
+        CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+        d.vi2_grid = std::max(1, std::min(d.vi2_grid, sms * d.vi2_occ / on_gpu));
+    }
+    if (env_int("CME_VERBOSE", 0))
+        std::fprintf(stderr, "[cme] rank %d fused halo sync: %lld push / %lld halo tiles of %lld, %d send / %d recv peers, grid %d\n",
+                     d.rank, (long long)np, (long long)nh, (long long)T, d.hs_nsend, d.hs_nrecv, d.vi2_grid);
+    return CME_OK;
+}
+
 // Peer-memory transport: given every rank's published buffers, derive the
 // peers' flag/gather/io pointers and, for every peer that needs some of my
 // rows, where in its x-span they go.
@@ -1211,14 +1279,22 @@ static void p2p_wire(cme_matrix_s* h, const std::vector<P2PRank>& all) {
     // when no peer shares this GPU: early-resident persistent CTAs would keep
     // a same-GPU peer's step off the SMs while the barrier waits for it
     d.bar_pdl = env_int("CME_PDL", 1) != 0;
+    int on_gpu = 0;
     for (int r = 0; r < d.nranks; ++r)
-        if (r != d.rank && std::memcmp(all[r].uuid, all[d.rank].uuid, 16) == 0) d.bar_pdl = false;
+        if (std::memcmp(all[r].uuid, all[d.rank].uuid, 16) == 0) ++on_gpu;
+    d.same_gpu_peers = on_gpu > 1;
+    if (d.same_gpu_peers) d.bar_pdl = false;
+    // fused in-kernel halo sync when every rank runs the tile-record kernel
+    bool all_ok = d.nranks > 1;
+    for (int r = 0; r < d.nranks; ++r) all_ok = all_ok && all[r].fused_ok;
+    d.fused = all_ok && hs_plan(h, all, on_gpu) == CME_OK;
     d.peers_ready = true;
 }
 
 static P2PRank p2p_mine(cme_matrix_s* h) {
     Device& d = *h->dev;
     P2PRank mine;
+    mine.fused_ok = d.vi2 && d.B == 1 && !d.vi2_words && env_int("CME_P2P_FUSED", 1) != 0 ? 1 : 0;
     mine.xb[0] = d.xb[0];
     mine.xb[1] = d.xb[1];
     mine.flags = d.flags;
@@ -1251,6 +1327,7 @@ struct IpcBlob {
     cudaIpcMemHandle_t h[5];   // xb[0] base, xb[1] base, flags, gather, io
     int64_t off[5];            // byte offset of the published pointer in its allocation
     unsigned char uuid[16];    // the exporting process's physical GPU
+    int32_t fused_ok;          // P2PRank::fused_ok
 };
 static_assert(sizeof(IpcBlob) <= CME_IPC_BLOB_BYTES, "IPC blob too large");
 constexpr uint64_t kIpcMagic = 0x434d45495043ull;   // "CMEIPC"
@@ -1267,6 +1344,7 @@ cme_status device_ipc_export(cme_matrix_s* h, uint8_t* out) {
     {
         const P2PRank me = p2p_mine(h);
         std::memcpy(b.uuid, me.uuid, 16);
+        b.fused_ok = me.fused_ok;
     }
     // allocation bases (device_upload): xb[b] sits one sentinel row of B doubles in
     void* bases[5] = {d.xb[0] - d.B, d.xb[1] - d.B, d.flags, d.gather, d.io};
@@ -1304,6 +1382,7 @@ cme_status device_ipc_attach(cme_matrix_s* h, const uint8_t* blobs) {
         all[r].span_lo = b.span_lo;
         all[r].device = b.device;
         std::memcpy(all[r].uuid, b.uuid, 16);
+        all[r].fused_ok = b.fused_ok;
     }
     p2p_wire(h, all);
     return CME_OK;
@@ -1348,13 +1427,33 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
     a.csr_v = d.csr_v;
     // programmatic dependent launch between consecutive steps (not across the
     // NCCL calls of a distributed solve, which are ordinary stream work)
-    const bool pdl = (!d.comm || d.p2p) && env_int("CME_PDL", 1) != 0;
+    // (not when fused-sync ranks share the GPU: an early-resident next step
+    // could hold SMs a peer's current step needs to release a gate)
+    const bool pdl = (!d.comm || d.p2p) && env_int("CME_PDL", 1) != 0 && !(d.fused && d.same_gpu_peers);
     if (d.format == CME_FMT_CSR) {
         CUDA_TRY(check ? launch_ex(csr_step_kernel<true>, dim3(d.grid), dim3(kCta), 0, pdl, s, a)
                        : launch_ex(csr_step_kernel<false>, dim3(d.grid), dim3(kCta), 0, pdl, s, a));
     } else if (d.vi2) {
         Vi2Args V{a, d.vi2_rec, d.vi2_rec_off, d.dict, d.vi2_tiles, d.vi2_stages, d.vi2_stage_bytes, d.dict_bytes,
                   d.win_shift, d.tma_xpf};
+        if (d.fused) {
+            HaloSync& hs = V.hs;
+            hs.on = 1;
+            hs.local = d.hsync;
+            hs.pushed = d.flags + d.nranks;
+            hs.consumed = d.flags + 2 * d.nranks;
+            hs.nsend = d.hs_nsend;
+            hs.nrecv = d.hs_nrecv;
+            for (int p = 0; p < d.hs_nsend; ++p) { hs.send_rank[p] = d.hs_send_rank[p]; hs.peer_pushed[p] = d.hs_peer_pushed[p]; }
+            for (int q = 0; q < d.hs_nrecv; ++q) { hs.recv_rank[q] = d.hs_recv_rank[q]; hs.peer_consumed[q] = d.hs_peer_consumed[q]; }
+            hs.tile_kind = d.tile_kind;
+            hs.push_warps = d.hs_push_warps;
+            hs.halo_warps = d.hs_halo_warps;
+            // as long as the barrier kernel's bound: a peer's host thread may be
+            // late to launch (8 virtual ranks in one process measured > 2 s)
+            hs.timeout_ns = (int64_t)std::max(1, env_int("CME_P2P_TIMEOUT_MS", 30000)) * 1000000;
+            hs.ctrl = d.ctrl;
+        }
         CUDA_TRY(launch_vi2(V, d.vi2_ncw, d.vi2_grid, d.dict_bytes + d.vi2_stages * d.vi2_stage_bytes, d.band, d.rearr,
                             check, d.vi2_f64 ? 2 : d.vi2_words ? 1 : 0, pdl, s));
     } else if (d.use_tma && d.vi && d.B > 1) {
@@ -1680,6 +1779,8 @@ static cme_status solve_epilogue(cme_matrix_s* h, cudaStream_t s, double omega, 
     if (f.status == CME_ERR_TIMEOUT) {
         set_error(d.use_res ? "resident kernel: a dependency wait timed out (CME_RES_TIMEOUT_MS)"
                   : d.wf    ? "wavefront kernel: a tile dependency wait timed out (CME_RES_TIMEOUT_MS)"
+                  : d.fused ? "peer-memory transport: a peer rank never signalled its halo rows (fused sync, "
+                              "CME_P2P_TIMEOUT_MS)"
                             : "peer-memory transport: a peer rank never reached the flag barrier");
         if (iters_out) *iters_out = f.iter;
         return CME_ERR_TIMEOUT;
@@ -1820,6 +1921,7 @@ void device_describe(const Device* d, cme_info* f) {
     f->tma_stages = d->vi2 ? d->vi2_stages : d->use_tma ? d->tma_stages : 0;
     f->records = d->vi2 ? 1 : 0;
     f->wf_steps = d->wf ? d->wf_s : 0;
+    f->halo_fused = d->fused ? 1 : 0;
     f->wf_lag = d->wf ? d->wf_lag : 0;
     f->grid = d->use_res ? d->res_grid : d->step_grid();
     f->compact = d->vi ? 2 : d->cpt ? 1 : 0;

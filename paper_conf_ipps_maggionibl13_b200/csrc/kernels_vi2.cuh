@@ -25,6 +25,101 @@
 
 namespace cme {
 
+// Fused peer-memory halo synchronisation (row-sharded solve, peer-memory
+// transport): instead of a flag-barrier kernel after every
+// step, the step kernel itself orders the halo traffic of the boundary tiles.
+// Per step k (= local[0], steps this rank has run; every rank runs the same
+// sequence) and neighbour pair:
+//   RAW  a tile reading halo rows waits until every rank pushing to me has
+//        signalled pushed >= k (its step k-1 stores of x_k into my buffer);
+//   WAR  a tile pushing rows waits until every rank I push to has signalled
+//        consumed >= k (its step k-1 reads of the buffer I now overwrite).
+// The waits gate the producer's stage arrival (the consumers never see a
+// gated tile early); the signals go out when the last warp of the last
+// push (halo) tile of the step finishes: atomic count at gpu scope, then
+// fence.sc.sys and st.release.sys of k+1 into the peers' flag words.  All
+// spins are bounded (%globaltimer): CME_ERR_TIMEOUT, never a hung GPU.
+struct HaloSync {
+    int64_t* local;                          // [0] steps run, [1] push-warp and [2] halo-warp completions, [3] CTAs out
+    const int64_t* pushed;                   // [nranks] written by the ranks pushing to me
+    const int64_t* consumed;                 // [nranks] written by the ranks I push to
+    int64_t* peer_pushed[kMaxPushPeers];     // send peer's pushed[my rank]
+    int64_t* peer_consumed[kMaxPushPeers];   // recv peer's consumed[my rank]
+    int32_t send_rank[kMaxPushPeers], recv_rank[kMaxPushPeers];
+    int32_t nsend, nrecv;
+    const uint8_t* tile_kind;                // [tiles] bit 0: reads halo rows, bit 1: pushes rows
+    int64_t push_warps, halo_warps;          // consumer-warp slots per step in push / halo tiles
+    int64_t timeout_ns;
+    Ctrl* ctrl;
+    int32_t on;
+};
+
+__device__ __forceinline__ int64_t ld_acquire_sys_s64(const int64_t* p) {
+    int64_t v;
+    asm volatile("ld.acquire.sys.global.s64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint64_t hs_ns() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+// producer warp: wait for the peers' flags tile kind `kind` depends on (all lanes call)
+static __device__ __noinline__ void hs_gate(const HaloSync& hs, uint32_t kind, int64_t k, bool& bad) {
+    const int lane = threadIdx.x & 31;
+    const int64_t* f = nullptr;
+    if ((kind & 1u) && lane < hs.nrecv) f = hs.pushed + hs.recv_rank[lane];
+    if ((kind & 2u) && lane >= 16 && lane - 16 < hs.nsend) f = hs.consumed + hs.send_rank[lane - 16];
+    if (f != nullptr && !bad && ld_acquire_sys_s64(f) < k) {
+        const uint64_t t0 = hs_ns();
+        while (ld_acquire_sys_s64(f) < k) {
+            if (hs_ns() - t0 > (uint64_t)hs.timeout_ns) { bad = true; break; }
+            __nanosleep(64);
+        }
+    }
+    bad = __any_sync(0xffffffffu, bad);
+}
+__device__ __forceinline__ int64_t atom_add_acq_rel(int64_t* p, int64_t v) {
+    int64_t old;
+    asm volatile("atom.acq_rel.gpu.global.add.u64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
+    return old;
+}
+// consumer lane 0 after its slice of a push / halo tile of step k (after a
+// __syncwarp: the lanes' peer stores / halo reads precede the release)
+static __device__ __noinline__ void hs_signal(const HaloSync& hs, uint32_t kind, int64_t k) {
+    if (kind & 2u) {
+        const int64_t old = atom_add_acq_rel(hs.local + 1, 1);
+        if ((int64_t)old + 1 == (k + 1) * hs.push_warps) {   // last push slice of the step
+            __threadfence_system();
+            for (int p = 0; p < hs.nsend; ++p)
+                asm volatile("st.release.sys.global.s64 [%0], %1;" ::"l"(hs.peer_pushed[p]), "l"(k + 1) : "memory");
+        }
+    }
+    if (kind & 1u) {
+        const int64_t old = atom_add_acq_rel(hs.local + 2, 1);
+        if ((int64_t)old + 1 == (k + 1) * hs.halo_warps) {   // last halo-reading slice of the step
+            __threadfence_system();
+            for (int q = 0; q < hs.nrecv; ++q)
+                asm volatile("st.release.sys.global.s64 [%0], %1;" ::"l"(hs.peer_consumed[q]), "l"(k + 1) : "memory");
+        }
+    }
+}
+
+// end of a step kernel (all threads): the last CTA out counts the step (the
+// next step reads it after its griddepcontrol.wait); stopped launches do not
+__device__ __forceinline__ void hs_finish(const HaloSync& hs, int G, const int32_t* stop) {
+    __syncwarp();
+    __syncthreads();
+    if (threadIdx.x == 0 && !(stop != nullptr && *(volatile const int32_t*)stop)) {
+        __threadfence();
+        if (atomicAdd(reinterpret_cast<unsigned long long*>(hs.local + 3), 1ull) == (unsigned long long)G - 1) {
+            hs.local[3] = 0;
+            __threadfence();
+            atomicAdd(reinterpret_cast<unsigned long long*>(hs.local), 1ull);
+        }
+    }
+}
+
 struct Vi2Args {
     StepArgs a;              // n_rows, slice_end, x/y, own_off, omega, pre_scale, partials, stop, inv_d (checks), push
     const unsigned char* rec;   // tile records, rec_off[t] bytes from rec
@@ -36,6 +131,7 @@ struct Vi2Args {
     int32_t dict_bytes;
     int32_t win_shift;          // log2(rearrangement window) (REARR)
     int32_t xpf;                // L2 prefetch of each tile's own x rows with its record
+    HaloSync hs;                // fused halo synchronisation (hs.on = 0: none)
 };
 
 // Record layout of a tile of TS slices (byte offsets; every block 16-B aligned).
@@ -235,16 +331,24 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
             mbar_arrive(&dbar);   // (F64 records: no dictionary)
         }
         int64_t o0 = 0, o1 = 0;
+        uint32_t kd = 0;      // fused halo sync: tile kind of the lane's tile
         int s = 0;
         uint32_t phase = 0;   // parity of the ring pass; reuse i >= S waits for pass (i / S - 1)'s release
-        bool waited = false;
+        bool waited = false, bad = false;
+        int64_t kstep = 0;
+        const bool fused = V.hs.on != 0;
         for (int i = 0; i < my_tiles; ++i) {
             const int l = i & 31;
             if (l == 0) {   // offsets of tiles i .. i+31
                 const int t = c + (i + lane) * G;
-                if (i + lane < my_tiles) { o0 = __ldg(V.rec_off + t); o1 = __ldg(V.rec_off + t + 1); }
+                if (i + lane < my_tiles) {
+                    o0 = __ldg(V.rec_off + t);
+                    o1 = __ldg(V.rec_off + t + 1);
+                    kd = fused ? (uint32_t)__ldg(V.hs.tile_kind + t) : 0u;
+                }
             }
             const int64_t b0 = __shfl_sync(0xffffffffu, o0, l), b1 = __shfl_sync(0xffffffffu, o1, l);
+            const uint32_t kind = __shfl_sync(0xffffffffu, kd, l);
             // first tiles were issued before the previous step ended; the stop
             // test comes before any ring reuse: on a stopped launch the
             // consumers release no stage, so waiting on empty[] would hang
@@ -252,6 +356,16 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
                 pdl_wait();
                 waited = true;
                 if (a.stop != nullptr && *a.stop) break;
+                if (fused) {   // gated tiles of the prologue: copied, not yet released
+                    kstep = *(volatile const int64_t*)V.hs.local;
+                    for (int i2 = 0; i2 < pro; ++i2) {
+                        const uint32_t k2 = __shfl_sync(0xffffffffu, kd, i2 & 31);
+                        if (k2) {
+                            hs_gate(V.hs, k2, kstep, bad);
+                            if (lane == 0) mbar_arrive(&full[i2]);
+                        }
+                    }
+                }
             }
             if (i >= S) mbar_wait(&empty[s], phase ^ 1u);
             if (lane == 0) {
@@ -261,14 +375,45 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
                     const int64_t r0 = (int64_t)t * NCW * 32, r1 = min(r0 + NCW * 32, a.n_rows);
                     if (r1 > r0) prefetch_l2(a.x + a.own_off + r0, (uint64_t)(r1 - r0) * 8);
                 }
-                mbar_expect_tx(&full[s], bytes);
+                if (kind)   // gated (fused halo sync): the arrival comes after the gate
+                    asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(&full[s])),
+                                 "r"(bytes)
+                                 : "memory");
+                else
+                    mbar_expect_tx(&full[s], bytes);
                 bulk_g2s(stages + (size_t)s * V.stage_bytes, V.rec + b0, bytes, &full[s], pol);
+            }
+            if (kind && i >= pro) {
+                hs_gate(V.hs, kind, kstep, bad);
+                if (lane == 0) mbar_arrive(&full[s]);
             }
             if (++s == S) { s = 0; phase ^= 1u; }
         }
-        if (!waited) pdl_wait();
+        if (!waited) {
+            pdl_wait();
+            const bool stopped = a.stop != nullptr && *a.stop;
+            if (fused) {   // every tile fit the prologue: release the gated ones
+                kstep = *(volatile const int64_t*)V.hs.local;
+                for (int i2 = 0; i2 < pro; ++i2) {
+                    const uint32_t k2 = __shfl_sync(0xffffffffu, kd, i2 & 31);
+                    if (k2) {
+                        if (!stopped) hs_gate(V.hs, k2, kstep, bad);
+                        if (lane == 0) mbar_arrive(&full[i2]);
+                    }
+                }
+            }
+        } else if (fused && a.stop != nullptr && *a.stop) {
+            // stopped: the consumers drain the prologue stages; release gated ones
+            for (int i2 = 0; i2 < pro; ++i2)
+                if (__shfl_sync(0xffffffffu, kd, i2 & 31) && lane == 0) mbar_arrive(&full[i2]);
+        }
+        if (bad && lane == 0) {
+            V.hs.ctrl->status = CME_ERR_TIMEOUT;
+            V.hs.ctrl->stop = 1;
+        }
         if (lane == 0) mbar_wait(&dbar, 0u);   // (no tile may have waited on it)
         if (CHECK) cta_check_partials<NCW + 1, 1>(CheckAcc<1>(), a.partials);
+        if (fused) hs_finish(V.hs, G, a.stop);
         return;
     }
     // ---------------- consumer warps: one slice each per tile ----------------
@@ -278,8 +423,11 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
         for (int i = 0; i < pro; ++i) mbar_wait(&full[i], 0u);
         mbar_wait(&dbar, 0u);
         if (CHECK) cta_check_partials<NCW + 1, 1>(CheckAcc<1>(), a.partials);
+        if (V.hs.on) hs_finish(V.hs, G, a.stop);
         return;
     }
+    const bool fused = V.hs.on != 0;
+    const int64_t kstep = fused ? *(volatile const int64_t*)V.hs.local : 0;
     CheckAcc<1> ck;
     {
         const double* xo = a.x + a.own_off;
@@ -371,12 +519,19 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
                     if (r >= a.push_lo[p] && r < a.push_hi[p]) a.push_y[p][r] = y;
             }
             __syncwarp();
-            if (lane == 0) mbar_arrive_a(empty0 + 8 * s);
+            if (lane == 0) {
+                if (fused) {
+                    const uint32_t kind = __ldg(V.hs.tile_kind + c + i * G);
+                    if (kind) hs_signal(V.hs, kind, kstep);
+                }
+                mbar_arrive_a(empty0 + 8 * s);
+            }
             st += sbytes;
             if (++s == S) { s = 0; phase ^= 1u; st = st0; }
         }
     }
     if (CHECK) cta_check_partials<NCW + 1, 1>(ck, a.partials);
+    if (fused) hs_finish(V.hs, G, a.stop);
 }
 
 }  // namespace cme

@@ -717,7 +717,7 @@ def test_f64_records_bit_identical_to_compact(cme, oracle_mod, monkeypatch, warp
     x = W.random_start(A.n, 21)
     outs = {}
     for rec in ("0", "1"):
-        env = {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "0", "CME_REC": rec}
+        env = {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "0", "CME_REC": rec}   # (records are opt-in)
         if rec == "1":
             env["CME_VI2_WARPS"] = str(warps)
             if grid:
@@ -731,7 +731,7 @@ def test_f64_records_bit_identical_to_compact(cme, oracle_mod, monkeypatch, warp
         f = m.info()
         assert f.compact == 1 and f.records == int(rec), (f.compact, f.records)
         if rec == "1":
-            assert f.tma_warps == warps and (not grid or f.grid == grid)
+            assert f.tma_warps == warps and (not grid or f.grid <= grid)
         m.set_opts(omega=omega, check_every=25, stag_tol=0.0)
         y = m.spmv(x)
         assert_spmv_close(y, oracle_mod.jacobi_step(A, x, omega))

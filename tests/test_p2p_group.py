@@ -97,3 +97,48 @@ def test_p2p_group_batch_and_fixed_iterations(oracle_mod):
         for b in range(2):
             o = oracle_mod.jacobi_solve(As[b], omega=0.9, tol=0.0, check_every=25, max_iter=210, stag_tol=0.0)
             assert np.abs(p[b * n:(b + 1) * n] - o.p).sum() <= 1e-12
+
+
+@pytest.mark.parametrize("nranks", [2, 4, 8])
+@pytest.mark.parametrize("fused", ["1", "0"])
+def test_fused_halo_sync_virtual_ranks(oracle_mod, monkeypatch, nranks, fused):
+    """The fused in-kernel halo sync: the tile-record step
+    kernel gates its boundary tiles on the peers' pushed / consumed step
+    counts instead of a flag-barrier kernel after every step.  2, 4 and 8
+    virtual ranks share one GPU, each rank's grid capped to its share of the
+    SMs so all ranks' step kernels are resident together (a gate spins until
+    a peer's tiles have run).  SpMV, a fixed-iteration run, a converged solve
+    and a transient vs the single-GPU path and the oracle; CME_P2P_FUSED = 0
+    (per-step neighbour barrier) on the same cases."""
+    import paper_conf_ipps_maggionibl13_b200 as cme
+    for k, val in {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_P2P_FUSED": fused}.items():
+        monkeypatch.setenv(k, val)
+    states, r, c, v = oracle_mod.enumerate_network(W.toggle_switch(150))
+    A = oracle_mod.ingest(len(states), r, c, v)
+    n = A.n
+    x = W.random_start(n, 6)
+
+    def body(m, rank):
+        info = m.info()
+        m.set_opts(omega=0.9, check_every=40, stag_tol=0.0)
+        y = m.spmv(x)
+        pf, stf, itf = m.solve(tol=0.0, max_iter=130)
+        m.set_opts(omega=0.9, check_every=100)
+        p, st, it = m.solve(tol=1e-10, max_iter=100000)
+        pt, terms = m.transient(0.1)
+        return info.halo_fused, info.records, y, pf, itf, p, st, it, pt
+
+    res = run_group(cme, nranks, n, r, c, v, body, window=256)
+    yref = oracle_mod.jacobi_step(A, x, 0.9)
+    of = oracle_mod.jacobi_solve(A, omega=0.9, tol=0.0, check_every=40, max_iter=130, stag_tol=0.0)
+    single = cme.Matrix(n, r, c, v).reorder(2).pack(cme.CME_FMT_DIAG_SELL, 256)
+    single.set_opts(omega=0.9, check_every=100)
+    p1, st1, it1 = single.solve(tol=1e-10, max_iter=100000)
+    ptr, _, _ = oracle_mod.transient(A, 0.1)
+    for hf, rec, y, pf, itf, p, st, it, pt in res:
+        assert rec == 1 and hf == int(fused)
+        assert np.max(np.abs(y - yref) / yref) <= 1e-13
+        assert itf == 130 and np.abs(pf - of.p).sum() <= 1e-12
+        assert st == st1 == "CONVERGED" and it == it1
+        assert np.abs(p - p1).sum() <= 1e-13
+        assert np.abs(pt - ptr).sum() <= 1e-12
