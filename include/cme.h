@@ -217,7 +217,9 @@ typedef struct cme_info {
     int32_t wf_lag;               /* wavefront lag L in tiles (0 when wf_steps = 0)     */
     int32_t halo_fused;           /* 1: row-sharded over peer memory with the halo ordered
                                      inside the step kernel (no per-step barrier, sec. 8) */
-    int32_t pad_;
+    int32_t xwin_kb;              /* > 0: the step kernel reads the iterate from a shared-memory
+                                     x window of this many KB per CTA, streamed with the tile
+                                     records (sec. 5f); 0: x gathers through L1/L2 */
 } cme_info;
 cme_status cme_get_info(cme_matrix h, cme_info* info);
 

@@ -73,7 +73,7 @@ class cme_info(C.Structure):
                 ("tma_stages", C.c_int32), ("grid", C.c_int32), ("batch", C.c_int32),
                 ("compact", C.c_int32), ("records", C.c_int32),
                 ("wf_steps", C.c_int32), ("wf_lag", C.c_int32), ("halo_fused", C.c_int32),
-                ("pad_", C.c_int32)]
+                ("xwin_kb", C.c_int32)]
 
 
 class cme_packed_view(C.Structure):

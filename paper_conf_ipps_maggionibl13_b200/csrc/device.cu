@@ -141,6 +141,12 @@ struct Device {
     int64_t vi2_tiles = 0;
     unsigned char* vi2_rec = nullptr;
     int64_t* vi2_rec_off = nullptr;
+    // x window in shared memory (XW; single GPU): per tile
+    // the iterate chunks it gathers, streamed with its record
+    bool xw = false;
+    int2* xw_ch = nullptr;           // [vi2 tiles] {first chunk, end chunk} (monotone)
+    int xw_mask = 0, xw_off = 0, xw_ring_bytes = 0;
+    int64_t xw_nx = 0;
     // wavefront s-step kernel over the tile records (kernels_wf.cuh): one
     // launch per s steps of a check block (single GPU, vi2 shapes)
     bool wf = false;
@@ -676,6 +682,128 @@ static cme_status configure_vi2(Device& d, const Packed& P, bool f64 = false) {
     return CME_OK;
 }
 
+// x-window plan (XW kernels) for tiles of ts slices:
+// per tile the iterate chunks (256 rows, chunk k = rows [256 k - xoff,
+// 256 k - xoff + 256) of the local x) holding its rows, band neighbours and
+// gathered columns, as a suffix-min of the first and a prefix-max of the end
+// chunk so the producer streams every chunk once, in order.  Returns the ring
+// chunks a CTA needs with S stages in flight: tiles j-S+1 .. j are live when
+// tile j's chunks are issued (tile j-S has released its stage).
+static int64_t xw_plan(const Packed& P, int ts, bool band, int64_t own_off, int xoff, int64_t nx, int S,
+                       std::vector<int2>& ch) {
+    const int64_t nt = (P.n_slices + ts - 1) / ts, n = P.n;
+    std::vector<int64_t> lo(nt), hi(nt);
+#pragma omp parallel for schedule(dynamic, 64)
+    for (int64_t t = 0; t < nt; ++t) {
+        int64_t mn = INT64_MAX, mx = INT64_MIN;
+        const int64_t q1 = std::min<int64_t>((t + 1) * ts, P.n_slices);
+        for (int64_t q = t * ts; q < q1; ++q)
+            for (int ln = 0; ln < 32; ++ln) {
+                const int64_t slot = q * 32 + ln;
+                if (slot >= n) break;
+                const int64_t r = P.row_of.empty() ? slot : P.row_of[slot];
+                mn = std::min(mn, r - (band ? 1 : 0));
+                mx = std::max(mx, r + (band ? 1 : 0));
+                for (int32_t u = 0; u < P.slice_w[q]; ++u) {
+                    const int64_t j = (int64_t)P.col[P.slice_off[q] + ln + 32 * u] - own_off;
+                    mn = std::min(mn, j);
+                    mx = std::max(mx, j);
+                }
+            }
+        if (mn > mx) mn = mx = 0;   // an all-padding tile
+        const int64_t last = (nx + xoff) >> 8;   // chunk of the sentinel row nx
+        lo[t] = std::max<int64_t>(0, (mn + xoff) >> 8);
+        hi[t] = std::min<int64_t>(last, (mx + xoff) >> 8) + 1;
+    }
+    for (int64_t t = nt - 2; t >= 0; --t) lo[t] = std::min(lo[t], lo[t + 1]);
+    for (int64_t t = 1; t < nt; ++t) hi[t] = std::max(hi[t], hi[t - 1]);
+    int64_t need = 1;
+    ch.resize(nt);
+    for (int64_t t = 0; t < nt; ++t) {
+        need = std::max(need, hi[t] - lo[std::max<int64_t>(0, t - S + 1)]);
+        ch[t] = make_int2((int)lo[t], (int)hi[t]);
+    }
+    return need;
+}
+
+// The x-window shape (single GPU; records of the value-indexed encoding, or
+// of the f64 compact one when there is no value index): the first of
+// (30 warps, 4 | 3 stages), (16, 4 | 3), (30, 2), (16, 2) whose stages,
+// dictionary and power-of-two x ring fit one CTA per SM.  CME_XW = 1 forces
+// it, 0 disables it; auto (-1) takes it for the f64 records when the ring is
+// <= 64 KB -- measured on config 5 (n = 16 M, mu = 10): width 1 024 290 us vs
+// 403 us on sell_cpt_kernel, width 32 283 vs 309 -- and not for the wide
+// windows of the CME orderings (cfg4 RCM: a 128 KB ring leaves 16 warps x 2
+// stages, 237 us vs 173; cfg3a: 21.2 vs 19.1 us).
+static cme_status configure_xw(Device& d, const Packed& P, bool f64, std::vector<int2>& plan) {
+    d.xw = false;
+    const int want = env_int("CME_XW", -1);
+    if (want == 0 || d.nranks > 1 || d.B != 1 || (want < 0 && !f64)) return CME_OK;
+    const int xoff = (int)((reinterpret_cast<uintptr_t>(d.xb[0] + d.own_off) >> 3) & 1);
+    if (xoff != (int)((reinterpret_cast<uintptr_t>(d.xb[1] + d.own_off) >> 3) & 1)) return CME_OK;
+    int dev = 0, smem_max = 0, sms = 0;
+    CUDA_TRY(cudaGetDevice(&dev));
+    CUDA_TRY(cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+    CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    const int cap = smem_max - 4096, enc = f64 ? 2 : 0;
+    const int dict = f64 ? 0 : d.dict_bytes;
+    const int force_w = env_int("CME_VI2_WARPS", 0), force_s = env_int("CME_VI2_STAGES", 0);
+    const int64_t nx = d.nx - d.own_off;
+    const int64_t ring_cap = want > 0 ? INT64_MAX : (int64_t)64 << 10;
+    int64_t stage_of[2] = {0, 0};   // [30 warps, 16 warps]
+    const int order[6][2] = {{30, 4}, {30, 3}, {16, 4}, {16, 3}, {30, 2}, {16, 2}};
+    for (const auto& sh : order) {
+        const int ncw = sh[0];
+        if (force_w && ncw != force_w) continue;
+        const int st = force_s > 0 ? std::min(force_s, 8) : sh[1];
+        if (force_s > 0 && sh[1] != 4) continue;   // one candidate per warp count when forced
+        const int64_t nt = (P.n_slices + ncw - 1) / ncw;
+        int64_t& stage = stage_of[ncw == 30 ? 0 : 1];
+        if (!stage) {
+            int64_t mx = 0;
+            for (int64_t t = 0; t < nt; ++t) mx = std::max(mx, vi2_record_bytes(P, ncw, d.band, d.rearr, t, f64));
+            stage = (mx + 127) / 128 * 128;
+            CUDA_TRY(vi2_xw_prepare(ncw, cap));
+        }
+        {
+            std::vector<int2> ch;
+            const int64_t need = xw_plan(P, ncw, d.band, d.own_off, xoff, nx, st, ch);
+            int64_t slots = 1;
+            while (slots < need) slots <<= 1;
+            const int64_t bytes = dict + st * stage + slots * 2048;
+            if (env_int("CME_VERBOSE", 0) > 1)
+                std::fprintf(stderr, "[cme] xw shape: ncw=%d stages=%d stage=%lld ring chunks=%lld (need %lld) smem=%lld\n",
+                             ncw, st, (long long)stage, (long long)slots, (long long)need, (long long)bytes);
+            if (bytes > cap || slots * 2048 > ring_cap) continue;
+            int occ = 0;
+            CUDA_TRY(vi2_xw_occupancy(ncw, (int)bytes, &occ, enc));
+            if (occ < 1) continue;
+            d.xw = true;
+            d.vi2 = true;
+            d.vi2_f64 = f64;
+            d.vi2_words = false;
+            if (f64) d.dict_bytes = 0;
+            d.vi2_ncw = ncw;
+            d.vi2_stages = st;
+            d.vi2_stage_bytes = (int)stage;
+            d.vi2_occ = occ;
+            d.vi2_tiles = nt;
+            d.vi2_grid = (int)std::min<int64_t>(nt, (int64_t)sms * occ);
+            if (env_int("CME_VI2_GRID", 0) > 0) d.vi2_grid = std::min(d.vi2_grid, env_int("CME_VI2_GRID", 0));
+            d.xw_mask = (int)(slots * 256 - 1);
+            d.xw_off = xoff;
+            d.xw_nx = nx;
+            d.xw_ring_bytes = (int)(slots * 2048);
+            plan.swap(ch);
+            if (env_int("CME_VERBOSE", 0))
+                std::fprintf(stderr, "[cme] xw: warps=%d stages=%d stage_bytes=%d ring=%d KB occ=%d grid=%d tiles=%lld\n",
+                             ncw, st, d.vi2_stage_bytes, d.xw_ring_bytes / 1024, occ, d.vi2_grid, (long long)nt);
+            return CME_OK;
+        }
+    }
+    return CME_OK;
+}
+
 // Wavefront plan (kernels_wf.cuh): per tile of ncw slices, the union of the
 // tiles holding the rows it gathers (RAW) and the tiles gathering its rows
 // (WAR), as one [first, last] range; then the (step, tile) items in wave
@@ -931,6 +1059,7 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
     h->Cpt = Compact();
     // (tried even when layout v0's stages were too wide for a TMA shape: the
     // compact and value-indexed stages are 2.5-3x smaller)
+    std::vector<int2> xwp;   // x-window chunk plan (sec. 5f), uploaded with the records
     const bool v0_tma = d->use_tma;
     const int v0_warps = v0_tma ? d->tma_ncw * d->tma_spw * d->tma_occ : 0;
     if (d->B == 1 && d->format == CME_FMT_DIAG_SELL && env_int("CME_COMPACT", 1) != 0 && env_int("CME_TMA", -1) != 0 &&
@@ -971,6 +1100,9 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
         // config 5 (w = 1024) 419 us vs 407)
         if (d->use_tma && d->cpt && !d->vi && env_int("CME_REC", 0) != 0 && (s = configure_vi2(*d, P, true)) != CME_OK)
             return fail(s);
+        // the x window in shared memory (sec. 5f) for narrow bands
+        if (d->use_tma && d->cpt && !comm && h->nranks == 1 && (s = configure_xw(*d, P, !d->vi, xwp)) != CME_OK)
+            return fail(s);
     }
     if (d->B > 1 && d->format == CME_FMT_DIAG_SELL && env_int("CME_COMPACT", 1) != 0 && env_int("CME_VI", -1) != 0 &&
         env_int("CME_TMA", -1) != 0 && encode_compact(P, d->own_off, h->Cpt) && encode_value_index(P, h->Cpt)) {
@@ -1004,6 +1136,7 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
                 dict.resize(d->dict_bytes / 8, 0.0);   // staged in shared memory, 128-B padded
                 UP(dict, dict);
             }
+            if (d->xw) UP(xw_ch, xwp);
             std::vector<unsigned char> rec;
             std::vector<int64_t> roff;
             vi2_build_records(P, h->Cpt, d->vi2_ncw, d->band, d->rearr, d->vi2_words, rec, roff, d->vi2_f64);
@@ -1012,7 +1145,7 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
             // wavefront s-step passes (CME_WF = s; single GPU, same grid as
             // the vi2 kernel so the check partials keep their layout)
             const int wf_s = env_int("CME_WF", 0);
-            if (wf_s >= 2 && wf_s <= 8 && !comm && h->nranks == 1 && (d->vi2_ncw == 30 || d->vi2_ncw == 16) &&
+            if (wf_s >= 2 && wf_s <= 8 && !comm && h->nranks == 1 && !d->xw && (d->vi2_ncw == 30 || d->vi2_ncw == 16) &&
                 !d->vi2_words && !d->vi2_f64 && d->vi2_tiles < (1 << 24)) {
                 const int smem = d->dict_bytes + d->vi2_stages * d->vi2_stage_bytes;
                 int occ = 0;
@@ -1454,8 +1587,18 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
             hs.timeout_ns = (int64_t)std::max(1, env_int("CME_P2P_TIMEOUT_MS", 30000)) * 1000000;
             hs.ctrl = d.ctrl;
         }
-        CUDA_TRY(launch_vi2(V, d.vi2_ncw, d.vi2_grid, d.dict_bytes + d.vi2_stages * d.vi2_stage_bytes, d.band, d.rearr,
-                            check, d.vi2_f64 ? 2 : d.vi2_words ? 1 : 0, pdl, s));
+        if (d.xw) {
+            V.xw_ch = d.xw_ch;
+            V.xw_mask = d.xw_mask;
+            V.xw_off = d.xw_off;
+            V.xw_nx = d.xw_nx;
+            V.xpf = 0;
+            CUDA_TRY(launch_vi2_xw(V, d.vi2_ncw, d.vi2_grid,
+                                   d.dict_bytes + d.vi2_stages * d.vi2_stage_bytes + d.xw_ring_bytes, d.band, d.rearr,
+                                   check, d.vi2_f64 ? 2 : 0, pdl, s));
+        } else
+            CUDA_TRY(launch_vi2(V, d.vi2_ncw, d.vi2_grid, d.dict_bytes + d.vi2_stages * d.vi2_stage_bytes, d.band,
+                                d.rearr, check, d.vi2_f64 ? 2 : d.vi2_words ? 1 : 0, pdl, s));
     } else if (d.use_tma && d.vi && d.B > 1) {
         ViArgs V{CptArgs{TmaArgs{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col,
                                  d.tma_contig, d.tma_xpf},
@@ -1922,6 +2065,7 @@ void device_describe(const Device* d, cme_info* f) {
     f->records = d->vi2 ? 1 : 0;
     f->wf_steps = d->wf ? d->wf_s : 0;
     f->halo_fused = d->fused ? 1 : 0;
+    f->xwin_kb = d->xw ? d->xw_ring_bytes / 1024 : 0;
     f->wf_lag = d->wf ? d->wf_lag : 0;
     f->grid = d->use_res ? d->res_grid : d->step_grid();
     f->compact = d->vi ? 2 : d->cpt ? 1 : 0;

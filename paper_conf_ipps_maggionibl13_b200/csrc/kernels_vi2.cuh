@@ -132,6 +132,14 @@ struct Vi2Args {
     int32_t win_shift;          // log2(rearrangement window) (REARR)
     int32_t xpf;                // L2 prefetch of each tile's own x rows with its record
     HaloSync hs;                // fused halo synchronisation (hs.on = 0: none)
+    // x window in shared memory (XW kernels): chunk k of
+    // the ring holds the iterate rows [256 k - xw_off, 256 k - xw_off + 256)
+    // (relative to x + own_off) at ring slot k & (xw_mask >> 8); tile t needs
+    // chunks [xw_ch[t].x, xw_ch[t].y) (suffix-min / prefix-max: both monotone)
+    const int2* xw_ch;
+    int32_t xw_mask;            // ring rows - 1 (a power of two >= 256)
+    int32_t xw_off;             // 1 when x + own_off is 8 mod 16 (bulk copies need 16-B sources)
+    int64_t xw_nx;              // iterate rows readable from x + own_off (a sentinel row at -1 and nx)
 };
 
 // Record layout of a tile of TS slices (byte offsets; every block 16-B aligned).
@@ -199,25 +207,41 @@ __device__ __forceinline__ int2 lds_v2(uint32_t a) {
     return v;
 }
 
+// x gathers: from global memory (L1/L2; the iterate row r is xr[0]) or from
+// the shared-memory x window (XW: ring index (r + off + xw_off) & mask)
+struct GatherG {
+    const double* xr;
+    __device__ __forceinline__ double operator()(int32_t o) const { return __ldg(xr + o); }
+};
+struct GatherS {
+    uint32_t xs;     // ring base (shared window)
+    uint32_t rx;     // r + xw_off
+    uint32_t mask;
+    __device__ __forceinline__ double operator()(int32_t o) const {
+        return lds_f64(xs + (((rx + (uint32_t)o) & mask) << 3));
+    }
+};
+
 // W entries of one slot: the W x gathers first (their latency is the step's
 // critical path), then per entry the dictionary value and the FMA in t order.
-template <int W>
-__device__ __forceinline__ double vi2_row(uint32_t pv, uint32_t pc, uint32_t sdict, const double* xr) {
+template <int W, class GX>
+__device__ __forceinline__ double vi2_row(uint32_t pv, uint32_t pc, uint32_t sdict, const GX& gx) {
     double xv[W];
 #pragma unroll
-    for (int u = 0; u < W; ++u) xv[u] = __ldg(xr + lds_s16(pc + 64 * u));
+    for (int u = 0; u < W; ++u) xv[u] = gx(lds_s16(pc + 64 * u));
     double acc = 0.0;
 #pragma unroll
     for (int u = 0; u < W; ++u) acc = fma(lds_f64(sdict + 8 * lds_u16(pv + 64 * u)), xv[u], acc);
     return acc;
 }
-__device__ __forceinline__ double vi2_row_wide(uint32_t pv, uint32_t pc, uint32_t sdict, const double* xr, int w) {
+template <class GX>
+__device__ __forceinline__ double vi2_row_wide(uint32_t pv, uint32_t pc, uint32_t sdict, const GX& gx, int w) {
     double acc = 0.0;
     for (int t0 = 0; t0 < w; t0 += 8) {
         double xv[8];
 #pragma unroll
         for (int u = 0; u < 8; ++u)
-            if (t0 + u < w) xv[u] = __ldg(xr + lds_s16(pc + 64 * (t0 + u)));
+            if (t0 + u < w) xv[u] = gx(lds_s16(pc + 64 * (t0 + u)));
 #pragma unroll
         for (int u = 0; u < 8; ++u)
             if (t0 + u < w) acc = fma(lds_f64(sdict + 8 * lds_u16(pv + 64 * (t0 + u))), xv[u], acc);
@@ -228,20 +252,21 @@ __device__ __forceinline__ double vi2_row_wide(uint32_t pv, uint32_t pc, uint32_
 // Packed-word variant (ENC = 1): entry u of a lane is one 32-bit word
 // vidx | col16 << 16 at pw + 128 u -- one shared-memory load per entry instead
 // of two (half the LSU wavefronts of the index reads).
-template <int W>
-__device__ __forceinline__ double vi2_row_w(uint32_t pw, uint32_t sdict, const double* xr) {
+template <int W, class GX>
+__device__ __forceinline__ double vi2_row_w(uint32_t pw, uint32_t sdict, const GX& gx) {
     uint32_t w[W];
 #pragma unroll
     for (int u = 0; u < W; ++u) w[u] = lds_u32(pw + 128 * u);
     double xv[W];
 #pragma unroll
-    for (int u = 0; u < W; ++u) xv[u] = __ldg(xr + ((int32_t)w[u] >> 16));
+    for (int u = 0; u < W; ++u) xv[u] = gx((int32_t)w[u] >> 16);
     double acc = 0.0;
 #pragma unroll
     for (int u = 0; u < W; ++u) acc = fma(lds_f64(sdict + 8 * (w[u] & 0xffffu)), xv[u], acc);
     return acc;
 }
-__device__ __forceinline__ double vi2_row_w_wide(uint32_t pw, uint32_t sdict, const double* xr, int wd) {
+template <class GX>
+__device__ __forceinline__ double vi2_row_w_wide(uint32_t pw, uint32_t sdict, const GX& gx, int wd) {
     double acc = 0.0;
     for (int t0 = 0; t0 < wd; t0 += 8) {
         uint32_t w[8];
@@ -251,7 +276,7 @@ __device__ __forceinline__ double vi2_row_w_wide(uint32_t pw, uint32_t sdict, co
             if (t0 + u < wd) w[u] = lds_u32(pw + 128 * (t0 + u));
 #pragma unroll
         for (int u = 0; u < 8; ++u)
-            if (t0 + u < wd) xv[u] = __ldg(xr + ((int32_t)w[u] >> 16));
+            if (t0 + u < wd) xv[u] = gx((int32_t)w[u] >> 16);
 #pragma unroll
         for (int u = 0; u < 8; ++u)
             if (t0 + u < wd) acc = fma(lds_f64(sdict + 8 * (w[u] & 0xffffu)), xv[u], acc);
@@ -261,28 +286,70 @@ __device__ __forceinline__ double vi2_row_w_wide(uint32_t pw, uint32_t sdict, co
 
 // F64 records (ENC = 2): entry u of a lane has its value at pv + 256 u and
 // its col16 at pc + 64 u; FMAs in t order (sell_cpt_kernel's arithmetic).
-template <int W>
-__device__ __forceinline__ double vi2_row_f(uint32_t pv, uint32_t pc, const double* xr) {
+template <int W, class GX>
+__device__ __forceinline__ double vi2_row_f(uint32_t pv, uint32_t pc, const GX& gx) {
     double xv[W];
 #pragma unroll
-    for (int u = 0; u < W; ++u) xv[u] = __ldg(xr + lds_s16(pc + 64 * u));
+    for (int u = 0; u < W; ++u) xv[u] = gx(lds_s16(pc + 64 * u));
     double acc = 0.0;
 #pragma unroll
     for (int u = 0; u < W; ++u) acc = fma(lds_f64(pv + 256 * u), xv[u], acc);
     return acc;
 }
-__device__ __forceinline__ double vi2_row_f_wide(uint32_t pv, uint32_t pc, const double* xr, int w) {
+template <class GX>
+__device__ __forceinline__ double vi2_row_f_wide(uint32_t pv, uint32_t pc, const GX& gx, int w) {
     double acc = 0.0;
     for (int t0 = 0; t0 < w; t0 += 8) {
         double xv[8];
 #pragma unroll
         for (int u = 0; u < 8; ++u)
-            if (t0 + u < w) xv[u] = __ldg(xr + lds_s16(pc + 64 * (t0 + u)));
+            if (t0 + u < w) xv[u] = gx(lds_s16(pc + 64 * (t0 + u)));
 #pragma unroll
         for (int u = 0; u < 8; ++u)
             if (t0 + u < w) acc = fma(lds_f64(pv + 256 * (t0 + u)), xv[u], acc);
     }
     return acc;
+}
+
+// The off-band sum of one slot, dispatched on the slice's (warp-uniform) width.
+template <int ENC, class GX>
+__device__ __forceinline__ double vi2_acc(int w, uint32_t pv, uint32_t pc, uint32_t sdict, const GX& gx) {
+    if (ENC == 2) switch (w) {
+        case 0: return 0.0;
+        case 1: return vi2_row_f<1>(pv, pc, gx);
+        case 2: return vi2_row_f<2>(pv, pc, gx);
+        case 3: return vi2_row_f<3>(pv, pc, gx);
+        case 4: return vi2_row_f<4>(pv, pc, gx);
+        case 5: return vi2_row_f<5>(pv, pc, gx);
+        case 6: return vi2_row_f<6>(pv, pc, gx);
+        case 7: return vi2_row_f<7>(pv, pc, gx);
+        case 8: return vi2_row_f<8>(pv, pc, gx);
+        default: return vi2_row_f_wide(pv, pc, gx, w);
+    }
+    if (ENC == 1) switch (w) {
+        case 0: return 0.0;
+        case 1: return vi2_row_w<1>(pv, sdict, gx);
+        case 2: return vi2_row_w<2>(pv, sdict, gx);
+        case 3: return vi2_row_w<3>(pv, sdict, gx);
+        case 4: return vi2_row_w<4>(pv, sdict, gx);
+        case 5: return vi2_row_w<5>(pv, sdict, gx);
+        case 6: return vi2_row_w<6>(pv, sdict, gx);
+        case 7: return vi2_row_w<7>(pv, sdict, gx);
+        case 8: return vi2_row_w<8>(pv, sdict, gx);
+        default: return vi2_row_w_wide(pv, sdict, gx, w);
+    }
+    switch (w) {
+        case 0: return 0.0;
+        case 1: return vi2_row<1>(pv, pc, sdict, gx);
+        case 2: return vi2_row<2>(pv, pc, sdict, gx);
+        case 3: return vi2_row<3>(pv, pc, sdict, gx);
+        case 4: return vi2_row<4>(pv, pc, sdict, gx);
+        case 5: return vi2_row<5>(pv, pc, sdict, gx);
+        case 6: return vi2_row<6>(pv, pc, sdict, gx);
+        case 7: return vi2_row<7>(pv, pc, sdict, gx);
+        case 8: return vi2_row<8>(pv, pc, sdict, gx);
+        default: return vi2_row_wide(pv, pc, sdict, gx, w);
+    }
 }
 
 template <int NCW>
@@ -292,9 +359,13 @@ struct Vi2Shape {
     static constexpr int kMinBlocks = NCW == 30 ? 1 : 2;
 };
 
-template <int NCW, bool BAND, bool REARR, bool CHECK, int ENC>
-__global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBlocks)
-    sell_vi2_kernel(const Vi2Args V) {
+// XW: the x window variant -- each CTA runs a contiguous
+// range of tiles and the producer streams the iterate rows those tiles gather
+// into a shared-memory ring with the tile records (same mbarriers), so every
+// x read of the step is a shared-memory load.  Single-GPU packs only.
+template <int NCW, bool BAND, bool REARR, bool CHECK, int ENC, bool XW = false>
+__global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, XW ? 1 : Vi2Shape<NCW>::kMinBlocks)
+    sell_vi2_kernel(const __grid_constant__ Vi2Args V) {
     constexpr bool F64 = ENC == 2;
     using R = Vi2Rec<NCW, BAND, REARR, F64>;
     const StepArgs& a = V.a;
@@ -303,6 +374,14 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
     __shared__ uint64_t full[8], empty[8], dbar;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int S = V.stages;
+    unsigned char* stages = smem + V.dict_bytes;
+    unsigned char* xring = stages + (size_t)S * V.stage_bytes;
+    if (XW) {   // rows the ring has not received (row -1 when xw_off = 0) read as 0
+        uint4* z = reinterpret_cast<uint4*>(xring);
+        const int nz = (V.xw_mask + 1) / 2;
+        for (int k = threadIdx.x; k < nz; k += blockDim.x) z[k] = make_uint4(0u, 0u, 0u, 0u);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // before the bulk copies overwrite it
+    }
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
             mbar_init(&full[s], 1);
@@ -314,9 +393,13 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
     __syncthreads();
     const int G = gridDim.x, c = blockIdx.x;
     const int n_tiles = (int)V.n_tiles;
-    const int my_tiles = c < n_tiles ? (n_tiles - 1 - c) / G + 1 : 0;
+    // tiles of this CTA: XW a contiguous range [t_begin, t_begin + my_tiles),
+    // else c, c + G, c + 2G, ...
+    const int t_begin = XW ? (int)((int64_t)c * n_tiles / G) : c;
+    const int t_step = XW ? 1 : G;
+    const int my_tiles = XW ? (int)((int64_t)(c + 1) * n_tiles / G) - t_begin
+                            : (c < n_tiles ? (n_tiles - 1 - c) / G + 1 : 0);
     const int pro = my_tiles < S ? my_tiles : S;
-    unsigned char* stages = smem + V.dict_bytes;
     if (warp == NCW) {
         // ---------------- producer warp: one bulk copy per tile record ----------------
         // the record offsets of the CTA's next 32 tiles are loaded by the 32
@@ -330,8 +413,31 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
         } else if (lane == 0) {
             mbar_arrive(&dbar);   // (F64 records: no dictionary)
         }
+        // XW: next iterate chunk to stream (chunks are issued in increasing order)
+        int32_t ch_hi = 0;
+        int32_t xk = XW && my_tiles > 0 ? __ldg(&V.xw_ch[t_begin].x) : 0;
+        const double* xsrc = a.x + a.own_off - V.xw_off;   // 16-B aligned: chunk k starts at xsrc + 256 k
+        const int32_t xw_slots = (V.xw_mask + 1) >> 8;
+        const int64_t x_avail = V.xw_nx + 1 + V.xw_off;    // rows readable from xsrc (through the sentinel at nx)
+        // bytes of chunks [xk, hi) (pure arithmetic; lane 0 then issues them)
+        auto x_bytes = [&](int32_t hi) -> uint32_t {
+            if (hi <= xk) return 0u;
+            const int64_t r0 = (int64_t)xk * 256, r1 = min((int64_t)hi * 256, x_avail & ~int64_t(1));
+            return r1 > r0 ? (uint32_t)((r1 - r0) * 8) : 0u;
+        };
+        auto x_issue = [&](int32_t hi, uint64_t* bar) {   // lane 0: chunks [xk, hi), split at the ring's end
+            while (xk < hi) {
+                const int32_t slot = xk & (xw_slots - 1);
+                const int32_t run = min(hi - xk, xw_slots - slot);
+                const int64_t r0 = (int64_t)xk * 256, r1 = min((int64_t)(xk + run) * 256, x_avail & ~int64_t(1));
+                if (r1 > r0)
+                    bulk_g2s(xring + (size_t)slot * 2048, xsrc + r0, (uint32_t)((r1 - r0) * 8), bar, pol);
+                xk += run;
+            }
+        };
         int64_t o0 = 0, o1 = 0;
         uint32_t kd = 0;      // fused halo sync: tile kind of the lane's tile
+        int32_t chd = 0;      // XW: chunk end of the lane's tile
         int s = 0;
         uint32_t phase = 0;   // parity of the ring pass; reuse i >= S waits for pass (i / S - 1)'s release
         bool waited = false, bad = false;
@@ -340,15 +446,17 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
         for (int i = 0; i < my_tiles; ++i) {
             const int l = i & 31;
             if (l == 0) {   // offsets of tiles i .. i+31
-                const int t = c + (i + lane) * G;
+                const int t = t_begin + (i + lane) * t_step;
                 if (i + lane < my_tiles) {
                     o0 = __ldg(V.rec_off + t);
                     o1 = __ldg(V.rec_off + t + 1);
                     kd = fused ? (uint32_t)__ldg(V.hs.tile_kind + t) : 0u;
+                    if (XW) chd = __ldg(&V.xw_ch[t].y);
                 }
             }
             const int64_t b0 = __shfl_sync(0xffffffffu, o0, l), b1 = __shfl_sync(0xffffffffu, o1, l);
             const uint32_t kind = __shfl_sync(0xffffffffu, kd, l);
+            if (XW) ch_hi = __shfl_sync(0xffffffffu, chd, l);
             // first tiles were issued before the previous step ended; the stop
             // test comes before any ring reuse: on a stopped launch the
             // consumers release no stage, so waiting on empty[] would hang
@@ -356,6 +464,17 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
                 pdl_wait();
                 waited = true;
                 if (a.stop != nullptr && *a.stop) break;
+                if (XW) {   // the prologue tiles' iterate chunks (x is the previous step's output)
+                    for (int i2 = 0; i2 < pro; ++i2) {
+                        const int32_t h2 = __shfl_sync(0xffffffffu, chd, i2);
+                        if (lane == 0) {
+                            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(&full[i2])),
+                                         "r"(x_bytes(h2))
+                                         : "memory");
+                            x_issue(h2, &full[i2]);
+                        }
+                    }
+                }
                 if (fused) {   // gated tiles of the prologue: copied, not yet released
                     kstep = *(volatile const int64_t*)V.hs.local;
                     for (int i2 = 0; i2 < pro; ++i2) {
@@ -369,19 +488,21 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
             }
             if (i >= S) mbar_wait(&empty[s], phase ^ 1u);
             if (lane == 0) {
-                const int t = c + i * G;
-                const uint32_t bytes = (uint32_t)(b1 - b0);
+                const int t = t_begin + i * t_step;
+                uint32_t bytes = (uint32_t)(b1 - b0);
+                if (XW && i >= pro) bytes += x_bytes(ch_hi);
                 if (V.xpf) {
                     const int64_t r0 = (int64_t)t * NCW * 32, r1 = min(r0 + NCW * 32, a.n_rows);
                     if (r1 > r0) prefetch_l2(a.x + a.own_off + r0, (uint64_t)(r1 - r0) * 8);
                 }
-                if (kind)   // gated (fused halo sync): the arrival comes after the gate
+                if (kind || (XW && i < pro))   // gated (fused halo sync; XW prologue): the arrival comes later
                     asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(&full[s])),
                                  "r"(bytes)
                                  : "memory");
                 else
                     mbar_expect_tx(&full[s], bytes);
-                bulk_g2s(stages + (size_t)s * V.stage_bytes, V.rec + b0, bytes, &full[s], pol);
+                bulk_g2s(stages + (size_t)s * V.stage_bytes, V.rec + b0, (uint32_t)(b1 - b0), &full[s], pol);
+                if (XW && i >= pro) x_issue(ch_hi, &full[s]);
             }
             if (kind && i >= pro) {
                 hs_gate(V.hs, kind, kstep, bad);
@@ -392,6 +513,16 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
         if (!waited) {
             pdl_wait();
             const bool stopped = a.stop != nullptr && *a.stop;
+            if (XW)   // every tile fit the prologue: its chunks now (a stopped launch: release only)
+                for (int i2 = 0; i2 < pro; ++i2) {
+                    const int32_t h2 = __shfl_sync(0xffffffffu, chd, i2);
+                    if (lane == 0) {
+                        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(&full[i2])),
+                                     "r"(stopped ? 0u : x_bytes(h2))
+                                     : "memory");
+                        if (!stopped) x_issue(h2, &full[i2]);
+                    }
+                }
             if (fused) {   // every tile fit the prologue: release the gated ones
                 kstep = *(volatile const int64_t*)V.hs.local;
                 for (int i2 = 0; i2 < pro; ++i2) {
@@ -402,10 +533,10 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
                     }
                 }
             }
-        } else if (fused && a.stop != nullptr && *a.stop) {
+        } else if ((fused || XW) && a.stop != nullptr && *a.stop) {
             // stopped: the consumers drain the prologue stages; release gated ones
             for (int i2 = 0; i2 < pro; ++i2)
-                if (__shfl_sync(0xffffffffu, kd, i2 & 31) && lane == 0) mbar_arrive(&full[i2]);
+                if ((XW || __shfl_sync(0xffffffffu, kd, i2 & 31)) && lane == 0) mbar_arrive(&full[i2]);
         }
         if (bad && lane == 0) {
             V.hs.ctrl->status = CME_ERR_TIMEOUT;
@@ -442,8 +573,9 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
         mbar_wait(&dbar, 0u);
         int s = 0;
         uint32_t phase = 0;
-        int q = c * NCW + warp;                    // this warp's slice of tile c + i G
-        const int dq = G * NCW;
+        int q = t_begin * NCW + warp;              // this warp's slice of tile t_begin + i t_step
+        const int dq = t_step * NCW;
+        const uint32_t sxw = smem_u32(xring);
         uint32_t st = st0;
         for (int i = 0; i < my_tiles; ++i, q += dq) {
             mbar_wait_a(full0 + 8 * s, phase);
@@ -453,50 +585,22 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
                 const int ls = warp * 32 + lane;
                 const int r = REARR ? ((slot >> V.win_shift) << V.win_shift) + (int)lds_u8(st + R::kRow + ls) : slot;
                 const double* xr = xo + r;
-                const double x_r = __ldg(xr);
                 const uint32_t pv = st + R::kEnt + R::kEntBytes * meta.x + (ENC == 1 ? 4 : ENC == 2 ? 8 : 2) * lane;
                 // (ENC 0: the col16 block follows the vidx block; ENC 2: it follows the val_c block)
                 const uint32_t pc = F64 ? st + R::kEnt + 10 * meta.x + 256 * meta.y + 2 * lane : pv + 64 * meta.y;
-                double acc = 0.0;
-                if (F64) switch (meta.y) {   // warp-uniform exact widths
-                    case 0: break;
-                    case 1: acc = vi2_row_f<1>(pv, pc, xr); break;
-                    case 2: acc = vi2_row_f<2>(pv, pc, xr); break;
-                    case 3: acc = vi2_row_f<3>(pv, pc, xr); break;
-                    case 4: acc = vi2_row_f<4>(pv, pc, xr); break;
-                    case 5: acc = vi2_row_f<5>(pv, pc, xr); break;
-                    case 6: acc = vi2_row_f<6>(pv, pc, xr); break;
-                    case 7: acc = vi2_row_f<7>(pv, pc, xr); break;
-                    case 8: acc = vi2_row_f<8>(pv, pc, xr); break;
-                    default: acc = vi2_row_f_wide(pv, pc, xr, meta.y);
-                }
-                else if (ENC) switch (meta.y) {   // warp-uniform exact widths
-                    case 0: break;
-                    case 1: acc = vi2_row_w<1>(pv, sdict, xr); break;
-                    case 2: acc = vi2_row_w<2>(pv, sdict, xr); break;
-                    case 3: acc = vi2_row_w<3>(pv, sdict, xr); break;
-                    case 4: acc = vi2_row_w<4>(pv, sdict, xr); break;
-                    case 5: acc = vi2_row_w<5>(pv, sdict, xr); break;
-                    case 6: acc = vi2_row_w<6>(pv, sdict, xr); break;
-                    case 7: acc = vi2_row_w<7>(pv, sdict, xr); break;
-                    case 8: acc = vi2_row_w<8>(pv, sdict, xr); break;
-                    default: acc = vi2_row_w_wide(pv, sdict, xr, meta.y);
-                }
-                else switch (meta.y) {   // warp-uniform exact widths
-                    case 0: break;
-                    case 1: acc = vi2_row<1>(pv, pc, sdict, xr); break;
-                    case 2: acc = vi2_row<2>(pv, pc, sdict, xr); break;
-                    case 3: acc = vi2_row<3>(pv, pc, sdict, xr); break;
-                    case 4: acc = vi2_row<4>(pv, pc, sdict, xr); break;
-                    case 5: acc = vi2_row<5>(pv, pc, sdict, xr); break;
-                    case 6: acc = vi2_row<6>(pv, pc, sdict, xr); break;
-                    case 7: acc = vi2_row<7>(pv, pc, sdict, xr); break;
-                    case 8: acc = vi2_row<8>(pv, pc, sdict, xr); break;
-                    default: acc = vi2_row_wide(pv, pc, sdict, xr, meta.y);
+                double acc, x_r, xl = 0.0, xu = 0.0;
+                if (XW) {
+                    const GatherS gx{sxw, (uint32_t)(r + V.xw_off), (uint32_t)V.xw_mask};
+                    x_r = gx(0);
+                    acc = vi2_acc<ENC>(meta.y, pv, pc, sdict, gx);
+                    if (BAND) { xl = gx(-1); xu = gx(1); }
+                } else {
+                    x_r = __ldg(xr);
+                    acc = vi2_acc<ENC>(meta.y, pv, pc, sdict, GatherG{xr});
+                    if (BAND) { xl = __ldg(xr - 1); xu = __ldg(xr + 1); }
                 }
                 double sum = acc;
                 if (BAND) {
-                    const double xl = __ldg(xr - 1), xu = __ldg(xr + 1);
                     const double lo = F64 ? lds_f64(st + R::kLoUp + 8 * ls)
                                           : lds_f64(sdict + 8 * lds_u16(st + R::kLoUp + 2 * ls));
                     const double up = F64 ? lds_f64(st + R::kLoUp + NCW * 256 + 8 * ls)
@@ -521,7 +625,7 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, Vi2Shape<NCW>::kMinBl
             __syncwarp();
             if (lane == 0) {
                 if (fused) {
-                    const uint32_t kind = __ldg(V.hs.tile_kind + c + i * G);
+                    const uint32_t kind = __ldg(V.hs.tile_kind + t_begin + i * t_step);
                     if (kind) hs_signal(V.hs, kind, kstep);
                 }
                 mbar_arrive_a(empty0 + 8 * s);

@@ -717,7 +717,8 @@ def test_f64_records_bit_identical_to_compact(cme, oracle_mod, monkeypatch, warp
     x = W.random_start(A.n, 21)
     outs = {}
     for rec in ("0", "1"):
-        env = {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "0", "CME_REC": rec}   # (records are opt-in)
+        env = {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "0", "CME_REC": rec,   # (records are opt-in)
+               "CME_XW": "0"}   # (the x-window kernel has its own tests: test_xw.py)
         if rec == "1":
             env["CME_VI2_WARPS"] = str(warps)
             if grid:
