@@ -153,15 +153,15 @@ def kernel_name(info):
         info.kernel, "?")
 
 
-def build_matrix(cme, name, dev_mode, batch=1):
+def build_matrix(cme, name, dev_mode, batch=1, first=0):
     cfg = DEFAULTS[name]
     t0 = time.perf_counter()
-    if batch > 1:   # batched sweep: B rate sets on one pattern
+    if batch > 1 or first > 0:   # sweep members first .. first+B-1: B rate sets on one pattern
         vs = []
-        for net in W.sweep_networks(name, batch):
+        for net in W.sweep_networks(name, batch, first):
             states, r, c, v = cme.cme_network_enumerate(net)
             vs.append(v)
-        v = np.stack(vs)
+        v = np.stack(vs) if batch > 1 else vs[0]
     else:
         states, r, c, v = cme.cme_network_enumerate(W.config_network(name))
     t1 = time.perf_counter()
@@ -333,6 +333,26 @@ def converge_closed_form(cme, name="cfg3a_schnakenberg_2m", tol=1e-12):
     return out
 
 
+def replica_members(rank, batch):
+    """Replicas (`--replicas`): rank r solves sweep members [r B, r B + B) on its
+    own GPU -- independent problems, no data-path collective (P:L5, L17, L83:
+    the same network under different conditions)."""
+    return list(range(rank * batch, rank * batch + batch))
+
+
+def aggregate(dist, world, dev, ms, work):
+    """Whole-job numbers of a multi-rank run: the slowest rank's time and the
+    work of all ranks (flops), so value = total work / max time."""
+    if world == 1:
+        return ms, work
+    import torch
+    t = torch.tensor([ms], device=dev, dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    w = torch.tensor([work], device=dev, dtype=torch.float64)
+    dist.all_reduce(w, op=dist.ReduceOp.SUM)
+    return float(t.item()), float(w.item())
+
+
 def self_launch(nproc):
     """`bench.py --gpus N` outside torchrun: launch the N ranks ourselves (one
     process per GPU, the launcher the driver uses, rendezvous on 127.0.0.1)
@@ -358,6 +378,9 @@ def main():
     ap.add_argument("--no-converge", action="store_true")
     ap.add_argument("--batch", type=int, default=1, choices=[1, 2, 4, 8],
                     help="solve a sweep of B rate sets on the workload's pattern (SURVEY NEXT-1)")
+    ap.add_argument("--replicas", action="store_true",
+                    help="with --gpus N: every rank solves its own members of a parameter sweep on its own GPU "
+                         "(weak scaling, no data-path collective) instead of row-sharding one matrix")
     ap.add_argument("--transport", choices=["p2p", "nccl"], default=os.environ.get("CME_TRANSPORT", "p2p"),
                     help="multi-rank halo/record exchange: peer-memory stores from the step kernel + flag "
                          "barriers over CUDA IPC (p2p), or NCCL send/recv + allgather in the graphs (nccl)")
@@ -391,12 +414,15 @@ def main():
     import paper_conf_ipps_maggionibl13_b200 as cme
 
     comm = None
+    replicas = args.replicas and dist_path
     if dist_path:
         if shared_gpus:
             dist.init_process_group("gloo")
         else:
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        if args.transport == "nccl":
+        if replicas:
+            pass   # independent problems: the process group only carries the timing reductions
+        elif args.transport == "nccl":
             obj = [cme.cme_comm_unique_id() if rank == 0 else None]
             dist.broadcast_object_list(obj, src=0)
             comm = cme.cme_comm_init(world, rank, obj[0], local)
@@ -406,7 +432,9 @@ def main():
     name = args.config
     B = args.batch
     log("[bench] building", args.config)
-    m, cfg, setup = build_matrix(cme, name, cme.CME_DEVICE_HOST_ONLY if dist_path else local, B)
+    members = replica_members(rank, B) if replicas else list(range(B))
+    m, cfg, setup = build_matrix(cme, name, cme.CME_DEVICE_HOST_ONLY if dist_path and not replicas else local, B,
+                                 members[0])
     log("[bench] built", setup)
     if comm is not None:
         cme.cme_matrix_distribute(m.h, comm)
@@ -436,14 +464,14 @@ def main():
             cme.cme_solver_run(m.h, 1)
         e1.record(stream)
         barrier()
-    ms = e0.elapsed_time(e1)
-    if world > 1:
-        t = torch.tensor([ms], device=coll_dev, dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
     iters = args.steps * C_BLOCK
+    # whole job: max time over ranks; the flops of every rank (a replica run
+    # solves world independent problems, a row-sharded one a single matrix)
+    ms, work = aggregate(dist, world, coll_dev, e0.elapsed_time(e1), 2.0 * nnz * B * iters)
+    if not replicas:
+        work = 2.0 * nnz * B * iters
     sec = ms * 1e-3
-    gflops = 2.0 * nnz * B * iters / sec / 1e9
+    gflops = work / sec / 1e9
     peak, peak_src = hbm_peak()
     t_iter = sec / iters
     achieved = info.bytes_alg / t_iter / 1e9        # algorithmic bytes per launch / launch time
@@ -482,7 +510,7 @@ def main():
         tt = torch.tensor([e2e_s], device=coll_dev, dtype=torch.float64)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         e2e_s = float(tt.item())
-    e2e_gflops = 2.0 * nnz * B * C_BLOCK * e2e_steps / e2e_s / 1e9
+    e2e_gflops = (world if replicas else 1) * 2.0 * nnz * B * C_BLOCK * e2e_steps / e2e_s / 1e9
     clocks = clk.summary()
 
     # time-to-converge of the benchmark workload itself (BASELINE metric), on
@@ -536,15 +564,17 @@ def main():
         line = {
             "metric": "fp64 Jacobi GFLOPS (2 nnz/iteration)", "value": round(gflops, 3), "unit": "GFLOPS",
             "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": round(ms / args.steps, 4), "higher_is_better": True, "scaling": "strong",
+            "ms_per_step": round(ms / args.steps, 4), "higher_is_better": True,
+            "scaling": "weak" if replicas else "strong",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": name if B == 1 else f"{name} x {B}-member sweep", "batch": B,
+            "config": {"workload": (f"{name} sweep, {B} member(s) per rank" if replicas else
+                                    name if B == 1 else f"{name} x {B}-member sweep"), "batch": B,
                        "n": n, "nnz": nnz, "order": cfg["order"], "format": "diag_sell",
                        "window": cfg["window"], "band_on": bool(info.band_on), "omega": cfg["omega"],
                        "check_every": C_BLOCK, "iters_per_step": C_BLOCK,
                        "l2": f"inputs larger than L2 ({info.bytes_alg / 1e9:.3f} GB/iteration vs 126 MB)",
-                       "parallelism": f"rows{world}", "setup": setup,
-                       "transport": args.transport if dist_path else None},
+                       "parallelism": f"replicas{world}" if replicas else f"rows{world}", "setup": setup,
+                       "transport": None if replicas or not dist_path else args.transport},
             "iters_per_s": round(iters / sec, 2),
             "pct_hbm_roofline": round(100.0 * fmt_frac, 2) if fmt_frac is not None else None,
             "roofline": {"bound": "hbm", "achieved": round(fmt_gbs, 1) if fmt_gbs else None,
@@ -584,6 +614,9 @@ def main():
         dist.barrier()   # peers may address this rank's buffers until everyone is done
         m.close()
         cme.cme_comm_destroy(comm)
+        dist.destroy_process_group()
+    elif dist_path:
+        dist.barrier()
         dist.destroy_process_group()
     return 0
 

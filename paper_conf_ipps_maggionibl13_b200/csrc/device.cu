@@ -143,9 +143,9 @@ struct Device {
     int64_t* vi2_rec_off = nullptr;
     // x window in shared memory (XW; single GPU): per tile
     // the iterate chunks it gathers, streamed with its record
-    bool xw = false;
+    int xw = 0;                      // 1 mirrored ring, 2 ring with a wrap per entry
     int2* xw_ch = nullptr;           // [vi2 tiles] {first chunk, end chunk} (monotone)
-    int xw_mask = 0, xw_off = 0, xw_ring_bytes = 0;
+    int xw_rows = 0, xw_mirror = 0, xw_off = 0, xw_ring_bytes = 0;
     int64_t xw_nx = 0;
     // wavefront s-step kernel over the tile records (kernels_wf.cuh): one
     // launch per s steps of a check block (single GPU, vi2 shapes)
@@ -690,7 +690,7 @@ static cme_status configure_vi2(Device& d, const Packed& P, bool f64 = false) {
 // chunks a CTA needs with S stages in flight: tiles j-S+1 .. j are live when
 // tile j's chunks are issued (tile j-S has released its stage).
 static int64_t xw_plan(const Packed& P, int ts, bool band, int64_t own_off, int xoff, int64_t nx, int S,
-                       std::vector<int2>& ch) {
+                       std::vector<int2>& ch, int64_t& span) {
     const int64_t nt = (P.n_slices + ts - 1) / ts, n = P.n;
     std::vector<int64_t> lo(nt), hi(nt);
 #pragma omp parallel for schedule(dynamic, 64)
@@ -718,29 +718,66 @@ static int64_t xw_plan(const Packed& P, int ts, bool band, int64_t own_off, int 
     for (int64_t t = nt - 2; t >= 0; --t) lo[t] = std::min(lo[t], lo[t + 1]);
     for (int64_t t = 1; t < nt; ++t) hi[t] = std::max(hi[t], hi[t - 1]);
     int64_t need = 1;
+    span = 1;
     ch.resize(nt);
     for (int64_t t = 0; t < nt; ++t) {
         need = std::max(need, hi[t] - lo[std::max<int64_t>(0, t - S + 1)]);
+        span = std::max(span, hi[t] - lo[t]);
         ch[t] = make_int2((int)lo[t], (int)hi[t]);
     }
     return need;
 }
 
+// Mean distinct 32-byte sectors per warp-wide x gather (32 lanes' t-th
+// entries of a slice), over every 16th slice: ~8-9 when consecutive rows
+// gather consecutive columns (the CME orderings, cfg3a's grid band), up to 32
+// for a random band (config 5).  Decides whether the x window pays.
+static double gather_sectors(const Packed& P) {
+    double sum = 0;
+    int64_t cnt = 0;
+#pragma omp parallel for schedule(dynamic, 64) reduction(+ : sum, cnt)
+    for (int64_t q = 0; q < P.n_slices; q += 16) {
+        for (int32_t t = 0; t < P.slice_w[q]; ++t) {
+            int64_t sec[32];
+            int k = 0;
+            for (int ln = 0; ln < 32; ++ln) {
+                if (q * 32 + ln >= P.n) break;
+                sec[k++] = (int64_t)P.col[P.slice_off[q] + ln + 32 * t] >> 2;
+            }
+            if (!k) continue;
+            std::sort(sec, sec + k);
+            sum += (double)(std::unique(sec, sec + k) - sec);
+            ++cnt;
+        }
+    }
+    return cnt ? sum / cnt : 0.0;
+}
+
 // The x-window shape (single GPU; records of the value-indexed encoding, or
 // of the f64 compact one when there is no value index): the first of
-// (30 warps, 4 | 3 stages), (16, 4 | 3), (30, 2), (16, 2) whose stages,
-// dictionary and power-of-two x ring fit one CTA per SM.  CME_XW = 1 forces
-// it, 0 disables it; auto (-1) takes it for the f64 records when the ring is
-// <= 64 KB -- measured on config 5 (n = 16 M, mu = 10): width 1 024 290 us vs
-// 403 us on sell_cpt_kernel, width 32 283 vs 309 -- and not for the wide
-// windows of the CME orderings (cfg4 RCM: a 128 KB ring leaves 16 warps x 2
-// stages, 237 us vs 173; cfg3a: 21.2 vs 19.1 us).
+// (30 warps, 4 | 3 stages), (16, 4 | 3), (30, 2), (16, 2) whose dictionary,
+// stages and ring fit one CTA per SM, for the mirrored ring (XWM 1) if any
+// shape fits it, else for the ring with a wrap per entry (XWM 2).  CME_XW = 1
+// forces the x window, 0 disables it; auto (-1) takes it for f64 records whose
+// x gathers are uncoalesced (>= 16 sectors per warp request) with a ring of at
+// most CME_XW_RING_KB (96) KB.  Measured (B200): config 5
+// (16 M rows, mu = 10, random band) width 1 024 291 us vs 410 on
+// sell_cpt_kernel, width 4 096 356 vs 643; coalesced gathers lose: cfg3a
+// 28.7 vs 19.1 us, toggle N = 2 200 (RCM) 133 vs 79 us.
 static cme_status configure_xw(Device& d, const Packed& P, bool f64, std::vector<int2>& plan) {
-    d.xw = false;
+    d.xw = 0;
     const int want = env_int("CME_XW", -1);
     if (want == 0 || d.nranks > 1 || d.B != 1 || (want < 0 && !f64)) return CME_OK;
-    const int xoff = (int)((reinterpret_cast<uintptr_t>(d.xb[0] + d.own_off) >> 3) & 1);
-    if (xoff != (int)((reinterpret_cast<uintptr_t>(d.xb[1] + d.own_off) >> 3) & 1)) return CME_OK;
+    if (want < 0) {
+        const double sec = gather_sectors(P);
+        if (env_int("CME_VERBOSE", 0)) std::fprintf(stderr, "[cme] xw: %.1f sectors per x gather\n", sec);
+        if (sec < 16.0) return CME_OK;
+    }
+    // chunk k starts at local row 256 k - 1: 16-B aligned when x + own_off is 8 mod 16 (the
+    // x-span buffers sit one sentinel row into 256-B aligned allocations), row -1 loadable
+    const int xoff = 1;
+    for (int b = 0; b < 2; ++b)
+        if (((reinterpret_cast<uintptr_t>(d.xb[b] + d.own_off) >> 3) & 1) != 1) return CME_OK;
     int dev = 0, smem_max = 0, sms = 0;
     CUDA_TRY(cudaGetDevice(&dev));
     CUDA_TRY(cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
@@ -749,10 +786,13 @@ static cme_status configure_xw(Device& d, const Packed& P, bool f64, std::vector
     const int dict = f64 ? 0 : d.dict_bytes;
     const int force_w = env_int("CME_VI2_WARPS", 0), force_s = env_int("CME_VI2_STAGES", 0);
     const int64_t nx = d.nx - d.own_off;
-    const int64_t ring_cap = want > 0 ? INT64_MAX : (int64_t)64 << 10;
+    const int64_t ring_cap = want > 0 ? INT64_MAX : (int64_t)env_int("CME_XW_RING_KB", 96) << 10;
     int64_t stage_of[2] = {0, 0};   // [30 warps, 16 warps]
     const int order[6][2] = {{30, 4}, {30, 3}, {16, 4}, {16, 3}, {30, 2}, {16, 2}};
+    const int force_m = env_int("CME_XW_MODE", 0);   // 1 mirror, 2 wrap (tests)
+    for (int mode = 1; mode <= 2; ++mode)
     for (const auto& sh : order) {
+        if (force_m && mode != force_m) continue;
         const int ncw = sh[0];
         if (force_w && ncw != force_w) continue;
         const int st = force_s > 0 ? std::min(force_s, 8) : sh[1];
@@ -767,18 +807,18 @@ static cme_status configure_xw(Device& d, const Packed& P, bool f64, std::vector
         }
         {
             std::vector<int2> ch;
-            const int64_t need = xw_plan(P, ncw, d.band, d.own_off, xoff, nx, st, ch);
-            int64_t slots = 1;
-            while (slots < need) slots <<= 1;
-            const int64_t bytes = dict + st * stage + slots * 2048;
+            int64_t span = 1;
+            const int64_t need = xw_plan(P, ncw, d.band, d.own_off, xoff, nx, st, ch, span);
+            const int64_t slots = need, mirror = mode == 1 ? span - 1 : 0;
+            const int64_t bytes = dict + st * stage + (slots + mirror) * 2048;
             if (env_int("CME_VERBOSE", 0) > 1)
                 std::fprintf(stderr, "[cme] xw shape: ncw=%d stages=%d stage=%lld ring chunks=%lld (need %lld) smem=%lld\n",
                              ncw, st, (long long)stage, (long long)slots, (long long)need, (long long)bytes);
-            if (bytes > cap || slots * 2048 > ring_cap) continue;
+            if (bytes > cap || (slots + mirror) * 2048 > ring_cap) continue;
             int occ = 0;
             CUDA_TRY(vi2_xw_occupancy(ncw, (int)bytes, &occ, enc));
             if (occ < 1) continue;
-            d.xw = true;
+            d.xw = mode;
             d.vi2 = true;
             d.vi2_f64 = f64;
             d.vi2_words = false;
@@ -790,14 +830,15 @@ static cme_status configure_xw(Device& d, const Packed& P, bool f64, std::vector
             d.vi2_tiles = nt;
             d.vi2_grid = (int)std::min<int64_t>(nt, (int64_t)sms * occ);
             if (env_int("CME_VI2_GRID", 0) > 0) d.vi2_grid = std::min(d.vi2_grid, env_int("CME_VI2_GRID", 0));
-            d.xw_mask = (int)(slots * 256 - 1);
+            d.xw_rows = (int)(slots * 256);
+            d.xw_mirror = (int)mirror;
             d.xw_off = xoff;
             d.xw_nx = nx;
-            d.xw_ring_bytes = (int)(slots * 2048);
+            d.xw_ring_bytes = (int)((slots + mirror) * 2048);
             plan.swap(ch);
             if (env_int("CME_VERBOSE", 0))
-                std::fprintf(stderr, "[cme] xw: warps=%d stages=%d stage_bytes=%d ring=%d KB occ=%d grid=%d tiles=%lld\n",
-                             ncw, st, d.vi2_stage_bytes, d.xw_ring_bytes / 1024, occ, d.vi2_grid, (long long)nt);
+                std::fprintf(stderr, "[cme] xw: mode=%d warps=%d stages=%d stage_bytes=%d ring=%d KB occ=%d grid=%d tiles=%lld\n",
+                             mode, ncw, st, d.vi2_stage_bytes, d.xw_ring_bytes / 1024, occ, d.vi2_grid, (long long)nt);
             return CME_OK;
         }
     }
@@ -1589,13 +1630,14 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
         }
         if (d.xw) {
             V.xw_ch = d.xw_ch;
-            V.xw_mask = d.xw_mask;
+            V.xw_rows = d.xw_rows;
+            V.xw_mirror = d.xw_mirror;
             V.xw_off = d.xw_off;
             V.xw_nx = d.xw_nx;
             V.xpf = 0;
             CUDA_TRY(launch_vi2_xw(V, d.vi2_ncw, d.vi2_grid,
                                    d.dict_bytes + d.vi2_stages * d.vi2_stage_bytes + d.xw_ring_bytes, d.band, d.rearr,
-                                   check, d.vi2_f64 ? 2 : 0, pdl, s));
+                                   check, d.vi2_f64 ? 2 : 0, d.xw, pdl, s));
         } else
             CUDA_TRY(launch_vi2(V, d.vi2_ncw, d.vi2_grid, d.dict_bytes + d.vi2_stages * d.vi2_stage_bytes, d.band,
                                 d.rearr, check, d.vi2_f64 ? 2 : d.vi2_words ? 1 : 0, pdl, s));

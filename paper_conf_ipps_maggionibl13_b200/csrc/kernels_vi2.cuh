@@ -134,11 +134,14 @@ struct Vi2Args {
     HaloSync hs;                // fused halo synchronisation (hs.on = 0: none)
     // x window in shared memory (XW kernels): chunk k of
     // the ring holds the iterate rows [256 k - xw_off, 256 k - xw_off + 256)
-    // (relative to x + own_off) at ring slot k & (xw_mask >> 8); tile t needs
-    // chunks [xw_ch[t].x, xw_ch[t].y) (suffix-min / prefix-max: both monotone)
+    // (relative to x + own_off) at ring slot k mod NX (NX = xw_rows / 256),
+    // and slots 0 .. xw_mirror-1 again at NX .. NX+xw_mirror-1, so that a
+    // tile's chunks are contiguous in shared memory (no wrap in the gathers);
+    // tile t needs chunks [xw_ch[t].x, xw_ch[t].y) (suffix-min / prefix-max)
     const int2* xw_ch;
-    int32_t xw_mask;            // ring rows - 1 (a power of two >= 256)
-    int32_t xw_off;             // 1 when x + own_off is 8 mod 16 (bulk copies need 16-B sources)
+    int32_t xw_rows;            // ring rows (a multiple of 256) without the mirror
+    int32_t xw_mirror;          // mirrored chunks (>= the widest tile's chunks - 1)
+    int32_t xw_off;             // 1: x + own_off is 8 mod 16 (bulk copies need 16-B sources; row -1 loadable)
     int64_t xw_nx;              // iterate rows readable from x + own_off (a sentinel row at -1 and nx)
 };
 
@@ -208,17 +211,23 @@ __device__ __forceinline__ int2 lds_v2(uint32_t a) {
 }
 
 // x gathers: from global memory (L1/L2; the iterate row r is xr[0]) or from
-// the shared-memory x window (XW: ring index (r + off + xw_off) & mask)
+// the shared-memory x window (XW)
 struct GatherG {
     const double* xr;
     __device__ __forceinline__ double operator()(int32_t o) const { return __ldg(xr + o); }
 };
 struct GatherS {
-    uint32_t xs;     // ring base (shared window)
-    uint32_t rx;     // r + xw_off
-    uint32_t mask;
+    uint32_t xr;     // shared-window address of row r in the (mirrored) ring
+    __device__ __forceinline__ double operator()(int32_t o) const { return lds_f64(xr + ((uint32_t)o << 3)); }
+};
+struct GatherW {     // ring without the mirror: one conditional wrap per entry
+    uint32_t xs;     // ring base
+    uint32_t rx;     // ring index of row r before the wrap (the tile's rows lie in [0, 2 rows))
+    uint32_t rows;
     __device__ __forceinline__ double operator()(int32_t o) const {
-        return lds_f64(xs + (((rx + (uint32_t)o) & mask) << 3));
+        uint32_t v = rx + (uint32_t)o;
+        v = v >= rows ? v - rows : v;
+        return lds_f64(xs + (v << 3));
     }
 };
 
@@ -363,22 +372,24 @@ struct Vi2Shape {
 // range of tiles and the producer streams the iterate rows those tiles gather
 // into a shared-memory ring with the tile records (same mbarriers), so every
 // x read of the step is a shared-memory load.  Single-GPU packs only.
-template <int NCW, bool BAND, bool REARR, bool CHECK, int ENC, bool XW = false>
-__global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, XW ? 1 : Vi2Shape<NCW>::kMinBlocks)
+template <int NCW, bool BAND, bool REARR, bool CHECK, int ENC, int XWM = 0>
+__global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, XWM ? 1 : Vi2Shape<NCW>::kMinBlocks)
     sell_vi2_kernel(const __grid_constant__ Vi2Args V) {
+    constexpr bool XW = XWM != 0;   // 1: mirrored ring, 2: ring with a wrap per entry
     constexpr bool F64 = ENC == 2;
     using R = Vi2Rec<NCW, BAND, REARR, F64>;
     const StepArgs& a = V.a;
     pdl_trigger();
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ uint64_t full[8], empty[8], dbar;
+    __shared__ int32_t xoffs[8];   // XW: per stage, ring index of row 0 of its tile's first chunk, minus 256 * chunk
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int S = V.stages;
     unsigned char* stages = smem + V.dict_bytes;
     unsigned char* xring = stages + (size_t)S * V.stage_bytes;
     if (XW) {   // rows the ring has not received (row -1 when xw_off = 0) read as 0
         uint4* z = reinterpret_cast<uint4*>(xring);
-        const int nz = (V.xw_mask + 1) / 2;
+        const int nz = (V.xw_rows + 256 * V.xw_mirror) / 2;
         for (int k = threadIdx.x; k < nz; k += blockDim.x) z[k] = make_uint4(0u, 0u, 0u, 0u);
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // before the bulk copies overwrite it
     }
@@ -414,30 +425,44 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, XW ? 1 : Vi2Shape<NCW
             mbar_arrive(&dbar);   // (F64 records: no dictionary)
         }
         // XW: next iterate chunk to stream (chunks are issued in increasing order)
-        int32_t ch_hi = 0;
+        int32_t ch_hi = 0, ch_lo = 0;
         int32_t xk = XW && my_tiles > 0 ? __ldg(&V.xw_ch[t_begin].x) : 0;
         const double* xsrc = a.x + a.own_off - V.xw_off;   // 16-B aligned: chunk k starts at xsrc + 256 k
-        const int32_t xw_slots = (V.xw_mask + 1) >> 8;
+        const int32_t xw_slots = V.xw_rows >> 8;
+        // lane 0, before the stage's arrival: where the tile's first chunk sits in the ring
+        auto x_base = [&](int st_, int32_t lo) { xoffs[st_] = V.xw_off + (lo % xw_slots - lo) * 256; };
         const int64_t x_avail = V.xw_nx + 1 + V.xw_off;    // rows readable from xsrc (through the sentinel at nx)
-        // bytes of chunks [xk, hi) (pure arithmetic; lane 0 then issues them)
-        auto x_bytes = [&](int32_t hi) -> uint32_t {
-            if (hi <= xk) return 0u;
-            const int64_t r0 = (int64_t)xk * 256, r1 = min((int64_t)hi * 256, x_avail & ~int64_t(1));
-            return r1 > r0 ? (uint32_t)((r1 - r0) * 8) : 0u;
-        };
-        auto x_issue = [&](int32_t hi, uint64_t* bar) {   // lane 0: chunks [xk, hi), split at the ring's end
-            while (xk < hi) {
-                const int32_t slot = xk & (xw_slots - 1);
-                const int32_t run = min(hi - xk, xw_slots - slot);
-                const int64_t r0 = (int64_t)xk * 256, r1 = min((int64_t)(xk + run) * 256, x_avail & ~int64_t(1));
-                if (r1 > r0)
-                    bulk_g2s(xring + (size_t)slot * 2048, xsrc + r0, (uint32_t)((r1 - r0) * 8), bar, pol);
-                xk += run;
+        // chunks [xk, hi): runs split at the ring's end, the slots below the
+        // mirror copied twice; issue = false only counts the bytes (lane 0)
+        auto x_chunks = [&](int32_t hi, uint64_t* bar, bool issue) -> uint32_t {
+            uint32_t bytes = 0;
+            for (int32_t k = xk; k < hi;) {
+                const int32_t slot = k % xw_slots;
+                const int32_t run = min(hi - k, xw_slots - slot);
+                const int64_t r0 = (int64_t)k * 256, r1 = min((int64_t)(k + run) * 256, x_avail & ~int64_t(1));
+                if (r1 > r0) {
+                    bytes += (uint32_t)((r1 - r0) * 8);
+                    if (issue) bulk_g2s(xring + (size_t)slot * 2048, xsrc + r0, (uint32_t)((r1 - r0) * 8), bar, pol);
+                }
+                if (slot < V.xw_mirror) {
+                    const int64_t m1 = min((int64_t)(k + min(run, V.xw_mirror - slot)) * 256, x_avail & ~int64_t(1));
+                    if (m1 > r0) {
+                        bytes += (uint32_t)((m1 - r0) * 8);
+                        if (issue)
+                            bulk_g2s(xring + (size_t)(xw_slots + slot) * 2048, xsrc + r0, (uint32_t)((m1 - r0) * 8),
+                                     bar, pol);
+                    }
+                }
+                k += run;
             }
+            if (issue) xk = max(xk, hi);
+            return bytes;
         };
+        auto x_bytes = [&](int32_t hi) -> uint32_t { return x_chunks(hi, nullptr, false); };
+        auto x_issue = [&](int32_t hi, uint64_t* bar) { x_chunks(hi, bar, true); };
         int64_t o0 = 0, o1 = 0;
         uint32_t kd = 0;      // fused halo sync: tile kind of the lane's tile
-        int32_t chd = 0;      // XW: chunk end of the lane's tile
+        int32_t chd = 0, chl = 0;   // XW: chunk range of the lane's tile
         int s = 0;
         uint32_t phase = 0;   // parity of the ring pass; reuse i >= S waits for pass (i / S - 1)'s release
         bool waited = false, bad = false;
@@ -451,12 +476,19 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, XW ? 1 : Vi2Shape<NCW
                     o0 = __ldg(V.rec_off + t);
                     o1 = __ldg(V.rec_off + t + 1);
                     kd = fused ? (uint32_t)__ldg(V.hs.tile_kind + t) : 0u;
-                    if (XW) chd = __ldg(&V.xw_ch[t].y);
+                    if (XW) {
+                        const int2 ch = __ldg(&V.xw_ch[t]);
+                        chl = ch.x;
+                        chd = ch.y;
+                    }
                 }
             }
             const int64_t b0 = __shfl_sync(0xffffffffu, o0, l), b1 = __shfl_sync(0xffffffffu, o1, l);
             const uint32_t kind = __shfl_sync(0xffffffffu, kd, l);
-            if (XW) ch_hi = __shfl_sync(0xffffffffu, chd, l);
+            if (XW) {
+                ch_hi = __shfl_sync(0xffffffffu, chd, l);
+                ch_lo = __shfl_sync(0xffffffffu, chl, l);
+            }
             // first tiles were issued before the previous step ended; the stop
             // test comes before any ring reuse: on a stopped launch the
             // consumers release no stage, so waiting on empty[] would hang
@@ -466,8 +498,9 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, XW ? 1 : Vi2Shape<NCW
                 if (a.stop != nullptr && *a.stop) break;
                 if (XW) {   // the prologue tiles' iterate chunks (x is the previous step's output)
                     for (int i2 = 0; i2 < pro; ++i2) {
-                        const int32_t h2 = __shfl_sync(0xffffffffu, chd, i2);
+                        const int32_t h2 = __shfl_sync(0xffffffffu, chd, i2), l2 = __shfl_sync(0xffffffffu, chl, i2);
                         if (lane == 0) {
+                            x_base(i2, l2);
                             asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(&full[i2])),
                                          "r"(x_bytes(h2))
                                          : "memory");
@@ -490,7 +523,10 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, XW ? 1 : Vi2Shape<NCW
             if (lane == 0) {
                 const int t = t_begin + i * t_step;
                 uint32_t bytes = (uint32_t)(b1 - b0);
-                if (XW && i >= pro) bytes += x_bytes(ch_hi);
+                if (XW && i >= pro) {
+                    bytes += x_bytes(ch_hi);
+                    x_base(s, ch_lo);
+                }
                 if (V.xpf) {
                     const int64_t r0 = (int64_t)t * NCW * 32, r1 = min(r0 + NCW * 32, a.n_rows);
                     if (r1 > r0) prefetch_l2(a.x + a.own_off + r0, (uint64_t)(r1 - r0) * 8);
@@ -515,8 +551,9 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, XW ? 1 : Vi2Shape<NCW
             const bool stopped = a.stop != nullptr && *a.stop;
             if (XW)   // every tile fit the prologue: its chunks now (a stopped launch: release only)
                 for (int i2 = 0; i2 < pro; ++i2) {
-                    const int32_t h2 = __shfl_sync(0xffffffffu, chd, i2);
+                    const int32_t h2 = __shfl_sync(0xffffffffu, chd, i2), l2 = __shfl_sync(0xffffffffu, chl, i2);
                     if (lane == 0) {
+                        x_base(i2, l2);
                         asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(&full[i2])),
                                      "r"(stopped ? 0u : x_bytes(h2))
                                      : "memory");
@@ -579,6 +616,7 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, XW ? 1 : Vi2Shape<NCW
         uint32_t st = st0;
         for (int i = 0; i < my_tiles; ++i, q += dq) {
             mbar_wait_a(full0 + 8 * s, phase);
+            const int32_t xo_t = XW ? xoffs[s] : 0;   // (written by the producer before the stage's arrival)
             const int slot = q * 32 + lane;
             if (q < slice_end && slot < n_rows) {
                 const int2 meta = lds_v2(st + 8 * warp);   // {entry offset in the tile, width}
@@ -589,8 +627,13 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, XW ? 1 : Vi2Shape<NCW
                 // (ENC 0: the col16 block follows the vidx block; ENC 2: it follows the val_c block)
                 const uint32_t pc = F64 ? st + R::kEnt + 10 * meta.x + 256 * meta.y + 2 * lane : pv + 64 * meta.y;
                 double acc, x_r, xl = 0.0, xu = 0.0;
-                if (XW) {
-                    const GatherS gx{sxw, (uint32_t)(r + V.xw_off), (uint32_t)V.xw_mask};
+                if (XWM == 1) {
+                    const GatherS gx{sxw + 8u * (uint32_t)(r + xo_t)};
+                    x_r = gx(0);
+                    acc = vi2_acc<ENC>(meta.y, pv, pc, sdict, gx);
+                    if (BAND) { xl = gx(-1); xu = gx(1); }
+                } else if (XWM == 2) {
+                    const GatherW gx{sxw, (uint32_t)(r + xo_t), (uint32_t)V.xw_rows};
                     x_r = gx(0);
                     acc = vi2_acc<ENC>(meta.y, pv, pc, sdict, gx);
                     if (BAND) { xl = gx(-1); xu = gx(1); }

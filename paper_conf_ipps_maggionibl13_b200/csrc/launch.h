@@ -70,7 +70,7 @@ cudaError_t vi2_prepare(int ncw, int smem);
 cudaError_t vi2_occupancy(int ncw, int smem, int* blocks_per_sm, int enc = 0);
 // the x-window variant (step_xw.cu): ncw = 16 or 30, enc 0 or 2
 cudaError_t launch_vi2_xw(const Vi2Args& V, int ncw, int grid, int smem, bool band, bool rearr, bool check, int enc,
-                          bool pdl, cudaStream_t s);
+                          int mode /* 1 mirrored ring, 2 wrap */, bool pdl, cudaStream_t s);
 cudaError_t vi2_xw_prepare(int ncw, int smem);
 cudaError_t vi2_xw_occupancy(int ncw, int smem, int* blocks_per_sm, int enc);
 struct ResArgs;

@@ -65,3 +65,38 @@ def test_gpus_flag_self_launches_ranks():
     assert len(lines) == 1
     assert json.loads(lines[0])["n_gpus"] == 2
     assert "launching" in r.stderr
+
+
+def _agg_worker(rank, world, port, outq):
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    sys.path.insert(0, ROOT)
+    import bench
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    ms, work = bench.aggregate(dist, world, "cpu", 10.0 + rank, 1e9 * (rank + 1))
+    outq.put((rank, ms, work, bench.replica_members(rank, 4)))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_replica_aggregation_gloo():
+    """`bench.py --replicas`: every rank solves its own sweep members (disjoint,
+    covering 0 .. world*B-1); the whole-job value is the work of all ranks over
+    the slowest rank's time (world_size 2 over gloo, 127.0.0.1)."""
+    import multiprocessing as mp
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    ps = [ctx.Process(target=_agg_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    out = sorted(q.get(timeout=120) for _ in ps)
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for rank, ms, work, members in out:
+        assert ms == 11.0 and work == 3e9
+    assert out[0][3] + out[1][3] == list(range(8))

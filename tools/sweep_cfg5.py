@@ -36,7 +36,8 @@ def points(quick):
     if quick:
         return [(1 * M, 10, 1024, False), (4 * M, 10, 32, False), (4 * M, 10, 4 * M, False)]
     pts = [(n, 10, 1024, False) for n in (1 * M, 4 * M, 16 * M, 64 * M, 100 * M)]
-    pts += [(16 * M, 10, w, False) for w in (32, 32768, 1 * M, 16 * M)]
+    pts += [(16 * M, 10, w, False) for w in (32, 4096, 8192, 32768, 1 * M, 16 * M)]
+    pts += [(16 * M, 10, 4096, True)]
     pts += [(16 * M, mu, 1024, irr) for mu in (5, 7, 15) for irr in (False, True)]
     pts += [(16 * M, 10, 1024, True), (64 * M, 10, 32768, True)]
     return pts
@@ -77,7 +78,7 @@ def run_point(n, mu, w, irr, blocks, C=100):
     torch.cuda.synchronize()
     ti = e0.elapsed_time(e1) * 1e-3 / (blocks * C)
     out = dict(n=n, mu=mu, width=w, irregular=irr, nnz=int(f.nnz), kernel=int(f.kernel), band_on=int(f.band_on),
-               encoding=int(f.compact),
+               encoding=int(f.compact), records=int(f.records), xwin_kb=int(f.xwin_kb),
                us_per_iter=ti * 1e6, gflops=2 * f.nnz / ti / 1e9, alg_gbs=f.bytes_alg / ti / 1e9,
                fmt_gbs=f.bytes_fmt / ti / 1e9, bytes_alg=int(f.bytes_alg), bytes_fmt=int(f.bytes_fmt),
                mass_invariant_rel=float(inv), gen_s=round(t_gen, 2), ingest_pack_s=round(t_pack, 2))
@@ -122,7 +123,10 @@ def main():
                 "fmt GB/s | % peak (fmt) |\n|---|---|---|---|---|---|---|---|---|---|---|---|\n")
         for o in rows:
             f.write(f"| {o['n']:,} | {o['mu']} | {o['width']:,} | {int(o['irregular'])} | {o['nnz']:,} | "
-                    f"{kn.get(o['kernel'], o['kernel'])}{enc.get(o.get('encoding', 0), '')} | {o['us_per_iter']:.1f} | {o['gflops']:.0f} | "
+                    f"{kn.get(o['kernel'], o['kernel'])}{enc.get(o.get('encoding', 0), '')}"
+                    f"{' + records' if o.get('records') else ''}"
+                    f"{(' + x window %d KB' % o['xwin_kb']) if o.get('xwin_kb') else ''} | "
+                    f"{o['us_per_iter']:.1f} | {o['gflops']:.0f} | "
                     f"{o['alg_gbs']:.0f} | {100 * o['frac_alg']:.1f} | {o['fmt_gbs']:.0f} | "
                     f"{100 * o['frac_fmt']:.1f} |\n")
 

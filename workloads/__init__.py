@@ -186,12 +186,13 @@ def config_network(name: str) -> Network:
 SWEEP_FACTORS = [1.0, 0.7, 1.3, 2.0, 0.5, 1.1, 0.9, 1.6]
 
 
-def sweep_networks(name: str, batch: int):
-    """`batch` variants of config `name`: reaction k of member b has rate
-    r_k * SWEEP_FACTORS[b] ** (+1 for even k, -0.5 for odd k)."""
+def sweep_networks(name: str, batch: int, first: int = 0):
+    """`batch` variants of config `name` (sweep members first .. first+batch-1):
+    reaction k of member b has rate r_k * SWEEP_FACTORS[b] ** (+1 for even k,
+    -0.5 for odd k); member 0 is the configuration itself."""
     base = config_network(name)
     out = []
-    for b in range(batch):
+    for b in range(first, first + batch):
         f = SWEEP_FACTORS[b % len(SWEEP_FACTORS)]
         rates = [r * (f if k % 2 == 0 else f ** -0.5) for k, r in enumerate(base.rates)]
         out.append(Network(name=f"{base.name}_sweep{b}", species=base.species, x0=base.x0,
