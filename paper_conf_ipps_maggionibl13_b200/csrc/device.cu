@@ -760,7 +760,7 @@ static double gather_sectors(const Packed& P) {
 // shape fits it, else for the ring with a wrap per entry (XWM 2).  CME_XW = 1
 // forces the x window, 0 disables it; auto (-1) takes it for f64 records whose
 // x gathers are uncoalesced (>= 16 sectors per warp request) with a ring of at
-// most CME_XW_RING_KB (96) KB.  Measured (B200): config 5
+// most CME_XW_RING_KB (160) KB.  Measured (B200): config 5
 // (16 M rows, mu = 10, random band) width 1 024 291 us vs 410 on
 // sell_cpt_kernel, width 4 096 356 vs 643; coalesced gathers lose: cfg3a
 // 28.7 vs 19.1 us, toggle N = 2 200 (RCM) 133 vs 79 us.
@@ -786,8 +786,10 @@ static cme_status configure_xw(Device& d, const Packed& P, bool f64, std::vector
     const int dict = f64 ? 0 : d.dict_bytes;
     const int force_w = env_int("CME_VI2_WARPS", 0), force_s = env_int("CME_VI2_STAGES", 0);
     const int64_t nx = d.nx - d.own_off;
-    const int64_t ring_cap = want > 0 ? INT64_MAX : (int64_t)env_int("CME_XW_RING_KB", 96) << 10;
+    const int64_t ring_cap = want > 0 ? INT64_MAX : (int64_t)env_int("CME_XW_RING_KB", 160) << 10;
     int64_t stage_of[2] = {0, 0};   // [30 warps, 16 warps]
+    // (8-warp tiles, for windows too wide for these: measured 587 vs 420 us on
+    // config 5 width 8 192 -- too few warps once the gathers are shared loads)
     const int order[6][2] = {{30, 4}, {30, 3}, {16, 4}, {16, 3}, {30, 2}, {16, 2}};
     const int force_m = env_int("CME_XW_MODE", 0);   // 1 mirror, 2 wrap (tests)
     for (int mode = 1; mode <= 2; ++mode)
@@ -1610,6 +1612,7 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
     } else if (d.vi2) {
         Vi2Args V{a, d.vi2_rec, d.vi2_rec_off, d.dict, d.vi2_tiles, d.vi2_stages, d.vi2_stage_bytes, d.dict_bytes,
                   d.win_shift, d.tma_xpf};
+        V.contig = env_int("CME_VI2_CONTIG", 0);
         if (d.fused) {
             HaloSync& hs = V.hs;
             hs.on = 1;

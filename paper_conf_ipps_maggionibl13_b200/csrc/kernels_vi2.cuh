@@ -143,6 +143,7 @@ struct Vi2Args {
     int32_t xw_mirror;          // mirrored chunks (>= the widest tile's chunks - 1)
     int32_t xw_off;             // 1: x + own_off is 8 mod 16 (bulk copies need 16-B sources; row -1 loadable)
     int64_t xw_nx;              // iterate rows readable from x + own_off (a sentinel row at -1 and nx)
+    int32_t contig;             // gather kernels: contiguous tile ranges per CTA (CME_VI2_CONTIG) instead of c + i G
 };
 
 // Record layout of a tile of TS slices (byte offsets; every block 16-B aligned).
@@ -406,10 +407,11 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, XWM ? 1 : Vi2Shape<NC
     const int n_tiles = (int)V.n_tiles;
     // tiles of this CTA: XW a contiguous range [t_begin, t_begin + my_tiles),
     // else c, c + G, c + 2G, ...
-    const int t_begin = XW ? (int)((int64_t)c * n_tiles / G) : c;
-    const int t_step = XW ? 1 : G;
-    const int my_tiles = XW ? (int)((int64_t)(c + 1) * n_tiles / G) - t_begin
-                            : (c < n_tiles ? (n_tiles - 1 - c) / G + 1 : 0);
+    const bool contig = XW || V.contig != 0;
+    const int t_begin = contig ? (int)((int64_t)c * n_tiles / G) : c;
+    const int t_step = contig ? 1 : G;
+    const int my_tiles = contig ? (int)((int64_t)(c + 1) * n_tiles / G) - t_begin
+                                : (c < n_tiles ? (n_tiles - 1 - c) / G + 1 : 0);
     const int pro = my_tiles < S ? my_tiles : S;
     if (warp == NCW) {
         // ---------------- producer warp: one bulk copy per tile record ----------------
