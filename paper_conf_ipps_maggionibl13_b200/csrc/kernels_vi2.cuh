@@ -222,13 +222,12 @@ struct GatherS {
     __device__ __forceinline__ double operator()(int32_t o) const { return lds_f64(xr + ((uint32_t)o << 3)); }
 };
 struct GatherW {     // ring without the mirror: one conditional wrap per entry
-    uint32_t xs;     // ring base
-    uint32_t rx;     // ring index of row r before the wrap (the tile's rows lie in [0, 2 rows))
-    uint32_t rows;
+    uint32_t xr;     // shared-window address of row r before the wrap
+    int32_t lim;     // offsets o >= lim lie past the ring's end (X - ring index of row r)
+    uint32_t back;   // 8 X
     __device__ __forceinline__ double operator()(int32_t o) const {
-        uint32_t v = rx + (uint32_t)o;
-        v = v >= rows ? v - rows : v;
-        return lds_f64(xs + (v << 3));
+        const uint32_t a = xr + ((uint32_t)o << 3);
+        return lds_f64(o >= lim ? a - back : a);
     }
 };
 
@@ -635,7 +634,7 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, XWM ? 1 : Vi2Shape<NC
                     acc = vi2_acc<ENC>(meta.y, pv, pc, sdict, gx);
                     if (BAND) { xl = gx(-1); xu = gx(1); }
                 } else if (XWM == 2) {
-                    const GatherW gx{sxw, (uint32_t)(r + xo_t), (uint32_t)V.xw_rows};
+                    const GatherW gx{sxw + 8u * (uint32_t)(r + xo_t), V.xw_rows - (r + xo_t), 8u * (uint32_t)V.xw_rows};
                     x_r = gx(0);
                     acc = vi2_acc<ENC>(meta.y, pv, pc, sdict, gx);
                     if (BAND) { xl = gx(-1); xu = gx(1); }

@@ -155,3 +155,35 @@ def test_xw_auto_rule(cme, monkeypatch):
     m = cme.Matrix(len(s), r, c, v).pack()
     assert m.info().xwin_kb == 0
     m.close()
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("width,mu,irr", [(1024, 10, False), (4096, 10, True)])
+def test_cfg5_full_size_xw_parity(cme, oracle_mod, width, mu, irr):
+    """Config 5 at the sweep's size (n = 16 M rows, 160 M entries; BASELINE
+    configs[4]) on the kernel the sweep times -- the auto rule's x-window
+    kernel (mirrored ring at width 1 024, the wrap mode at width 4 096): one
+    SpMV on every row vs the oracle's C Jacobi step, the |a_jj|-weighted mass
+    invariant, and 40 iterations of the landscape vs the oracle (all host
+    threads)."""
+    import os
+    n = 16_000_000
+    r, c, v = W.banded_markov_fast(n, mu, width, irr, seed=1)
+    A = oracle_mod.ingest(n, r, c, v)
+    m = cme.Matrix(n, r, c, v).pack()
+    del r, c, v
+    f = m.info()
+    assert f.xwin_kb > 0 and f.records == 1 and f.compact == 1, (f.xwin_kb, f.records, f.compact)
+    x = W.random_start(n, 23)
+    m.set_opts(omega=1.0)
+    y = m.spmv(x)
+    assert_spmv_close(y, oracle_mod.jacobi_step(A, x, 1.0))
+    d = -A.diag
+    assert abs((d * y).sum() - (d * x).sum()) <= 1e-12 * (d * x).sum()
+    m.set_opts(omega=1.0, check_every=20, stag_tol=0.0)
+    p, st, it = m.solve(tol=0.0, max_iter=40)
+    ref = oracle_mod.jacobi_solve(A, omega=1.0, tol=0.0, check_every=20, max_iter=40, stag_tol=0.0,
+                                  nthreads=len(os.sched_getaffinity(0)))
+    assert it == ref.iters == 40
+    assert np.abs(p - ref.p).sum() <= 1e-12
+    m.close()
