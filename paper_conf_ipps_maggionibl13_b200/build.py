@@ -81,18 +81,23 @@ def up_to_date(lib: str = LIB, defines=()) -> bool:
     if not os.path.exists(lib) or not os.path.exists(_stamp(lib)):
         return False
     with open(_stamp(lib)) as f:
-        return f.read().strip() == source_hash(defines)
+        return f.read().strip() == source_hash(tuple(defines))
 
 
-def build(force: bool = False, verbose: bool = False, out: str | None = None, defines=()) -> str:
-    """Compile libcme.so (or `out` with extra -D`defines`, for kernel A/B builds)."""
+SANITIZE = ["-Xcompiler", "-fsanitize=address", "-Xcompiler", "-fsanitize=undefined", "-Xcompiler",
+            "-fno-omit-frame-pointer", "-Xcompiler", "-fno-sanitize-recover=undefined"]   # (nvcc splits -Xcompiler at commas)
+
+
+def build(force: bool = False, verbose: bool = False, out: str | None = None, defines=(), sanitize=False) -> str:
+    """Compile libcme.so (or `out` with extra -D`defines`, for kernel A/B builds;
+    `sanitize`: the host code instrumented with ASan + UBSan, tools/asan_host.py)."""
     lib = out or LIB
-    digest = source_hash(defines)
+    digest = source_hash(tuple(defines) + (("SANITIZE",) if sanitize else ()))
     if not force and up_to_date(lib, defines):
         return lib
     obj_dir = OBJ if out is None else OBJ + "_" + os.path.basename(out).replace(".so", "")
     os.makedirs(obj_dir, exist_ok=True)
-    common = _common_flags(defines)
+    common = _common_flags(defines) + (SANITIZE if sanitize else [])
 
     def compile_one(src):
         obj = os.path.join(obj_dir, os.path.basename(src) + ".o")
@@ -111,7 +116,8 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None, de
     with ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 1)) as ex:
         objs = list(ex.map(compile_one, _sources()))
     tmp = lib + f".tmp{os.getpid()}"
-    cmd = [nvcc()] + ARCH + ["-shared", "-o", tmp] + objs + ["-Xcompiler", "-fopenmp", "-lgomp", "-ldl"]
+    cmd = [nvcc()] + ARCH + ["-shared", "-o", tmp] + objs + ["-Xcompiler", "-fopenmp", "-lgomp", "-ldl"] + \
+        (SANITIZE if sanitize else [])
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stderr}")
@@ -125,4 +131,4 @@ if __name__ == "__main__":
     args = sys.argv[1:]
     out = args[args.index("--out") + 1] if "--out" in args else None
     defs = [a[2:] for a in args if a.startswith("-D")]
-    print(build(force="--force" in args, verbose="-v" in args, out=out, defines=defs))
+    print(build(force="--force" in args, verbose="-v" in args, out=out, defines=defs, sanitize="--sanitize" in args))

@@ -9,6 +9,8 @@
 #include <cuda_runtime.h>
 
 #include "cme_internal.h"
+
+#include <nvtx3/nvToolsExt.h>
 #include "comm.h"
 
 namespace cme {
@@ -135,10 +137,22 @@ bool valid(cme_matrix h, int min_stage) { return h && h->stage >= min_stage; }
 
 using namespace cme;
 
+namespace {
+// NVTX range per C-ABI call (host phases in nsys/ncu timelines; header-only
+// NVTX v3: a no-op unless a tool injects itself)
+struct NvtxRange {
+    explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange&) = delete;
+    NvtxRange& operator=(const NvtxRange&) = delete;
+};
+}  // namespace
+
 extern "C" {
 
 cme_status cme_matrix_create_coo_batch(int64_t n, int64_t nnz, const int32_t* row, const int32_t* col,
                                        const double* rates, int32_t batch, uint32_t flags, cme_matrix* out) {
+    NvtxRange nvtx_("cme_matrix_create_coo_batch");
     if (!out) return CME_ERR_INVALID_ARG;
     *out = nullptr;
     if (batch != 1 && batch != 2 && batch != 4 && batch != 8) {
@@ -159,6 +173,7 @@ cme_status cme_matrix_create_coo_batch(int64_t n, int64_t nnz, const int32_t* ro
 
 cme_status cme_matrix_create_coo(int64_t n, int64_t nnz, const int32_t* row, const int32_t* col,
                                  const double* rate, uint32_t flags, cme_matrix* out) {
+    NvtxRange nvtx_("cme_matrix_create_coo");
     if (!out) return CME_ERR_INVALID_ARG;
     *out = nullptr;
     return guarded([&] {
@@ -175,6 +190,7 @@ cme_status cme_matrix_create_coo(int64_t n, int64_t nnz, const int32_t* row, con
 
 cme_status cme_matrix_create_csr(int64_t n, const int64_t* row_ptr, const int32_t* col, const double* rate,
                                  uint32_t flags, cme_matrix* out) {
+    NvtxRange nvtx_("cme_matrix_create_csr");
     if (!out || !row_ptr || n <= 0 || n > INT32_MAX) return CME_ERR_INVALID_ARG;
     *out = nullptr;
     return guarded([&] {
@@ -190,6 +206,7 @@ cme_status cme_matrix_create_csr(int64_t n, const int64_t* row_ptr, const int32_
 }
 
 cme_status cme_reorder(cme_matrix h, int method, int64_t root) {
+    NvtxRange nvtx_("cme_reorder");
     if (!valid(h, 1)) return CME_ERR_INVALID_ARG;
     if (h->stage != 1) { set_error("cme_reorder must precede cme_pack"); return CME_ERR_BAD_STATE; }
     if (method < CME_ORDER_NONE || method > CME_ORDER_RCM) return CME_ERR_INVALID_ARG;
@@ -208,6 +225,7 @@ cme_status cme_reorder(cme_matrix h, int method, int64_t root) {
 }
 
 cme_status cme_set_permutation(cme_matrix h, const int32_t* new_to_old) {
+    NvtxRange nvtx_("cme_set_permutation");
     if (!valid(h, 1) || !new_to_old) return CME_ERR_INVALID_ARG;
     if (h->stage != 1) { set_error("cme_set_permutation must precede cme_pack"); return CME_ERR_BAD_STATE; }
     return guarded([&] {
@@ -225,6 +243,7 @@ cme_status cme_set_permutation(cme_matrix h, const int32_t* new_to_old) {
 }
 
 cme_status cme_pack(cme_matrix h, int format, const cme_pack_opts* opts) {
+    NvtxRange nvtx_("cme_pack");
     if (!valid(h, 1)) return CME_ERR_INVALID_ARG;
     if (h->stage == 3) { set_error("matrix already distributed"); return CME_ERR_BAD_STATE; }
     cme_pack_opts o = opts ? *opts : cme_pack_opts{32, 256, CME_BAND_AUTO, -1};
@@ -283,6 +302,7 @@ cme_status cme_set_solver_opts(cme_matrix h, const cme_solver_opts* o) {
 
 cme_status cme_jacobi_solve(cme_matrix h, const double* p0, double tol, int64_t max_iter, double* p_out,
                             int64_t* iters_out) {
+    NvtxRange nvtx_("cme_jacobi_solve");
     if (iters_out) *iters_out = 0;
     if (!h || !p_out || max_iter < 0 || std::isnan(tol)) return CME_ERR_INVALID_ARG;
     if (h->stage < 2 || !h->dev) { set_error("solve before pack/distribute"); return CME_ERR_BAD_STATE; }
@@ -291,6 +311,7 @@ cme_status cme_jacobi_solve(cme_matrix h, const double* p0, double tol, int64_t 
 
 cme_status cme_transient(cme_matrix h, const double* p0, double t, double eps, double* p_out,
                          int64_t* terms_out) {
+    NvtxRange nvtx_("cme_transient");
     if (terms_out) *terms_out = 0;
     if (!h || !p_out || !(t >= 0.0) || std::isinf(t) || !(eps > 0.0 && eps < 1.0)) return CME_ERR_INVALID_ARG;
     if (h->stage < 2 || !h->dev) { set_error("transient before pack/distribute"); return CME_ERR_BAD_STATE; }
@@ -315,24 +336,28 @@ cme_status cme_get_batch_report(cme_matrix h, cme_report* reports, int32_t count
 }
 
 cme_status cme_spmv(cme_matrix h, const double* x, double* y) {
+    NvtxRange nvtx_("cme_spmv");
     if (!h || !x || !y) return CME_ERR_INVALID_ARG;
     if (h->stage < 2 || !h->dev) return CME_ERR_BAD_STATE;
     return guarded([&] { return device_spmv(h, x, y); });
 }
 
 cme_status cme_solver_load(cme_matrix h, const double* p0) {
+    NvtxRange nvtx_("cme_solver_load");
     if (!h) return CME_ERR_INVALID_ARG;
     if (h->stage < 2 || !h->dev) return CME_ERR_BAD_STATE;
     return guarded([&] { return device_load(h, p0); });
 }
 
 cme_status cme_solver_run(cme_matrix h, int64_t blocks) {
+    NvtxRange nvtx_("cme_solver_run");
     if (!h || blocks < 0) return CME_ERR_INVALID_ARG;
     if (h->stage < 2 || !h->dev) return CME_ERR_BAD_STATE;
     return guarded([&] { return device_run(h, blocks); });
 }
 
 cme_status cme_solver_fetch(cme_matrix h, double* p_out) {
+    NvtxRange nvtx_("cme_solver_fetch");
     if (!h || !p_out) return CME_ERR_INVALID_ARG;
     if (h->stage < 2 || !h->dev) return CME_ERR_BAD_STATE;
     return guarded([&] { return device_fetch(h, p_out); });
@@ -458,6 +483,7 @@ cme_status cme_period(cme_matrix h, int64_t root, int64_t* out) {
 }
 
 cme_status cme_matrix_plan_partition(cme_matrix h, int nranks, int rank) {
+    NvtxRange nvtx_("cme_matrix_plan_partition");
     if (!h || nranks < 1 || rank < 0 || rank >= nranks) return CME_ERR_INVALID_ARG;
     if (h->stage < 2) { set_error("plan_partition needs a packed matrix"); return CME_ERR_BAD_STATE; }
     return guarded([&] {
@@ -471,6 +497,7 @@ cme_status cme_matrix_plan_partition(cme_matrix h, int nranks, int rank) {
 }
 
 cme_status cme_matrix_distribute(cme_matrix h, cme_comm c) {
+    NvtxRange nvtx_("cme_matrix_distribute");
     if (!h || !c) return CME_ERR_INVALID_ARG;
     if (h->stage < 2) { set_error("distribute needs a packed matrix"); return CME_ERR_BAD_STATE; }
     return guarded([&] {
@@ -491,6 +518,7 @@ cme_status cme_matrix_ipc_export(cme_matrix h, uint8_t* blob) {
 }
 
 cme_status cme_matrix_ipc_attach(cme_matrix h, const uint8_t* blobs) {
+    NvtxRange nvtx_("cme_matrix_ipc_attach");
     if (!h || !blobs) return CME_ERR_INVALID_ARG;
     if (h->stage != 3 || !h->dev) return CME_ERR_BAD_STATE;
     return guarded([&] { return device_ipc_attach(h, blobs); });
