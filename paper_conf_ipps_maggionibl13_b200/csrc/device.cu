@@ -143,6 +143,7 @@ struct Device {
     int64_t* vi2_rec_off = nullptr;
     // x window in shared memory (XW; single GPU): per tile
     // the iterate chunks it gathers, streamed with its record
+    bool vi2b = false;               // batched tile records (sell_vi2b_kernel, B > 1; vi2_* shape fields)
     int xw = 0;                      // 1 mirrored ring, 2 ring with a wrap per entry
     int2* xw_ch = nullptr;           // [vi2 tiles] {first chunk, end chunk} (monotone)
     int xw_rows = 0, xw_mirror = 0, xw_off = 0, xw_ring_bytes = 0;
@@ -186,7 +187,7 @@ struct Device {
         if (!h.empty()) CUDA_TRY(cudaMemcpy(p, h.data(), h.size() * sizeof(T), cudaMemcpyHostToDevice));
         return CME_OK;
     }
-    int step_grid() const { return vi2 ? vi2_grid : use_tma ? tma_grid : grid; }
+    int step_grid() const { return vi2 || vi2b ? vi2_grid : use_tma ? tma_grid : grid; }
 };
 
 // ------------------------------------------------------------------------------
@@ -682,6 +683,88 @@ static cme_status configure_vi2(Device& d, const Packed& P, bool f64 = false) {
     return CME_OK;
 }
 
+// Batched tile records (sell_vi2b_kernel): the B = 1
+// record with a B-wide inv_d block (member-minor per slot).
+static int64_t vi2b_record_bytes(const Packed& P, int ts, int B, bool band, bool rearr, int64_t t) {
+    const int64_t q0 = t * ts, q1 = std::min<int64_t>(q0 + ts, P.n_slices);
+    return vi2b_fixed_bytes(ts, B, band, rearr) + 4 * (P.slice_off[q1] - P.slice_off[q0]);
+}
+
+static void vi2b_build_records(const Packed& P, const Compact& C, int ts, int B, bool band, bool rearr,
+                               std::vector<unsigned char>& rec, std::vector<int64_t>& off) {
+    const int64_t nt = (P.n_slices + ts - 1) / ts;
+    off.assign(nt + 1, 0);
+    for (int64_t t = 0; t < nt; ++t) off[t + 1] = off[t] + vi2b_record_bytes(P, ts, B, band, rearr, t);
+    rec.assign((size_t)off[nt], 0);
+    const int kMeta = ((ts + 1) & ~1) * 8;
+    const int kRow = kMeta, kLoUp = kRow + (rearr ? ts * 32 : 0), kInv = kLoUp + (band ? ts * 128 : 0),
+              kEnt = kInv + ts * 256 * B;
+#pragma omp parallel for schedule(static)
+    for (int64_t t = 0; t < nt; ++t) {
+        unsigned char* R = rec.data() + off[t];
+        const int64_t q0 = t * ts, q1 = std::min<int64_t>(q0 + ts, P.n_slices);
+        const int64_t e0 = P.slice_off[q0];
+        for (int64_t q = q0; q < q1; ++q) {
+            const int32_t m[2] = {(int32_t)(P.slice_off[q] - e0), (int32_t)P.slice_w[q]};
+            std::memcpy(R + 8 * (q - q0), m, 8);
+            const int64_t sl0 = q * 32, ls0 = (q - q0) * 32;
+            if (rearr) std::memcpy(R + kRow + ls0, C.row8.data() + sl0, 32);
+            if (band) {
+                std::memcpy(R + kLoUp + 2 * ls0, C.loi.data() + sl0, 64);
+                std::memcpy(R + kLoUp + ts * 64 + 2 * ls0, C.upi.data() + sl0, 64);
+            }
+            std::memcpy(R + kInv + 8 * B * ls0, P.inv_d.data() + (size_t)sl0 * B, (size_t)256 * B);
+            const int64_t ne = P.slice_off[q + 1] - P.slice_off[q];
+            unsigned char* E = R + kEnt + 4 * (P.slice_off[q] - e0);
+            std::memcpy(E, C.vidx.data() + P.slice_off[q], 2 * ne);
+            std::memcpy(E + 2 * ne, C.col16.data() + P.slice_off[q], 2 * ne);
+        }
+    }
+}
+
+// Shape of the batched tile-record kernel (vi2b_warps: B = 2 16 warps, B = 4
+// 16, B = 8 15), the deepest ring (<= 4 stages) that fits one CTA per SM.
+// Auto (CME_VI2B = -1) only at B = 2, where it was measured faster on cfg4
+// (333 vs 375 us per iteration); B = 4 573 vs 563 and B = 8 1 676 vs 1 364
+// (the 404 KB tuple dictionary misses L1 either way) keep sell_vib_kernel.
+// CME_VI2B = 1 forces it at any B, 0 disables it.
+static cme_status configure_vi2b(Device& d, const Packed& P) {
+    d.vi2b = false;
+    const int want = env_int("CME_VI2B", -1);
+    if (want == 0 || d.B < 2 || d.nranks > 1 || (want < 0 && d.B != 2)) return CME_OK;
+    int dev = 0, smem_max = 0, sms = 0;
+    CUDA_TRY(cudaGetDevice(&dev));
+    CUDA_TRY(cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+    CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    const int cap = smem_max - 4096;
+    const int ncw = vi2b_warps(d.B, env_int("CME_VI2_WARPS", 0));
+    const int64_t nt = (P.n_slices + ncw - 1) / ncw;
+    int64_t mx = 0;
+    for (int64_t t = 0; t < nt; ++t) mx = std::max(mx, vi2b_record_bytes(P, ncw, d.B, d.band, d.rearr, t));
+    const int64_t stage = (mx + 127) / 128 * 128;
+    CUDA_TRY(vi2b_prepare(d.B, ncw, cap));
+    const int force_s = env_int("CME_VI2_STAGES", 0);
+    for (int st = force_s > 0 ? std::min(force_s, 8) : 4; st >= 2; --st) {
+        if (st * stage > cap) continue;
+        int occ = 0;
+        CUDA_TRY(vi2b_occupancy(d.B, ncw, (int)(st * stage), &occ));
+        if (occ < 1) continue;
+        d.vi2b = true;
+        d.vi2_ncw = ncw;
+        d.vi2_stages = st;
+        d.vi2_stage_bytes = (int)stage;
+        d.vi2_occ = occ;
+        d.vi2_tiles = nt;
+        d.vi2_grid = (int)std::min<int64_t>(nt, (int64_t)sms * occ);
+        if (env_int("CME_VI2_GRID", 0) > 0) d.vi2_grid = std::min(d.vi2_grid, env_int("CME_VI2_GRID", 0));
+        if (env_int("CME_VERBOSE", 0))
+            std::fprintf(stderr, "[cme] vi2b: B=%d warps=%d stages=%d stage_bytes=%d occ=%d grid=%d tiles=%lld\n", d.B,
+                         ncw, st, d.vi2_stage_bytes, occ, d.vi2_grid, (long long)nt);
+        return CME_OK;
+    }
+    return CME_OK;
+}
+
 // x-window plan (XW kernels) for tiles of ts slices:
 // per tile the iterate chunks (256 rows, chunk k = rows [256 k - xoff,
 // 256 k - xoff + 256) of the local x) holding its rows, band neighbours and
@@ -1161,6 +1244,8 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
             h->Cpt = Compact();
             if (was_tma && (s = configure_tma(*d, P)) != CME_OK) return fail(s);
         }
+        // the batch's tile records (single GPU)
+        if (d->use_tma && d->vi && !comm && h->nranks == 1 && (s = configure_vi2b(*d, P)) != CME_OK) return fail(s);
     }
     if ((s = configure_resident(*d, P, comm != nullptr || h->nranks > 1)) != CME_OK) return fail(s);
     if ((s = preload_kernels(B)) != CME_OK) return fail(s);
@@ -1213,6 +1298,13 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
                                      (long long)d->vi2_tiles, items.size());
                 }
             }
+        } else if (d->vi2b) {   // batched tile records + the tuple dictionary (read through L1)
+            UP(dict, h->Cpt.dict);
+            std::vector<unsigned char> rec;
+            std::vector<int64_t> roff;
+            vi2b_build_records(P, h->Cpt, d->vi2_ncw, d->B, d->band, d->rearr, rec, roff);
+            UP(vi2_rec, rec);
+            UP(vi2_rec_off, roff);
         } else if (d->vi) {
             std::vector<double> dict(h->Cpt.dict);
             if (d->B == 1) dict.resize(d->dict_bytes / 8, 0.0);   // (B = 1: staged in shared memory, 128-B padded)
@@ -1235,7 +1327,7 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
         }
     }
 #undef UP
-    d->part_blocks = std::max(std::max(d->grid, d->res_grid), grid_for(d->n_own));
+    d->part_blocks = std::max(std::max(std::max(d->grid, d->res_grid), grid_for(d->n_own)), d->step_grid());
     if ((s = d->alloc(d->partials, (size_t)d->part_blocks * B * kPartials)) != CME_OK) return fail(s);
     if ((s = d->alloc(d->gather, (size_t)d->nranks * B * 8)) != CME_OK) return fail(s);
     if ((s = d->alloc(d->local8, (size_t)B * 8)) != CME_OK) return fail(s);
@@ -1644,6 +1736,11 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
         } else
             CUDA_TRY(launch_vi2(V, d.vi2_ncw, d.vi2_grid, d.dict_bytes + d.vi2_stages * d.vi2_stage_bytes, d.band,
                                 d.rearr, check, d.vi2_f64 ? 2 : d.vi2_words ? 1 : 0, pdl, s));
+    } else if (d.vi2b) {
+        Vi2Args V{a, d.vi2_rec, d.vi2_rec_off, d.dict, d.vi2_tiles, d.vi2_stages, d.vi2_stage_bytes, 0,
+                  d.win_shift, d.tma_xpf};
+        CUDA_TRY(launch_vi2b(V, d.B, d.vi2_ncw, d.vi2_grid, d.vi2_stages * d.vi2_stage_bytes, d.band, d.rearr, check,
+                             pdl, s));
     } else if (d.use_tma && d.vi && d.B > 1) {
         ViArgs V{CptArgs{TmaArgs{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col,
                                  d.tma_contig, d.tma_xpf},
@@ -2105,9 +2202,9 @@ cme_status device_transient(cme_matrix_s* h, const double* p0, double t, double 
 void device_describe(const Device* d, cme_info* f) {
     if (!d) { f->kernel = -1; return; }
     f->kernel = d->format == CME_FMT_CSR ? 2 : d->use_res ? 3 : d->use_tma ? 1 : 0;
-    f->tma_warps = d->vi2 ? d->vi2_ncw : d->use_tma ? d->tma_ncw : 0;
-    f->tma_stages = d->vi2 ? d->vi2_stages : d->use_tma ? d->tma_stages : 0;
-    f->records = d->vi2 ? 1 : 0;
+    f->tma_warps = d->vi2 || d->vi2b ? d->vi2_ncw : d->use_tma ? d->tma_ncw : 0;
+    f->tma_stages = d->vi2 || d->vi2b ? d->vi2_stages : d->use_tma ? d->tma_stages : 0;
+    f->records = d->vi2 || d->vi2b ? 1 : 0;
     f->wf_steps = d->wf ? d->wf_s : 0;
     f->halo_fused = d->fused ? 1 : 0;
     f->xwin_kb = d->xw ? d->xw_ring_bytes / 1024 : 0;

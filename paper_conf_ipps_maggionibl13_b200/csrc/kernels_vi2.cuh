@@ -682,4 +682,161 @@ __global__ void __launch_bounds__(Vi2Shape<NCW>::kThreads, XWM ? 1 : Vi2Shape<NC
     if (fused) hs_finish(V.hs, G, a.stop);
 }
 
+
+// ---------------------------------------------------------------------------
+// Batched tile records (B = 2, 4, 8 rate sets on one pattern; DESIGN.md
+// sec. 9): sell_vib_kernel's arithmetic -- per entry the B-tuple of rates from
+// the dictionary (global memory, L1-cached) times the B-wide x gather, FMAs
+// in t order per member, row sum times inv_d -- over one contiguous record
+// per tile of TS slices:
+//   [meta | row8 | loi, upi | inv_d (B per slot, member-minor) | per slice:
+//    vidx[32 W], col16[32 W]]
+// (the B = 1 record with a B-wide inv_d block), moved by one bulk copy; inv_d
+// is read from shared memory.  Single-GPU packs.
+template <int TS, int B, bool BAND, bool REARR>
+struct Vi2bRec {
+    static constexpr int kMeta = ((TS + 1) & ~1) * 8;
+    static constexpr int kRow = kMeta;
+    static constexpr int kLoUp = kRow + (REARR ? TS * 32 : 0);
+    static constexpr int kInv = kLoUp + (BAND ? TS * 128 : 0);
+    static constexpr int kEnt = kInv + TS * 256 * B;
+};
+__host__ __device__ constexpr int vi2b_fixed_bytes(int ts, int b, bool band, bool rearr) {
+    return ((ts + 1) & ~1) * 8 + (rearr ? ts * 32 : 0) + (band ? ts * 128 : 0) + ts * 256 * b;
+}
+
+template <int NCW, int B>
+struct Vi2bShape {
+    static constexpr int kThreads = 32 * (NCW + 1);
+};
+
+template <int NCW, int B, bool BAND, bool REARR, bool CHECK>
+__global__ void __launch_bounds__(Vi2bShape<NCW, B>::kThreads, 1)
+    sell_vi2b_kernel(const __grid_constant__ Vi2Args V) {
+    using R = Vi2bRec<NCW, B, BAND, REARR>;
+    constexpr int U = Chunk<B>::U;   // entries whose loads are in flight together
+    const StepArgs& a = V.a;
+    pdl_trigger();
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ uint64_t full[8], empty[8];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int S = V.stages;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < S; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], NCW);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    const int G = gridDim.x, c = blockIdx.x;
+    const int n_tiles = (int)V.n_tiles;
+    const int my_tiles = c < n_tiles ? (n_tiles - 1 - c) / G + 1 : 0;
+    const int pro = my_tiles < S ? my_tiles : S;
+    unsigned char* stages = smem;
+    if (warp == NCW) {
+        // ---------------- producer warp: one bulk copy per tile record ----------------
+        const uint64_t pol = evict_first_policy();
+        int64_t o0 = 0, o1 = 0;
+        int s = 0;
+        uint32_t phase = 0;
+        bool waited = false;
+        for (int i = 0; i < my_tiles; ++i) {
+            const int l = i & 31;
+            if (l == 0 && i + lane < my_tiles) {   // offsets of tiles i .. i+31
+                const int t = c + (i + lane) * G;
+                o0 = __ldg(V.rec_off + t);
+                o1 = __ldg(V.rec_off + t + 1);
+            }
+            const int64_t b0 = __shfl_sync(0xffffffffu, o0, l), b1 = __shfl_sync(0xffffffffu, o1, l);
+            // the first S records were issued before the previous step ended
+            // (they are constant); the stop test precedes any ring reuse
+            if (i == pro && !waited) {
+                pdl_wait();
+                waited = true;
+                if (a.stop != nullptr && *a.stop) break;
+            }
+            if (i >= S) mbar_wait(&empty[s], phase ^ 1u);
+            if (lane == 0) {
+                const uint32_t bytes = (uint32_t)(b1 - b0);
+                if (V.xpf) {
+                    const int64_t t = c + (int64_t)i * G;
+                    const int64_t r0 = t * NCW * 32, r1 = min(r0 + NCW * 32, a.n_rows);
+                    if (r1 > r0) prefetch_l2(a.x + (a.own_off + r0) * B, (uint64_t)(r1 - r0) * 8 * B);
+                }
+                mbar_expect_tx(&full[s], bytes);
+                bulk_g2s(stages + (size_t)s * V.stage_bytes, V.rec + b0, bytes, &full[s], pol);
+            }
+            if (++s == S) { s = 0; phase ^= 1u; }
+        }
+        if (!waited) pdl_wait();
+        if (CHECK) cta_check_partials<NCW + 1, B>(CheckAcc<B>(), a.partials);
+        return;
+    }
+    // ---------------- consumer warps: one slice each per tile ----------------
+    pdl_wait();
+    if (a.stop != nullptr && *a.stop) {   // drain the prologue copies before exit
+        for (int i = 0; i < pro; ++i) mbar_wait(&full[i], 0u);
+        if (CHECK) cta_check_partials<NCW + 1, B>(CheckAcc<B>(), a.partials);
+        return;
+    }
+    CheckAcc<B> ck;
+    {
+        const double* xo = a.x + a.own_off * B;
+        double* yo = a.y + a.own_off * B;
+        const double* dict = V.dict;
+        const int n_rows = (int)a.n_rows, slice_end = (int)a.slice_end;
+        const uint32_t full0 = smem_u32(full), empty0 = smem_u32(empty);
+        const uint32_t st0 = smem_u32(stages), sbytes = (uint32_t)V.stage_bytes;
+        int s = 0;
+        uint32_t phase = 0;
+        int q = c * NCW + warp;
+        const int dq = G * NCW;
+        uint32_t st = st0;
+        for (int i = 0; i < my_tiles; ++i, q += dq) {
+            mbar_wait_a(full0 + 8 * s, phase);
+            const int slot = q * 32 + lane;
+            if (q < slice_end && slot < n_rows) {
+                const int2 meta = lds_v2(st + 8 * warp);   // {entry offset in the tile, width}
+                const int ls = warp * 32 + lane;
+                const int r = REARR ? ((slot >> V.win_shift) << V.win_shift) + (int)lds_u8(st + R::kRow + ls) : slot;
+                RowX<B, BAND> X;
+                X.load(xo, r);
+                double id[B];
+#pragma unroll
+                for (int b = 0; b < B; ++b) id[b] = lds_f64(st + R::kInv + 8 * (B * ls + b));
+                const uint32_t pv = st + R::kEnt + 4 * meta.x + 2 * lane, pc = pv + 64 * meta.y;
+                double acc[B];
+#pragma unroll
+                for (int b = 0; b < B; ++b) acc[b] = 0.0;
+                for (int t0 = 0; t0 < meta.y; t0 += U) {
+                    double xv[U][B], vv[U][B];
+#pragma unroll
+                    for (int u = 0; u < U; ++u)
+                        if (t0 + u < meta.y) {
+                            ld_vec<B>(xo + (int64_t)(r + lds_s16(pc + 64 * (t0 + u))) * B, xv[u]);
+                            ld_vec<B>(dict + (int64_t)lds_u16(pv + 64 * (t0 + u)) * B, vv[u]);
+                        }
+#pragma unroll
+                    for (int u = 0; u < U; ++u)
+                        if (t0 + u < meta.y)
+#pragma unroll
+                            for (int b = 0; b < B; ++b) acc[b] = fma(vv[u][b], xv[u][b], acc[b]);
+                }
+                double lo[B], up[B];
+                if (BAND) {
+                    ld_vec<B>(dict + (int64_t)lds_u16(st + R::kLoUp + 2 * ls) * B, lo);
+                    ld_vec<B>(dict + (int64_t)lds_u16(st + R::kLoUp + NCW * 64 + 2 * ls) * B, up);
+                }
+                finish_row_x<B, BAND, CHECK>(a, r, yo, acc, lo, up, id, a.pre_scale, ck, X);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive_a(empty0 + 8 * s);
+            st += sbytes;
+            if (++s == S) { s = 0; phase ^= 1u; st = st0; }
+        }
+    }
+    if (CHECK) cta_check_partials<NCW + 1, B>(ck, a.partials);
+}
+
 }  // namespace cme

@@ -68,6 +68,12 @@ cudaError_t launch_vi2(const Vi2Args& V, int ncw, int grid, int smem, bool band,
                        bool pdl, cudaStream_t s);
 cudaError_t vi2_prepare(int ncw, int smem);
 cudaError_t vi2_occupancy(int ncw, int smem, int* blocks_per_sm, int enc = 0);
+// batched tile records (step_vi2b.cu, B = 2, 4, 8)
+int vi2b_warps(int B, int force);
+cudaError_t launch_vi2b(const Vi2Args& V, int B, int ncw, int grid, int smem, bool band, bool rearr, bool check,
+                        bool pdl, cudaStream_t s);
+cudaError_t vi2b_prepare(int B, int ncw, int smem);
+cudaError_t vi2b_occupancy(int B, int ncw, int smem, int* blocks_per_sm);
 // the x-window variant (step_xw.cu): ncw = 16 or 30, enc 0 or 2
 cudaError_t launch_vi2_xw(const Vi2Args& V, int ncw, int grid, int smem, bool band, bool rearr, bool check, int enc,
                           int mode /* 1 mirrored ring, 2 wrap */, bool pdl, cudaStream_t s);

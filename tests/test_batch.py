@@ -117,8 +117,13 @@ def test_batch_errors():
 # ------------------------------------------------------------------ GPU -------
 
 KNOBS = [{"CME_TMA": "0"}, {"CME_TMA": "1", "CME_VI": "0"}, {"CME_TMA": "1", "CME_TMA_WARPS": "8", "CME_VI": "0"},
-         {"CME_TMA": "1"}, {"CME_TMA": "1", "CME_TMA_WARPS": "8"},
-         {"CME_TMA": "1", "CME_TMA_WARPS": "15"}]   # the last three: batched value index
+         {"CME_TMA": "1", "CME_VI2B": "0"}, {"CME_TMA": "1", "CME_TMA_WARPS": "8", "CME_VI2B": "0"},
+         {"CME_TMA": "1", "CME_TMA_WARPS": "15", "CME_VI2B": "0"},   # batched value index (sell_vib_kernel)
+         {"CME_TMA": "1"},                                            # auto: the records at B = 2
+         {"CME_TMA": "1", "CME_VI2B": "1"},                           # its tile records (sell_vi2b_kernel)
+         {"CME_TMA": "1", "CME_VI2B": "1", "CME_VI2_WARPS": "alt"},
+         {"CME_TMA": "1", "CME_VI2B": "1", "CME_VI2_GRID": "3", "CME_VI2_STAGES": "2"}]   # ring wraps many times
+ALT_WARPS = {2: "30", 4: "30", 8: "8"}   # sell_vi2b_kernel's second shape per B
 
 
 @pytest.mark.gpu
@@ -126,13 +131,21 @@ KNOBS = [{"CME_TMA": "0"}, {"CME_TMA": "1", "CME_VI": "0"}, {"CME_TMA": "1", "CM
 @pytest.mark.parametrize("knobs", KNOBS, ids=lambda k: ",".join(f"{a}={b}" for a, b in k.items()))
 def test_batch_spmv_and_landscape_parity(oracle_mod, monkeypatch, B, knobs):
     for k, v in knobs.items():
-        monkeypatch.setenv(k, v)
+        monkeypatch.setenv(k, ALT_WARPS[B] if v == "alt" else v)
     n, r, c, rates, As = batch_inputs(oracle_mod, toggle_members(26, B))
     m = cme.Matrix(n, r, c, rates).reorder(cme.CME_ORDER_RCM).pack()
-    assert m.info().kernel == (1 if knobs["CME_TMA"] == "1" else 0)
-    assert m.info().compact == (2 if knobs["CME_TMA"] == "1" and knobs.get("CME_VI") != "0" else 0)
+    f = m.info()
+    assert f.kernel == (1 if knobs["CME_TMA"] == "1" else 0)
+    assert f.compact == (2 if knobs["CME_TMA"] == "1" and knobs.get("CME_VI") != "0" else 0)
     if "CME_TMA_WARPS" in knobs:
-        assert m.info().tma_warps == int(knobs["CME_TMA_WARPS"])
+        assert f.tma_warps == int(knobs["CME_TMA_WARPS"])
+    records = knobs["CME_TMA"] == "1" and knobs.get("CME_VI") != "0" and (
+        knobs.get("CME_VI2B") == "1" or (knobs.get("CME_VI2B") is None and B == 2))
+    assert f.records == int(records), (f.records, knobs)
+    if knobs.get("CME_VI2_WARPS") == "alt":
+        assert f.tma_warps == int(ALT_WARPS[B])
+    if "CME_VI2_GRID" in knobs:
+        assert f.grid <= 3
     m.set_opts(omega=0.9, check_every=7, stag_tol=0.0)
     x = np.concatenate([W.random_start(n, 30 + b) for b in range(B)])
     y = m.spmv(x)
@@ -167,3 +180,23 @@ def test_batch_p0_and_device_vectors(oracle_mod):
         o = oracle_mod.jacobi_solve(As[b], p0=p0[b * n:(b + 1) * n].cpu().numpy(), omega=0.9, tol=0.0,
                                     check_every=50, max_iter=333, stag_tol=0.0)
         assert np.abs(out[b * n:(b + 1) * n] - o.p).sum() <= 1e-12
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("B", [2, 4, 8])
+def test_batch_records_bit_identical_to_sell_vib(oracle_mod, monkeypatch, B):
+    """The batched tile records (sell_vi2b_kernel) do sell_vib_kernel's
+    arithmetic exactly (same tuples, FMA order, row sum times inv_d): their
+    SpMVs agree bit for bit."""
+    n, r, c, rates, _ = batch_inputs(oracle_mod, toggle_members(30, B))
+    x = np.concatenate([W.random_start(n, 40 + b) for b in range(B)])
+    out = {}
+    for rec in ("0", "1"):
+        monkeypatch.setenv("CME_TMA", "1")
+        monkeypatch.setenv("CME_VI2B", rec)   # (1 forces the records at every B)
+        m = cme.Matrix(n, r, c, rates).reorder(cme.CME_ORDER_RCM).pack()
+        assert m.info().records == int(rec)
+        m.set_opts(omega=0.9)
+        out[rec] = m.spmv(x)
+        m.close()
+    assert np.array_equal(out["0"], out["1"])

@@ -1,5 +1,6 @@
-# vi2 shapes: stage depth for the 30-warp CTA, and ncu captures of the 30- and 16-warp kernels on cfg4
+# batched tile records (sell_vi2b_kernel): parity, then cfg4 B = 2/4/8 against sell_vib_kernel
 mkdir -p gpurun_out
-timeout 900 python tools/kbench.py --config cfg4_toggle_20m --blocks 10 "CME_VI2_WARPS=30" "CME_VI2_WARPS=30,CME_VI2_STAGES=5" "CME_VI2_WARPS=30,CME_VI2_STAGES=3" "CME_VI2_WARPS=16,CME_VI2_STAGES=2" 2>&1 | grep "^\["
-timeout 600 ncu --set full --import-source on --clock-control none -k regex:sell_vi2 -s 20 -c 1 -o gpurun_out/prof_vi2w30 python tools/kbench.py --config cfg4_toggle_20m --blocks 1 CME_VI2_WARPS=30 > gpurun_out/ncu_vi2w30.log 2>&1; tail -2 gpurun_out/ncu_vi2w30.log
-timeout 600 ncu --set full --import-source on --clock-control none -k regex:sell_vi2 -s 20 -c 1 -o gpurun_out/prof_vi2w16 python tools/kbench.py --config cfg4_toggle_20m --blocks 1 CME_VI2_WARPS=16 > gpurun_out/ncu_vi2w16.log 2>&1; tail -2 gpurun_out/ncu_vi2w16.log
+python paper_conf_ipps_maggionibl13_b200/build.py
+timeout 1500 python -m pytest tests/test_batch.py -q -p no:cacheprovider -x > gpurun_out/pytest_batch.log 2>&1; tail -3 gpurun_out/pytest_batch.log
+export CME_VERBOSE=1
+for b in 2 4 8; do timeout 900 python tools/kbench.py --config cfg4_toggle_20m --batch $b --blocks 5 "CME_VI2B=0" "" "CME_VI2_WARPS=$( [ $b = 2 ] && echo 16 || ( [ $b = 4 ] && echo 30 || echo 8 ) )" 2>&1 | grep "^\[\|rror" | grep -v "tma:" | tee -a gpurun_out/vi2b_kbench.txt; done
