@@ -769,11 +769,9 @@ static cme_status configure_vi2b(Device& d, const Packed& P) {
 // per tile the iterate chunks (256 rows, chunk k = rows [256 k - xoff,
 // 256 k - xoff + 256) of the local x) holding its rows, band neighbours and
 // gathered columns, as a suffix-min of the first and a prefix-max of the end
-// chunk so the producer streams every chunk once, in order.  Returns the ring
-// chunks a CTA needs with S stages in flight: tiles j-S+1 .. j are live when
-// tile j's chunks are issued (tile j-S has released its stage).
-static int64_t xw_plan(const Packed& P, int ts, bool band, int64_t own_off, int xoff, int64_t nx, int S,
-                       std::vector<int2>& ch, int64_t& span) {
+// chunk so the producer streams every chunk once, in order.
+static void xw_plan(const Packed& P, int ts, bool band, int64_t own_off, int xoff, int64_t nx,
+                    std::vector<int2>& ch) {
     const int64_t nt = (P.n_slices + ts - 1) / ts, n = P.n;
     std::vector<int64_t> lo(nt), hi(nt);
 #pragma omp parallel for schedule(dynamic, 64)
@@ -800,13 +798,19 @@ static int64_t xw_plan(const Packed& P, int ts, bool band, int64_t own_off, int 
     }
     for (int64_t t = nt - 2; t >= 0; --t) lo[t] = std::min(lo[t], lo[t + 1]);
     for (int64_t t = 1; t < nt; ++t) hi[t] = std::max(hi[t], hi[t - 1]);
+    ch.resize(nt);
+    for (int64_t t = 0; t < nt; ++t) ch[t] = make_int2((int)lo[t], (int)hi[t]);
+}
+
+// Ring chunks a CTA needs with S stages in flight: tiles j-S+1 .. j are live
+// when tile j's chunks are issued (tile j-S has released its stage); and the
+// widest tile's chunk count (the mirror).
+static int64_t xw_need(const std::vector<int2>& ch, int S, int64_t& span) {
     int64_t need = 1;
     span = 1;
-    ch.resize(nt);
-    for (int64_t t = 0; t < nt; ++t) {
-        need = std::max(need, hi[t] - lo[std::max<int64_t>(0, t - S + 1)]);
-        span = std::max(span, hi[t] - lo[t]);
-        ch[t] = make_int2((int)lo[t], (int)hi[t]);
+    for (int64_t t = 0; t < (int64_t)ch.size(); ++t) {
+        need = std::max<int64_t>(need, ch[t].y - ch[std::max<int64_t>(0, t - S + 1)].x);
+        span = std::max<int64_t>(span, ch[t].y - ch[t].x);
     }
     return need;
 }
@@ -871,6 +875,7 @@ static cme_status configure_xw(Device& d, const Packed& P, bool f64, std::vector
     const int64_t nx = d.nx - d.own_off;
     const int64_t ring_cap = want > 0 ? INT64_MAX : (int64_t)env_int("CME_XW_RING_KB", 160) << 10;
     int64_t stage_of[2] = {0, 0};   // [30 warps, 16 warps]
+    std::vector<int2> plan_of[2];   // chunk ranges per tile, by warp count
     // (8-warp tiles, for windows too wide for these: measured 587 vs 420 us on
     // config 5 width 8 192 -- too few warps once the gathers are shared loads)
     const int order[6][2] = {{30, 4}, {30, 3}, {16, 4}, {16, 3}, {30, 2}, {16, 2}};
@@ -891,9 +896,10 @@ static cme_status configure_xw(Device& d, const Packed& P, bool f64, std::vector
             CUDA_TRY(vi2_xw_prepare(ncw, cap));
         }
         {
-            std::vector<int2> ch;
+            std::vector<int2>& ch = plan_of[ncw == 30 ? 0 : 1];
+            if (ch.empty()) xw_plan(P, ncw, d.band, d.own_off, xoff, nx, ch);
             int64_t span = 1;
-            const int64_t need = xw_plan(P, ncw, d.band, d.own_off, xoff, nx, st, ch, span);
+            const int64_t need = xw_need(ch, st, span);
             const int64_t slots = need, mirror = mode == 1 ? span - 1 : 0;
             const int64_t bytes = dict + st * stage + (slots + mirror) * 2048;
             if (env_int("CME_VERBOSE", 0) > 1)
@@ -920,7 +926,7 @@ static cme_status configure_xw(Device& d, const Packed& P, bool f64, std::vector
             d.xw_off = xoff;
             d.xw_nx = nx;
             d.xw_ring_bytes = (int)((slots + mirror) * 2048);
-            plan.swap(ch);
+            plan = ch;
             if (env_int("CME_VERBOSE", 0))
                 std::fprintf(stderr, "[cme] xw: mode=%d warps=%d stages=%d stage_bytes=%d ring=%d KB occ=%d grid=%d tiles=%lld\n",
                              mode, ncw, st, d.vi2_stage_bytes, d.xw_ring_bytes / 1024, occ, d.vi2_grid, (long long)nt);
