@@ -849,7 +849,7 @@ static double gather_sectors(const Packed& P) {
 // x gathers are uncoalesced (>= 16 sectors per warp request) with a ring of at
 // most CME_XW_RING_KB (160) KB.  Measured (B200): config 5
 // (16 M rows, mu = 10, random band) width 1 024 291 us vs 410 on
-// sell_cpt_kernel, width 4 096 356 vs 643; coalesced gathers lose: cfg3a
+// sell_cpt_kernel, width 4 096 330 vs 640 (wrap mode); coalesced gathers lose: cfg3a
 // 28.7 vs 19.1 us, toggle N = 2 200 (RCM) 133 vs 79 us.
 static cme_status configure_xw(Device& d, const Packed& P, bool f64, std::vector<int2>& plan) {
     d.xw = 0;
