@@ -282,6 +282,18 @@ cme_status cme_export_compact(cme_matrix h, cme_compact_view* v);
 /* Directed period of the ingested graph from `root` (R1); host-only. */
 cme_status cme_period(cme_matrix h, int64_t root, int64_t* period_out);
 
+/* The x-window plan of a packed single-GPU DIAG_SELL
+ * matrix (B = 1; a CME_DEVICE_HOST_ONLY pack suffices) for tiles of `ncw`
+ * slices with `stages` records in flight -- host logic exported for tests.
+ * Iterate chunk k = local rows [256 k - 1, 256 k + 255).  plan[2 t], plan[2 t + 1]
+ * (caller-allocated, 2 * tiles int32, tiles = ceil(n_slices / ncw)) receive tile
+ * t's chunk range [first, end): every row, band neighbour and gathered column of
+ * the tile lies in it; both ends are non-decreasing in t.  *need = the ring
+ * chunks a CTA needs (max over t of end(t) - first(t - stages + 1)), *span =
+ * the widest tile's chunk count.  BAD_STATE before pack or when distributed. */
+cme_status cme_export_xw_plan(cme_matrix h, int32_t ncw, int32_t stages, int64_t tiles, int32_t* plan,
+                              int64_t* need, int64_t* span);
+
 /* ---- multi-GPU -------------------------------------------- */
 /* Rank 0 creates the id; it is broadcast over the caller's process group
  * (torch.distributed) and every rank calls cme_comm_init.  NCCL is loaded

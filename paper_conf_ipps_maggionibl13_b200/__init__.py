@@ -120,6 +120,7 @@ _SIGS = {
     "cme_get_permutation": [vp, i32p],
     "cme_export_packed": [vp, _p(cme_packed_view)],
     "cme_period": [vp, C.c_int64, i64p],
+    "cme_export_xw_plan": [vp, C.c_int32, C.c_int32, C.c_int64, i32p, i64p, i64p],
     "cme_export_compact": [vp, _p(cme_compact_view)],
     "cme_comm_unique_id": [u8p],
     "cme_comm_init": [C.c_int, C.c_int, u8p, C.c_int, _p(vp)],
@@ -348,6 +349,16 @@ def cme_period(h, root=0):
     g = C.c_int64()
     _chk(_lib.cme_period(h, root, C.byref(g)), "cme_period")
     return g.value
+
+
+def cme_export_xw_plan(h, ncw, stages, n_slices):
+    """The x-window chunk plan (tiles x 2 int32), ring chunks needed, widest tile."""
+    tiles = (n_slices + ncw - 1) // ncw
+    plan = np.zeros(2 * tiles, np.int32)
+    need, span = C.c_int64(0), C.c_int64(0)
+    _chk(_lib.cme_export_xw_plan(h, ncw, stages, tiles, plan.ctypes.data_as(i32p), C.byref(need), C.byref(span)),
+         "cme_export_xw_plan")
+    return plan.reshape(tiles, 2), need.value, span.value
 
 
 def cme_comm_unique_id() -> bytes:

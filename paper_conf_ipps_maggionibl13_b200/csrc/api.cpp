@@ -477,6 +477,24 @@ cme_status cme_export_compact(cme_matrix h, cme_compact_view* v) {
     });
 }
 
+cme_status cme_export_xw_plan(cme_matrix h, int32_t ncw, int32_t stages, int64_t tiles, int32_t* plan,
+                              int64_t* need, int64_t* span) {
+    if (!h || !plan || !need || !span || ncw < 1 || ncw > 64 || stages < 1 || stages > 8) return CME_ERR_INVALID_ARG;
+    if (h->stage != 2 || h->format != CME_FMT_DIAG_SELL || h->P.B != 1 || h->nranks > 1) {
+        set_error("x-window plan: a packed single-GPU DIAG_SELL matrix with B = 1");
+        return CME_ERR_BAD_STATE;
+    }
+    const int64_t nt = (h->P.n_slices + ncw - 1) / ncw;
+    if (tiles != nt) { set_error("x-window plan: tiles must be ceil(n_slices / ncw)"); return CME_ERR_INVALID_ARG; }
+    return guarded([&] {
+        std::vector<int2> ch;
+        xw_plan(h->P, ncw, h->P.band_on != 0, 0, 1, h->P.n, ch);
+        *need = xw_need(ch, stages, *span);
+        for (int64_t t = 0; t < nt; ++t) { plan[2 * t] = ch[t].x; plan[2 * t + 1] = ch[t].y; }
+        return CME_OK;
+    });
+}
+
 cme_status cme_period(cme_matrix h, int64_t root, int64_t* out) {
     if (!h || !out || h->stage < 1 || root < 0 || root >= h->A.n) return CME_ERR_INVALID_ARG;
     return guarded([&] { *out = directed_period(h->A, root); return CME_OK; });

@@ -86,6 +86,12 @@ bool encode_compact(const Packed& P, int64_t own_off, Compact& C);
 // Value-index P's layout-v0 values into C (needs C.valid); false when the
 // pack holds more than 65536 distinct values.
 bool encode_value_index(const Packed& P, Compact& C);
+// x-window plan (device.cu): per tile of ts slices the
+// monotone chunk range [ch.x, ch.y) of 256-row iterate chunks (chunk k = rows
+// [256 k - xoff, 256 k - xoff + 256)); xw_need = ring chunks with S stages in
+// flight, span = the widest tile's chunk count.
+void xw_plan(const Packed& P, int ts, bool band, int64_t own_off, int xoff, int64_t nx, std::vector<int2>& ch);
+int64_t xw_need(const std::vector<int2>& ch, int S, int64_t& span);
 
 struct Device;  // device state (device.cu)
 

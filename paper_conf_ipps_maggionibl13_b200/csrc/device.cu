@@ -770,8 +770,8 @@ static cme_status configure_vi2b(Device& d, const Packed& P) {
 // 256 k - xoff + 256) of the local x) holding its rows, band neighbours and
 // gathered columns, as a suffix-min of the first and a prefix-max of the end
 // chunk so the producer streams every chunk once, in order.
-static void xw_plan(const Packed& P, int ts, bool band, int64_t own_off, int xoff, int64_t nx,
-                    std::vector<int2>& ch) {
+void xw_plan(const Packed& P, int ts, bool band, int64_t own_off, int xoff, int64_t nx,
+             std::vector<int2>& ch) {
     const int64_t nt = (P.n_slices + ts - 1) / ts, n = P.n;
     std::vector<int64_t> lo(nt), hi(nt);
 #pragma omp parallel for schedule(dynamic, 64)
@@ -805,7 +805,7 @@ static void xw_plan(const Packed& P, int ts, bool band, int64_t own_off, int xof
 // Ring chunks a CTA needs with S stages in flight: tiles j-S+1 .. j are live
 // when tile j's chunks are issued (tile j-S has released its stage); and the
 // widest tile's chunk count (the mirror).
-static int64_t xw_need(const std::vector<int2>& ch, int S, int64_t& span) {
+int64_t xw_need(const std::vector<int2>& ch, int S, int64_t& span) {
     int64_t need = 1;
     span = 1;
     for (int64_t t = 0; t < (int64_t)ch.size(); ++t) {

@@ -254,3 +254,59 @@ def test_info_bytes_model(oracle_mod):
     assert f.band_on == 1 and f.band_density > 0.99
     assert 0.9 < f.ell_efficiency <= 1.0
     assert f.bytes_fmt < f.bytes_alg                     # DIA band + separate diagonal save bytes
+
+
+def _xw_case(name):
+    if name == "banded-w300-irregular":
+        n = 30000
+        r, c, v = W.banded_markov(n, 10, 300, True, seed=5)
+        return cme.Matrix(n, r, c, v), cme.CME_ORDER_NONE
+    net = {"toggle90": W.toggle_switch(90), "schnakenberg40": W.schnakenberg(40)}[name]
+    s, r, c, v = cme.cme_network_enumerate(net)
+    return cme.Matrix(len(s), r, c, v), cme.CME_ORDER_RCM if name == "toggle90" else cme.CME_ORDER_NONE
+
+
+@pytest.mark.parametrize("name", ["banded-w300-irregular", "toggle90", "schnakenberg40"])
+@pytest.mark.parametrize("ncw,stages", [(16, 2), (16, 3), (30, 4)])
+def test_xw_plan_invariants(name, ncw, stages):
+    """The x-window plan, checked against the packed layout
+    it is derived from: every row, band neighbour and gathered column of a tile
+    lies in the tile's chunk range (chunk k = rows [256k - 1, 256k + 255)); both
+    ends are monotone; and a replay of the producer -- tiles issued in order,
+    `stages` records in flight, chunks written to slot k mod need -- never
+    overwrites a chunk a live tile still reads."""
+    m, order = _xw_case(name)
+    m.reorder(order).pack(cme.CME_FMT_DIAG_SELL, 256, cme.CME_BAND_AUTO, cme.CME_DEVICE_HOST_ONLY)
+    P = m.packed()
+    plan, need, span = cme.cme_export_xw_plan(m.h, ncw, stages, P["n_slices"])
+    lo, hi = plan[:, 0].astype(np.int64), plan[:, 1].astype(np.int64)
+    n, T = P["n"], len(plan)
+    assert np.all(np.diff(lo) >= 0) and np.all(np.diff(hi) >= 0) and np.all(hi > lo)
+    chunk = lambda rows: (np.asarray(rows, np.int64) + 1) >> 8   # noqa: E731
+    for t in range(T):
+        q0, q1 = t * ncw, min((t + 1) * ncw, P["n_slices"])
+        slots = np.arange(q0 * 32, min(q1 * 32, n))
+        rows = P["row_of"][slots].astype(np.int64) if P["row_of"].size else slots
+        need_rows = [rows]
+        if P["band_on"]:
+            need_rows += [np.maximum(rows - 1, -1), np.minimum(rows + 1, n - 1)]
+        e0, e1 = P["slice_off"][q0], P["slice_off"][q1]
+        need_rows.append(P["col"][e0:e1])
+        k = chunk(np.concatenate(need_rows))
+        assert k.min() >= lo[t] and k.max() < hi[t], (t, k.min(), k.max(), lo[t], hi[t])
+    ref_need = max(hi[t] - lo[max(0, t - stages + 1)] for t in range(T))
+    assert need == max(1, ref_need) and span == max(1, int((hi - lo).max()))
+    # replay: ring of `need` slots, slot -> chunk currently held
+    held = {}
+    issued = lo[0]
+    for j in range(T):
+        oldest = lo[max(0, j - stages + 1)]   # tiles j-stages+1 .. j are live
+        while issued < hi[j]:
+            slot = issued % need
+            prev = held.get(slot)
+            assert prev is None or prev < oldest, (j, issued, prev, oldest)
+            held[slot] = issued
+            issued += 1
+        for kk in range(lo[j], hi[j]):       # tile j reads chunks it finds in place
+            assert held.get(kk % need) == kk
+    m.close()
