@@ -80,7 +80,8 @@ for cfg in a.configs.split(","):
         torch.cuda.synchronize()
         ti = e0.elapsed_time(e1) * 1e-3 / (100 * a.blocks)
         row = dict(config=cfg, variant=name, order=order, n=f.n, nnz=f.nnz, band_on=bool(f.band_on),
-                   ell_efficiency=round(f.ell_efficiency, 4), kernel=int(f.kernel),
+                   ell_efficiency=round(f.ell_efficiency, 4), kernel=int(f.kernel), encoding=int(f.compact),
+                   records=int(f.records), xwin_kb=int(f.xwin_kb),
                    packed_mib=round(f.packed_bytes / 2 ** 20, 2), bytes_fmt=f.bytes_fmt,
                    us_per_iter=round(ti * 1e6, 2), gflops=round(2 * f.nnz / ti / 1e9, 1),
                    alg_gbs=round(f.bytes_alg / ti / 1e9, 1), pct_peak=round(100 * f.bytes_alg / ti / 1e9 / PEAK, 1),
