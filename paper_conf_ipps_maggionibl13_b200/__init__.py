@@ -353,12 +353,12 @@ def cme_period(h, root=0):
 
 def cme_export_xw_plan(h, ncw, stages, n_slices):
     """The x-window chunk plan (tiles x 2 int32), ring chunks needed, widest tile."""
-    tiles = (n_slices + ncw - 1) // ncw
-    plan = np.zeros(2 * tiles, np.int32)
+    tiles = (n_slices + ncw - 1) // ncw if ncw > 0 else 0   # (the library rejects ncw < 1)
+    plan = np.zeros(max(2 * tiles, 2), np.int32)
     need, span = C.c_int64(0), C.c_int64(0)
     _chk(_lib.cme_export_xw_plan(h, ncw, stages, tiles, plan.ctypes.data_as(i32p), C.byref(need), C.byref(span)),
          "cme_export_xw_plan")
-    return plan.reshape(tiles, 2), need.value, span.value
+    return plan[:2 * tiles].reshape(tiles, 2), need.value, span.value
 
 
 def cme_comm_unique_id() -> bytes:

@@ -310,3 +310,24 @@ def test_xw_plan_invariants(name, ncw, stages):
         for kk in range(lo[j], hi[j]):       # tile j reads chunks it finds in place
             assert held.get(kk % need) == kk
     m.close()
+
+
+def test_xw_plan_errors():
+    s, r, c, v = cme.cme_network_enumerate(W.toggle_switch(20))
+    m = cme.Matrix(len(s), r, c, v)
+    with pytest.raises(cme.CmeError) as e:          # before pack
+        cme.cme_export_xw_plan(m.h, 16, 3, 1)
+    assert e.value.status == cme.CME_ERR_BAD_STATE
+    m.pack(device=cme.CME_DEVICE_HOST_ONLY)
+    ns = m.packed()["n_slices"]
+    buf = np.zeros(2 * (ns + 7), np.int32)
+    need, span = cme.C.c_int64(), cme.C.c_int64()
+    st = cme._lib.cme_export_xw_plan(m.h, 16, 3, ns + 7, buf.ctypes.data_as(cme.i32p), cme.C.byref(need),
+                                     cme.C.byref(span))
+    assert st == cme.CME_ERR_INVALID_ARG            # tiles must be ceil(n_slices / ncw)
+    with pytest.raises(cme.CmeError) as e:          # ncw out of range
+        cme.cme_export_xw_plan(m.h, 0, 3, ns)
+    assert e.value.status == cme.CME_ERR_INVALID_ARG
+    plan, need, span = cme.cme_export_xw_plan(m.h, 16, 3, ns)
+    assert plan.shape == ((ns + 15) // 16, 2) and need >= span >= 1
+    m.close()
