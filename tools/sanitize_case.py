@@ -31,9 +31,13 @@ KNOBS = [
     ("vi2-16", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_VI2_WARPS": "16"}),
     ("vi2-words", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_VI2_WORDS": "1"}),
     ("vi2-grid2", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_VI": "1", "CME_VI2_GRID": "2"}),
+    # x window in shared memory (sell_vi2_kernel XWM 1 / 2): mirrored ring and
+    # wrap mode, capped grid so each CTA's ring wraps
+    ("xw-mirror", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_XW": "1", "CME_XW_MODE": "1", "CME_VI2_GRID": "3"}),
+    ("xw-wrap", {"CME_TMA": "1", "CME_RESIDENT": "0", "CME_XW": "1", "CME_XW_MODE": "2", "CME_VI2_GRID": "3"}),
     ("resident", {"CME_TMA": "-1", "CME_RESIDENT": "1"}),
 ]
-ALL_KEYS = sorted({k for _, kn in KNOBS for k in kn} | {"CME_TMA_WARPS", "CME_VI2_WARPS"})
+ALL_KEYS = sorted({k for _, kn in KNOBS for k in kn} | {"CME_TMA_WARPS", "CME_VI2_WARPS", "CME_XW", "CME_VI2B"})
 
 
 def set_knobs(kn):
@@ -55,10 +59,11 @@ for label, knobs in KNOBS:
               float(p.sum()), terms, flush=True)
         m.close()
 
-# batches: the batched value-indexed kernel (B = 2 default shape, B = 8 on 15-warp tiles)
+# batches: the batched tile records (B = 2 default, B = 4 forced) and the
+# batched value-indexed kernel (B = 8 on 15-warp tiles)
 states, r, c, v = cme.cme_network_enumerate(W.toggle_switch(20))
-for B, warps in ((2, None), (8, "15")):
-    set_knobs({"CME_TMA": "1", "CME_RESIDENT": "-1"} | ({"CME_TMA_WARPS": warps} if warps else {}))
+for B, warps, extra in ((2, None, {}), (8, "15", {}), (4, None, {"CME_VI2B": "1"})):
+    set_knobs({"CME_TMA": "1", "CME_RESIDENT": "-1"} | ({"CME_TMA_WARPS": warps} if warps else {}) | extra)
     vs = np.stack([v * (1.0 + 0.1 * b) for b in range(B)])
     m = cme.Matrix(len(states), r, c, vs).reorder(cme.CME_ORDER_RCM).pack()
     m.set_opts(omega=0.9, check_every=10)
