@@ -144,6 +144,7 @@ struct Device {
     // x window in shared memory (XW; single GPU): per tile
     // the iterate chunks it gathers, streamed with its record
     bool vi2b = false;               // batched tile records (sell_vi2b_kernel, B > 1; vi2_* shape fields)
+    int vi2b_dict_bytes = 0;         // > 0: its tuple dictionary staged in shared memory (B = 2)
     int xw = 0;                      // 1 mirrored ring, 2 ring with a wrap per entry
     int2* xw_ch = nullptr;           // [vi2 tiles] {first chunk, end chunk} (monotone)
     int xw_rows = 0, xw_mirror = 0, xw_off = 0, xw_ring_bytes = 0;
@@ -728,8 +729,9 @@ static void vi2b_build_records(const Packed& P, const Compact& C, int ts, int B,
 // (333 vs 375 us per iteration); B = 4 573 vs 563 and B = 8 1 676 vs 1 364
 // (the 404 KB tuple dictionary misses L1 either way) keep sell_vib_kernel.
 // CME_VI2B = 1 forces it at any B, 0 disables it.
-static cme_status configure_vi2b(Device& d, const Packed& P) {
+static cme_status configure_vi2b(Device& d, const Packed& P, int64_t dict_doubles) {
     d.vi2b = false;
+    d.vi2b_dict_bytes = 0;
     const int want = env_int("CME_VI2B", -1);
     if (want == 0 || d.B < 2 || d.nranks > 1 || (want < 0 && d.B != 2)) return CME_OK;
     int dev = 0, smem_max = 0, sms = 0;
@@ -744,12 +746,23 @@ static cme_status configure_vi2b(Device& d, const Packed& P) {
     const int64_t stage = (mx + 127) / 128 * 128;
     CUDA_TRY(vi2b_prepare(d.B, ncw, cap));
     const int force_s = env_int("CME_VI2_STAGES", 0);
+    // B = 2 on 16-warp tiles: the tuple dictionary in shared memory when it fits
+    // beside >= 3 stages (CME_VI2B_SD = 0 keeps it in global memory)
+    const int64_t sd = d.B == 2 && ncw == 16 && env_int("CME_VI2B_SD", 1) != 0 ? (dict_doubles * 8 + 127) / 128 * 128 : 0;
+    // first the staged-dictionary shapes (>= 3 stages), then the L1 ones
+    for (int pass = sd > 0 ? 0 : 1; pass < 2; ++pass)
     for (int st = force_s > 0 ? std::min(force_s, 8) : 4; st >= 2; --st) {
-        if (st * stage > cap) continue;
+        const int64_t dict = pass == 0 ? sd : 0;
+        if (pass == 0 && st < 3 && force_s <= 0) continue;
+        if (dict + st * stage > cap) continue;
         int occ = 0;
-        CUDA_TRY(vi2b_occupancy(d.B, ncw, (int)(st * stage), &occ));
+        CUDA_TRY(vi2b_occupancy(d.B, ncw, (int)(dict + st * stage), &occ));
+        if (env_int("CME_VERBOSE", 0) > 1)
+            std::fprintf(stderr, "[cme] vi2b shape: stages=%d stage=%lld dict=%lld (tuples %lld doubles) occ=%d\n", st,
+                         (long long)stage, (long long)dict, (long long)dict_doubles, occ);
         if (occ < 1) continue;
         d.vi2b = true;
+        d.vi2b_dict_bytes = (int)dict;
         d.vi2_ncw = ncw;
         d.vi2_stages = st;
         d.vi2_stage_bytes = (int)stage;
@@ -758,8 +771,8 @@ static cme_status configure_vi2b(Device& d, const Packed& P) {
         d.vi2_grid = (int)std::min<int64_t>(nt, (int64_t)sms * occ);
         if (env_int("CME_VI2_GRID", 0) > 0) d.vi2_grid = std::min(d.vi2_grid, env_int("CME_VI2_GRID", 0));
         if (env_int("CME_VERBOSE", 0))
-            std::fprintf(stderr, "[cme] vi2b: B=%d warps=%d stages=%d stage_bytes=%d occ=%d grid=%d tiles=%lld\n", d.B,
-                         ncw, st, d.vi2_stage_bytes, occ, d.vi2_grid, (long long)nt);
+            std::fprintf(stderr, "[cme] vi2b: B=%d warps=%d stages=%d stage_bytes=%d dict_smem=%d occ=%d grid=%d tiles=%lld\n",
+                         d.B, ncw, st, d.vi2_stage_bytes, d.vi2b_dict_bytes, occ, d.vi2_grid, (long long)nt);
         return CME_OK;
     }
     return CME_OK;
@@ -1251,7 +1264,8 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
             if (was_tma && (s = configure_tma(*d, P)) != CME_OK) return fail(s);
         }
         // the batch's tile records (single GPU)
-        if (d->use_tma && d->vi && !comm && h->nranks == 1 && (s = configure_vi2b(*d, P)) != CME_OK) return fail(s);
+        if (d->use_tma && d->vi && !comm && h->nranks == 1 && (s = configure_vi2b(*d, P, (int64_t)h->Cpt.dict.size())) != CME_OK)
+            return fail(s);
     }
     if ((s = configure_resident(*d, P, comm != nullptr || h->nranks > 1)) != CME_OK) return fail(s);
     if ((s = preload_kernels(B)) != CME_OK) return fail(s);
@@ -1304,8 +1318,10 @@ cme_status device_upload(cme_matrix_s* h, int want_dev, const HaloPlan* halo, cm
                                      (long long)d->vi2_tiles, items.size());
                 }
             }
-        } else if (d->vi2b) {   // batched tile records + the tuple dictionary (read through L1)
-            UP(dict, h->Cpt.dict);
+        } else if (d->vi2b) {   // batched tile records + the tuple dictionary (L1, or staged: 128-B padded)
+            std::vector<double> dict(h->Cpt.dict);
+            if (d->vi2b_dict_bytes > 0) dict.resize(d->vi2b_dict_bytes / 8, 0.0);
+            UP(dict, dict);
             std::vector<unsigned char> rec;
             std::vector<int64_t> roff;
             vi2b_build_records(P, h->Cpt, d->vi2_ncw, d->B, d->band, d->rearr, rec, roff);
@@ -1743,10 +1759,10 @@ static cme_status launch_step(Device& d, cudaStream_t s, int src, int dst, bool 
             CUDA_TRY(launch_vi2(V, d.vi2_ncw, d.vi2_grid, d.dict_bytes + d.vi2_stages * d.vi2_stage_bytes, d.band,
                                 d.rearr, check, d.vi2_f64 ? 2 : d.vi2_words ? 1 : 0, pdl, s));
     } else if (d.vi2b) {
-        Vi2Args V{a, d.vi2_rec, d.vi2_rec_off, d.dict, d.vi2_tiles, d.vi2_stages, d.vi2_stage_bytes, 0,
-                  d.win_shift, d.tma_xpf};
-        CUDA_TRY(launch_vi2b(V, d.B, d.vi2_ncw, d.vi2_grid, d.vi2_stages * d.vi2_stage_bytes, d.band, d.rearr, check,
-                             pdl, s));
+        Vi2Args V{a, d.vi2_rec, d.vi2_rec_off, d.dict, d.vi2_tiles, d.vi2_stages, d.vi2_stage_bytes,
+                  d.vi2b_dict_bytes, d.win_shift, d.tma_xpf};
+        CUDA_TRY(launch_vi2b(V, d.B, d.vi2_ncw, d.vi2_grid, d.vi2b_dict_bytes + d.vi2_stages * d.vi2_stage_bytes, d.band,
+                             d.rearr, check, pdl, s));
     } else if (d.use_tma && d.vi && d.B > 1) {
         ViArgs V{CptArgs{TmaArgs{a, d.n_tiles, d.tma_stages, d.tma_stage_bytes, d.tma_off_val, d.tma_off_col,
                                  d.tma_contig, d.tma_xpf},

@@ -15,15 +15,15 @@ int vi2b_warps(int B, int force) {
     return force == 8 ? 8 : 15;
 }
 
-template <int W, int B>
+template <int W, int B, bool SD = false>
 static cudaError_t launch_w(const Vi2Args& V, int grid, int smem, bool band, bool rearr, bool check, bool pdl,
                             cudaStream_t s) {
     const int key = (band ? 4 : 0) | (rearr ? 2 : 0) | (check ? 1 : 0);
     switch (key) {
 #define K_(bd, r, c)                                                                                           \
     case bd * 4 + r * 2 + c:                                                                                   \
-        return launch_ex(sell_vi2b_kernel<W, B, bd, r, c>, dim3(grid), dim3(Vi2bShape<W, B>::kThreads), smem, pdl, \
-                         s, V);
+        return launch_ex(sell_vi2b_kernel<W, B, bd, r, c, SD>, dim3(grid), dim3(Vi2bShape<W, B>::kThreads), smem, \
+                         pdl, s, V);
         K_(0, 0, 0) K_(0, 0, 1) K_(0, 1, 0) K_(0, 1, 1) K_(1, 0, 0) K_(1, 0, 1) K_(1, 1, 0) K_(1, 1, 1)
 #undef K_
     }
@@ -32,6 +32,9 @@ static cudaError_t launch_w(const Vi2Args& V, int grid, int smem, bool band, boo
 
 cudaError_t launch_vi2b(const Vi2Args& V, int B, int ncw, int grid, int smem, bool band, bool rearr, bool check,
                         bool pdl, cudaStream_t s) {
+    const bool sd = V.dict_bytes > 0;   // the tuple dictionary in shared memory (B = 2, 16 warps)
+    if (B == 2 && sd) return ncw == 16 ? launch_w<16, 2, true>(V, grid, smem, band, rearr, check, pdl, s)
+                                       : cudaErrorInvalidValue;
     if (B == 2) return ncw == 16 ? launch_w<16, 2>(V, grid, smem, band, rearr, check, pdl, s)
                                  : launch_w<30, 2>(V, grid, smem, band, rearr, check, pdl, s);
     if (B == 4) return ncw == 30 ? launch_w<30, 4>(V, grid, smem, band, rearr, check, pdl, s)
@@ -41,18 +44,23 @@ cudaError_t launch_vi2b(const Vi2Args& V, int B, int ncw, int grid, int smem, bo
     return cudaErrorInvalidValue;
 }
 
-template <int W, int B>
+template <int W, int B, bool SD = false>
 static cudaError_t prepare_w(int smem) {
     cudaError_t e = cudaSuccess;
 #define A_(bd, r, c)                                                                                       \
     if (e == cudaSuccess)                                                                                  \
-        e = cudaFuncSetAttribute(sell_vi2b_kernel<W, B, bd, r, c>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        e = cudaFuncSetAttribute(sell_vi2b_kernel<W, B, bd, r, c, SD>, cudaFuncAttributeMaxDynamicSharedMemorySize, \
+                                 smem);
     A_(0, 0, 0) A_(0, 0, 1) A_(0, 1, 0) A_(0, 1, 1) A_(1, 0, 0) A_(1, 0, 1) A_(1, 1, 0) A_(1, 1, 1)
 #undef A_
     return e;
 }
 
 cudaError_t vi2b_prepare(int B, int ncw, int smem) {
+    if (B == 2 && ncw == 16) {
+        const cudaError_t e = prepare_w<16, 2, true>(smem);
+        if (e != cudaSuccess) return e;
+    }
     if (B == 2) return ncw == 16 ? prepare_w<16, 2>(smem) : prepare_w<30, 2>(smem);
     if (B == 4) return ncw == 30 ? prepare_w<30, 4>(smem) : prepare_w<16, 4>(smem);
     if (B == 8) return ncw == 8 ? prepare_w<8, 8>(smem) : prepare_w<15, 8>(smem);

@@ -121,6 +121,7 @@ KNOBS = [{"CME_TMA": "0"}, {"CME_TMA": "1", "CME_VI": "0"}, {"CME_TMA": "1", "CM
          {"CME_TMA": "1", "CME_TMA_WARPS": "15", "CME_VI2B": "0"},   # batched value index (sell_vib_kernel)
          {"CME_TMA": "1"},                                            # auto: the records at B = 2
          {"CME_TMA": "1", "CME_VI2B": "1"},                           # its tile records (sell_vi2b_kernel)
+         {"CME_TMA": "1", "CME_VI2B": "1", "CME_VI2B_SD": "0"},       # (B = 2: tuples through L1, not staged)
          {"CME_TMA": "1", "CME_VI2B": "1", "CME_VI2_WARPS": "alt"},
          {"CME_TMA": "1", "CME_VI2B": "1", "CME_VI2_GRID": "3", "CME_VI2_STAGES": "2"}]   # ring wraps many times
 ALT_WARPS = {2: "30", 4: "30", 8: "8"}   # sell_vi2b_kernel's second shape per B
